@@ -1,0 +1,209 @@
+"""Pins for oracle steps O12-O14: boundary flux (paper-literal Fig. 2/3 transcription,
+delta currents, symmetry, linearity, self-term invariance), the interior Grad-Shafranov
+solve (exact discrete Solov'ev identity, manufactured solutions, O(h^2) consistency with
+the free-space Green's sum) and the fit iteration (twin fixed point)."""
+import math
+
+import numpy as np
+import pytest
+
+import synth
+
+MU0 = 4e-7 * math.pi
+
+
+@pytest.fixture(scope="module")
+def g17(oracle_mod):
+    cfg = synth.small_config(17)
+    return cfg, oracle_mod.Oracle.from_config(cfg)
+
+
+def test_literal_fig2_equals_plain_sum(oracle_mod, g17):
+    """or_pflux_literal (Fig. 2/3 loops, + the second nest, Q2) returns -sum G I."""
+    cfg, orc = g17
+    I = synth.random_current(cfg.grid, seed=3, signed=True)
+    psib = orc.boundary(I)
+    lit = orc.pflux_literal(I)
+    edge = orc.edge_nodes()
+    vals = np.array([lit[i * cfg.grid.nh + j] for i, j in edge])
+    np.testing.assert_allclose(-vals, psib, rtol=0, atol=1e-14 * np.abs(psib).max())
+    # interior entries untouched
+    mask = np.ones(cfg.grid.n, bool)
+    mask[[i * cfg.grid.nh + j for i, j in edge]] = False
+    assert np.all(lit[mask] == 0)
+
+
+def test_boundary_delta_current(oracle_mod, g17):
+    """I = delta at an interior node g => psi_b(p) = G(x_p; x_g) from the plain formula."""
+    cfg, orc = g17
+    ii, jj = 5, 9
+    I = np.zeros(cfg.grid.n); I[ii * cfg.grid.nh + jj] = 1.0
+    psib = orc.boundary(I)
+    R, Z = cfg.grid.r(), cfg.grid.z()
+    for p, (i, j) in enumerate(orc.edge_nodes()):
+        ref = oracle_mod.green_psi(R[i], Z[j], R[ii], Z[jj])
+        assert abs(psib[p] - ref) <= 1e-14 * abs(ref)
+
+
+def test_boundary_updown_symmetry_and_linearity(oracle_mod, g17):
+    cfg, orc = g17
+    nw, nh = cfg.grid.nw, cfg.grid.nh
+    I = synth.random_current(cfg.grid, seed=2).reshape(nw, nh)
+    Isym = (I + I[:, ::-1]).reshape(-1)
+    psib = orc.boundary(Isym)
+    left, right = psib[:nh], psib[nh:2 * nh]
+    bot, top = psib[2 * nh:2 * nh + nw - 2], psib[2 * nh + nw - 2:]
+    np.testing.assert_allclose(left, left[::-1], rtol=1e-14)
+    np.testing.assert_allclose(right, right[::-1], rtol=1e-14)
+    np.testing.assert_allclose(bot, top, rtol=1e-14)
+    I1 = synth.random_current(cfg.grid, seed=8, signed=True)
+    I2 = synth.random_current(cfg.grid, seed=9, signed=True)
+    a, b, ab = orc.boundary(I1), orc.boundary(I2), orc.boundary(0.3 * I1 - 1.7 * I2)
+    np.testing.assert_allclose(ab, 0.3 * a - 1.7 * b, rtol=0, atol=1e-14 * np.abs(ab).max())
+
+
+def test_boundary_memo_equals_direct(oracle_mod, g17):
+    cfg, orc = g17
+    I = synth.random_current(cfg.grid, seed=3, signed=True)
+    psib = orc.boundary(I)
+    tg = list(range(orc.n_edge))
+    direct = orc.boundary_targets(I, tg)
+    np.testing.assert_allclose(direct, psib, rtol=0, atol=1e-15 * np.abs(psib).max())
+
+
+def test_self_term_never_reaches_results(oracle_mod):
+    """Q5: perturbing G_self by 10% changes no output when the edge ring carries no current."""
+    cfg = synth.small_config(17)
+    a = oracle_mod.Oracle.from_config(cfg)
+    b = oracle_mod.Oracle.from_config(cfg)
+    b.set_self_scale(1.1)
+    I = synth.random_current(cfg.grid, seed=2)
+    assert np.array_equal(a.boundary(I), b.boundary(I))
+    T1, T2 = a.table_T(), b.table_T()
+    assert not np.array_equal(T1, T2)
+
+
+# ------------------------------------------------------------------ interior solve (O13)
+
+@pytest.mark.parametrize("n", [9, 33, 65])
+def test_apply_gs_exact_solovev(oracle_mod, n):
+    """Delta*_h [A R^2 Z^2 + B (R^2-R0^2)^2 + C Z^2] = (2A+8B) R^2 + 2C - 2 B dR^2 exactly."""
+    cfg = synth.small_config(n)
+    orc = oracle_mod.Oracle.from_config(cfg)
+    A, B, C, R0 = 1.2346, 1.0, 0.05, 1.67
+    psi = synth.solovev_poly(cfg.grid, A, B, C, R0)
+    out = orc.apply_gs(psi).reshape(n, n)
+    R = cfg.grid.r()
+    exp = (2 * A + 8 * B) * R ** 2 + 2 * C - 2 * B * cfg.grid.dr ** 2
+    inner = out[1:-1, 1:-1]
+    np.testing.assert_allclose(inner, np.broadcast_to(exp[1:-1, None], inner.shape), rtol=2e-11)
+
+
+@pytest.mark.parametrize("n", [9, 33, 65])
+def test_solve_recovers_solovev(oracle_mod, n):
+    """Exact discrete identity => solve(I from the Solov'ev RHS, edge values of psi_S) = psi_S."""
+    cfg = synth.small_config(n)
+    orc = oracle_mod.Oracle.from_config(cfg)
+    A, B, C, R0 = 1.2346, 1.0, 0.05, 1.67
+    psi = synth.solovev_poly(cfg.grid, A, B, C, R0)
+    R = np.repeat(cfg.grid.r(), n)
+    rhs = np.tile(((2 * A + 8 * B) * cfg.grid.r() ** 2 + 2 * C - 2 * B * cfg.grid.dr ** 2)[:, None], (1, n)).reshape(-1)
+    I = -rhs * cfg.grid.dr * cfg.grid.dz / (MU0 * R)
+    psib = np.array([psi[i * n + j] for i, j in orc.edge_nodes()])
+    sol = orc.interior_solve(I, psib)
+    assert np.max(np.abs(sol - psi)) <= 1e-12 * np.max(np.abs(psi))
+
+
+def test_solve_manufactured_random(oracle_mod):
+    cfg = synth.small_config(33)
+    orc = oracle_mod.Oracle.from_config(cfg)
+    n = 33
+    psi = np.random.default_rng(11).standard_normal(n * n)
+    lap = orc.apply_gs(psi)
+    R = np.repeat(cfg.grid.r(), n)
+    I = -lap * cfg.grid.dr * cfg.grid.dz / (MU0 * R)
+    psib = np.array([psi[i * n + j] for i, j in orc.edge_nodes()])
+    sol = orc.interior_solve(I, psib)
+    assert np.max(np.abs(sol - psi)) <= 1e-11 * np.max(np.abs(psi))
+
+
+def test_solve_continuous_solovev_order2(oracle_mod):
+    """Continuous Solov'ev RHS (no -2B dR^2 term) => error vs psi_S is O(h^2)."""
+    A, B, C, R0 = 1.2346, 1.0, 0.05, 1.67
+    errs = []
+    for n in [17, 33, 65]:
+        cfg = synth.small_config(n)
+        orc = oracle_mod.Oracle.from_config(cfg)
+        psi = synth.solovev_poly(cfg.grid, A, B, C, R0)
+        R = np.repeat(cfg.grid.r(), n)
+        rhs = (2 * A + 8 * B) * R ** 2 + 2 * C
+        I = -rhs * cfg.grid.dr * cfg.grid.dz / (MU0 * R)
+        psib = np.array([psi[i * n + j] for i, j in orc.edge_nodes()])
+        errs.append(np.max(np.abs(orc.interior_solve(I, psib) - psi)))
+    r1, r2 = errs[0] / errs[1], errs[1] / errs[2]
+    assert 3.6 < r1 < 4.4 and 3.6 < r2 < 4.4
+
+
+def test_green_sum_consistent_with_solve(oracle_mod):
+    """Free-space flux of a smooth current (sum_g G I_g at interior nodes, the same G as the
+    boundary step) vs the interior solve fed with that boundary: agreement improves ~h^2.
+    Pins the relative sign and scale of O12 and O13 (mu0, dR dZ, R weighting)."""
+    errs = []
+    for n in [17, 33, 65]:
+        cfg = synth.small_config(n)
+        orc = oracle_mod.Oracle.from_config(cfg)
+        R, Z = cfg.grid.r()[:, None], cfg.grid.z()[None, :]
+        J = np.exp(-((R - 1.7) ** 2 + (Z / 1.5) ** 2) / 0.08)
+        I = (J * cfg.grid.dr * cfg.grid.dz).reshape(-1)
+        T = orc.table_T()  # T[i][ii][m] = G(R_i, m dZ; R_ii, 0)
+        nh = n
+        idx = np.abs(np.arange(nh)[:, None] - np.arange(nh)[None, :])
+        full = np.einsum("iajb,ab->ij", T[:, :, idx], I.reshape(n, n))
+        psib = orc.boundary(I)
+        sol = orc.interior_solve(I, psib).reshape(n, n)
+        errs.append(np.max(np.abs(sol - full)) / np.max(np.abs(full)))
+    assert errs[0] < 0.05
+    assert errs[1] < errs[0] / 3 and errs[2] < errs[1] / 3
+
+
+# ------------------------------------------------------------------ fit iteration (O14)
+
+@pytest.fixture(scope="module")
+def twin33(oracle_mod):
+    cfg = synth.small_config(33)
+    orc = oracle_mod.Oracle.from_config(cfg)
+    psi_s = synth.solovev_psi(cfg.grid)
+    ct = synth.c_true(cfg.basis)
+    tw = orc.twin(psi_s, ct)
+    return cfg, orc, psi_s, ct, tw
+
+
+def test_twin_is_fixed_point(oracle_mod, twin33):
+    cfg, orc, psi_s, ct, tw = twin33
+    st, psi, coef, chi2, eps = orc.fit_step(psi_s, tw["psi_ext"], tw["y"], tw["sigma"])
+    assert st == 0
+    assert np.max(np.abs(psi - psi_s)) <= 1e-12 * np.max(np.abs(psi_s))
+    # coefficient error relative to max|c| (scaled cond(A) ~ 3e3 for the 2+3 basis)
+    assert np.max(np.abs(coef - ct) / np.abs(ct).max()) < 1e-10
+    assert chi2 < 1e-10
+    assert eps < 1e-11
+
+
+def test_twin_perturbed_converges(oracle_mod):
+    """Full loop (iterate until the max psi residual < eps = 1e-5) from a
+    0.1%-perturbed psi_S on 65^2 with the 2+3 basis converges in ~10 iterations."""
+    cfg = synth.small_config(65)
+    orc = oracle_mod.Oracle.from_config(cfg)
+    psi_s = synth.solovev_psi(cfg.grid)
+    tw = orc.twin(psi_s, synth.c_true(cfg.basis))
+    psi = synth.perturbed_psi(cfg.grid, seed=5, rel=1e-3)
+    epss = []
+    for it in range(60):
+        st, psi, coef, chi2, eps = orc.fit_step(psi, tw["psi_ext"], tw["y"], tw["sigma"])
+        assert st == 0
+        epss.append(eps)
+        if eps < 1e-5:
+            break
+    assert epss[-1] < 1e-5, epss
+    # converges to a nearby discrete fixed point (the mask is piecewise constant in psi)
+    assert np.max(np.abs(psi - psi_s)) < 1e-2 * np.max(np.abs(psi_s))
