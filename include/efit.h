@@ -1,0 +1,190 @@
+/*
+ * efit.h -- C ABI of the B200-native EFIT fitting-iteration hot path
+ *           (library: paper_conf_sc_anteparawkbml23_b200/libefit_b200.so, sm_100a).
+ *
+ * The method is the per-iteration Green's-function work of EFIT's fitting call fit_
+ * (Antepara et al., SC-W 2023; "P:L<n>" = /root/reference/PAPER.md line n):
+ *   green_   diagnostic response of each current basis function
+ *   current_ toroidal current on the grid, Eq. (2)
+ *   pflux_   computational-boundary flux (the O(N^3) nests of Fig. 2/3,
+ *            P:L187, L205-L230, L259-L285) + interior Grad-Shafranov solve, Eq. (1)
+ *   steps_   normalised flux and plasma boundary
+ *   fit_     one Picard iteration, convergence max|dpsi| < eps
+ *
+ * Conventions (every call):
+ *   - fp64 (IEEE binary64) everywhere; SI units (m, A, Wb/rad, T); mu0 = 4 pi 1e-7.
+ *   - Uniform grid R_i = rmin + i dR, Z_j = zmin + j dZ, i < nw, j < nh; node index
+ *     g = i*nh + j (Z fastest), the paper's (ii-1)*nh+jj flattening.
+ *   - psi is poloidal flux per radian.  pcurr is amperes per grid cell.
+ *   - Edge ("computational boundary") order, n_edge = 2*nh + 2*(nw-2):
+ *       left i=0, j=0..nh-1 | right i=nw-1, j=0..nh-1 | bottom j=0, i=1..nw-2 | top j=nh-1, i=1..nw-2
+ *   - Diagnostic (response row) order: flux loops | magnetic probes | internal B_Z points.
+ *   - Basis column order: n_pp P' terms (weight R) | n_ff FF' terms (weight mu0/(4 pi^2 R)).
+ *
+ * Memory & ownership: every d_* pointer is caller-owned DEVICE memory on the context's
+ *   device, 16-byte aligned, never freed by the library.  Host arrays passed to
+ *   efit_green_init are copied before it returns.  The workspace (all Green's tables
+ *   and scratch) is caller-allocated device memory of efit_workspace_bytes() bytes
+ *   that must stay alive until efit_destroy().
+ * Asynchrony: compute calls only enqueue work on `stream` (a cudaStream_t; NULL = the
+ *   legacy default stream) and never synchronise the host.  Outputs are valid once the
+ *   stream reaches the call.  Data-dependent failures (empty plasma mask, singular
+ *   least-squares matrix, non-finite input) are recorded in a device status word and
+ *   reported by efit_status(); the affected outputs are set to NaN.
+ * Errors: arguments are validated on the host before any launch; a failing call returns
+ *   a negative EFIT_E_* code, launches nothing and leaves outputs untouched.
+ *   efit_last_error() gives a one-line reason.  A context is not thread-safe.
+ * Multi-GPU (efit_dist.world > 1): each rank owns a contiguous slice of the targets
+ *   (boundary rows i, response rows m); see efit_shard().  The compute calls write only
+ *   the rank's slice of d_resp / d_psib; the caller exchanges the slices.
+ */
+#ifndef EFIT_H
+#define EFIT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct efit_ctx efit_ctx;
+typedef void* efit_stream_t; /* cudaStream_t */
+
+/* Uniform R-Z grid.  Requires 3 <= nw, nh <= 4097, 0 < rmin < rmax, zmin < zmax. */
+typedef struct {
+    int32_t nw, nh;
+    double rmin, rmax, zmin, zmax;
+} efit_grid;
+
+/* Current-density basis for P'(psihat) and FF'(psihat), Eq. (2).
+ * kind 0: monomials psihat^k, k = 0..n-1.  kind 1: clamped cubic B-splines on the knot
+ * vector {0,0,0,0, knots[0..n_knots-1], 1,1,1,1} (knots strictly increasing in (0,1));
+ * then n_pp = n_ff = n_knots + 4.  1 <= n_pp + n_ff <= 24.  knots: host array, copied. */
+typedef struct {
+    int32_t kind;
+    int32_t n_pp, n_ff;
+    int32_t n_knots;
+    const double* knots;
+} efit_basis;
+
+/* Machine geometry (host arrays, copied).  Flux loops measure psi; magnetic probes measure
+ * B_R cos(ang) + B_Z sin(ang); internal points measure B_Z.  No diagnostic may sit on a
+ * grid node.  The limiter is a closed polygon (vertices not repeated), n_lim >= 3.
+ * ip_sign = +1 if psi is maximal on the magnetic axis (positive plasma current), -1 otherwise. */
+typedef struct {
+    int32_t n_fl;  const double *fl_r, *fl_z;
+    int32_t n_mp;  const double *mp_r, *mp_z, *mp_ang;
+    int32_t n_int; const double *int_r, *int_z;
+    int32_t n_lim; const double *lim_r, *lim_z;
+    int32_t ip_sign;
+} efit_geometry;
+
+/* Target sharding across `world` ranks (one process per GPU).  {0, 1} = single GPU. */
+typedef struct {
+    int32_t rank, world;
+} efit_dist;
+
+/* Sizes derived from the configuration (filled by efit_info). */
+typedef struct {
+    int32_t nw, nh, ndiag, nbasis, n_edge;
+    int32_t mode;
+    int32_t rank, world;
+    int32_t resp_row_lo, resp_row_hi;   /* this rank's response rows [lo, hi)          */
+    int32_t bnd_row_lo, bnd_row_hi;     /* this rank's top/bottom target rows i [lo, hi) */
+    int32_t lr_blk_lo, lr_blk_hi;       /* this rank's left/right source blocks          */
+    int64_t slab_stride;                /* doubles between Green's-table slabs           */
+    size_t workspace_bytes;
+} efit_info_t;
+
+enum { EFIT_GREEN_TABLE = 0, EFIT_GREEN_ONTHEFLY = 1 };
+
+enum {
+    EFIT_OK = 0,
+    EFIT_E_INVAL = -1,     /* bad argument (host-side validation)                 */
+    EFIT_E_NOMEM = -2,     /* workspace too small / host allocation failed        */
+    EFIT_E_CUDA = -3,      /* CUDA runtime error (possibly from earlier async work) */
+    EFIT_E_NCCL = -4,      /* reserved for the collective layer                    */
+    EFIT_E_SINGULAR = -5,  /* least-squares: |R_kk| < 1e-13 max|R_jj|              */
+    EFIT_E_NOPLASMA = -6,  /* empty plasma mask / psi_axis == psi_bdry             */
+    EFIT_E_NONFINITE = -7, /* NaN/Inf met in a reduction                           */
+    EFIT_E_STATE = -8      /* call not valid in this context state / mode          */
+};
+
+/* Bytes of device workspace efit_green_init needs for this configuration. */
+int efit_workspace_bytes(const efit_grid* grid, const efit_basis* basis,
+                         const efit_geometry* geom, const efit_dist* dist, int mode,
+                         size_t* bytes_out);
+
+/* Validate, carve the workspace and build every Green's table on `stream` (the
+ * precomputed gridpc of P:L217-L221 re-laid out as T[i][ii][m] = G(R_i, m dZ; R_ii, 0),
+ * m fastest, plus the diagnostic tables Gd[m][g]).  mode = EFIT_GREEN_ONTHEFLY skips T
+ * and recomputes G inside efit_boundary_flux.  On success *out owns host state only. */
+int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit_basis* basis,
+                    const efit_geometry* geom, const efit_dist* dist, int mode,
+                    void* d_workspace, size_t ws_bytes, efit_stream_t stream);
+
+int efit_info(const efit_ctx* ctx, efit_info_t* info);
+
+/* steps_ + green_: psi_axis/psi_bdry from d_psi[nw*nh], then
+ * d_resp[m*nbasis + k] = sum_g Gd[m][g] dR dZ mask_g w_k(R_g) phi_k(psihat_g)
+ * for this rank's rows m (all rows if world == 1).  d_axbd[2] (may be NULL) receives
+ * {psi_axis, psi_bdry}. */
+int efit_response(efit_ctx* ctx, const double* d_psi, double* d_resp, double* d_axbd,
+                  efit_stream_t stream);
+
+/* current_ (Eq. (2)): d_pcurr[g] = dR dZ mask_g sum_k coef_k w_k(R_g) phi_k(psihat_g)
+ * with the mask and psihat of d_psi. */
+int efit_current(efit_ctx* ctx, const double* d_psi, const double* d_coef, double* d_pcurr,
+                 efit_stream_t stream);
+
+/* pflux_ O(N^3) part (Fig. 2/3): d_psib[p] = sum_g G(x_p; x_g) d_pcurr[g] for the
+ * n_edge edge nodes p in the edge order above, physical sign (+; the paper stores the
+ * negated sum).  The self term G(x_p; x_p) is the point-to-cell average
+ * (reading Q5).  world > 1: only this rank's targets are written. */
+int efit_boundary_flux(efit_ctx* ctx, const double* d_pcurr, double* d_psib,
+                       efit_stream_t stream);
+
+/* pflux_ O(N^2) part, Eq. (1): solve Delta*_h psi = -mu0 R pcurr/(dR dZ) on the interior
+ * nodes (5-point operator, reading Q17) with psi = d_psib on the edge.
+ * Writes all nw*nh nodes of d_psi_p. */
+int efit_interior_solve(efit_ctx* ctx, const double* d_pcurr, const double* d_psib,
+                        double* d_psi_p, efit_stream_t stream);
+
+/* Weighted least squares: minimise sum_m ((meas_m - sum_k resp_mk c_k)/sigma_m)^2
+ * over all ndiag rows.  d_coef[nbasis], d_chi2[1]. */
+int efit_lsq(efit_ctx* ctx, const double* d_resp, const double* d_meas, const double* d_sigma,
+             double* d_coef, double* d_chi2, efit_stream_t stream);
+
+/* fit_: one Picard iteration, entirely on the device (a captured CUDA graph
+ * after the first call with the same pointers):
+ *   response(psi) -> lsq -> current -> boundary flux -> interior solve ->
+ *   psi <- psi_p + d_psi_ext (in place);  d_eps[0] = max|psi_new - psi_old| / |psi_bdry - psi_axis|.
+ * d_meas: measurements with the external-coil contribution already removed.
+ * world > 1 is not supported by this fused call (EFIT_E_STATE): use the step calls. */
+int efit_fit_step(efit_ctx* ctx, double* d_psi, const double* d_psi_ext, const double* d_meas,
+                  const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps,
+                  efit_stream_t stream);
+
+/* Synchronise `stream` and return the first data-dependent failure recorded since the last
+ * efit_status() call (EFIT_OK, EFIT_E_NOPLASMA, EFIT_E_SINGULAR, EFIT_E_NONFINITE), or
+ * EFIT_E_CUDA.  Clears the status word. */
+int efit_status(efit_ctx* ctx, efit_stream_t stream);
+
+/* Test/inspection access: device pointers into the workspace.  which = 0: T (slab i at
+ * T + (i - bnd_row_lo_or_0)*slab_stride, see efit_info), 1: Gd (row m at Gd + (m-resp_row_lo)*slab_stride),
+ * 2: in-limiter flags (uint8[nw*nh]).  Returns EFIT_E_STATE if the table is not built. */
+int efit_table(const efit_ctx* ctx, int which, const void** d_ptr);
+
+/* This rank's share of n targets: [lo, hi), contiguous and balanced (host logic, no GPU). */
+void efit_shard(int32_t n, int32_t rank, int32_t world, int32_t* lo, int32_t* hi);
+
+int efit_destroy(efit_ctx* ctx);
+const char* efit_strerror(int status);
+const char* efit_last_error(const efit_ctx* ctx);
+const char* efit_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* EFIT_H */

@@ -1,0 +1,317 @@
+"""B200-native EFIT fitting-iteration hot path -- thin Python binding of include/efit.h.
+
+Argument marshalling only: every step runs inside libefit_b200.so (hand-written sm_100a
+kernels).  PyTorch provides device memory (tensors), streams and process groups.  There
+is no CPU fallback: importing this package without the built library, or calling it
+without a CUDA device, raises.
+
+Names follow the C ABI (efit_green_init, efit_response, efit_boundary_flux, efit_fit_step,
+...).  `EfitContext` bundles the workspace tensor and the opaque handle.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional
+
+import numpy as np
+
+__all__ = [
+    "EfitError", "lib", "lib_path", "efit_workspace_bytes", "efit_green_init", "efit_info", "efit_response",
+    "efit_current", "efit_boundary_flux", "efit_interior_solve", "efit_lsq", "efit_fit_step", "efit_status",
+    "efit_table", "efit_shard", "efit_destroy", "efit_strerror", "efit_last_error", "efit_version",
+    "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY",
+]
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+lib_path = os.path.join(_HERE, "libefit_b200.so")
+
+EFIT_GREEN_TABLE = 0
+EFIT_GREEN_ONTHEFLY = 1
+EFIT_OK, EFIT_E_INVAL, EFIT_E_NOMEM, EFIT_E_CUDA, EFIT_E_NCCL = 0, -1, -2, -3, -4
+EFIT_E_SINGULAR, EFIT_E_NOPLASMA, EFIT_E_NONFINITE, EFIT_E_STATE = -5, -6, -7, -8
+
+_dp = ctypes.POINTER(ctypes.c_double)
+
+
+class efit_grid(ctypes.Structure):
+    _fields_ = [("nw", ctypes.c_int32), ("nh", ctypes.c_int32), ("rmin", ctypes.c_double),
+                ("rmax", ctypes.c_double), ("zmin", ctypes.c_double), ("zmax", ctypes.c_double)]
+
+
+class efit_basis(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("n_pp", ctypes.c_int32), ("n_ff", ctypes.c_int32),
+                ("n_knots", ctypes.c_int32), ("knots", _dp)]
+
+
+class efit_geometry(ctypes.Structure):
+    _fields_ = [("n_fl", ctypes.c_int32), ("fl_r", _dp), ("fl_z", _dp),
+                ("n_mp", ctypes.c_int32), ("mp_r", _dp), ("mp_z", _dp), ("mp_ang", _dp),
+                ("n_int", ctypes.c_int32), ("int_r", _dp), ("int_z", _dp),
+                ("n_lim", ctypes.c_int32), ("lim_r", _dp), ("lim_z", _dp),
+                ("ip_sign", ctypes.c_int32)]
+
+
+class efit_dist(ctypes.Structure):
+    _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32)]
+
+
+class efit_info_t(ctypes.Structure):
+    _fields_ = [("nw", ctypes.c_int32), ("nh", ctypes.c_int32), ("ndiag", ctypes.c_int32),
+                ("nbasis", ctypes.c_int32), ("n_edge", ctypes.c_int32), ("mode", ctypes.c_int32),
+                ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("resp_row_lo", ctypes.c_int32), ("resp_row_hi", ctypes.c_int32),
+                ("bnd_row_lo", ctypes.c_int32), ("bnd_row_hi", ctypes.c_int32),
+                ("lr_blk_lo", ctypes.c_int32), ("lr_blk_hi", ctypes.c_int32),
+                ("slab_stride", ctypes.c_int64), ("workspace_bytes", ctypes.c_size_t)]
+
+
+class EfitError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"EFIT error {code}: {msg}")
+        self.code = code
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libefit_b200.so (in-tree).  Fails loudly if it has not been built."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(lib_path):
+            raise ImportError(f"{lib_path} is missing: run `python -c 'import __graft_entry__ as g; g.build()'`")
+        L = ctypes.CDLL(lib_path)
+        P, I, vp = ctypes.POINTER, ctypes.c_int, ctypes.c_void_p
+        sig = {
+            "efit_workspace_bytes": (I, [P(efit_grid), P(efit_basis), P(efit_geometry), P(efit_dist), I,
+                                         P(ctypes.c_size_t)]),
+            "efit_green_init": (I, [P(vp), P(efit_grid), P(efit_basis), P(efit_geometry), P(efit_dist), I, vp,
+                                    ctypes.c_size_t, vp]),
+            "efit_info": (I, [vp, P(efit_info_t)]),
+            "efit_response": (I, [vp, vp, vp, vp, vp]),
+            "efit_current": (I, [vp, vp, vp, vp, vp]),
+            "efit_boundary_flux": (I, [vp, vp, vp, vp]),
+            "efit_interior_solve": (I, [vp, vp, vp, vp, vp]),
+            "efit_lsq": (I, [vp, vp, vp, vp, vp, vp, vp]),
+            "efit_fit_step": (I, [vp, vp, vp, vp, vp, vp, vp, vp, vp]),
+            "efit_status": (I, [vp, vp]),
+            "efit_table": (I, [vp, I, P(vp)]),
+            "efit_shard": (None, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int32),
+                                  P(ctypes.c_int32)]),
+            "efit_destroy": (I, [vp]),
+            "efit_strerror": (ctypes.c_char_p, [I]),
+            "efit_last_error": (ctypes.c_char_p, [vp]),
+            "efit_version": (ctypes.c_char_p, []),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def _check(code: int, ctx=None) -> None:
+    if code != EFIT_OK:
+        msg = lib().efit_last_error(ctx)
+        raise EfitError(code, (msg or b"").decode() or lib().efit_strerror(code).decode())
+
+
+def _ptr(t) -> Optional[int]:
+    """Device pointer of a torch tensor (must be contiguous fp64 on CUDA), or None."""
+    if t is None:
+        return None
+    if not t.is_cuda:
+        raise ValueError("expected a CUDA tensor")
+    if not t.is_contiguous():
+        raise ValueError("expected a contiguous tensor")
+    return t.data_ptr()
+
+
+def _stream(stream) -> Optional[int]:
+    import torch
+    if stream is None:
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+# ------------------------------------------------------------------------ struct builders
+
+def _arr(a) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(a, dtype=np.float64))
+
+
+class _Config:
+    """Holds the ctypes structs + the numpy arrays they point into (kept alive)."""
+
+    def __init__(self, grid, basis, geometry, rank: int = 0, world: int = 1):
+        self.keep = []
+
+        def P(a):
+            a = _arr(a)
+            self.keep.append(a)
+            return a.ctypes.data_as(_dp)
+
+        self.grid = efit_grid(grid.nw, grid.nh, grid.rmin, grid.rmax, grid.zmin, grid.zmax)
+        self.basis = efit_basis(basis.kind, basis.n_pp, basis.n_ff, len(basis.knots), P(basis.knots))
+        g = geometry
+        self.geom = efit_geometry(len(g.fl_r), P(g.fl_r), P(g.fl_z), len(g.mp_r), P(g.mp_r), P(g.mp_z),
+                                  P(g.mp_ang), len(g.int_r), P(g.int_r), P(g.int_z), len(g.lim_r), P(g.lim_r),
+                                  P(g.lim_z), int(g.ip_sign))
+        self.dist = efit_dist(rank, world)
+
+
+# ------------------------------------------------------------------------ ABI functions
+
+def efit_workspace_bytes(grid, basis, geom, dist, mode: int = EFIT_GREEN_TABLE) -> int:
+    n = ctypes.c_size_t()
+    _check(lib().efit_workspace_bytes(ctypes.byref(grid), ctypes.byref(basis), ctypes.byref(geom),
+                                      ctypes.byref(dist), mode, ctypes.byref(n)))
+    return n.value
+
+
+def efit_green_init(grid, basis, geom, dist, mode, workspace, stream=None) -> ctypes.c_void_p:
+    h = ctypes.c_void_p()
+    _check(lib().efit_green_init(ctypes.byref(h), ctypes.byref(grid), ctypes.byref(basis), ctypes.byref(geom),
+                                 ctypes.byref(dist), mode, _ptr(workspace), workspace.numel(), _stream(stream)))
+    return h
+
+
+def efit_info(ctx) -> efit_info_t:
+    info = efit_info_t()
+    _check(lib().efit_info(ctx, ctypes.byref(info)), ctx)
+    return info
+
+
+def efit_response(ctx, psi, resp, axbd=None, stream=None) -> None:
+    _check(lib().efit_response(ctx, _ptr(psi), _ptr(resp), _ptr(axbd), _stream(stream)), ctx)
+
+
+def efit_current(ctx, psi, coef, pcurr, stream=None) -> None:
+    _check(lib().efit_current(ctx, _ptr(psi), _ptr(coef), _ptr(pcurr), _stream(stream)), ctx)
+
+
+def efit_boundary_flux(ctx, pcurr, psib, stream=None) -> None:
+    _check(lib().efit_boundary_flux(ctx, _ptr(pcurr), _ptr(psib), _stream(stream)), ctx)
+
+
+def efit_interior_solve(ctx, pcurr, psib, psi_p, stream=None) -> None:
+    _check(lib().efit_interior_solve(ctx, _ptr(pcurr), _ptr(psib), _ptr(psi_p), _stream(stream)), ctx)
+
+
+def efit_lsq(ctx, resp, meas, sigma, coef, chi2, stream=None) -> None:
+    _check(lib().efit_lsq(ctx, _ptr(resp), _ptr(meas), _ptr(sigma), _ptr(coef), _ptr(chi2), _stream(stream)), ctx)
+
+
+def efit_fit_step(ctx, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None) -> None:
+    _check(lib().efit_fit_step(ctx, _ptr(psi), _ptr(psi_ext), _ptr(meas), _ptr(sigma), _ptr(coef), _ptr(chi2),
+                               _ptr(eps), _stream(stream)), ctx)
+
+
+def efit_status(ctx, stream=None) -> int:
+    return lib().efit_status(ctx, _stream(stream))
+
+
+def efit_table(ctx, which: int) -> int:
+    p = ctypes.c_void_p()
+    _check(lib().efit_table(ctx, which, ctypes.byref(p)), ctx)
+    return p.value
+
+
+def efit_shard(n: int, rank: int, world: int):
+    lo, hi = ctypes.c_int32(), ctypes.c_int32()
+    lib().efit_shard(n, rank, world, ctypes.byref(lo), ctypes.byref(hi))
+    return lo.value, hi.value
+
+
+def efit_destroy(ctx) -> None:
+    lib().efit_destroy(ctx)
+
+
+def efit_strerror(code: int) -> str:
+    return lib().efit_strerror(code).decode()
+
+
+def efit_last_error(ctx=None) -> str:
+    return (lib().efit_last_error(ctx) or b"").decode()
+
+
+def efit_version() -> str:
+    return lib().efit_version().decode()
+
+
+# ------------------------------------------------------------------------ convenience context
+
+class EfitContext:
+    """Owns the device workspace (a torch uint8 tensor) and the library handle."""
+
+    def __init__(self, grid, basis, geometry, mode: int = EFIT_GREEN_TABLE, rank: int = 0, world: int = 1,
+                 device=None, stream=None):
+        import torch
+        self.cfg = _Config(grid, basis, geometry, rank, world)
+        self.device = torch.device(device if device is not None else "cuda")
+        nbytes = efit_workspace_bytes(self.cfg.grid, self.cfg.basis, self.cfg.geom, self.cfg.dist, mode)
+        # 256-byte alignment: allocate a little extra and offset
+        raw = torch.empty(nbytes + 256, dtype=torch.uint8, device=self.device)
+        off = (-raw.data_ptr()) % 256
+        self._raw = raw
+        self.workspace = raw[off:off + nbytes]
+        self.handle = efit_green_init(self.cfg.grid, self.cfg.basis, self.cfg.geom, self.cfg.dist, mode,
+                                      self.workspace, stream)
+        self.info = efit_info(self.handle)
+        self.nw, self.nh = self.info.nw, self.info.nh
+        self.ndiag, self.nbasis, self.n_edge = self.info.ndiag, self.info.nbasis, self.info.n_edge
+
+    def close(self) -> None:
+        if getattr(self, "handle", None):
+            efit_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _t(self, n: int):
+        import torch
+        return torch.zeros(n, dtype=torch.float64, device=self.device)
+
+    # tensor-returning helpers (allocation + one ABI call each)
+    def response(self, psi, stream=None):
+        resp = self._t(self.ndiag * self.nbasis)
+        axbd = self._t(2)
+        efit_response(self.handle, psi, resp, axbd, stream)
+        return resp.view(self.ndiag, self.nbasis), axbd
+
+    def current(self, psi, coef, stream=None):
+        out = self._t(self.nw * self.nh)
+        efit_current(self.handle, psi, coef, out, stream)
+        return out
+
+    def boundary_flux(self, pcurr, stream=None):
+        out = self._t(self.n_edge)
+        efit_boundary_flux(self.handle, pcurr, out, stream)
+        return out
+
+    def interior_solve(self, pcurr, psib, stream=None):
+        out = self._t(self.nw * self.nh)
+        efit_interior_solve(self.handle, pcurr, psib, out, stream)
+        return out
+
+    def lsq(self, resp, meas, sigma, stream=None):
+        coef, chi2 = self._t(self.nbasis), self._t(1)
+        efit_lsq(self.handle, resp.reshape(-1).contiguous(), meas, sigma, coef, chi2, stream)
+        return coef, chi2
+
+    def fit_step(self, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None):
+        efit_fit_step(self.handle, psi, psi_ext, meas, sigma, coef, chi2, eps, stream)
+
+    def status(self, stream=None) -> int:
+        return efit_status(self.handle, stream)
+
+    def table_ptr(self, which: int) -> int:
+        return efit_table(self.handle, which)

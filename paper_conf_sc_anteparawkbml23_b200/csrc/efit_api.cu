@@ -1,0 +1,471 @@
+// efit_api.cu -- C ABI (include/efit.h): validation, tiling plan, workspace carve, CUDA-graph
+// capture of the fit step.  Host code only; kernels live in efit_kernels.cu.
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "efit_internal.h"
+
+using efit::Ctx;
+
+struct efit_ctx {
+    Ctx c;
+};
+
+namespace efit {
+cudaError_t prepare_kernels(Ctx& c);
+cudaError_t launch_make_pair(Ctx& c, const double* pcurr, cudaStream_t s);
+}  // namespace efit
+
+static thread_local char g_err[256] = "";
+
+static int fail(Ctx* c, int code, const char* fmt, ...) {
+    char* dst = c ? c->err : g_err;
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(dst, 256, fmt, ap);
+    va_end(ap);
+    if (c) std::snprintf(g_err, sizeof(g_err), "%s", c->err);
+    return code;
+}
+
+static int cuda_fail(Ctx* c, cudaError_t e, const char* where) {
+    return fail(c, EFIT_E_CUDA, "%s: %s", where, cudaGetErrorString(e));
+}
+
+static inline long long round_up(long long x, long long m) { return (x + m - 1) / m * m; }
+
+extern "C" void efit_shard(int32_t n, int32_t rank, int32_t world, int32_t* lo, int32_t* hi) {
+    if (world < 1) world = 1;
+    int32_t base = n / world, rem = n % world;
+    int32_t l = rank * base + (rank < rem ? rank : rem);
+    *lo = l;
+    *hi = l + base + (rank < rem ? 1 : 0);
+}
+
+static bool finite_arr(const double* p, int n) {
+    for (int i = 0; i < n; ++i)
+        if (!std::isfinite(p[i])) return false;
+    return true;
+}
+
+static int validate(const efit_grid* g, const efit_basis* b, const efit_geometry* geo, const efit_dist* d, int mode) {
+    if (!g || !b || !geo) return fail(nullptr, EFIT_E_INVAL, "null grid/basis/geometry");
+    if (g->nw < 3 || g->nh < 3 || g->nw > efit::kMaxN || g->nh > efit::kMaxN)
+        return fail(nullptr, EFIT_E_INVAL, "grid size %dx%d outside [3, %d]", g->nw, g->nh, efit::kMaxN);
+    int nm = g->nh - 1;
+    if ((nm & (nm - 1)) != 0)
+        return fail(nullptr, EFIT_E_INVAL, "nh-1 = %d must be a power of two (FFT-based interior solve)", nm);
+    if (!(g->rmin > 0.0) || !(g->rmax > g->rmin) || !(g->zmax > g->zmin) || !std::isfinite(g->rmax) ||
+        !std::isfinite(g->zmin) || !std::isfinite(g->zmax))
+        return fail(nullptr, EFIT_E_INVAL, "need 0 < rmin < rmax and zmin < zmax (finite)");
+    if (b->kind != 0 && b->kind != 1) return fail(nullptr, EFIT_E_INVAL, "basis kind %d", b->kind);
+    if (b->n_pp < 0 || b->n_ff < 0 || b->n_pp + b->n_ff < 1 || b->n_pp + b->n_ff > efit::kMaxBasis)
+        return fail(nullptr, EFIT_E_INVAL, "need 1 <= n_pp + n_ff <= %d", efit::kMaxBasis);
+    if (b->kind == 1) {
+        if (b->n_knots < 0 || b->n_knots > efit::kMaxKnots || (b->n_knots > 0 && !b->knots))
+            return fail(nullptr, EFIT_E_INVAL, "spline: 0 <= n_knots <= %d", efit::kMaxKnots);
+        if (b->n_pp != b->n_knots + 4 || b->n_ff != b->n_knots + 4)
+            return fail(nullptr, EFIT_E_INVAL, "spline: n_pp = n_ff = n_knots + 4 required");
+        for (int k = 0; k < b->n_knots; ++k) {
+            double lo = k ? b->knots[k - 1] : 0.0;
+            if (!(b->knots[k] > lo) || !(b->knots[k] < 1.0))
+                return fail(nullptr, EFIT_E_INVAL, "spline knots must increase strictly inside (0,1)");
+        }
+    }
+    if (geo->n_fl < 0 || geo->n_mp < 0 || geo->n_int < 0 || geo->n_fl + geo->n_mp + geo->n_int < 1)
+        return fail(nullptr, EFIT_E_INVAL, "need at least one diagnostic");
+    if (geo->n_fl + geo->n_mp + geo->n_int > efit::kLsqMaxRowsHost)
+        return fail(nullptr, EFIT_E_INVAL, "at most %d diagnostics", efit::kLsqMaxRowsHost);
+    if (geo->n_fl + geo->n_mp + geo->n_int < b->n_pp + b->n_ff)
+        return fail(nullptr, EFIT_E_INVAL, "fewer diagnostics than basis functions");
+    if ((geo->n_fl && (!geo->fl_r || !geo->fl_z)) || (geo->n_mp && (!geo->mp_r || !geo->mp_z || !geo->mp_ang)) ||
+        (geo->n_int && (!geo->int_r || !geo->int_z)))
+        return fail(nullptr, EFIT_E_INVAL, "null diagnostic array");
+    if (geo->n_lim < 3 || !geo->lim_r || !geo->lim_z) return fail(nullptr, EFIT_E_INVAL, "limiter needs >= 3 vertices");
+    if (!finite_arr(geo->fl_r, geo->n_fl) || !finite_arr(geo->fl_z, geo->n_fl) || !finite_arr(geo->mp_r, geo->n_mp) ||
+        !finite_arr(geo->mp_z, geo->n_mp) || !finite_arr(geo->mp_ang, geo->n_mp) ||
+        !finite_arr(geo->int_r, geo->n_int) || !finite_arr(geo->int_z, geo->n_int) ||
+        !finite_arr(geo->lim_r, geo->n_lim) || !finite_arr(geo->lim_z, geo->n_lim))
+        return fail(nullptr, EFIT_E_INVAL, "non-finite geometry");
+    for (int m = 0; m < geo->n_fl; ++m) if (!(geo->fl_r[m] > 0)) return fail(nullptr, EFIT_E_INVAL, "flux loop R <= 0");
+    for (int m = 0; m < geo->n_mp; ++m) if (!(geo->mp_r[m] > 0)) return fail(nullptr, EFIT_E_INVAL, "probe R <= 0");
+    for (int m = 0; m < geo->n_int; ++m) if (!(geo->int_r[m] > 0)) return fail(nullptr, EFIT_E_INVAL, "internal point R <= 0");
+    if (geo->ip_sign != 1 && geo->ip_sign != -1) return fail(nullptr, EFIT_E_INVAL, "ip_sign must be +1 or -1");
+    if (mode != EFIT_GREEN_TABLE && mode != EFIT_GREEN_ONTHEFLY) return fail(nullptr, EFIT_E_INVAL, "mode %d", mode);
+    if (d && (d->world < 1 || d->rank < 0 || d->rank >= d->world))
+        return fail(nullptr, EFIT_E_INVAL, "rank %d / world %d", d->rank, d->world);
+    return EFIT_OK;
+}
+
+// Tiling + sharding plan (host logic; DESIGN.md §"Tiling").
+static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geometry* geo, const efit_dist* d,
+                 int mode) {
+    c.nw = g->nw; c.nh = g->nh;
+    c.rmin = g->rmin; c.rmax = g->rmax; c.zmin = g->zmin; c.zmax = g->zmax;
+    c.dr = (g->rmax - g->rmin) / (double)(g->nw - 1);
+    c.dz = (g->zmax - g->zmin) / (double)(g->nh - 1);
+    c.kind = b->kind; c.n_pp = b->n_pp; c.n_ff = b->n_ff; c.nb = b->n_pp + b->n_ff;
+    c.n_knots = b->kind == 1 ? b->n_knots : 0;
+    for (int k = 0; k < efit::kMaxKnots; ++k) c.knots[k] = k < c.n_knots ? b->knots[k] : 1.0;
+    c.n_fl = geo->n_fl; c.n_mp = geo->n_mp; c.n_int = geo->n_int;
+    c.ndiag = geo->n_fl + geo->n_mp + geo->n_int;
+    c.n_lim = geo->n_lim; c.ip_sign = geo->ip_sign;
+    c.mode = mode;
+    c.rank = d ? d->rank : 0;
+    c.world = d ? d->world : 1;
+    c.n_edge = 2 * c.nh + 2 * (c.nw - 2);
+    c.ni = c.nw - 2;
+    c.nmode = c.nh - 2;
+    c.fft_m = 2 * (c.nh - 1);
+    c.fft_log2 = 0;
+    while ((1 << c.fft_log2) < c.fft_m) ++c.fft_log2;
+    const long long n = (long long)c.nw * c.nh;
+    c.S = round_up(n, 64);
+    efit::Tiling& t = c.t;
+    t.resp_gc = c.nb <= 12 ? 512 : 256;
+    t.resp_nchunk = (int)((n + t.resp_gc - 1) / t.resp_gc);
+    t.tb_ch = 2048;
+    t.tb_nchunk = (int)((n + t.tb_ch - 1) / t.tb_ch);
+    t.tb_gi = 8;
+    t.lr_jt = 16;
+    t.lr_njt = (c.nh + 8 * t.lr_jt - 1) / (8 * t.lr_jt);
+    t.lr_iib = 8;
+    t.lr_nblk = (c.nw + t.lr_iib - 1) / t.lr_iib;
+    t.red_blocks = 148;
+    // shards (targets only => bitwise identical results for any world size)
+    int lo, hi;
+    efit_shard(c.ndiag, c.rank, c.world, &lo, &hi);
+    c.m_lo = lo; c.m_hi = hi;
+    efit_shard(c.nw - 2, c.rank, c.world, &lo, &hi);
+    c.i_lo = 1 + lo; c.i_hi = 1 + hi;
+    efit_shard(t.lr_njt, c.rank, c.world, &lo, &hi);
+    c.jt_lo = lo; c.jt_hi = hi;
+    t.tb_ngroup = (c.i_hi - c.i_lo + t.tb_gi - 1) / t.tb_gi;
+    if (t.tb_ngroup < 1) t.tb_ngroup = 1;
+    // response rows per warp block: fewest rows on the busiest warp, registers MB*NB <= 40
+    const int nrows = c.m_hi - c.m_lo;
+    int best_mb = 1, best_cost = 1 << 30;
+    for (int mb = 4; mb >= 1; --mb) {
+        if (mb * c.nb > 40 && mb > 1) continue;
+        int nblk = (nrows + mb - 1) / mb;
+        int cost = ((nblk + 7) / 8) * mb;
+        if (cost < best_cost) { best_cost = cost; best_mb = mb; }
+    }
+    t.resp_mb = best_mb;
+}
+
+// Carve the workspace (base == nullptr: sizing only).  Returns total bytes.
+static size_t carve(Ctx& c, char* base) {
+    size_t off = 0;
+    auto take = [&](size_t bytes) -> char* {
+        off = (size_t)round_up((long long)off, 256);
+        char* p = base ? base + off : nullptr;
+        off += bytes;
+        return p;
+    };
+    const long long n = (long long)c.nw * c.nh;
+    const int nrows = c.m_hi - c.m_lo;
+    const int nslab = c.i_hi - c.i_lo;
+    c.T = (c.mode == EFIT_GREEN_TABLE && nslab > 0) ? (double*)take(sizeof(double) * (size_t)nslab * c.S) : nullptr;
+    c.Tedge = (double*)take(sizeof(double) * 2 * (size_t)c.S);
+    c.Gd = (double*)take(sizeof(double) * (size_t)(nrows > 0 ? nrows : 1) * c.S);
+    c.inlim = (uint8_t*)take((size_t)n);
+    c.dgeo = (double*)take(sizeof(double) * 4 * c.ndiag);
+    c.dkind = (int*)take(sizeof(int) * c.ndiag);
+    c.lim = (double*)take(sizeof(double) * 2 * c.n_lim);
+    c.tri_a = (double*)take(sizeof(double) * c.ni);
+    c.tri_cp = (double*)take(sizeof(double) * (size_t)c.ni * c.nmode);
+    c.tri_inv = (double*)take(sizeof(double) * (size_t)c.ni * c.nmode);
+    c.twiddle = (double2*)take(sizeof(double2) * (size_t)(c.fft_m / 2));
+    c.axbd = (double*)take(sizeof(double) * 2);
+    c.status = (int*)take(sizeof(int) * 4);
+    c.tickets = (unsigned*)take(sizeof(unsigned) * 8);
+    c.norm_part = (double*)take(sizeof(double) * 2 * c.t.red_blocks);
+    c.resp_part = (double*)take(sizeof(double) * (size_t)c.t.resp_nchunk * (nrows > 0 ? nrows : 1) * c.nb);
+    c.resp_cnt = (double*)take(sizeof(double) * c.t.resp_nchunk);
+    c.resp = (double*)take(sizeof(double) * (size_t)c.ndiag * c.nb);
+    c.coef = (double*)take(sizeof(double) * 32);
+    c.chi2 = (double*)take(sizeof(double) * 4);
+    c.pcurr = (double*)take(sizeof(double) * (size_t)n);
+    c.ipair = (double2*)take(sizeof(double2) * (size_t)round_up(n, c.t.tb_ch));
+    c.tb_part = (double*)take(sizeof(double) * (size_t)c.t.tb_nchunk * c.nw * 2);
+    c.lr_part = (double*)take(sizeof(double) * (size_t)c.t.lr_nblk * 2 * c.nh);
+    c.psib = (double*)take(sizeof(double) * c.n_edge);
+    c.fhat = (double*)take(sizeof(double) * (size_t)c.ni * c.nmode);
+    c.psip = (double*)take(sizeof(double) * (size_t)n);
+    c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 1));
+    c.scratch_meas = (double*)take(sizeof(double) * c.ndiag);
+    return (size_t)round_up((long long)off, 256);
+}
+
+static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
+
+extern "C" int efit_workspace_bytes(const efit_grid* grid, const efit_basis* basis, const efit_geometry* geom,
+                                    const efit_dist* dist, int mode, size_t* bytes_out) {
+    int st = validate(grid, basis, geom, dist, mode);
+    if (st) return st;
+    if (!bytes_out) return fail(nullptr, EFIT_E_INVAL, "bytes_out is null");
+    Ctx* c = new (std::nothrow) Ctx();
+    if (!c) return fail(nullptr, EFIT_E_NOMEM, "host allocation");
+    plan(*c, grid, basis, geom, dist, mode);
+    *bytes_out = carve(*c, nullptr);
+    delete c;
+    return EFIT_OK;
+}
+
+extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit_basis* basis,
+                               const efit_geometry* geom, const efit_dist* dist, int mode, void* d_workspace,
+                               size_t ws_bytes, efit_stream_t stream) {
+    if (!out) return fail(nullptr, EFIT_E_INVAL, "out is null");
+    *out = nullptr;
+    int st = validate(grid, basis, geom, dist, mode);
+    if (st) return st;
+    if (!d_workspace || ((uintptr_t)d_workspace & 255u))
+        return fail(nullptr, EFIT_E_INVAL, "workspace must be non-null and 256-byte aligned");
+    efit_ctx* h = new (std::nothrow) efit_ctx();
+    if (!h) return fail(nullptr, EFIT_E_NOMEM, "host allocation");
+    Ctx& c = h->c;
+    plan(c, grid, basis, geom, dist, mode);
+    size_t need = carve(c, nullptr);
+    if (ws_bytes < need) {
+        delete h;
+        return fail(nullptr, EFIT_E_NOMEM, "workspace %zu bytes < required %zu", ws_bytes, need);
+    }
+    c.ws_bytes = carve(c, (char*)d_workspace);
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = cudaGetDevice(&c.device);
+    if (e) { delete h; return cuda_fail(nullptr, e, "cudaGetDevice"); }
+    cudaPointerAttributes pa;
+    e = cudaPointerGetAttributes(&pa, d_workspace);
+    if (e || pa.type != cudaMemoryTypeDevice) {
+        cudaGetLastError();
+        delete h;
+        return fail(nullptr, EFIT_E_INVAL, "workspace is not device memory");
+    }
+    // geometry to the device
+    std::vector<double> dgeo(4 * (size_t)c.ndiag);
+    std::vector<int> dkind(c.ndiag);
+    int m = 0;
+    for (int k = 0; k < geom->n_fl; ++k, ++m) {
+        dgeo[4 * m] = geom->fl_r[k]; dgeo[4 * m + 1] = geom->fl_z[k]; dgeo[4 * m + 2] = 0; dgeo[4 * m + 3] = 0; dkind[m] = 0;
+    }
+    for (int k = 0; k < geom->n_mp; ++k, ++m) {
+        dgeo[4 * m] = geom->mp_r[k]; dgeo[4 * m + 1] = geom->mp_z[k];
+        dgeo[4 * m + 2] = std::cos(geom->mp_ang[k]); dgeo[4 * m + 3] = std::sin(geom->mp_ang[k]); dkind[m] = 1;
+    }
+    for (int k = 0; k < geom->n_int; ++k, ++m) {
+        dgeo[4 * m] = geom->int_r[k]; dgeo[4 * m + 1] = geom->int_z[k]; dgeo[4 * m + 2] = 0; dgeo[4 * m + 3] = 0; dkind[m] = 2;
+    }
+    std::vector<double> lim(2 * (size_t)c.n_lim);
+    for (int k = 0; k < c.n_lim; ++k) { lim[k] = geom->lim_r[k]; lim[c.n_lim + k] = geom->lim_z[k]; }
+    if ((e = cudaMemcpyAsync(c.dgeo, dgeo.data(), sizeof(double) * dgeo.size(), cudaMemcpyHostToDevice, s)) ||
+        (e = cudaMemcpyAsync(c.dkind, dkind.data(), sizeof(int) * dkind.size(), cudaMemcpyHostToDevice, s)) ||
+        (e = cudaMemcpyAsync(c.lim, lim.data(), sizeof(double) * lim.size(), cudaMemcpyHostToDevice, s))) {
+        delete h;
+        return cuda_fail(nullptr, e, "geometry upload");
+    }
+    if ((e = efit::prepare_kernels(c)) || (e = efit::launch_init_tables(c, s)) || (e = cudaStreamSynchronize(s))) {
+        delete h;
+        return cuda_fail(nullptr, e, "table build");
+    }
+    c.gexec = nullptr;
+    c.use_graph = getenv("EFIT_NO_GRAPH") == nullptr;
+    c.err[0] = 0;
+    *out = h;
+    return EFIT_OK;
+}
+
+extern "C" int efit_info(const efit_ctx* h, efit_info_t* info) {
+    if (!h || !info) return fail(nullptr, EFIT_E_INVAL, "null argument");
+    const Ctx& c = h->c;
+    info->nw = c.nw; info->nh = c.nh; info->ndiag = c.ndiag; info->nbasis = c.nb; info->n_edge = c.n_edge;
+    info->mode = c.mode; info->rank = c.rank; info->world = c.world;
+    info->resp_row_lo = c.m_lo; info->resp_row_hi = c.m_hi;
+    info->bnd_row_lo = c.i_lo; info->bnd_row_hi = c.i_hi;
+    info->lr_blk_lo = c.jt_lo; info->lr_blk_hi = c.jt_hi;
+    info->slab_stride = c.S;
+    info->workspace_bytes = c.ws_bytes;
+    return EFIT_OK;
+}
+
+#define EFIT_CHECK_PTR(c, p, name)                                                                  \
+    do {                                                                                            \
+        if (!(p)) return fail(&(c), EFIT_E_INVAL, "%s is null", name);                              \
+        if (!aligned16(p)) return fail(&(c), EFIT_E_INVAL, "%s is not 16-byte aligned", name);      \
+    } while (0)
+
+extern "C" int efit_response(efit_ctx* h, const double* d_psi, double* d_resp, double* d_axbd,
+                             efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    EFIT_CHECK_PTR(c, d_psi, "d_psi");
+    EFIT_CHECK_PTR(c, d_resp, "d_resp");
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    if ((e = efit::launch_normalize(c, d_psi, s))) return cuda_fail(&c, e, "normalize");
+    if ((e = efit::launch_response(c, d_psi, d_resp + (size_t)c.m_lo * c.nb, s))) return cuda_fail(&c, e, "response");
+    if (d_axbd && (e = cudaMemcpyAsync(d_axbd, c.axbd, 2 * sizeof(double), cudaMemcpyDeviceToDevice, s)))
+        return cuda_fail(&c, e, "axbd copy");
+    return EFIT_OK;
+}
+
+extern "C" int efit_current(efit_ctx* h, const double* d_psi, const double* d_coef, double* d_pcurr,
+                            efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    EFIT_CHECK_PTR(c, d_psi, "d_psi");
+    EFIT_CHECK_PTR(c, d_coef, "d_coef");
+    EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    if ((e = efit::launch_normalize(c, d_psi, s))) return cuda_fail(&c, e, "normalize");
+    if ((e = efit::launch_current(c, d_psi, d_coef, d_pcurr, false, s))) return cuda_fail(&c, e, "current");
+    return EFIT_OK;
+}
+
+extern "C" int efit_boundary_flux(efit_ctx* h, const double* d_pcurr, double* d_psib, efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
+    EFIT_CHECK_PTR(c, d_psib, "d_psib");
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    if ((e = efit::launch_make_pair(c, d_pcurr, s))) return cuda_fail(&c, e, "pair");
+    if ((e = efit::launch_boundary(c, d_pcurr, d_psib, s))) return cuda_fail(&c, e, "boundary");
+    return EFIT_OK;
+}
+
+extern "C" int efit_interior_solve(efit_ctx* h, const double* d_pcurr, const double* d_psib, double* d_psi_p,
+                                   efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
+    EFIT_CHECK_PTR(c, d_psib, "d_psib");
+    EFIT_CHECK_PTR(c, d_psi_p, "d_psi_p");
+    cudaError_t e = efit::launch_solve(c, d_pcurr, d_psib, d_psi_p, nullptr, nullptr, nullptr, (cudaStream_t)stream);
+    if (e) return cuda_fail(&c, e, "interior solve");
+    return EFIT_OK;
+}
+
+extern "C" int efit_lsq(efit_ctx* h, const double* d_resp, const double* d_meas, const double* d_sigma,
+                        double* d_coef, double* d_chi2, efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    EFIT_CHECK_PTR(c, d_resp, "d_resp");
+    EFIT_CHECK_PTR(c, d_meas, "d_meas");
+    EFIT_CHECK_PTR(c, d_sigma, "d_sigma");
+    EFIT_CHECK_PTR(c, d_coef, "d_coef");
+    EFIT_CHECK_PTR(c, d_chi2, "d_chi2");
+    cudaError_t e = efit::launch_lsq(c, d_resp, d_meas, d_sigma, d_coef, d_chi2, (cudaStream_t)stream);
+    if (e) return cuda_fail(&c, e, "lsq");
+    return EFIT_OK;
+}
+
+static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, const double* meas,
+                                    const double* sigma, double* coef, double* chi2, double* eps, cudaStream_t s) {
+    cudaError_t e;
+    if ((e = efit::launch_normalize(c, psi, s))) return e;
+    if ((e = efit::launch_response(c, psi, c.resp, s))) return e;
+    if ((e = efit::launch_lsq(c, c.resp, meas, sigma, coef, chi2, s))) return e;
+    if ((e = efit::launch_current(c, psi, coef, c.pcurr, true, s))) return e;
+    if ((e = efit::launch_boundary(c, c.pcurr, c.psib, s))) return e;
+    if ((e = efit::launch_solve(c, c.pcurr, c.psib, nullptr, psi, psi_ext, eps, s))) return e;
+    return cudaSuccess;
+}
+
+extern "C" int efit_fit_step(efit_ctx* h, double* d_psi, const double* d_psi_ext, const double* d_meas,
+                             const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps,
+                             efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    if (c.world != 1) return fail(&c, EFIT_E_STATE, "efit_fit_step needs world == 1 (use the step calls)");
+    EFIT_CHECK_PTR(c, d_psi, "d_psi");
+    EFIT_CHECK_PTR(c, d_psi_ext, "d_psi_ext");
+    EFIT_CHECK_PTR(c, d_meas, "d_meas");
+    EFIT_CHECK_PTR(c, d_sigma, "d_sigma");
+    EFIT_CHECK_PTR(c, d_coef, "d_coef");
+    EFIT_CHECK_PTR(c, d_chi2, "d_chi2");
+    EFIT_CHECK_PTR(c, d_eps, "d_eps");
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    const void* key[8] = {d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, (const void*)s};
+    if (!c.use_graph || s == nullptr) {
+        if ((e = enqueue_fit_step(c, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, s)))
+            return cuda_fail(&c, e, "fit step");
+        return EFIT_OK;
+    }
+    if (!c.gexec || std::memcmp(key, c.gkey, sizeof(key)) != 0) {
+        if (c.gexec) { cudaGraphExecDestroy(c.gexec); c.gexec = nullptr; }
+        cudaGraph_t graph = nullptr;
+        if ((e = cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal))) return cuda_fail(&c, e, "begin capture");
+        cudaError_t e2 = enqueue_fit_step(c, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, s);
+        e = cudaStreamEndCapture(s, &graph);
+        if (e2) { if (graph) cudaGraphDestroy(graph); return cuda_fail(&c, e2, "fit step capture"); }
+        if (e) return cuda_fail(&c, e, "end capture");
+        e = cudaGraphInstantiateWithFlags(&c.gexec, graph, 0);
+        cudaGraphDestroy(graph);
+        if (e) { c.gexec = nullptr; return cuda_fail(&c, e, "graph instantiate"); }
+        std::memcpy(c.gkey, key, sizeof(key));
+    }
+    if ((e = cudaGraphLaunch(c.gexec, s))) return cuda_fail(&c, e, "graph launch");
+    return EFIT_OK;
+}
+
+extern "C" int efit_status(efit_ctx* h, efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    cudaStream_t s = (cudaStream_t)stream;
+    int st = 0;
+    cudaError_t e;
+    if ((e = cudaMemcpyAsync(&st, c.status, sizeof(int), cudaMemcpyDeviceToHost, s)) ||
+        (e = cudaMemsetAsync(c.status, 0, sizeof(int), s)) || (e = cudaStreamSynchronize(s)))
+        return cuda_fail(&c, e, "status");
+    if (st & EFIT_ST_NONFINITE) return fail(&c, EFIT_E_NONFINITE, "non-finite psi");
+    if (st & EFIT_ST_NOPLASMA) return fail(&c, EFIT_E_NOPLASMA, "empty plasma mask or psi_axis == psi_bdry");
+    if (st & EFIT_ST_SINGULAR) return fail(&c, EFIT_E_SINGULAR, "singular least-squares matrix");
+    return EFIT_OK;
+}
+
+extern "C" int efit_table(const efit_ctx* h, int which, const void** d_ptr) {
+    if (!h || !d_ptr) return fail(nullptr, EFIT_E_INVAL, "null argument");
+    const Ctx& c = h->c;
+    switch (which) {
+        case 0: *d_ptr = c.T; break;
+        case 1: *d_ptr = c.Gd; break;
+        case 2: *d_ptr = c.inlim; break;
+        case 3: *d_ptr = c.Tedge; break;
+        default: return fail(nullptr, EFIT_E_INVAL, "which = %d", which);
+    }
+    if (!*d_ptr) return fail(nullptr, EFIT_E_STATE, "table %d not built in this mode", which);
+    return EFIT_OK;
+}
+
+extern "C" int efit_destroy(efit_ctx* h) {
+    if (!h) return EFIT_OK;
+    if (h->c.gexec) cudaGraphExecDestroy(h->c.gexec);
+    delete h;
+    return EFIT_OK;
+}
+
+extern "C" const char* efit_strerror(int status) {
+    switch (status) {
+        case EFIT_OK: return "ok";
+        case EFIT_E_INVAL: return "invalid argument";
+        case EFIT_E_NOMEM: return "out of memory / workspace too small";
+        case EFIT_E_CUDA: return "CUDA error";
+        case EFIT_E_NCCL: return "collective error";
+        case EFIT_E_SINGULAR: return "singular least-squares matrix";
+        case EFIT_E_NOPLASMA: return "no plasma (empty mask)";
+        case EFIT_E_NONFINITE: return "non-finite value";
+        case EFIT_E_STATE: return "invalid state for this call";
+        default: return "unknown status";
+    }
+}
+
+extern "C" const char* efit_last_error(const efit_ctx* h) { return h ? h->c.err : g_err; }
+
+extern "C" const char* efit_version(void) { return "efit_b200 0.1 (sm_100a)"; }

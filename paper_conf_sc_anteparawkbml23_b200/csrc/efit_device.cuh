@@ -1,0 +1,164 @@
+// efit_device.cuh -- device-side math of the B200 EFIT path (Green's functions, grid,
+// basis).  Written for sm_100a from the definitions cited below; shares nothing with the
+// CPU oracle.  All fp64.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace efit {
+
+constexpr double kPi = 3.141592653589793238462643383279502884;
+constexpr double kMu0 = 4.0e-7 * kPi;     // mu0 = 4 pi 1e-7 (reading Q7)
+constexpr double kMu0Over2Pi = 2.0e-7;    // mu0 / (2 pi)
+constexpr int kAgmIters = 10;             // enough for m1 >= 1e-15 (quadratic convergence)
+
+// Grid coordinates without FMA contraction (R_i = rmin + i*dR rounded twice), so that
+// discrete decisions (limiter test, bilinear cell) are reproducible bit for bit.
+__device__ __forceinline__ double grid_coord(double lo, int i, double d) {
+    return __dadd_rn(lo, __dmul_rn((double)i, d));
+}
+
+// Complete elliptic integrals by the arithmetic-geometric mean (Gauss; A&S 17.6):
+//   a0 = 1, b0 = sqrt(m1), c0^2 = m;  a' = (a+b)/2, b' = sqrt(ab), c' = c^2/(4a')
+//   K = pi/(2 a_inf),  E = K (1 - sum_{n>=0} 2^(n-1) c_n^2).
+// Returns K and S1 = sum_{n>=1} 2^(n-1) c_n^2, so that
+//   (1 - m/2) K - E = K * S1        (no cancellation; all terms positive)
+//   E = K (1 - m/2 - S1).
+// c1 = (1 - sqrt(m1))/2 is formed as m / (2 (1 + sqrt(m1))) (cancellation-free).
+__device__ __forceinline__ void agm_ks1(double m, double m1, double& K, double& S1) {
+    double b = sqrt(m1);
+    double c = m / (2.0 * (1.0 + b));  // c1
+    double a = 0.5 * (1.0 + b);        // a1
+    b = sqrt(b);                       // b1 = sqrt(a0 b0) = sqrt(sqrt(m1))
+    double s = c * c;                  // 2^0 c1^2
+    double p = 1.0;
+#pragma unroll
+    for (int n = 1; n < kAgmIters; ++n) {
+        double an = 0.5 * (a + b);
+        double bn = sqrt(a * b);
+        c = c * c / (4.0 * an);
+        p *= 2.0;
+        s += p * c * c;
+        a = an;
+        b = bn;
+    }
+    K = kPi / (2.0 * a);
+    S1 = s;
+}
+
+// Flux per radian at (R, Z) from a 1 A filament at (Rs, Zs):
+//   G = (mu0/2pi) sqrt((R+Rs)^2 + dz^2) [(1 - m/2) K(m) - E(m)],  m = 4 R Rs / den.
+__device__ __forceinline__ double green_psi(double R, double Z, double Rs, double Zs) {
+    double dz = Z - Zs;
+    double dz2 = dz * dz;
+    double sp = R + Rs, sm = R - Rs;
+    double den = sp * sp + dz2;
+    double inv = 1.0 / den;
+    double m = 4.0 * R * Rs * inv;
+    double m1 = (sm * sm + dz2) * inv;
+    double K, S1;
+    agm_ks1(m, m1, K, S1);
+    return kMu0Over2Pi * sqrt(den) * K * S1;
+}
+
+// Self term: point-to-cell average of (mu0/2pi) R (ln(8R/rho) - 2) over a dR x dZ cell
+// (reading Q5).
+__device__ __forceinline__ double green_self(double R, double dR, double dZ) {
+    double p = 0.5 * dR, q = 0.5 * dZ;
+    double lnrho = (p * q * log(p * p + q * q) - 3.0 * p * q + p * p * atan(q / p) + q * q * atan(p / q))
+                   / (2.0 * p * q);
+    return kMu0Over2Pi * R * (log(8.0 * R) - lnrho - 2.0);
+}
+
+// Field of a 1 A filament at (Rs, Zs) measured at (R, Z) (Smythe; a = Rs, z = Z - Zs):
+//   B_Z = (mu0/2pi) [K + (a^2 - R^2 - z^2)/((a-R)^2 + z^2) E] / sqrt((a+R)^2 + z^2)
+//   B_R = (mu0/2pi) z [-K + (a^2 + R^2 + z^2)/((a-R)^2 + z^2) E] / (R sqrt((a+R)^2 + z^2))
+__device__ __forceinline__ void green_field(double R, double Z, double Rs, double Zs,
+                                            double& BR, double& BZ) {
+    double z = Z - Zs;
+    double z2 = z * z;
+    double sp = Rs + R, sm = Rs - R;
+    double den = sp * sp + z2;
+    double dm = sm * sm + z2;
+    double m = 4.0 * R * Rs / den;
+    double m1 = dm / den;
+    double K, S1;
+    agm_ks1(m, m1, K, S1);
+    double E = K * ((1.0 - 0.5 * m) - S1);
+    double isq = 1.0 / sqrt(den);
+    BZ = kMu0Over2Pi * isq * (K + (Rs * Rs - R * R - z2) / dm * E);
+    BR = kMu0Over2Pi * z * isq / R * (-K + (Rs * Rs + R * R + z2) / dm * E);
+}
+
+// Basis evaluation: out[k] = w_k(R) phi_k(psihat), columns [P' (w = R) | FF' (w = mu0/(4 pi^2 R))].
+// kind 0: psihat^k.  kind 1: clamped cubic B-splines -- only the 4 non-zero functions on
+// the knot span are formed (Cox-de Boor triangle), the rest are zero.
+struct BasisParams {
+    int kind, n_pp, n_ff, n_knots;
+    double knots[20];
+};
+
+template <int NB>
+__device__ __forceinline__ void basis_eval(const BasisParams& bp, double h, double R, double* out) {
+    double wpp = R;
+    double wff = kMu0 / (4.0 * kPi * kPi * R);
+    if (bp.kind == 0) {
+        double p = 1.0;
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+            // columns k < n_pp: P' term k;  k >= n_pp: FF' term k - n_pp
+            out[k] = 0.0;
+        }
+        int nmax = bp.n_pp > bp.n_ff ? bp.n_pp : bp.n_ff;
+        double pw[NB];
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+            pw[k] = p;
+            if (k + 1 < nmax) p *= h;
+        }
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+            if (k < bp.n_pp) out[k] = wpp * pw[k];
+            else if (k < bp.n_pp + bp.n_ff) out[k] = wff * pw[k - bp.n_pp];
+        }
+    } else {
+        // knot vector t: 0,0,0,0, k_1..k_n, 1,1,1,1;  span s with t_s <= h < t_{s+1}, 3 <= s <= n+3
+        int n = bp.n_knots;
+        int s = 3;
+        for (int q = 0; q < n; ++q)
+            if (h >= bp.knots[q]) s = 4 + q;
+        // t(idx) accessor
+        auto t = [&](int idx) -> double {
+            if (idx <= 3) return 0.0;
+            if (idx >= n + 4) return 1.0;
+            return bp.knots[idx - 4];
+        };
+        double N0[4], left[4], right[4];
+        N0[0] = 1.0;
+        for (int j = 1; j <= 3; ++j) {
+            left[j] = h - t(s + 1 - j);
+            right[j] = t(s + j) - h;
+            double saved = 0.0;
+            for (int r = 0; r < j; ++r) {
+                double tmp = N0[r] / (right[r + 1] + left[j - r]);
+                N0[r] = saved + right[r + 1] * tmp;
+                saved = left[j - r] * tmp;
+            }
+            N0[j] = saved;
+        }
+        // non-zero functions: indices s-3 .. s  (0-based basis index)
+#pragma unroll
+        for (int k = 0; k < NB; ++k) out[k] = 0.0;
+        int nf = n + 4;
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            int idx = s - 3 + r;
+            if (idx >= 0 && idx < nf) {
+                if (idx < bp.n_pp) out[idx] = wpp * N0[r];
+                if (bp.n_pp + idx < NB) out[bp.n_pp + idx] = wff * N0[r];
+            }
+        }
+    }
+}
+
+}  // namespace efit

@@ -1,0 +1,105 @@
+// efit_internal.h -- private state of the B200 EFIT library (not part of the ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stddef.h>
+
+#include "efit.h"
+
+namespace efit {
+
+constexpr int kMaxBasis = 24;
+constexpr int kMaxKnots = 20;
+constexpr int kMaxN = 4097;
+constexpr int kLsqMaxRowsHost = 1024;
+
+// device status-word bits
+#define EFIT_ST_NOPLASMA 1
+#define EFIT_ST_SINGULAR 2
+#define EFIT_ST_NONFINITE 4
+
+// Tiling parameters (chosen on the host from the configuration).
+struct Tiling {
+    // response: chunks of `resp_gc` grid nodes, partial sums per chunk
+    int resp_gc, resp_nchunk, resp_mb;
+    // top/bottom boundary: chunks of `tb_ch` doubles of each slab, groups of `tb_gi` slabs
+    int tb_ch, tb_nchunk, tb_gi, tb_ngroup;
+    // left/right boundary: j-tiles of `lr_jt` targets per CTA, `lr_iib` source rows per CTA
+    int lr_jt, lr_njt, lr_iib, lr_nblk;
+    // normalisation / eps reductions
+    int red_blocks;
+};
+
+struct Ctx {
+    // configuration (host copy)
+    int nw, nh;
+    double rmin, rmax, zmin, zmax, dr, dz;
+    int kind, n_pp, n_ff, nb, n_knots;
+    double knots[kMaxKnots];
+    int n_fl, n_mp, n_int, ndiag, n_lim, ip_sign;
+    int mode, rank, world;
+    int n_edge, ni, nmode;       // ni = nw-2 interior rows, nmode = nh-2 sine modes
+    int fft_m, fft_log2;         // complex FFT length 2(nh-1) and its log2
+    int m_lo, m_hi;              // response rows of this rank
+    int i_lo, i_hi;              // top/bottom target rows of this rank (within [1, nw-1))
+    int jt_lo, jt_hi;            // left/right j-tiles of this rank
+    long long S;                 // slab / row stride (doubles), multiple of 32
+    Tiling t;
+    size_t ws_bytes;
+    int device;
+
+    // device pointers carved from the workspace
+    double* T;          // [i_hi-i_lo][S]   top/bottom Green's slabs (table mode)
+    double* Tedge;      // [2][S]           slabs i = 0 and i = nw-1 (left/right)
+    double* Gd;         // [m_hi-m_lo][S]   diagnostic Green's rows
+    uint8_t* inlim;     // [nw*nh]
+    double* dgeo;       // [ndiag][4]       r, z, cos(ang), sin(ang); kind in dkind
+    int* dkind;         // [ndiag]          0 flux loop, 1 probe, 2 internal B_Z
+    double* lim;        // [2*n_lim]        r then z
+    double* tri_a;      // [ni]             sub-diagonal coefficient a_i
+    double* tri_cp;     // [ni][nmode]      Thomas c'_i per mode
+    double* tri_inv;    // [ni][nmode]      1/den_i per mode
+    double2* twiddle;   // [fft_m/2]        exp(-2 pi i k/M)
+
+    // per-iteration scratch
+    double* axbd;       // [2] psi_axis, psi_bdry
+    int* status;        // [1] sticky data-dependent failure
+    unsigned* tickets;  // [8] last-block counters
+    double* norm_part;  // [red_blocks][2]  (value, index) partials
+    double* resp_part;  // [resp_nchunk][rows][nb]
+    double* resp_cnt;   // [resp_nchunk]    masked-node counts
+    double* resp;       // [ndiag][nb]      full response (fit step)
+    double* coef;       // [nb]
+    double* chi2;       // [1]
+    double* pcurr;      // [nw*nh]
+    double2* ipair;     // [S]              (I[g], I[ii][nh-1-m])
+    double* tb_part;    // [tb_nchunk][nw][2]
+    double* lr_part;    // [lr_nblk][2][nh]
+    double* psib;       // [n_edge]
+    double* fhat;       // [ni][nmode]  DST coefficients (in place: Thomas solution)
+    double* psip;       // [nw*nh]
+    double* eps_part;   // [red_blocks]
+    double* scratch_meas;  // [ndiag] (unused placeholder)
+
+    // CUDA graph cache for efit_fit_step
+    cudaGraphExec_t gexec;
+    const void* gkey[8];
+    cudaStream_t gstream;
+    bool use_graph;
+
+    char err[256];
+};
+
+// ---- launchers (efit_kernels.cu) -------------------------------------------------
+cudaError_t launch_init_tables(Ctx& c, cudaStream_t s);
+cudaError_t launch_normalize(Ctx& c, const double* psi, cudaStream_t s);
+cudaError_t launch_response(Ctx& c, const double* psi, double* resp_rows, cudaStream_t s);
+cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const double* sigma,
+                       double* coef, double* chi2, cudaStream_t s);
+cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double* pcurr,
+                           bool pair, cudaStream_t s);
+cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s);
+cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out,
+                         double* psi_inout, const double* psi_ext, double* eps, cudaStream_t s);
+
+}  // namespace efit

@@ -140,11 +140,14 @@ def diagnostics(n_fl: int = 44, n_mp: int = 76, n_int: int = 0, grid: Optional[G
         dr, dz = grid.dr, grid.dz
         i0 = int(math.ceil((1.75 - grid.rmin) / dr - 0.5))
         i1 = int(math.floor((2.25 - grid.rmin) / dr - 0.5))
-        idx = np.unique(np.round(np.linspace(i0, i1, n_int)).astype(int))
-        assert len(idx) == n_int, "grid too coarse for the requested MSE-like points"
-        int_r = grid.rmin + (idx + 0.5) * dr
+        idx = np.round(np.linspace(i0, i1, n_int)).astype(int)
+        # alternate the cell row just above / below the midplane so no two points coincide
+        # on coarse grids (129^2 has fewer than 40 cells in [1.75, 2.25])
         j0 = (grid.nh - 1) // 2
-        int_z = np.full(n_int, grid.zmin + (j0 + 0.5) * dz)
+        rows = np.where(np.arange(n_int) % 2 == 0, j0, j0 - 1)
+        int_r = grid.rmin + (idx + 0.5) * dr
+        int_z = grid.zmin + (rows + 0.5) * dz
+        assert len(set(zip(idx.tolist(), rows.tolist()))) == n_int, "grid too coarse for the MSE-like points"
     else:
         int_r = np.zeros(0)
         int_z = np.zeros(0)
