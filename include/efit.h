@@ -166,14 +166,33 @@ int efit_fit_step(efit_ctx* ctx, double* d_psi, const double* d_psi_ext, const d
                   const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps,
                   efit_stream_t stream);
 
+/* Tail of a fit iteration for the sharded (world > 1) path, after the caller has exchanged the
+ * boundary slices: interior solve of d_pcurr with edge values d_psib, then
+ * psi <- psi_p + d_psi_ext (in place) and d_eps[0] = max|psi_new - psi_old| / |psi_bdry - psi_axis|,
+ * with psi_axis/psi_bdry from the most recent efit_response or efit_current call on this ctx. */
+int efit_solve_update(efit_ctx* ctx, const double* d_pcurr, const double* d_psib, const double* d_psi_ext,
+                      double* d_psi, double* d_eps, efit_stream_t stream);
+
+/* Per-step kernel timing (the measurement hook used by bench.py).  After efit_profile_begin(ctx, n),
+ * the next n efit_fit_step calls record CUDA events at nine marks in stream order (they run
+ * eagerly, or as nodes of the caller's graph when the caller is capturing the stream);
+ * efit_profile_end synchronises and returns, summed over the recorded steps, milliseconds for
+ *   ms[0] whole step, ms[1] normalise, ms[2] response (k_response + reduce), ms[3] lsq,
+ *   ms[4] current, ms[5] k_bnd_tb, ms[6] k_bnd_lr, ms[7] boundary reduce, ms[8] interior solve + update.
+ * nout >= 9.  *nsteps_out = number of steps recorded. */
+int efit_profile_begin(efit_ctx* ctx, int32_t nsteps);
+int efit_profile_end(efit_ctx* ctx, double* ms_out, int32_t nout, int32_t* nsteps_out);
+
 /* Synchronise `stream` and return the first data-dependent failure recorded since the last
  * efit_status() call (EFIT_OK, EFIT_E_NOPLASMA, EFIT_E_SINGULAR, EFIT_E_NONFINITE), or
  * EFIT_E_CUDA.  Clears the status word. */
 int efit_status(efit_ctx* ctx, efit_stream_t stream);
 
-/* Test/inspection access: device pointers into the workspace.  which = 0: T (slab i at
- * T + (i - bnd_row_lo_or_0)*slab_stride, see efit_info), 1: Gd (row m at Gd + (m-resp_row_lo)*slab_stride),
- * 2: in-limiter flags (uint8[nw*nh]).  Returns EFIT_E_STATE if the table is not built. */
+/* Test/inspection access: device pointers into the workspace.  which = 0: top/bottom Green's
+ * slabs (slab of target row i at T + (i - bnd_row_lo)*slab_stride, entry ii*nh + m),
+ * 1: Gd (row m at Gd + (m - resp_row_lo)*slab_stride, entry g), 2: in-limiter flags
+ * (uint8[nw*nh]), 3: the two edge slabs i = 0 and i = nw-1 (at 0 and slab_stride).
+ * Returns EFIT_E_STATE if the table is not built in this mode. */
 int efit_table(const efit_ctx* ctx, int which, const void** d_ptr);
 
 /* This rank's share of n targets: [lo, hi), contiguous and balanced (host logic, no GPU). */

@@ -19,6 +19,7 @@ import numpy as np
 __all__ = [
     "EfitError", "lib", "lib_path", "efit_workspace_bytes", "efit_green_init", "efit_info", "efit_response",
     "efit_current", "efit_boundary_flux", "efit_interior_solve", "efit_lsq", "efit_fit_step", "efit_status",
+    "efit_solve_update", "efit_profile_begin", "efit_profile_end",
     "efit_table", "efit_shard", "efit_destroy", "efit_strerror", "efit_last_error", "efit_version",
     "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY",
 ]
@@ -96,6 +97,9 @@ def lib() -> ctypes.CDLL:
             "efit_lsq": (I, [vp, vp, vp, vp, vp, vp, vp]),
             "efit_fit_step": (I, [vp, vp, vp, vp, vp, vp, vp, vp, vp]),
             "efit_status": (I, [vp, vp]),
+            "efit_solve_update": (I, [vp, vp, vp, vp, vp, vp, vp]),
+            "efit_profile_begin": (I, [vp, ctypes.c_int32]),
+            "efit_profile_end": (I, [vp, P(ctypes.c_double), ctypes.c_int32, P(ctypes.c_int32)]),
             "efit_table": (I, [vp, I, P(vp)]),
             "efit_shard": (None, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int32),
                                   P(ctypes.c_int32)]),
@@ -209,6 +213,26 @@ def efit_lsq(ctx, resp, meas, sigma, coef, chi2, stream=None) -> None:
 def efit_fit_step(ctx, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None) -> None:
     _check(lib().efit_fit_step(ctx, _ptr(psi), _ptr(psi_ext), _ptr(meas), _ptr(sigma), _ptr(coef), _ptr(chi2),
                                _ptr(eps), _stream(stream)), ctx)
+
+
+def efit_solve_update(ctx, pcurr, psib, psi_ext, psi, eps, stream=None) -> None:
+    _check(lib().efit_solve_update(ctx, _ptr(pcurr), _ptr(psib), _ptr(psi_ext), _ptr(psi), _ptr(eps),
+                                   _stream(stream)), ctx)
+
+
+PROFILE_FIELDS = ("step", "normalize", "response", "lsq", "current", "bnd_tb", "bnd_lr", "bnd_reduce", "solve")
+
+
+def efit_profile_begin(ctx, nsteps: int) -> None:
+    _check(lib().efit_profile_begin(ctx, nsteps), ctx)
+
+
+def efit_profile_end(ctx):
+    """Returns ({field: total ms over the recorded steps}, nsteps)."""
+    out = (ctypes.c_double * len(PROFILE_FIELDS))()
+    n = ctypes.c_int32()
+    _check(lib().efit_profile_end(ctx, out, len(PROFILE_FIELDS), ctypes.byref(n)), ctx)
+    return dict(zip(PROFILE_FIELDS, list(out))), n.value
 
 
 def efit_status(ctx, stream=None) -> int:

@@ -119,6 +119,7 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     c.world = d ? d->world : 1;
     c.n_edge = 2 * c.nh + 2 * (c.nw - 2);
     c.ni = c.nw - 2;
+    c.ni_pad = 32 * ((c.ni + 31) / 32);  // segment-interleaved solve layout: 32 lanes x L rows
     c.nmode = c.nh - 2;
     c.fft_m = 2 * (c.nh - 1);
     c.fft_log2 = 0;
@@ -126,16 +127,20 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     const long long n = (long long)c.nw * c.nh;
     c.S = round_up(n, 64);
     efit::Tiling& t = c.t;
-    t.resp_gc = c.nb <= 12 ? 512 : 256;
+    t.resp_gc = c.nb <= 8 ? 1024 : (c.nb <= 16 ? 512 : 256);
     t.resp_nchunk = (int)((n + t.resp_gc - 1) / t.resp_gc);
     t.tb_ch = 2048;
     t.tb_nchunk = (int)((n + t.tb_ch - 1) / t.tb_ch);
     t.tb_gi = 8;
-    t.lr_jt = 16;
-    t.lr_njt = (c.nh + 8 * t.lr_jt - 1) / (8 * t.lr_jt);
-    t.lr_iib = 8;
+    t.lr_jt = c.nh <= 96 ? 3 : (c.nh <= 160 ? 5 : (c.nh <= 288 ? 9 : 17));
+    t.lr_njt = (c.nh + 32 * t.lr_jt - 1) / (32 * t.lr_jt);
+    t.lr_iib = 2;
     t.lr_nblk = (c.nw + t.lr_iib - 1) / t.lr_iib;
-    t.red_blocks = 148;
+    {
+        const int q = (c.nh + 3) / 4;  // sources per warp (one quarter), multiple of lr_jt
+        t.lr_jj = (q + t.lr_jt - 1) / t.lr_jt * t.lr_jt;
+    }
+    t.red_blocks = 592;  // 4 per SM: enough loads in flight for the psi scans
     // shards (targets only => bitwise identical results for any world size)
     int lo, hi;
     efit_shard(c.ndiag, c.rank, c.world, &lo, &hi);
@@ -148,11 +153,13 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     if (t.tb_ngroup < 1) t.tb_ngroup = 1;
     // response rows per warp block: fewest rows on the busiest warp, registers MB*NB <= 40
     const int nrows = c.m_hi - c.m_lo;
+    // a CTA covers 8*MB rows (one MB-row block per warp); pick MB (<= 5, MB*NB <= 40 registers'
+    // worth of accumulators) minimising padded rows, then preferring more rows per warp
     int best_mb = 1, best_cost = 1 << 30;
-    for (int mb = 4; mb >= 1; --mb) {
-        if (mb * c.nb > 40 && mb > 1) continue;
-        int nblk = (nrows + mb - 1) / mb;
-        int cost = ((nblk + 7) / 8) * mb;
+    for (int mb = 1; mb <= 4; ++mb) {
+        if (16 * mb + 2 * mb * c.nb > 90 && mb > 1) continue;  // loads + accumulators under 128 regs
+        int groups = (nrows + 8 * mb - 1) / (8 * mb);
+        int cost = groups * 8 * mb + 4 * groups;  // padded rows + per-CTA basis work
         if (cost < best_cost) { best_cost = cost; best_mb = mb; }
     }
     t.resp_mb = best_mb;
@@ -178,8 +185,9 @@ static size_t carve(Ctx& c, char* base) {
     c.dkind = (int*)take(sizeof(int) * c.ndiag);
     c.lim = (double*)take(sizeof(double) * 2 * c.n_lim);
     c.tri_a = (double*)take(sizeof(double) * c.ni);
-    c.tri_cp = (double*)take(sizeof(double) * (size_t)c.ni * c.nmode);
-    c.tri_inv = (double*)take(sizeof(double) * (size_t)c.ni * c.nmode);
+    c.tri_cp = (double*)take(sizeof(double) * (size_t)c.ni_pad * c.nmode);
+    c.tri_inv = (double*)take(sizeof(double) * (size_t)c.ni_pad * c.nmode);
+    c.tri_alpha = (double*)take(sizeof(double) * (size_t)c.ni_pad * c.nmode);
     c.twiddle = (double2*)take(sizeof(double2) * (size_t)(c.fft_m / 2));
     c.axbd = (double*)take(sizeof(double) * 2);
     c.status = (int*)take(sizeof(int) * 4);
@@ -187,15 +195,16 @@ static size_t carve(Ctx& c, char* base) {
     c.norm_part = (double*)take(sizeof(double) * 2 * c.t.red_blocks);
     c.resp_part = (double*)take(sizeof(double) * (size_t)c.t.resp_nchunk * (nrows > 0 ? nrows : 1) * c.nb);
     c.resp_cnt = (double*)take(sizeof(double) * c.t.resp_nchunk);
+    c.bmat = (double*)take(sizeof(double) * (size_t)c.nb * c.t.resp_nchunk * c.t.resp_gc);
     c.resp = (double*)take(sizeof(double) * (size_t)c.ndiag * c.nb);
     c.coef = (double*)take(sizeof(double) * 32);
     c.chi2 = (double*)take(sizeof(double) * 4);
-    c.pcurr = (double*)take(sizeof(double) * (size_t)n);
-    c.ipair = (double2*)take(sizeof(double2) * (size_t)round_up(n, c.t.tb_ch));
+    c.pcurr = (double*)take(sizeof(double) * (size_t)round_up(n, c.t.tb_ch));
+    c.pflip = (double*)take(sizeof(double) * (size_t)round_up(n, c.t.tb_ch));
     c.tb_part = (double*)take(sizeof(double) * (size_t)c.t.tb_nchunk * c.nw * 2);
     c.lr_part = (double*)take(sizeof(double) * (size_t)c.t.lr_nblk * 2 * c.nh);
     c.psib = (double*)take(sizeof(double) * c.n_edge);
-    c.fhat = (double*)take(sizeof(double) * (size_t)c.ni * c.nmode);
+    c.fhat = (double*)take(sizeof(double) * (size_t)c.ni_pad * c.nmode);
     c.psip = (double*)take(sizeof(double) * (size_t)n);
     c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 1));
     c.scratch_meas = (double*)take(sizeof(double) * c.ndiag);
@@ -272,7 +281,19 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
         delete h;
         return cuda_fail(nullptr, e, "table build");
     }
+    c.side = nullptr; c.ev_fork = nullptr; c.ev_join = nullptr;
+    if ((e = cudaStreamCreateWithFlags(&c.side, cudaStreamNonBlocking)) ||
+        (e = cudaEventCreateWithFlags(&c.ev_fork, cudaEventDisableTiming)) ||
+        (e = cudaEventCreateWithFlags(&c.ev_join, cudaEventDisableTiming))) {
+        if (c.side) cudaStreamDestroy(c.side);
+        if (c.ev_fork) cudaEventDestroy(c.ev_fork);
+        delete h;
+        return cuda_fail(nullptr, e, "side stream");
+    }
     c.gexec = nullptr;
+    c.prof_on = false;
+    c.prof_ev = nullptr;
+    c.prof_slots = c.prof_next = 0;
     c.use_graph = getenv("EFIT_NO_GRAPH") == nullptr;
     c.err[0] = 0;
     *out = h;
@@ -365,15 +386,35 @@ extern "C" int efit_lsq(efit_ctx* h, const double* d_resp, const double* d_meas,
     return EFIT_OK;
 }
 
+namespace efit {
+void mark(Ctx& c, cudaStream_t s, int id) {
+    if (!c.prof_on || c.prof_next >= c.prof_slots) return;
+    cudaEvent_t ev = c.prof_ev[(size_t)c.prof_next * kNumMarks + id];
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    cudaStreamIsCapturing(s, &cs);
+    if (cs == cudaStreamCaptureStatusActive) cudaEventRecordWithFlags(ev, s, cudaEventRecordExternal);
+    else cudaEventRecord(ev, s);
+}
+}  // namespace efit
+
 static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, const double* meas,
                                     const double* sigma, double* coef, double* chi2, double* eps, cudaStream_t s) {
+    using namespace efit;
     cudaError_t e;
-    if ((e = efit::launch_normalize(c, psi, s))) return e;
-    if ((e = efit::launch_response(c, psi, c.resp, s))) return e;
-    if ((e = efit::launch_lsq(c, c.resp, meas, sigma, coef, chi2, s))) return e;
-    if ((e = efit::launch_current(c, psi, coef, c.pcurr, true, s))) return e;
-    if ((e = efit::launch_boundary(c, c.pcurr, c.psib, s))) return e;
-    if ((e = efit::launch_solve(c, c.pcurr, c.psib, nullptr, psi, psi_ext, eps, s))) return e;
+    mark(c, s, M_BEGIN);
+    if ((e = launch_normalize(c, psi, s))) return e;
+    mark(c, s, M_NORM);
+    if ((e = launch_response(c, psi, c.resp, s))) return e;
+    mark(c, s, M_RESP);
+    if ((e = launch_lsq(c, c.resp, meas, sigma, coef, chi2, s))) return e;
+    mark(c, s, M_LSQ);
+    if ((e = launch_current(c, psi, coef, c.pcurr, true, s))) return e;
+    mark(c, s, M_CUR);
+    if ((e = launch_boundary(c, c.pcurr, c.psib, s))) return e;  // marks M_TB, M_LR inside
+    mark(c, s, M_BRED);
+    if ((e = launch_solve(c, c.pcurr, c.psib, nullptr, psi, psi_ext, eps, s))) return e;
+    mark(c, s, M_SOLVE);
+    if (c.prof_on && c.prof_next < c.prof_slots) ++c.prof_next;
     return cudaSuccess;
 }
 
@@ -393,7 +434,11 @@ extern "C" int efit_fit_step(efit_ctx* h, double* d_psi, const double* d_psi_ext
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e;
     const void* key[8] = {d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, (const void*)s};
-    if (!c.use_graph || s == nullptr) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (s != nullptr && (e = cudaStreamIsCapturing(s, &cs))) return cuda_fail(&c, e, "capture query");
+    // eager enqueue when profiling, when the caller is capturing the stream itself (the kernels
+    // then become nodes of the caller's graph), or on the legacy stream (not capturable)
+    if (!c.use_graph || s == nullptr || c.prof_on || cs == cudaStreamCaptureStatusActive) {
         if ((e = enqueue_fit_step(c, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, s)))
             return cuda_fail(&c, e, "fit step");
         return EFIT_OK;
@@ -413,6 +458,70 @@ extern "C" int efit_fit_step(efit_ctx* h, double* d_psi, const double* d_psi_ext
     }
     if ((e = cudaGraphLaunch(c.gexec, s))) return cuda_fail(&c, e, "graph launch");
     return EFIT_OK;
+}
+
+extern "C" int efit_solve_update(efit_ctx* h, const double* d_pcurr, const double* d_psib, const double* d_psi_ext,
+                                 double* d_psi, double* d_eps, efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
+    EFIT_CHECK_PTR(c, d_psib, "d_psib");
+    EFIT_CHECK_PTR(c, d_psi_ext, "d_psi_ext");
+    EFIT_CHECK_PTR(c, d_psi, "d_psi");
+    EFIT_CHECK_PTR(c, d_eps, "d_eps");
+    cudaError_t e = efit::launch_solve(c, d_pcurr, d_psib, nullptr, d_psi, d_psi_ext, d_eps, (cudaStream_t)stream);
+    if (e) return cuda_fail(&c, e, "solve update");
+    return EFIT_OK;
+}
+
+extern "C" int efit_profile_begin(efit_ctx* h, int32_t nsteps) {
+    if (!h || nsteps < 1) return fail(nullptr, EFIT_E_INVAL, "profile_begin: bad argument");
+    Ctx& c = h->c;
+    if (c.prof_ev) return fail(&c, EFIT_E_STATE, "profiling already active");
+    size_t n = (size_t)nsteps * efit::kNumMarks;
+    c.prof_ev = new (std::nothrow) cudaEvent_t[n];
+    if (!c.prof_ev) return fail(&c, EFIT_E_NOMEM, "events");
+    for (size_t i = 0; i < n; ++i) {
+        cudaError_t e = cudaEventCreate(&c.prof_ev[i]);
+        if (e) {
+            for (size_t k = 0; k < i; ++k) cudaEventDestroy(c.prof_ev[k]);
+            delete[] c.prof_ev;
+            c.prof_ev = nullptr;
+            return cuda_fail(&c, e, "event create");
+        }
+    }
+    c.prof_slots = nsteps;
+    c.prof_next = 0;
+    c.prof_on = true;
+    return EFIT_OK;
+}
+
+extern "C" int efit_profile_end(efit_ctx* h, double* ms_out, int32_t nout, int32_t* nsteps_out) {
+    if (!h || !ms_out || nout < efit::kNumMarks) return fail(nullptr, EFIT_E_INVAL, "profile_end: bad argument");
+    Ctx& c = h->c;
+    if (!c.prof_ev) return fail(&c, EFIT_E_STATE, "profiling not active");
+    for (int k = 0; k < nout; ++k) ms_out[k] = 0.0;
+    int rc = EFIT_OK;
+    for (int st = 0; st < c.prof_next && rc == EFIT_OK; ++st) {
+        cudaEvent_t* ev = c.prof_ev + (size_t)st * efit::kNumMarks;
+        if (cudaEventSynchronize(ev[efit::M_SOLVE])) { rc = cuda_fail(&c, cudaGetLastError(), "event sync"); break; }
+        using namespace efit;
+        // (from, to) mark pairs of the nine reported intervals; k_bnd_tb and k_bnd_lr both
+        // start at the fork after the current kernel and run concurrently
+        static const int pairs[9][2] = {{M_BEGIN, M_SOLVE}, {M_BEGIN, M_NORM}, {M_NORM, M_RESP}, {M_RESP, M_LSQ},
+                                        {M_LSQ, M_CUR},     {M_CUR, M_TB},     {M_CUR, M_LR},   {M_TB, M_BRED},
+                                        {M_BRED, M_SOLVE}};
+        float t;
+        for (int k = 0; k < 9; ++k)
+            if (cudaEventElapsedTime(&t, ev[pairs[k][0]], ev[pairs[k][1]]) == cudaSuccess) ms_out[k] += t;
+    }
+    if (nsteps_out) *nsteps_out = c.prof_next;
+    for (size_t i = 0; i < (size_t)c.prof_slots * efit::kNumMarks; ++i) cudaEventDestroy(c.prof_ev[i]);
+    delete[] c.prof_ev;
+    c.prof_ev = nullptr;
+    c.prof_on = false;
+    c.prof_slots = c.prof_next = 0;
+    return rc;
 }
 
 extern "C" int efit_status(efit_ctx* h, efit_stream_t stream) {
@@ -447,6 +556,13 @@ extern "C" int efit_table(const efit_ctx* h, int which, const void** d_ptr) {
 extern "C" int efit_destroy(efit_ctx* h) {
     if (!h) return EFIT_OK;
     if (h->c.gexec) cudaGraphExecDestroy(h->c.gexec);
+    if (h->c.side) cudaStreamDestroy(h->c.side);
+    if (h->c.ev_fork) cudaEventDestroy(h->c.ev_fork);
+    if (h->c.ev_join) cudaEventDestroy(h->c.ev_join);
+    if (h->c.prof_ev) {
+        for (size_t i = 0; i < (size_t)h->c.prof_slots * efit::kNumMarks; ++i) cudaEventDestroy(h->c.prof_ev[i]);
+        delete[] h->c.prof_ev;
+    }
     delete h;
     return EFIT_OK;
 }

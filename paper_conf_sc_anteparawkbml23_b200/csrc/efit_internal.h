@@ -24,8 +24,9 @@ struct Tiling {
     int resp_gc, resp_nchunk, resp_mb;
     // top/bottom boundary: chunks of `tb_ch` doubles of each slab, groups of `tb_gi` slabs
     int tb_ch, tb_nchunk, tb_gi, tb_ngroup;
-    // left/right boundary: j-tiles of `lr_jt` targets per CTA, `lr_iib` source rows per CTA
-    int lr_jt, lr_njt, lr_iib, lr_nblk;
+    // left/right boundary: lr_jt targets per lane (odd), j-tiles of 32*lr_jt targets, 4 source
+    // rows per CTA (lr_nblk blocks), source loop padded to lr_jj = roundup(nh, lr_jt)
+    int lr_jt, lr_njt, lr_iib, lr_nblk, lr_jj;
     // normalisation / eps reductions
     int red_blocks;
 };
@@ -39,6 +40,7 @@ struct Ctx {
     int n_fl, n_mp, n_int, ndiag, n_lim, ip_sign;
     int mode, rank, world;
     int n_edge, ni, nmode;       // ni = nw-2 interior rows, nmode = nh-2 sine modes
+    int ni_pad;                  // row stride of the mode-major solve arrays (even)
     int fft_m, fft_log2;         // complex FFT length 2(nh-1) and its log2
     int m_lo, m_hi;              // response rows of this rank
     int i_lo, i_hi;              // top/bottom target rows of this rank (within [1, nw-1))
@@ -57,8 +59,9 @@ struct Ctx {
     int* dkind;         // [ndiag]          0 flux loop, 1 probe, 2 internal B_Z
     double* lim;        // [2*n_lim]        r then z
     double* tri_a;      // [ni]             sub-diagonal coefficient a_i
-    double* tri_cp;     // [ni][nmode]      Thomas c'_i per mode
-    double* tri_inv;    // [ni][nmode]      1/den_i per mode
+    double* tri_cp;     // [nmode][ld]      Thomas c'_i per mode (mode-major, ld = ni_pad)
+    double* tri_inv;    // [nmode][ld]      1/den_i per mode
+    double* tri_alpha;  // [nmode][ld]      -a_i/den_i (forward-sweep recurrence coefficient)
     double2* twiddle;   // [fft_m/2]        exp(-2 pi i k/M)
 
     // per-iteration scratch
@@ -68,18 +71,28 @@ struct Ctx {
     double* norm_part;  // [red_blocks][2]  (value, index) partials
     double* resp_part;  // [resp_nchunk][rows][nb]
     double* resp_cnt;   // [resp_nchunk]    masked-node counts
+    double* bmat;       // [nb][resp_nchunk*resp_gc]  basis values of this iteration (k-major)
     double* resp;       // [ndiag][nb]      full response (fit step)
     double* coef;       // [nb]
     double* chi2;       // [1]
-    double* pcurr;      // [nw*nh]
-    double2* ipair;     // [S]              (I[g], I[ii][nh-1-m])
+    double* pcurr;      // [roundup(nw*nh, tb_ch)]  current per cell, zero tail
+    double* pflip;      // [roundup(nw*nh, tb_ch)]  I[ii][nh-1-m] (vertically mirrored), zero tail
     double* tb_part;    // [tb_nchunk][nw][2]
     double* lr_part;    // [lr_nblk][2][nh]
     double* psib;       // [n_edge]
-    double* fhat;       // [ni][nmode]  DST coefficients (in place: Thomas solution)
+    double* fhat;       // [nmode][ld]  DST coefficients, mode-major (in place: tridiagonal solution)
     double* psip;       // [nw*nh]
     double* eps_part;   // [red_blocks]
     double* scratch_meas;  // [ndiag] (unused placeholder)
+
+    // profiling: CUDA events recorded at marks inside the fit step (efit_profile_begin/end)
+    bool prof_on;
+    int prof_slots, prof_next;
+    cudaEvent_t* prof_ev;  // [prof_slots][kNumMarks]
+
+    // side stream + events: k_bnd_lr (FP64-bound) runs concurrently with k_bnd_tb (HBM-bound)
+    cudaStream_t side;
+    cudaEvent_t ev_fork, ev_join;
 
     // CUDA graph cache for efit_fit_step
     cudaGraphExec_t gexec;
@@ -89,6 +102,10 @@ struct Ctx {
 
     char err[256];
 };
+
+// Marks recorded (as CUDA events) inside a profiled fit step, in stream order.
+enum Mark { M_BEGIN = 0, M_NORM, M_RESP, M_LSQ, M_CUR, M_TB, M_LR, M_BRED, M_SOLVE, kNumMarks };
+void mark(Ctx& c, cudaStream_t s, int id);  // efit_api.cu; no-op unless profiling
 
 // ---- launchers (efit_kernels.cu) -------------------------------------------------
 cudaError_t launch_init_tables(Ctx& c, cudaStream_t s);

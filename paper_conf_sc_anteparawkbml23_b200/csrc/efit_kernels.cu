@@ -45,6 +45,32 @@ __device__ __forceinline__ double2 ldg_stream(const double* p) {
     return v;
 }
 
+struct d4 {
+    double x, y, z, w;
+};
+
+// 256-bit streaming load (LDG.E.NA.EFL2.256): read-only, no L1 allocation, L2 evict-first.
+// Used for data read exactly once per iteration (Green's tables).  32-byte aligned.
+__device__ __forceinline__ d4 ld256_stream(const double* p) {
+    d4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::evict_first.v4.f64 {%0, %1, %2, %3}, [%4];"
+                 : "=d"(v.x), "=d"(v.y), "=d"(v.z), "=d"(v.w) : "l"(p));
+    return v;
+}
+
+__device__ __forceinline__ d4 lds256(const double* p) {  // two 128-bit shared loads
+    const double2 a = reinterpret_cast<const double2*>(p)[0];
+    const double2 b = reinterpret_cast<const double2*>(p)[1];
+    return d4{a.x, a.y, b.x, b.y};
+}
+
+__device__ __forceinline__ double dot4(const d4& a, const d4& b, double acc) {
+    acc = fma(a.x, b.x, acc);
+    acc = fma(a.y, b.y, acc);
+    acc = fma(a.z, b.z, acc);
+    return fma(a.w, b.w, acc);
+}
+
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
@@ -160,10 +186,13 @@ __global__ void k_inlim(uint8_t* __restrict__ inlim, const double* __restrict__ 
     }
 }
 
-// Thomas factors of the radial tridiagonal systems, one per sine mode k = 1..nmode:
+// Factors of the radial tridiagonal systems, one per sine mode k = 1..nmode:
 //   a_i x_{i-1} + (-2/dR^2 + lambda_k) x_i + c_i x_{i+1},  lambda_k = -4 sin^2(pi k/(2(n+1)))/dZ^2
+// LU (Thomas) factors den_i = b - a_i c'_{i-1}, c'_i = c_i/den_i, stored mode-major with the
+// forward-sweep coefficients  d_i = inv_i f_i + alpha_i d_{i-1},  alpha_i = -a_i/den_i.
 __global__ void k_tri_factors(double* __restrict__ tri_a, double* __restrict__ cp, double* __restrict__ inv,
-                              int ni, int nmode, double rmin, double dr, double dz) {
+                              double* __restrict__ alpha, int ni, int ld, int nmode, double rmin, double dr,
+                              double dz) {
     int k = blockIdx.x * blockDim.x + threadIdx.x;  // mode index 0..nmode-1 (mode k+1)
     double idr2 = 1.0 / (dr * dr);
     if (k == 0) {
@@ -183,8 +212,11 @@ __global__ void k_tri_factors(double* __restrict__ tri_a, double* __restrict__ c
         double c = idr2 - 1.0 / (2.0 * R * dr);
         double den = (i == 1) ? b : b - a * cprev;
         double cpi = c / den;
-        cp[(long long)(i - 1) * nmode + k] = cpi;
-        inv[(long long)(i - 1) * nmode + k] = 1.0 / den;
+        const int r = i - 1, L = ld >> 5;  // segment-interleaved position of row r
+        const long long o = (long long)k * ld + (long long)(r % L) * 32 + r / L;
+        cp[o] = (i == ni) ? 0.0 : cpi;
+        inv[o] = 1.0 / den;
+        alpha[o] = (i == 1) ? 0.0 : -a / den;
         cprev = cpi;
     }
 }
@@ -211,8 +243,11 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
         e = cudaMemsetAsync(c.Gd, 0, sizeof(double) * (size_t)(c.m_hi - c.m_lo) * c.S, s);
         if (e) return e;
     }
-    e = cudaMemsetAsync(c.ipair, 0, sizeof(double2) * (size_t)(((n + c.t.tb_ch - 1) / c.t.tb_ch) * c.t.tb_ch), s);
-    if (e) return e;
+    {
+        const size_t padn = (size_t)(((n + c.t.tb_ch - 1) / c.t.tb_ch) * c.t.tb_ch);
+        if ((e = cudaMemsetAsync(c.pcurr, 0, sizeof(double) * padn, s))) return e;
+        if ((e = cudaMemsetAsync(c.pflip, 0, sizeof(double) * padn, s))) return e;
+    }
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c.device);
     const int bs = 256;
@@ -223,7 +258,8 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
         k_green_diag<<<sms * 16, bs, 0, s>>>(c.Gd, c.S, c.m_hi - c.m_lo, c.m_lo, c.dgeo, c.dkind, nw, nh,
                                               c.rmin, c.dr, c.zmin, c.dz);
     k_inlim<<<(int)((n + bs - 1) / bs), bs, 0, s>>>(c.inlim, c.lim, c.n_lim, nw, nh, c.rmin, c.dr, c.zmin, c.dz);
-    k_tri_factors<<<(c.nmode + 63) / 64, 64, 0, s>>>(c.tri_a, c.tri_cp, c.tri_inv, c.ni, c.nmode, c.rmin, c.dr, c.dz);
+    k_tri_factors<<<(c.nmode + 63) / 64, 64, 0, s>>>(c.tri_a, c.tri_cp, c.tri_inv, c.tri_alpha, c.ni, c.ni_pad,
+                                                     c.nmode, c.rmin, c.dr, c.dz);
     k_twiddles<<<(c.fft_m / 2 + 255) / 256, 256, 0, s>>>(c.twiddle, c.fft_m);
     e = cudaMemsetAsync(c.status, 0, sizeof(int), s);
     if (e) return e;
@@ -250,10 +286,13 @@ __global__ void __launch_bounds__(256) k_normalize(const double* __restrict__ ps
     double best = -DBL_MAX;
     long long bi = LLONG_MAX;
     bool bad = false;
-    for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += gridDim.x * blockDim.x) {
-        double p = psi[g];
+    const int stride = gridDim.x * blockDim.x;
+#pragma unroll 4
+    for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += stride) {
+        const double p = __ldg(psi + g);
+        const uint8_t in = __ldg(inlim + g);
         if (!isfinite(p)) bad = true;
-        if (inlim[g]) argmax_merge(best, bi, s * p, (long long)g);
+        if (in) argmax_merge(best, bi, s * p, (long long)g);
     }
     if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(status, EFIT_ST_NONFINITE);
     warp_argmax(best, bi);
@@ -333,101 +372,132 @@ __device__ __forceinline__ bool node_psihat(const double* psi, const uint8_t* in
 
 // ================================================================================ response
 
-// One CTA per chunk of `gc` nodes: basis values of the chunk (fused basis evaluation, never
-// materialised in HBM) into shared memory Bs[k][q], then warps stream the Gd rows of the chunk
-// with 128-bit loads, MB rows at a time, accumulating MB x NB dot products in registers.
-template <int NB, int MB>
-__global__ void __launch_bounds__(256) k_response(const double* __restrict__ Gd, long long S, int nrows,
-                                                  const double* __restrict__ psi, const uint8_t* __restrict__ inlim,
-                                                  const double* __restrict__ axbd, int nw, int nh,
-                                                  double rmin, double dr, double cell, BasisParams bp, int gc,
-                                                  double* __restrict__ part, double* __restrict__ cnt_part) {
-    extern __shared__ __align__(16) double Bs[];  // [NB][gc]
-    __shared__ int cnt_s[8];
+// Basis values of every node for this iteration: Bm[k][g] = dR dZ mask_g w_k(R_g) phi_k(psihat_g)
+// (k-major, zero-padded to whole chunks), plus the masked-node count per chunk.  ~10 MB at 513^2,
+// written once and read by k_response from L2.
+template <int NB>
+__global__ void __launch_bounds__(1024) k_basis(const double* __restrict__ psi, const uint8_t* __restrict__ inlim,
+                                               const double* __restrict__ axbd, int nw, int nh, double rmin,
+                                               double dr, double cell, BasisParams bp, int gc, long long ldb,
+                                               double* __restrict__ Bm, double* __restrict__ cnt_part) {
+    __shared__ int cnt_s[32];
     const int n = nw * nh;
-    const int c = blockIdx.x;
-    const int g0 = c * gc;
+    const int g0 = blockIdx.x * gc;
     const double pa = axbd[0], pb = axbd[1];
     int cnt = 0;
     for (int q = threadIdx.x; q < gc; q += blockDim.x) {
-        int g = g0 + q;
+        const int g = g0 + q;
         double f[NB];
 #pragma unroll
         for (int k = 0; k < NB; ++k) f[k] = 0.0;
         double h;
         if (g < n && node_psihat(psi, inlim, g, pa, pb, h)) {
-            double R = grid_coord(rmin, g / nh, dr);
-            basis_eval<NB>(bp, h, R, f);
+            basis_eval<NB>(bp, h, grid_coord(rmin, g / nh, dr), f);
             ++cnt;
         }
 #pragma unroll
-        for (int k = 0; k < NB; ++k) Bs[k * gc + q] = cell * f[k];
+        for (int k = 0; k < NB; ++k) Bm[k * ldb + g] = cell * f[k];
     }
-    int wc = __reduce_add_sync(0xffffffffu, cnt);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int wc = __reduce_add_sync(0xffffffffu, cnt);
     if (lane == 0) cnt_s[warp] = wc;
     __syncthreads();
     if (threadIdx.x == 0) {
         int t = 0;
         for (int q = 0; q < (int)(blockDim.x >> 5); ++q) t += cnt_s[q];
-        cnt_part[c] = (double)t;
+        cnt_part[blockIdx.x] = (double)t;
     }
-    const int nwarps = blockDim.x >> 5;
-    const int nmb = (nrows + MB - 1) / MB;
-    const int qend = min(gc, n - g0);  // valid nodes in this chunk (pairs may read 1 padding entry)
-    for (int mb = warp; mb < nmb; mb += nwarps) {
-        double acc[MB][NB];
+}
+
+// Grid (chunk of `gc` nodes) x (group of 8*MB diagnostic rows).  The CTA stages the chunk's
+// basis values in shared memory, permuted so that the 4 values a lane needs (nodes q..q+3) are
+// two 16-byte words at stride 512 B across lanes (conflict-free).  Each warp streams MB Gd rows:
+// per step it issues all 2*MB 256-bit loads (2 positions of 128 nodes, 192-256 B per thread in
+// flight), then does the 2*MB*NB*4 FMAs; the MB x NB dot products are reduced once per chunk
+// with a fixed butterfly.  Every Gd byte is read from HBM exactly once.
+__device__ __forceinline__ int bperm(int q) {  // node q of a chunk -> permuted shared offset (per k)
+    const int blk = q >> 7, lane = (q >> 2) & 31, h = (q >> 1) & 1, w = q & 1;
+    return (blk << 7) + (h << 6) + (lane << 1) + w;
+}
+
+template <int NB, int MB>
+__global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ Gd, long long S, int nrows, int n,
+                                                     const double* __restrict__ Bm, long long ldb, int gc,
+                                                     double* __restrict__ part) {
+    extern __shared__ __align__(16) double Bs[];  // [NB][gc] permuted
+    const int c = blockIdx.x;
+    const int g0 = c * gc;
+    for (int e = 2 * threadIdx.x; e < NB * gc; e += 2 * blockDim.x) {
+        const int k = e / gc, q = e - (e / gc) * gc;
+        const double2 v = __ldg(reinterpret_cast<const double2*>(Bm + k * ldb + g0 + q));
+        *reinterpret_cast<double2*>(Bs + k * gc + bperm(q)) = v;
+    }
+    __syncthreads();
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int row0 = (blockIdx.y * 8 + warp) * MB;
+    if (row0 >= nrows) return;
+    const int qend = min(gc, n - g0);  // valid nodes; a 4-wide load may read up to 3 zero pads
+    double acc[MB][NB];
 #pragma unroll
-        for (int r = 0; r < MB; ++r)
+    for (int r = 0; r < MB; ++r)
 #pragma unroll
-            for (int k = 0; k < NB; ++k) acc[r][k] = 0.0;
-        const double* rowp[MB];
+        for (int k = 0; k < NB; ++k) acc[r][k] = 0.0;
+    const double* rowp[MB];
+#pragma unroll
+    for (int r = 0; r < MB; ++r) rowp[r] = Gd + (long long)min(row0 + r, nrows - 1) * S + g0;
+    for (int q0 = 0; q0 < qend; q0 += 256) {
+        const int qa = q0 + 4 * lane, qb = qa + 128;
+        const bool va = qa < qend, vb = qb < qend;
+        d4 ga[MB], gb[MB];
 #pragma unroll
         for (int r = 0; r < MB; ++r) {
-            int row = mb * MB + r;
-            rowp[r] = Gd + (long long)(row < nrows ? row : nrows - 1) * S + g0;
-        }
-#pragma unroll 2
-        for (int q = 2 * lane; q < qend; q += 64) {
-            double2 gv[MB];
-#pragma unroll
-            for (int r = 0; r < MB; ++r) gv[r] = ldg_stream(rowp[r] + q);
-#pragma unroll
-            for (int k = 0; k < NB; ++k) {
-                double2 b = *reinterpret_cast<const double2*>(&Bs[k * gc + q]);
-#pragma unroll
-                for (int r = 0; r < MB; ++r) {
-                    acc[r][k] = fma(gv[r].x, b.x, acc[r][k]);
-                    acc[r][k] = fma(gv[r].y, b.y, acc[r][k]);
-                }
-            }
+            ga[r] = va ? ld256_stream(rowp[r] + qa) : d4{0.0, 0.0, 0.0, 0.0};
+            gb[r] = vb ? ld256_stream(rowp[r] + qb) : d4{0.0, 0.0, 0.0, 0.0};
         }
 #pragma unroll
-        for (int r = 0; r < MB; ++r) {
-            int row = mb * MB + r;
+        for (int k = 0; k < NB; ++k) {
+            const double* bk = Bs + k * gc + q0 + 2 * lane;
+            const double2 a0 = *reinterpret_cast<const double2*>(bk);
+            const double2 a1 = *reinterpret_cast<const double2*>(bk + 64);
+            const double2 b0 = *reinterpret_cast<const double2*>(bk + 128);
+            const double2 b1 = *reinterpret_cast<const double2*>(bk + 192);
+            const d4 ba{a0.x, a0.y, a1.x, a1.y}, bb{b0.x, b0.y, b1.x, b1.y};
 #pragma unroll
-            for (int k = 0; k < NB; ++k) {
-                double v = warp_sum(acc[r][k]);
-                if (lane == 0 && row < nrows) part[((long long)c * nrows + row) * NB + k] = v;
+            for (int r = 0; r < MB; ++r) {
+                acc[r][k] = dot4(ga[r], ba, acc[r][k]);
+                acc[r][k] = dot4(gb[r], bb, acc[r][k]);
             }
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < MB; ++r) {
+        const int row = row0 + r;
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+            double v = warp_sum(acc[r][k]);
+            if (lane == 0 && row < nrows) part[((long long)row * NB + k) * gridDim.x + c] = v;
         }
     }
 }
 
-// out[r][k] = sum over chunks in index order; total masked count -> status.
+// out[r][k] = sum over chunks (partials stored chunk-fastest): one warp per output, lanes take
+// chunks lane, lane+32, ... and a fixed butterfly combines them => deterministic.  The total
+// masked-node count decides EFIT_ST_NOPLASMA.
 __global__ void k_resp_reduce(const double* __restrict__ part, const double* __restrict__ cnt_part, int nchunk,
-                              int nrows, int nb, double* __restrict__ out, int* status) {
-    int t = blockIdx.x * blockDim.x + threadIdx.x;
-    int total = nrows * nb;
-    if (t < total) {
+                              int total, double* __restrict__ out, int* status) {
+    const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+    if (w < total) {
+        const double* p = part + (long long)w * nchunk;
         double s = 0.0;
-        for (int c = 0; c < nchunk; ++c) s += part[(long long)c * total + t];
-        out[t] = s;
+        for (int c = lane; c < nchunk; c += 32) s += p[c];
+        s = warp_sum(s);
+        if (lane == 0) out[w] = s;
     }
-    if (t == 0) {
+    if (blockIdx.x == 0 && threadIdx.x < 32) {
         double cnt = 0.0;
-        for (int c = 0; c < nchunk; ++c) cnt += cnt_part[c];
-        if (cnt == 0.0) atomicOr(status, EFIT_ST_NOPLASMA);
+        for (int c = lane; c < nchunk; c += 32) cnt += cnt_part[c];
+        cnt = warp_sum(cnt);
+        if (lane == 0 && cnt == 0.0) atomicOr(status, EFIT_ST_NOPLASMA);
     }
 }
 
@@ -435,15 +505,19 @@ template <int NB>
 static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t s, int nrows, bool prepare) {
     const int gc = c.t.resp_gc;
     const size_t smem = sizeof(double) * NB * gc;
-    BasisParams bp = basis_params(c);
-    const double* Gd = c.Gd;
+    const long long ldb = (long long)c.t.resp_nchunk * gc;
+    if (!prepare) {
+        BasisParams bp = basis_params(c);
+        k_basis<NB><<<c.t.resp_nchunk, gc <= 1024 ? gc : 1024, 0, s>>>(psi, c.inlim, c.axbd, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp,
+                                                    gc, ldb, c.bmat, c.resp_cnt);
+    }
     int mb = c.t.resp_mb;
 #define EFIT_RESP_LAUNCH(MBV)                                                                              \
     do {                                                                                                   \
         auto kern = k_response<NB, MBV>;                                                                   \
-        if (prepare) { raise_smem_limit((const void*)kern, smem); break; } \
-        kern<<<c.t.resp_nchunk, 256, smem, s>>>(Gd, c.S, nrows, psi, c.inlim, c.axbd, c.nw, c.nh, c.rmin, c.dr, \
-                                                c.dr * c.dz, bp, gc, part, c.resp_cnt);                  \
+        if (prepare) { raise_smem_limit((const void*)kern, smem); break; }                               \
+        dim3 grid(c.t.resp_nchunk, (nrows + 8 * MBV - 1) / (8 * MBV));                                    \
+        kern<<<grid, 256, smem, s>>>(c.Gd, c.S, nrows, c.nw * c.nh, c.bmat, ldb, gc, part);               \
     } while (0)
     if (mb >= 4) EFIT_RESP_LAUNCH(4);
     else if (mb == 3) EFIT_RESP_LAUNCH(3);
@@ -467,8 +541,8 @@ static cudaError_t response_impl(Ctx& c, const double* psi, double* resp_rows, c
     cudaError_t e = cudaGetLastError();
     if (e || prepare) return e;
     const int total = nrows * c.nb;
-    k_resp_reduce<<<(total + 255) / 256, 256, 0, s>>>(c.resp_part, c.resp_cnt, c.t.resp_nchunk, nrows, c.nb,
-                                                      resp_rows, c.status);
+    k_resp_reduce<<<(total + 7) / 8, 256, 0, s>>>(c.resp_part, c.resp_cnt, c.t.resp_nchunk, total, resp_rows,
+                                                  c.status);
     return cudaGetLastError();
 }
 
@@ -478,106 +552,98 @@ cudaError_t launch_response(Ctx& c, const double* psi, double* resp_rows, cudaSt
 
 // ================================================================================ least squares
 
-// One CTA: rows scaled by 1/sigma, columns to unit 2-norm, Householder QR (reflectors
-// v = x + sign(x_0)|x| e_0), back substitution, unscale; chi2 = sum((meas - A c)/sigma)^2.
-// Reductions are fixed-order (warp shuffles + one ordered pass), so the result is deterministic.
-
-__global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, const double* __restrict__ meas,
+// One CTA of 4 warps: rows scaled by 1/sigma, columns to unit 2-norm, Householder QR (reflectors
+// v = x - alpha e_k, alpha = -sign(x_k)|x|, H = I - v v^T/(|x|(|x| + |x_k|))), back substitution,
+// unscale; chi2 = sum((meas - A c)/sigma)^2.  Per reflection: warp 0 forms alpha and v, then the
+// remaining columns (and b) are updated by different warps in parallel -- two barriers per
+// reflection.  Lane-strided sums + fixed butterflies => deterministic.
+__global__ void __launch_bounds__(128) k_lsq(const double* __restrict__ resp, const double* __restrict__ meas,
                                              const double* __restrict__ sigma, int nd, int nb,
                                              double* __restrict__ coef, double* __restrict__ chi2, int* status) {
     extern __shared__ __align__(16) double sm[];
-    double* A = sm;                      // [nb][nd] column-major (scaled)
-    double* b = A + (size_t)nb * nd;     // [nd]
-    double* v = b + nd;                  // [nd]
-    double* red = v + nd;                // [32 + 64]
-    double* scale = red + 96;            // [nb]
-    double* x = scale + 32;              // [nb]
+    double* A = sm;                   // [nb+1][nd] column-major (scaled); column nb = b
+    double* isg = A + (size_t)(nb + 1) * nd;  // [nd] 1/sigma
+    double* sc = isg + nd;            // [32] column scales
+    double* x = sc + 32;              // [32] solution
+    double* red = x + 32;             // [8]
+    __shared__ double s_alpha, s_vtv2;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarp = blockDim.x >> 5;
-    __shared__ int bad;
-    if (tid == 0) bad = (*status & (EFIT_ST_NOPLASMA | EFIT_ST_NONFINITE)) ? 1 : 0;
-    for (int e = tid; e < nd * nb; e += blockDim.x) {
-        int m = e / nb, k = e - (e / nb) * nb;
-        A[(size_t)k * nd + m] = resp[e] / sigma[m];
+    for (int m = tid; m < nd; m += blockDim.x) {
+        const double is = 1.0 / sigma[m];
+        isg[m] = is;
+        for (int k = 0; k < nb; ++k) A[(size_t)k * nd + m] = resp[(size_t)m * nb + k] * is;
+        A[(size_t)nb * nd + m] = meas[m] * is;
     }
-    for (int m = tid; m < nd; m += blockDim.x) b[m] = meas[m] / sigma[m];
     __syncthreads();
-    // column norms: warp per column
     for (int k = warp; k < nb; k += nwarp) {
+        double* col = A + (size_t)k * nd;
         double s = 0.0;
-        for (int m = lane; m < nd; m += 32) { double a = A[(size_t)k * nd + m]; s += a * a; }
-        s = warp_sum(s);
-        if (lane == 0) scale[k] = sqrt(s);
-    }
-    __syncthreads();
-    for (int e = tid; e < nd * nb; e += blockDim.x) {
-        int k = e / nd;
-        double sc = scale[k];
-        A[e] = sc > 0.0 ? A[e] / sc : 0.0;
+        for (int m = lane; m < nd; m += 32) s = fma(col[m], col[m], s);
+        s = sqrt(warp_sum(s));
+        const double is = s > 0.0 ? 1.0 / s : 0.0;
+        for (int m = lane; m < nd; m += 32) col[m] *= is;
+        if (lane == 0) sc[k] = s;
     }
     __syncthreads();
     for (int k = 0; k < nb; ++k) {
-        // norm of column k below (and incl.) the diagonal: warp 0
+        double* ck = A + (size_t)k * nd;
         if (warp == 0) {
             double s = 0.0;
-            for (int m = k + lane; m < nd; m += 32) { double a = A[(size_t)k * nd + m]; s += a * a; }
-            s = warp_sum(s);
+            for (int m = k + lane; m < nd; m += 32) s = fma(ck[m], ck[m], s);
+            const double nx = sqrt(warp_sum(s));
             if (lane == 0) {
-                double nx = sqrt(s);
-                double x0 = A[(size_t)k * nd + k];
-                double alpha = x0 >= 0.0 ? -nx : nx;      // R_kk = alpha
-                red[0] = alpha;
-                red[1] = nx * (nx + fabs(x0));            // v^T v / 2 with v = x - alpha e_k
+                const double x0 = ck[k];
+                const double alpha = x0 >= 0.0 ? -nx : nx;
+                s_alpha = alpha;
+                s_vtv2 = nx * (nx + fabs(x0));
+                ck[k] = x0 - alpha;  // ck[k..nd) now holds v
             }
         }
         __syncthreads();
-        double alpha = red[0], vtv2 = red[1];
-        for (int m = tid; m < nd; m += blockDim.x) v[m] = (m < k) ? 0.0 : (m == k ? A[(size_t)k * nd + k] - alpha : A[(size_t)k * nd + m]);
-        __syncthreads();
-        // apply H = I - v v^T / vtv2 to columns j > k and to b (warp per column)
+        const double vtv2 = s_vtv2;
         for (int j = k + 1 + warp; j <= nb; j += nwarp) {
-            double* col = (j < nb) ? A + (size_t)j * nd : b;
-            double s = 0.0;
-            for (int m = k + lane; m < nd; m += 32) s += v[m] * col[m];
-            s = warp_sum(s);
-            double f = vtv2 > 0.0 ? s / vtv2 : 0.0;
-            for (int m = k + lane; m < nd; m += 32) col[m] -= f * v[m];
+            double* cj = A + (size_t)j * nd;
+            double d = 0.0;
+            for (int m = k + lane; m < nd; m += 32) d = fma(ck[m], cj[m], d);
+            d = warp_sum(d);
+            const double f = vtv2 > 0.0 ? d / vtv2 : 0.0;
+            for (int m = k + lane; m < nd; m += 32) cj[m] = fma(-f, ck[m], cj[m]);
         }
         __syncthreads();
-        if (tid == 0) {
-            A[(size_t)k * nd + k] = alpha;
-            for (int m = k + 1; m < nd; ++m) A[(size_t)k * nd + m] = 0.0;
-        }
-        __syncthreads();
+        if (tid == 0) ck[k] = s_alpha;  // R_kk (rows below k of column k are no longer read)
     }
+    __syncthreads();
     if (tid == 0) {
         double rmax = 0.0;
         for (int k = 0; k < nb; ++k) rmax = fmax(rmax, fabs(A[(size_t)k * nd + k]));
         bool sing = false;
         for (int k = 0; k < nb; ++k)
-            if (!(fabs(A[(size_t)k * nd + k]) >= 1e-13 * rmax) || !(scale[k] > 0.0)) sing = true;
-        if (sing) { atomicOr(status, EFIT_ST_SINGULAR); bad = 1; }
+            if (!(fabs(A[(size_t)k * nd + k]) >= 1e-13 * rmax) || !(sc[k] > 0.0)) sing = true;
+        const double* bq = A + (size_t)nb * nd;
         for (int k = nb - 1; k >= 0; --k) {
-            double s = b[k];
+            double s = bq[k];
             for (int j = k + 1; j < nb; ++j) s -= A[(size_t)j * nd + k] * x[j];
             x[k] = s / A[(size_t)k * nd + k];
         }
-        for (int k = 0; k < nb; ++k) x[k] = x[k] / scale[k];
+        for (int k = 0; k < nb; ++k) x[k] = x[k] / sc[k];
+        if (sing) atomicOr(status, EFIT_ST_SINGULAR);
+        red[7] = sing ? 1.0 : 0.0;
     }
     __syncthreads();
-    // chi2 with the unscaled matrix
     double s = 0.0;
     for (int m = tid; m < nd; m += blockDim.x) {
         double r = meas[m];
-        for (int k = 0; k < nb; ++k) r -= resp[(size_t)m * nb + k] * x[k];
-        r /= sigma[m];
-        s += r * r;
+        for (int k = 0; k < nb; ++k) r = fma(-resp[(size_t)m * nb + k], x[k], r);
+        r *= isg[m];
+        s = fma(r, r, s);
     }
     s = warp_sum(s);
-    if (lane == 0) red[32 + warp] = s;
+    if (lane == 0) red[warp] = s;
     __syncthreads();
     if (tid == 0) {
         double t = 0.0;
-        for (int q = 0; q < nwarp; ++q) t += red[32 + q];
+        for (int q = 0; q < nwarp; ++q) t += red[q];
+        const bool bad = (*status & (EFIT_ST_NOPLASMA | EFIT_ST_NONFINITE)) != 0 || red[7] != 0.0;
         const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
         *chi2 = bad ? nanv : t;
         for (int k = 0; k < nb; ++k) coef[k] = bad ? nanv : x[k];
@@ -585,13 +651,13 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
 }
 
 static size_t lsq_smem(const Ctx& c) {
-    return sizeof(double) * ((size_t)c.nb * c.ndiag + 2 * (size_t)c.ndiag + 96 + 32 + 32);
+    return sizeof(double) * ((size_t)(c.nb + 2) * c.ndiag + 72);
 }
 
 cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const double* sigma, double* coef,
                        double* chi2, cudaStream_t s) {
     size_t smem = lsq_smem(c);
-    k_lsq<<<1, 256, smem, s>>>(resp, meas, sigma, c.ndiag, c.nb, coef, chi2, c.status);
+    k_lsq<<<1, 128, smem, s>>>(resp, meas, sigma, c.ndiag, c.nb, coef, chi2, c.status);
     return cudaGetLastError();
 }
 
@@ -615,33 +681,65 @@ template <int NB>
 __global__ void k_current(const double* __restrict__ psi, const uint8_t* __restrict__ inlim,
                           const double* __restrict__ axbd, const double* __restrict__ coef, int nw, int nh,
                           double rmin, double dr, double cell, BasisParams bp, double* __restrict__ pcurr,
-                          double2* __restrict__ ipair) {
+                          double* __restrict__ pflip) {
     const int n = nw * nh;
     const double pa = axbd[0], pb = axbd[1];
     double cf[NB];
 #pragma unroll
     for (int k = 0; k < NB; ++k) cf[k] = coef[k];
     for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += gridDim.x * blockDim.x) {
-        double I = current_at<NB>(psi, inlim, g, nh, pa, pb, rmin, dr, cell, bp, cf);
-        if (pcurr) pcurr[g] = I;
-        if (ipair) {
-            int ii = g / nh, m = g - (g / nh) * nh;
-            int gf = ii * nh + (nh - 1 - m);
-            double If = current_at<NB>(psi, inlim, gf, nh, pa, pb, rmin, dr, cell, bp, cf);
-            ipair[g] = make_double2(I, If);
+        const double I = current_at<NB>(psi, inlim, g, nh, pa, pb, rmin, dr, cell, bp, cf);
+        pcurr[g] = I;
+        if (pflip) {  // I at the vertically mirrored node, for the top-target dot products
+            const int ii = g / nh, m = g - (g / nh) * nh;
+            pflip[ii * nh + (nh - 1 - m)] = I;
         }
+    }
+}
+
+// Fit-step current from this iteration's basis matrix (already masked and scaled by dR dZ):
+// I_g = sum_k c_k Bm[k][g]  -- no second basis evaluation.
+template <int NB>
+__global__ void k_current_from_basis(const double* __restrict__ Bm, long long ldb, const double* __restrict__ coef,
+                                     int nw, int nh, double* __restrict__ pcurr, double* __restrict__ pflip) {
+    const int n = nw * nh;
+    double cf[NB];
+#pragma unroll
+    for (int k = 0; k < NB; ++k) cf[k] = coef[k];
+    for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += gridDim.x * blockDim.x) {
+        double I = 0.0;
+#pragma unroll
+        for (int k = 0; k < NB; ++k) I = fma(cf[k], Bm[k * ldb + g], I);
+        pcurr[g] = I;
+        const int ii = g / nh, m = g - (g / nh) * nh;
+        pflip[ii * nh + (nh - 1 - m)] = I;
     }
 }
 
 cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double* pcurr, bool pair,
                            cudaStream_t s) {
     BasisParams bp = basis_params(c);
+    if (pair) {  // fit step: the basis matrix of this iteration is in c.bmat (k_basis ran in response)
+        const int n = c.nw * c.nh;
+        const long long ldb = (long long)c.t.resp_nchunk * c.t.resp_gc;
+        switch (c.nb) {
+#define EFIT_NB_CASE(V) \
+    case V: k_current_from_basis<V><<<(n + 255) / 256, 256, 0, s>>>(c.bmat, ldb, coef, c.nw, c.nh, pcurr, c.pflip); break;
+            EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
+            EFIT_NB_CASE(7) EFIT_NB_CASE(8) EFIT_NB_CASE(9) EFIT_NB_CASE(10) EFIT_NB_CASE(11) EFIT_NB_CASE(12)
+            EFIT_NB_CASE(13) EFIT_NB_CASE(14) EFIT_NB_CASE(15) EFIT_NB_CASE(16) EFIT_NB_CASE(17) EFIT_NB_CASE(18)
+            EFIT_NB_CASE(19) EFIT_NB_CASE(20) EFIT_NB_CASE(21) EFIT_NB_CASE(22) EFIT_NB_CASE(23) EFIT_NB_CASE(24)
+#undef EFIT_NB_CASE
+            default: return cudaErrorInvalidValue;
+        }
+        return cudaGetLastError();
+    }
     const int n = c.nw * c.nh;
     const int blocks = (n + 255) / 256;
-    double2* ip = pair ? c.ipair : nullptr;
+    double* fl = pair ? c.pflip : nullptr;
     switch (c.nb) {
 #define EFIT_NB_CASE(V) \
-    case V: k_current<V><<<blocks, 256, 0, s>>>(psi, c.inlim, c.axbd, coef, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp, pcurr, ip); break;
+    case V: k_current<V><<<blocks, 256, 0, s>>>(psi, c.inlim, c.axbd, coef, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp, pcurr, fl); break;
         EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
         EFIT_NB_CASE(7) EFIT_NB_CASE(8) EFIT_NB_CASE(9) EFIT_NB_CASE(10) EFIT_NB_CASE(11) EFIT_NB_CASE(12)
         EFIT_NB_CASE(13) EFIT_NB_CASE(14) EFIT_NB_CASE(15) EFIT_NB_CASE(16) EFIT_NB_CASE(17) EFIT_NB_CASE(18)
@@ -657,38 +755,54 @@ cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double
 // Top/bottom targets (the second O(N^3) nest, reading Q2): for target row i,
 //   psi_b(i, 0)    = sum_{ii,m} T[i][ii][m] I[ii][m]
 //   psi_b(i, nh-1) = sum_{ii,m} T[i][ii][m] I[ii][nh-1-m]
-// i.e. two dot products of slab T[i] with the (I, I_flipped) pair array.  A CTA owns a chunk of
-// `ch` slab entries (its pair values staged once in shared memory) and GI slabs; every T byte is
-// read from HBM exactly once with 128-bit streaming loads.
-template <int GI>
-__global__ void __launch_bounds__(256) k_bnd_tb(const double* __restrict__ T, long long S, int nslab, int row_lo,
-                                                int n, const double2* __restrict__ ipair, int ch,
-                                                double* __restrict__ part, int nw) {
-    extern __shared__ __align__(16) double2 ips[];  // [ch]
+// i.e. two dot products of slab T[i] with I and with the vertically mirrored I (F).  A CTA owns
+// a chunk of `ch` slab entries (its I and F values staged once in shared memory, consecutive
+// lanes -> consecutive 32-byte words, conflict-free) and GI slabs; every T byte is read from HBM
+// exactly once with 256-bit streaming loads, UNR slabs x 2 positions (256 B per thread) in flight.
+template <int GI, int UNR>
+__global__ void __launch_bounds__(256, 2) k_bnd_tb(const double* __restrict__ T, long long S, int nslab,
+                                                   int row_lo, int n, const double* __restrict__ Ib,
+                                                   const double* __restrict__ Fb, int ch,
+                                                   double* __restrict__ part) {
+    extern __shared__ __align__(16) double sm_tb[];
+    double* sI = sm_tb;        // [ch]
+    double* sF = sm_tb + ch;   // [ch]
     __shared__ double red[8][2 * GI];
     const int c = blockIdx.x, grp = blockIdx.y;
     const long long e0 = (long long)c * ch;
-    const int len = (int)min((long long)ch, (long long)n - e0);  // valid entries in this chunk
-    for (int q = threadIdx.x; q < ch; q += blockDim.x) ips[q] = ipair[e0 + q];
+    const int len = (int)min((long long)ch, (long long)n - e0);
+    for (int q = 4 * threadIdx.x; q < ch; q += 4 * blockDim.x) {
+        *reinterpret_cast<double2*>(sI + q) = __ldg(reinterpret_cast<const double2*>(Ib + e0 + q));
+        *reinterpret_cast<double2*>(sI + q + 2) = __ldg(reinterpret_cast<const double2*>(Ib + e0 + q + 2));
+        *reinterpret_cast<double2*>(sF + q) = __ldg(reinterpret_cast<const double2*>(Fb + e0 + q));
+        *reinterpret_cast<double2*>(sF + q + 2) = __ldg(reinterpret_cast<const double2*>(Fb + e0 + q + 2));
+    }
     __syncthreads();
     double a0[GI], a1[GI];
 #pragma unroll
     for (int t = 0; t < GI; ++t) { a0[t] = 0.0; a1[t] = 0.0; }
     const int s0 = grp * GI;
+    const int q0 = 4 * threadIdx.x, q1 = q0 + 4 * blockDim.x;  // two 4-wide positions per slab (ch = 2048)
+    const bool v0 = q0 < len, v1 = q1 < len;
 #pragma unroll
-    for (int t = 0; t < GI; ++t) {
-        const int sl = s0 + t;
-        if (sl < nslab) {
-            const double* base = T + (long long)sl * S + e0;
-#pragma unroll 4
-            for (int q = 2 * threadIdx.x; q < len; q += 2 * blockDim.x) {
-                double2 tv = ldg_stream(base + q);
-                double2 p0 = ips[q], p1 = ips[q + 1];
-                a0[t] = fma(tv.x, p0.x, a0[t]);
-                a1[t] = fma(tv.x, p0.y, a1[t]);
-                a0[t] = fma(tv.y, p1.x, a0[t]);
-                a1[t] = fma(tv.y, p1.y, a1[t]);
-            }
+    for (int t = 0; t < GI; t += UNR) {
+        d4 tv[UNR][2];
+#pragma unroll
+        for (int u = 0; u < UNR; ++u) {
+            const int sl = s0 + t + u;
+            const double* base = T + (long long)min(sl, nslab - 1) * S + e0;
+            const bool ok = sl < nslab;
+            tv[u][0] = (ok && v0) ? ld256_stream(base + q0) : d4{0.0, 0.0, 0.0, 0.0};
+            tv[u][1] = (ok && v1) ? ld256_stream(base + q1) : d4{0.0, 0.0, 0.0, 0.0};
+        }
+        const d4 i0 = lds256(sI + q0), i1 = lds256(sI + q1);
+        const d4 f0 = lds256(sF + q0), f1 = lds256(sF + q1);
+#pragma unroll
+        for (int u = 0; u < UNR; ++u) {
+            a0[t + u] = dot4(tv[u][0], i0, a0[t + u]);
+            a1[t + u] = dot4(tv[u][0], f0, a1[t + u]);
+            a0[t + u] = dot4(tv[u][1], i1, a0[t + u]);
+            a1[t + u] = dot4(tv[u][1], f1, a1[t + u]);
         }
     }
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -703,151 +817,158 @@ __global__ void __launch_bounds__(256) k_bnd_tb(const double* __restrict__ T, lo
         const int t = threadIdx.x >> 1, side = threadIdx.x & 1;
         const int sl = s0 + t;
         if (sl < nslab) {
-            double s = 0.0;
-            for (int w = 0; w < (int)(blockDim.x >> 5); ++w) s += red[w][threadIdx.x];
-            part[((long long)c * nw + row_lo + sl) * 2 + side] = s;
+            double sum = 0.0;
+            for (int w = 0; w < (int)(blockDim.x >> 5); ++w) sum += red[w][threadIdx.x];
+            part[((long long)(row_lo + sl) * 2 + side) * gridDim.x + c] = sum;
         }
     }
 }
 
 // Left/right targets (the printed Fig. 2 nest): for side s (slab i = 0 or nw-1),
-//   psi_b(s, j) = sum_ii sum_jj T[s][ii][|j - jj|] I[ii][jj].
-// Each row ii is a symmetric Toeplitz product.  A warp owns JT consecutive targets j0..j0+JT-1,
-// lanes own contiguous jj ranges and keep the JT kernel values t[|j - jj|] in a register
-// window that slides by one per jj step (one new shared-memory load per step, slot index
-// (a - u) mod JT resolved at compile time by unrolling).  CTA = 8 warps x JT targets, one block
-// of `iib` source rows; partial sums per block are reduced in block order by k_bnd_reduce.
+//   psi_b(s, j) = sum_ii sum_jj T[s][ii][|j - jj|] I[ii][jj]
+// (a symmetric Toeplitz product per source row ii).  A warp owns one source row ii and one
+// quarter of its sources jj; lane l owns JT consecutive targets j = jt0 + JT l + a (JT odd => the
+// lane stride is conflict-free in shared memory) and the whole warp steps through jj together
+// (x[jj] is a broadcast).  The kernel row is staged mirrored and zero-padded, so target a at step u
+// needs tx[JT l + a - u + JQ - 1]: a register window sliding by one per step with one new shared
+// load, slot (a - u) mod JT resolved at compile time by unrolling by JT, and no bounds checks
+// (sources zero-padded to 4*JQ).  17 FMA per 2 shared loads.  CTA = 2 rows x 4 quarters; the 8
+// warps are summed in fixed order, the per-row-pair partials in pair order by k_bnd_reduce.
 template <int JT>
 __global__ void __launch_bounds__(256) k_bnd_lr(const double* __restrict__ Tedge, long long S,
-                                                const double* __restrict__ I, int nw, int nh, int iib,
+                                                const double* __restrict__ I, int nw, int nh, int JQ,
                                                 int jt_lo, double* __restrict__ part) {
-    extern __shared__ __align__(16) double sm[];
-    double* ts = sm;                    // [iib][nh] kernel rows
-    double* xs = sm + (size_t)iib * nh; // [iib][nh] current rows
-    const int tile = jt_lo + blockIdx.x;
-    const int blk = blockIdx.y;
-    const int side = blockIdx.z;
-    const int ii0 = blk * iib;
-    const int nrow = min(iib, nw - ii0);
-    const double* tsrc = Tedge + (long long)side * S + (long long)ii0 * nh;
-    const double* xsrc = I + (long long)ii0 * nh;
-    for (int e = threadIdx.x; e < nrow * nh; e += blockDim.x) {
-        ts[e] = tsrc[e];
-        xs[e] = xsrc[e];
-    }
-    __syncthreads();
+    extern __shared__ __align__(16) double sm_lr[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int j0 = (tile * 8 + warp) * JT;
-    if (j0 >= nh) return;
-    const int L = (nh + 31) / 32;
-    const int jb = lane * L;
-    const int je = min(nh, jb + L);
-    double acc[JT];
+    const int TL = 32 * JT + JQ + 1;  // mirrored row window incl. one front pad
+    double* tx = sm_lr + (size_t)warp * (TL + JQ);
+    double* xs = tx + TL;
+    const int side = blockIdx.z, blk = blockIdx.y;
+    const int ii = blk * 2 + (warp >> 2);
+    const int jb0 = (warp & 3) * JQ;
+    const int jt0 = (jt_lo + blockIdx.x) * 32 * JT;
+    const bool live = ii < nw;
+    const double* t = Tedge + (long long)side * S + (long long)(live ? ii : 0) * nh;
+    const double* x = I + (long long)(live ? ii : 0) * nh;
+    for (int k = lane; k < TL; k += 32) {
+        double v = 0.0;
+        if (live && k >= 1) {
+            int d = jt0 - jb0 + (k - 1) - (JQ - 1);
+            d = d < 0 ? -d : d;
+            if (d < nh) v = t[d];
+        }
+        tx[k] = v;
+    }
+    for (int k = lane; k < JQ; k += 32) xs[k] = (live && jb0 + k < nh) ? x[jb0 + k] : 0.0;
+    __syncwarp();
+    const double* tl = tx + 1 + JT * lane + (JQ - 1);
+    double w[JT], acc[JT];
 #pragma unroll
-    for (int a = 0; a < JT; ++a) acc[a] = 0.0;
-    if (jb < je) {
-        for (int r = 0; r < nrow; ++r) {
-            const double* t = ts + (size_t)r * nh;
-            const double* x = xs + (size_t)r * nh;
-            double w[JT];
-            // slot (a - u) mod JT holds t[|j0 + a - jj|] at step u (jj = jb + u)
+    for (int a = 0; a < JT; ++a) { w[a] = tl[a]; acc[a] = 0.0; }
+    for (int ub = 0; ub < JQ; ub += JT) {
 #pragma unroll
-            for (int a = 0; a < JT; ++a) {
-                int d = j0 + a - jb;
-                d = d < 0 ? -d : d;
-                w[a] = d < nh ? t[d] : 0.0;
-            }
-            for (int jj = jb; jj < je; jj += JT) {
+        for (int u = 0; u < JT; ++u) {
+            const int uu = ub + u;
+            const double xv = xs[uu];
 #pragma unroll
-                for (int u = 0; u < JT; ++u) {
-                    if (jj + u < je) {
-                        const double xv = x[jj + u];
-#pragma unroll
-                        for (int a = 0; a < JT; ++a) acc[a] = fma(w[(a - u + JT) % JT], xv, acc[a]);
-                        // next step needs t[|j0 - (jj+u+1)|] in slot (-(u+1)) mod JT
-                        int d = j0 - (jj + u + 1);
-                        d = d < 0 ? -d : d;
-                        w[(2 * JT - 1 - u) % JT] = d < nh ? t[d] : 0.0;
-                    }
-                }
-            }
+            for (int a = 0; a < JT; ++a) acc[a] = fma(w[(a - u + JT) % JT], xv, acc[a]);
+            w[(2 * JT - 1 - u) % JT] = tl[-uu - 1];  // target a = 0 at step uu + 1
         }
     }
+    __syncthreads();
+    double* red = sm_lr;  // [8][32 JT]
 #pragma unroll
-    for (int a = 0; a < JT; ++a) {
-        double v = warp_sum(acc[a]);
-        const int j = j0 + a;
-        if (lane == 0 && j < nh) part[((long long)blk * 2 + side) * nh + j] = v;
+    for (int a = 0; a < JT; ++a) red[warp * 32 * JT + JT * lane + a] = acc[a];
+    __syncthreads();
+    for (int q = threadIdx.x; q < 32 * JT; q += blockDim.x) {
+        const int j = jt0 + q;
+        if (j < nh) {
+            double v = 0.0;
+#pragma unroll
+            for (int w8 = 0; w8 < 8; ++w8) v += red[w8 * 32 * JT + q];
+            part[((long long)side * nh + j) * gridDim.y + blk] = v;
+        }
     }
 }
 
-// psi_b in edge order from the partials (fixed block order).
+// psi_b in edge order from the partials: one warp per edge target, chunk-fastest partials,
+// fixed lane assignment + butterfly => deterministic and independent of the rank count.
 __global__ void k_bnd_reduce(const double* __restrict__ tb_part, int tb_nchunk, const double* __restrict__ lr_part,
                              int lr_nblk, int nw, int nh, int i_lo, int i_hi, int jlo, int jhi,
                              double* __restrict__ psib) {
     const int n_edge = 2 * nh + 2 * (nw - 2);
-    int p = blockIdx.x * blockDim.x + threadIdx.x;
+    const int p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
     if (p >= n_edge) return;
-    double s = 0.0;
+    const double* src;
+    int cnt;
     if (p < 2 * nh) {
         const int side = p < nh ? 0 : 1;
         const int j = p - side * nh;
         if (j < jlo || j >= jhi) return;
-        for (int b = 0; b < lr_nblk; ++b) s += lr_part[((long long)b * 2 + side) * nh + j];
+        src = lr_part + ((long long)side * nh + j) * lr_nblk;
+        cnt = lr_nblk;
     } else {
         const int q = p - 2 * nh;
         const int side = q < nw - 2 ? 0 : 1;
         const int i = q - side * (nw - 2) + 1;
         if (i < i_lo || i >= i_hi) return;
-        for (int c = 0; c < tb_nchunk; ++c) s += tb_part[((long long)c * nw + i) * 2 + side];
+        src = tb_part + ((long long)i * 2 + side) * tb_nchunk;
+        cnt = tb_nchunk;
     }
-    psib[p] = s;
+    double s = 0.0;
+    for (int c = lane; c < cnt; c += 32) s += src[c];
+    s = warp_sum(s);
+    if (lane == 0) psib[p] = s;
 }
 
 // On-the-fly variant of k_bnd_tb: G recomputed from (R_i, R_ii, m dZ) with the same device
-// function as the table build and the same summation order => bitwise equal to table mode.
+// function as the table build, same decomposition and summation order => bitwise equal to the
+// table mode.  FP64-bound (AGM: 10 square roots per entry).
 template <int GI>
 __global__ void __launch_bounds__(256) k_bnd_tb_otf(int row_lo, int nslab, int nw, int nh, double rmin, double dr,
-                                                    double dz, const double2* __restrict__ ipair, int ch,
+                                                    double dz, const double* __restrict__ Ib,
+                                                    const double* __restrict__ Fb, int ch,
                                                     double* __restrict__ part) {
-    extern __shared__ __align__(16) double2 ips[];
+    extern __shared__ __align__(16) double sm_tb[];
+    double* sI = sm_tb;
+    double* sF = sm_tb + ch;
     __shared__ double red[8][2 * GI];
     const int n = nw * nh;
     const int c = blockIdx.x, grp = blockIdx.y;
     const long long e0 = (long long)c * ch;
     const int len = (int)min((long long)ch, (long long)n - e0);
-    for (int q = threadIdx.x; q < ch; q += blockDim.x) ips[q] = ipair[e0 + q];
+    for (int q = threadIdx.x; q < ch; q += blockDim.x) { sI[q] = Ib[e0 + q]; sF[q] = Fb[e0 + q]; }
     __syncthreads();
     double a0[GI], a1[GI];
 #pragma unroll
     for (int t = 0; t < GI; ++t) { a0[t] = 0.0; a1[t] = 0.0; }
     const int s0 = grp * GI;
-#pragma unroll
+    const int qs[2] = {4 * (int)threadIdx.x, 4 * (int)threadIdx.x + 4 * (int)blockDim.x};
     for (int t = 0; t < GI; ++t) {
         const int sl = s0 + t;
-        if (sl < nslab) {
-            const int i = row_lo + sl;
-            const double Ri = grid_coord(rmin, i, dr);
-            for (int q = 2 * threadIdx.x; q < len; q += 2 * blockDim.x) {
-                double tv[2];
+        if (sl >= nslab) break;
+        const int i = row_lo + sl;
+        const double Ri = grid_coord(rmin, i, dr);
 #pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                    long long e = e0 + q + h;
-                    if (e < n) {
-                        int ii = (int)(e / nh), m = (int)(e - (long long)ii * nh);
-                        double Rs = grid_coord(rmin, ii, dr);
-                        tv[h] = (i == ii && m == 0) ? green_self(Ri, dr, dz)
-                                                    : green_psi(Ri, __dmul_rn((double)m, dz), Rs, 0.0);
-                    } else {
-                        tv[h] = 0.0;
-                    }
+        for (int p = 0; p < 2; ++p) {
+            const int q = qs[p];
+            if (q >= len) continue;
+            double tv[4];
+#pragma unroll
+            for (int h = 0; h < 4; ++h) {
+                const long long e = e0 + q + h;
+                if (e < n) {
+                    const int ii = (int)(e / nh), m = (int)(e - (long long)ii * nh);
+                    const double Rs = grid_coord(rmin, ii, dr);
+                    tv[h] = (i == ii && m == 0) ? green_self(Ri, dr, dz)
+                                                : green_psi(Ri, __dmul_rn((double)m, dz), Rs, 0.0);
+                } else {
+                    tv[h] = 0.0;
                 }
-                double2 p0 = ips[q], p1 = ips[q + 1];
-                a0[t] = fma(tv[0], p0.x, a0[t]);
-                a1[t] = fma(tv[0], p0.y, a1[t]);
-                a0[t] = fma(tv[1], p1.x, a0[t]);
-                a1[t] = fma(tv[1], p1.y, a1[t]);
             }
+            const d4 tt{tv[0], tv[1], tv[2], tv[3]};
+            a0[t] = dot4(tt, lds256(sI + q), a0[t]);
+            a1[t] = dot4(tt, lds256(sF + q), a1[t]);
         }
     }
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -862,42 +983,70 @@ __global__ void __launch_bounds__(256) k_bnd_tb_otf(int row_lo, int nslab, int n
         const int t = threadIdx.x >> 1, side = threadIdx.x & 1;
         const int sl = s0 + t;
         if (sl < nslab) {
-            double s = 0.0;
-            for (int w = 0; w < (int)(blockDim.x >> 5); ++w) s += red[w][threadIdx.x];
-            part[((long long)c * nw + row_lo + sl) * 2 + side] = s;
+            double sum = 0.0;
+            for (int w = 0; w < (int)(blockDim.x >> 5); ++w) sum += red[w][threadIdx.x];
+            part[((long long)(row_lo + sl) * 2 + side) * gridDim.x + c] = sum;
         }
     }
 }
 
 constexpr int kTbGI = 8;
-constexpr int kLrJT = 16;
+constexpr int kTbUnroll = 4;
+
+static size_t lr_smem(const Ctx& c) {
+    const int JT = c.t.lr_jt, JQ = c.t.lr_jj;
+    return sizeof(double) * 8 * (size_t)(32 * JT + JQ + 1 + JQ);
+}
+
+static cudaError_t launch_lr(Ctx& c, cudaStream_t s, bool prepare) {
+    const int ntile = c.jt_hi - c.jt_lo;
+    const size_t smem = lr_smem(c);
+    const void* f = nullptr;
+    switch (c.t.lr_jt) {
+        case 3: f = (const void*)k_bnd_lr<3>; break;
+        case 5: f = (const void*)k_bnd_lr<5>; break;
+        case 9: f = (const void*)k_bnd_lr<9>; break;
+        case 17: f = (const void*)k_bnd_lr<17>; break;
+        default: return cudaErrorInvalidValue;
+    }
+    if (prepare) return raise_smem_limit(f, smem);
+    if (ntile <= 0) return cudaSuccess;
+    dim3 grid(ntile, c.t.lr_nblk, 2);
+    switch (c.t.lr_jt) {
+#define EFIT_LR_CASE(V) \
+    case V: k_bnd_lr<V><<<grid, 256, smem, s>>>(c.Tedge, c.S, c.pcurr, c.nw, c.nh, c.t.lr_jj, c.jt_lo, c.lr_part); break;
+        EFIT_LR_CASE(3) EFIT_LR_CASE(5) EFIT_LR_CASE(9) EFIT_LR_CASE(17)
+#undef EFIT_LR_CASE
+    }
+    return cudaGetLastError();
+}
 
 cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s) {
+    cudaError_t e;
+    // fork: the FP64-bound left/right kernel runs on the side stream, concurrently with the
+    // HBM-bound top/bottom stream (both only read pcurr / ipair); join before the reduce.
+    if ((e = cudaEventRecord(c.ev_fork, s)) || (e = cudaStreamWaitEvent(c.side, c.ev_fork, 0))) return e;
+    if ((e = launch_lr(c, c.side, false))) return e;
+    mark(c, c.side, M_LR);
+    if ((e = cudaEventRecord(c.ev_join, c.side))) return e;
     const int nslab = c.i_hi - c.i_lo;
-    const size_t smem_tb = sizeof(double2) * c.t.tb_ch;
+    const size_t smem_tb = 2 * sizeof(double) * c.t.tb_ch;
     if (nslab > 0) {
         dim3 grid(c.t.tb_nchunk, c.t.tb_ngroup);
         if (c.mode == EFIT_GREEN_TABLE) {
-            k_bnd_tb<kTbGI><<<grid, 256, smem_tb, s>>>(c.T, c.S, nslab, c.i_lo, c.nw * c.nh, c.ipair, c.t.tb_ch,
-                                                       c.tb_part, c.nw);
+            k_bnd_tb<kTbGI, kTbUnroll><<<grid, 256, smem_tb, s>>>(c.T, c.S, nslab, c.i_lo, c.nw * c.nh, c.pcurr,
+                                                                  c.pflip, c.t.tb_ch, c.tb_part);
         } else {
-            k_bnd_tb_otf<kTbGI><<<grid, 256, smem_tb, s>>>(c.i_lo, nslab, c.nw, c.nh, c.rmin, c.dr, c.dz, c.ipair,
-                                                           c.t.tb_ch, c.tb_part);
+            k_bnd_tb_otf<kTbGI><<<grid, 256, smem_tb, s>>>(c.i_lo, nslab, c.nw, c.nh, c.rmin, c.dr, c.dz, c.pcurr,
+                                                           c.pflip, c.t.tb_ch, c.tb_part);
         }
-        cudaError_t e = cudaGetLastError();
-        if (e) return e;
+        if ((e = cudaGetLastError())) return e;
     }
-    const int ntile = c.jt_hi - c.jt_lo;
-    if (ntile > 0) {
-        const size_t smem_lr = sizeof(double) * 2 * (size_t)c.t.lr_iib * c.nh;
-        dim3 grid(ntile, c.t.lr_nblk, 2);
-        k_bnd_lr<kLrJT><<<grid, 256, smem_lr, s>>>(c.Tedge, c.S, pcurr, c.nw, c.nh, c.t.lr_iib, c.jt_lo, c.lr_part);
-        cudaError_t e = cudaGetLastError();
-        if (e) return e;
-    }
-    const int jlo = c.jt_lo * 8 * kLrJT, jhi = min(c.nh, c.jt_hi * 8 * kLrJT);
-    k_bnd_reduce<<<(c.n_edge + 255) / 256, 256, 0, s>>>(c.tb_part, c.t.tb_nchunk, c.lr_part, c.t.lr_nblk, c.nw,
-                                                        c.nh, c.i_lo, c.i_hi, jlo, jhi, psib);
+    mark(c, s, M_TB);
+    if ((e = cudaStreamWaitEvent(s, c.ev_join, 0))) return e;
+    const int jlo = c.jt_lo * 32 * c.t.lr_jt, jhi = min(c.nh, c.jt_hi * 32 * c.t.lr_jt);
+    k_bnd_reduce<<<(c.n_edge + 7) / 8, 256, 0, s>>>(c.tb_part, c.t.tb_nchunk, c.lr_part, c.t.lr_nblk, c.nw, c.nh,
+                                                    c.i_lo, c.i_hi, jlo, jhi, psib);
     return cudaGetLastError();
 }
 
@@ -905,7 +1054,7 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
 
 // In-place radix-2 complex FFT (forward, exp(-2 pi i jk/M)) of M = 2^log2m points in shared
 // memory; input must already be in bit-reversed order.  Twiddles W[k] = exp(-2 pi i k/M).
-__device__ void fft_smem(double2* a, int M, int log2m, const double2* __restrict__ W) {
+__device__ void fft_smem(double2* a, int M, int log2m, const double2* W) {
     for (int st = 1; st <= log2m; ++st) {
         const int half = 1 << (st - 1);
         const int tstride = M >> st;
@@ -914,7 +1063,7 @@ __device__ void fft_smem(double2* a, int M, int log2m, const double2* __restrict
             const int pos = b & (half - 1);
             const int i0 = (grp << st) + pos;
             const int i1 = i0 + half;
-            const double2 w = __ldg(W + pos * tstride);
+            const double2 w = W[pos * tstride];
             const double2 u = a[i0], v = a[i1];
             const double2 t = make_double2(w.x * v.x - w.y * v.y, w.x * v.y + w.y * v.x);
             a[i0] = make_double2(u.x + t.x, u.y + t.y);
@@ -933,13 +1082,16 @@ __device__ __forceinline__ int bitrev(int x, int log2m) { return (int)(__brev((u
 __global__ void __launch_bounds__(256) k_dst_fwd(const double* __restrict__ pcurr, const double* __restrict__ psib,
                                                  const double* __restrict__ tri_a, int nw, int nh, double rmin,
                                                  double dr, double dz, const double2* __restrict__ W, int M,
-                                                 int log2m, double* __restrict__ fhat) {
-    extern __shared__ __align__(16) double2 a2[];  // [M]
+                                                 int log2m, double* __restrict__ fhat, int ld) {
+    extern __shared__ __align__(16) double2 a2[];  // [M] data, then [M/2] twiddles
+    double2* Ws = a2 + M;
     const int n = nh - 2, ni = nw - 2;
     const int r0 = 1 + 2 * blockIdx.x;  // first row of the pair
     const double idz2 = 1.0 / (dz * dz);
     const double cellinv = 1.0 / (dr * dz);
-    for (int j = threadIdx.x; j < M; j += blockDim.x) {
+    for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = __ldg(W + k);
+    for (int p = threadIdx.x; p < M; p += blockDim.x) {
+        const int j = bitrev(p, log2m);  // a2[p] = z[bitrev(p)]: contiguous shared stores
         double v[2] = {0.0, 0.0};
         int jj = 0;
         double sgn = 0.0;
@@ -959,33 +1111,81 @@ __global__ void __launch_bounds__(256) k_dst_fwd(const double* __restrict__ pcur
                 v[h] = sgn * f;
             }
         }
-        a2[bitrev(j, log2m)] = make_double2(v[0], v[1]);
+        a2[p] = make_double2(v[0], v[1]);
     }
     __syncthreads();
-    fft_smem(a2, M, log2m, W);
+    fft_smem(a2, M, log2m, Ws);
+    // mode-major, segment-interleaved output (see k_tridiag): row r at (r % L)*32 + r / L
+    const int L = ld >> 5;
+    const int ra = r0 - 1, rb = r0;
+    const long long pa = (long long)(ra % L) * 32 + ra / L, pb = (long long)(rb % L) * 32 + rb / L;
     for (int k = 1 + threadIdx.x; k <= n; k += blockDim.x) {
         const double2 z = a2[k];
-        fhat[(long long)(r0 - 1) * n + (k - 1)] = -0.5 * z.y;
-        if (r0 + 1 <= ni) fhat[(long long)r0 * n + (k - 1)] = 0.5 * z.x;
+        double* dst = fhat + (long long)(k - 1) * ld;
+        dst[pa] = -0.5 * z.y;
+        if (r0 + 1 <= ni) dst[pb] = 0.5 * z.x;
     }
 }
 
-// Radial tridiagonal solve per sine mode (Thomas with precomputed factors), in place.
-__global__ void k_tridiag(double* __restrict__ fhat, const double* __restrict__ tri_a,
-                          const double* __restrict__ cp, const double* __restrict__ inv, int ni, int nmode) {
-    const int k = blockIdx.x * blockDim.x + threadIdx.x;
-    if (k >= nmode) return;
-    double d = 0.0;
-    for (int i = 0; i < ni; ++i) {
-        const long long o = (long long)i * nmode + k;
-        d = (fhat[o] - (i > 0 ? tri_a[i] * d : 0.0)) * inv[o];
-        fhat[o] = d;
+// Radial tridiagonal solve per sine mode, one warp per mode, in place.  Row r of a mode lives at
+// (r % L)*32 + r / L (L = ld/32): lane l owns the contiguous rows [l L, (l+1) L) and element e of
+// every lane is one coalesced 256-byte line.  Both Thomas sweeps are first-order linear
+// recurrences,  forward d_r = inv_r f_r + alpha_r d_{r-1} (d_{-1} = 0),  backward
+// x_r = d_r - c'_r x_{r+1} (x_ni = 0): each lane composes the affine map of its segment, a 5-step
+// shuffle scan composes the maps of the preceding (following) lanes, and each lane replays its
+// segment from the exact incoming value.  Padding rows (r >= ni) have alpha = inv = c' = 0 and
+// only follow the real rows.  |alpha|, |c'| < 1 (diagonal dominance) keeps the reassociation as
+// accurate as the sequential sweep.
+__global__ void __launch_bounds__(128) k_tridiag(double* __restrict__ fhat, const double* __restrict__ alpha,
+                                                 const double* __restrict__ inv, const double* __restrict__ cp,
+                                                 int ld, int nmode) {
+    const int mode = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (mode >= nmode) return;
+    const int L = ld >> 5;
+    double* f = fhat + (long long)mode * ld + lane;
+    const double* al = alpha + (long long)mode * ld + lane;
+    const double* iv = inv + (long long)mode * ld + lane;
+    const double* c = cp + (long long)mode * ld + lane;
+    double A = 1.0, B = 0.0;
+#pragma unroll 4
+    for (int e = 0; e < L; ++e) {
+        const double a = al[32 * e];
+        B = fma(a, B, iv[32 * e] * f[32 * e]);
+        A *= a;
     }
-    double x = 0.0;
-    for (int i = ni - 1; i >= 0; --i) {
-        const long long o = (long long)i * nmode + k;
-        x = fhat[o] - (i < ni - 1 ? cp[o] * x : 0.0);
-        fhat[o] = x;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        const double Ap = __shfl_up_sync(0xffffffffu, A, off);
+        const double Bp = __shfl_up_sync(0xffffffffu, B, off);
+        if (lane >= off) { B = fma(A, Bp, B); A *= Ap; }
+    }
+    double d = __shfl_up_sync(0xffffffffu, B, 1);
+    if (lane == 0) d = 0.0;
+#pragma unroll 4
+    for (int e = 0; e < L; ++e) {
+        d = fma(al[32 * e], d, iv[32 * e] * f[32 * e]);
+        f[32 * e] = d;
+    }
+    double C = 1.0, D = 0.0;
+#pragma unroll 4
+    for (int e = L - 1; e >= 0; --e) {
+        const double q = -c[32 * e];
+        D = fma(q, D, f[32 * e]);
+        C *= q;
+    }
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        const double Cn = __shfl_down_sync(0xffffffffu, C, off);
+        const double Dn = __shfl_down_sync(0xffffffffu, D, off);
+        if (lane + off < 32) { D = fma(C, Dn, D); C *= Cn; }
+    }
+    double x = __shfl_down_sync(0xffffffffu, D, 1);
+    if (lane == 31) x = 0.0;
+#pragma unroll 4
+    for (int e = L - 1; e >= 0; --e) {
+        x = fma(-c[32 * e], x, f[32 * e]);
+        f[32 * e] = x;
     }
 }
 
@@ -993,13 +1193,15 @@ __global__ void k_tridiag(double* __restrict__ fhat, const double* __restrict__ 
 //   psi_out = psi_p                                  (efit_interior_solve), or
 //   psi_inout <- psi_p + psi_ext, eps partial max     (efit_fit_step),
 // edges (j = 0, nh-1, and rows 0, nw-1 in the extra last block) take psi_b.
-__global__ void __launch_bounds__(256) k_dst_inv(const double* __restrict__ fhat, const double* __restrict__ psib,
+__global__ void __launch_bounds__(256) k_dst_inv(const double* __restrict__ fhat, int ld,
+                                                 const double* __restrict__ psib,
                                                  int nw, int nh, const double2* __restrict__ W, int M, int log2m,
                                                  double* __restrict__ psi_out, double* __restrict__ psi_inout,
                                                  const double* __restrict__ psi_ext, double* __restrict__ eps_part,
                                                  unsigned* ticket, const double* __restrict__ axbd,
                                                  double* __restrict__ eps) {
-    extern __shared__ __align__(16) double2 a2[];
+    extern __shared__ __align__(16) double2 a2[];  // [M] data, then [M/2] twiddles
+    double2* Ws = a2 + M;
     __shared__ double wmax[8];
     __shared__ bool last;
     const int n = nh - 2, ni = nw - 2;
@@ -1015,20 +1217,25 @@ __global__ void __launch_bounds__(256) k_dst_inv(const double* __restrict__ fhat
     };
     if ((int)blockIdx.x < npairs) {
         const int r0 = 1 + 2 * blockIdx.x;
-        for (int j = threadIdx.x; j < M; j += blockDim.x) {
+        for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = __ldg(W + k);
+        for (int p = threadIdx.x; p < M; p += blockDim.x) {
+            const int j = bitrev(p, log2m);
             double v[2] = {0.0, 0.0};
-            if (j >= 1 && j <= n) {
-                v[0] = fhat[(long long)(r0 - 1) * n + (j - 1)];
-                if (r0 + 1 <= ni) v[1] = fhat[(long long)r0 * n + (j - 1)];
-            } else if (j >= n + 2) {
-                const int jj = M - j;
-                v[0] = -fhat[(long long)(r0 - 1) * n + (jj - 1)];
-                if (r0 + 1 <= ni) v[1] = -fhat[(long long)r0 * n + (jj - 1)];
+            int jj = 0;
+            double sg = 0.0;
+            if (j >= 1 && j <= n) { jj = j; sg = 1.0; }
+            else if (j >= n + 2) { jj = M - j; sg = -1.0; }
+            if (sg != 0.0) {
+                const int L = ld >> 5;
+                const int ra = r0 - 1, rb = r0;
+                const double* src = fhat + (long long)(jj - 1) * ld;
+                v[0] = sg * src[(ra % L) * 32 + ra / L];
+                if (r0 + 1 <= ni) v[1] = sg * src[(rb % L) * 32 + rb / L];
             }
-            a2[bitrev(j, log2m)] = make_double2(v[0], v[1]);
+            a2[p] = make_double2(v[0], v[1]);
         }
         __syncthreads();
-        fft_smem(a2, M, log2m, W);
+        fft_smem(a2, M, log2m, Ws);
         const double sc = 2.0 / (double)(n + 1);
         for (int h = 0; h < 2; ++h) {
             const int i = r0 + h;
@@ -1082,31 +1289,35 @@ __global__ void __launch_bounds__(256) k_dst_inv(const double* __restrict__ fhat
 cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out, double* psi_inout,
                          const double* psi_ext, double* eps, cudaStream_t s) {
     const int npairs = (c.ni + 1) / 2;
-    const size_t smem = sizeof(double2) * c.fft_m;
+    const size_t smem = sizeof(double2) * (c.fft_m + c.fft_m / 2);
     k_dst_fwd<<<npairs, 256, smem, s>>>(pcurr, psib, c.tri_a, c.nw, c.nh, c.rmin, c.dr, c.dz, c.twiddle, c.fft_m,
-                                        c.fft_log2, c.fhat);
+                                        c.fft_log2, c.fhat, c.ni_pad);
     cudaError_t e = cudaGetLastError();
     if (e) return e;
-    k_tridiag<<<(c.nmode + 63) / 64, 64, 0, s>>>(c.fhat, c.tri_a, c.tri_cp, c.tri_inv, c.ni, c.nmode);
+    k_tridiag<<<(c.nmode + 3) / 4, 128, 0, s>>>(c.fhat, c.tri_alpha, c.tri_inv, c.tri_cp, c.ni_pad, c.nmode);
     e = cudaGetLastError();
     if (e) return e;
-    k_dst_inv<<<npairs + 1, 256, smem, s>>>(c.fhat, psib, c.nw, c.nh, c.twiddle, c.fft_m, c.fft_log2, psi_out,
+    k_dst_inv<<<npairs + 1, 256, smem, s>>>(c.fhat, c.ni_pad, psib, c.nw, c.nh, c.twiddle, c.fft_m, c.fft_log2, psi_out,
                                             psi_inout, psi_ext, c.eps_part, c.tickets + 1, c.axbd, eps);
     return cudaGetLastError();
 }
 
-// (I[g], I[ii][nh-1-m]) pairs for a caller-supplied current (efit_boundary_flux).
-__global__ void k_make_pair(const double* __restrict__ I, double2* __restrict__ ip, int nw, int nh) {
+// Caller-supplied current (efit_boundary_flux): copy into the internal zero-padded buffer and
+// build the vertically mirrored copy used by the top targets.
+__global__ void k_make_pair(const double* __restrict__ I, double* __restrict__ pc, double* __restrict__ pf,
+                            int nw, int nh) {
     const int n = nw * nh;
     for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += gridDim.x * blockDim.x) {
         const int ii = g / nh, m = g - (g / nh) * nh;
-        ip[g] = make_double2(I[g], I[ii * nh + (nh - 1 - m)]);
+        const double v = I[g];
+        pc[g] = v;
+        pf[ii * nh + (nh - 1 - m)] = v;
     }
 }
 
 cudaError_t launch_make_pair(Ctx& c, const double* pcurr, cudaStream_t s) {
     const int n = c.nw * c.nh;
-    k_make_pair<<<(n + 255) / 256, 256, 0, s>>>(pcurr, c.ipair, c.nw, c.nh);
+    k_make_pair<<<(n + 255) / 256, 256, 0, s>>>(pcurr, c.pcurr, c.pflip, c.nw, c.nh);
     return cudaGetLastError();
 }
 
@@ -1123,11 +1334,11 @@ cudaError_t prepare_kernels(Ctx& c) {
         return raise_smem_limit(f, need);
     };
     if ((e = big((const void*)k_lsq, lsq_smem(c)))) return e;
-    if ((e = big((const void*)k_bnd_lr<kLrJT>, sizeof(double) * 2 * (size_t)c.t.lr_iib * c.nh))) return e;
-    if ((e = big((const void*)k_bnd_tb<kTbGI>, sizeof(double2) * c.t.tb_ch))) return e;
-    if ((e = big((const void*)k_bnd_tb_otf<kTbGI>, sizeof(double2) * c.t.tb_ch))) return e;
-    if ((e = big((const void*)k_dst_fwd, sizeof(double2) * c.fft_m))) return e;
-    if ((e = big((const void*)k_dst_inv, sizeof(double2) * c.fft_m))) return e;
+    if ((e = launch_lr(c, nullptr, true))) return e;
+    if ((e = big((const void*)k_bnd_tb<kTbGI, kTbUnroll>, 2 * sizeof(double) * c.t.tb_ch))) return e;
+    if ((e = big((const void*)k_bnd_tb_otf<kTbGI>, 2 * sizeof(double) * c.t.tb_ch))) return e;
+    if ((e = big((const void*)k_dst_fwd, sizeof(double2) * (c.fft_m + c.fft_m / 2)))) return e;
+    if ((e = big((const void*)k_dst_inv, sizeof(double2) * (c.fft_m + c.fft_m / 2)))) return e;
     return cudaSuccess;
 }
 
