@@ -92,7 +92,8 @@ typedef struct {
     int32_t rank, world;
     int32_t resp_row_lo, resp_row_hi;   /* this rank's response rows [lo, hi)          */
     int32_t bnd_row_lo, bnd_row_hi;     /* this rank's top/bottom target rows i [lo, hi) */
-    int32_t lr_blk_lo, lr_blk_hi;       /* this rank's left/right source blocks          */
+    int32_t lr_blk_lo, lr_blk_hi;       /* this rank's left/right target tiles           */
+    int32_t lr_j_lo, lr_j_hi;           /* this rank's left/right targets j [lo, hi)     */
     int64_t slab_stride;                /* doubles between Green's-table slabs           */
     size_t workspace_bytes;
 } efit_info_t;
@@ -125,6 +126,11 @@ int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit_basis* bas
                     void* d_workspace, size_t ws_bytes, efit_stream_t stream);
 
 int efit_info(const efit_ctx* ctx, efit_info_t* info);
+
+/* Host-only: the same sizes and this rank's shard ranges for a configuration, without a device
+ * or a context (validates like efit_workspace_bytes). */
+int efit_plan_info(const efit_grid* grid, const efit_basis* basis, const efit_geometry* geom,
+                   const efit_dist* dist, int mode, efit_info_t* info);
 
 /* steps_ + green_: psi_axis/psi_bdry from d_psi[nw*nh], then
  * d_resp[m*nbasis + k] = sum_g Gd[m][g] dR dZ mask_g w_k(R_g) phi_k(psihat_g)
@@ -173,14 +179,16 @@ int efit_fit_step(efit_ctx* ctx, double* d_psi, const double* d_psi_ext, const d
 int efit_solve_update(efit_ctx* ctx, const double* d_pcurr, const double* d_psib, const double* d_psi_ext,
                       double* d_psi, double* d_eps, efit_stream_t stream);
 
-/* Per-step kernel timing (the measurement hook used by bench.py).  After efit_profile_begin(ctx, n),
- * the next n efit_fit_step calls record CUDA events at nine marks in stream order (they run
- * eagerly, or as nodes of the caller's graph when the caller is capturing the stream);
+/* Per-step kernel timing (the measurement hook used by bench.py).  After
+ * efit_profile_begin(ctx, n, every), every `every`-th efit_fit_step call (the 1st, (every+1)-th, ...)
+ * records CUDA events at seven marks, on the streams the kernels run on, until n steps are recorded.  The calls enqueue eagerly, or -- when the caller is capturing the stream into its own CUDA
+ * graph, as bench.py does for its timed region -- as external event-record nodes of that graph;
  * efit_profile_end synchronises and returns, summed over the recorded steps, milliseconds for
- *   ms[0] whole step, ms[1] normalise, ms[2] response (k_response + reduce), ms[3] lsq,
- *   ms[4] current, ms[5] k_bnd_tb, ms[6] k_bnd_lr, ms[7] boundary reduce, ms[8] interior solve + update.
- * nout >= 9.  *nsteps_out = number of steps recorded. */
-int efit_profile_begin(efit_ctx* ctx, int32_t nsteps);
+ *   ms[0] whole step, ms[1] normalise, ms[2] response (k_basis + k_response + reduce),
+ *   ms[3] lsq + current, ms[4] k_bnd_tb (from the fork), ms[5] k_bnd_lr (from the fork, concurrent),
+ *   ms[6] boundary reduce + interior solve + update (from the end of k_bnd_tb).
+ * nout >= 7.  *nsteps_out = number of steps recorded. */
+int efit_profile_begin(efit_ctx* ctx, int32_t nsteps, int32_t every);
 int efit_profile_end(efit_ctx* ctx, double* ms_out, int32_t nout, int32_t* nsteps_out);
 
 /* Synchronise `stream` and return the first data-dependent failure recorded since the last

@@ -21,7 +21,7 @@ __all__ = [
     "efit_current", "efit_boundary_flux", "efit_interior_solve", "efit_lsq", "efit_fit_step", "efit_status",
     "efit_solve_update", "efit_profile_begin", "efit_profile_end",
     "efit_table", "efit_shard", "efit_destroy", "efit_strerror", "efit_last_error", "efit_version",
-    "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY",
+    "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY", "efit_plan_info", "owned_targets", "exchange",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -64,6 +64,7 @@ class efit_info_t(ctypes.Structure):
                 ("resp_row_lo", ctypes.c_int32), ("resp_row_hi", ctypes.c_int32),
                 ("bnd_row_lo", ctypes.c_int32), ("bnd_row_hi", ctypes.c_int32),
                 ("lr_blk_lo", ctypes.c_int32), ("lr_blk_hi", ctypes.c_int32),
+                ("lr_j_lo", ctypes.c_int32), ("lr_j_hi", ctypes.c_int32),
                 ("slab_stride", ctypes.c_int64), ("workspace_bytes", ctypes.c_size_t)]
 
 
@@ -90,6 +91,7 @@ def lib() -> ctypes.CDLL:
             "efit_green_init": (I, [P(vp), P(efit_grid), P(efit_basis), P(efit_geometry), P(efit_dist), I, vp,
                                     ctypes.c_size_t, vp]),
             "efit_info": (I, [vp, P(efit_info_t)]),
+            "efit_plan_info": (I, [P(efit_grid), P(efit_basis), P(efit_geometry), P(efit_dist), I, P(efit_info_t)]),
             "efit_response": (I, [vp, vp, vp, vp, vp]),
             "efit_current": (I, [vp, vp, vp, vp, vp]),
             "efit_boundary_flux": (I, [vp, vp, vp, vp]),
@@ -98,7 +100,7 @@ def lib() -> ctypes.CDLL:
             "efit_fit_step": (I, [vp, vp, vp, vp, vp, vp, vp, vp, vp]),
             "efit_status": (I, [vp, vp]),
             "efit_solve_update": (I, [vp, vp, vp, vp, vp, vp, vp]),
-            "efit_profile_begin": (I, [vp, ctypes.c_int32]),
+            "efit_profile_begin": (I, [vp, ctypes.c_int32, ctypes.c_int32]),
             "efit_profile_end": (I, [vp, P(ctypes.c_double), ctypes.c_int32, P(ctypes.c_int32)]),
             "efit_table": (I, [vp, I, P(vp)]),
             "efit_shard": (None, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int32),
@@ -190,6 +192,31 @@ def efit_info(ctx) -> efit_info_t:
     return info
 
 
+def efit_plan_info(grid, basis, geom, dist, mode: int = EFIT_GREEN_TABLE) -> efit_info_t:
+    info = efit_info_t()
+    _check(lib().efit_plan_info(ctypes.byref(grid), ctypes.byref(basis), ctypes.byref(geom), ctypes.byref(dist),
+                                mode, ctypes.byref(info)))
+    return info
+
+
+def owned_targets(info):
+    """Host logic of the sharded step: the response rows and the edge positions (ABI edge order)
+    this rank writes.  Every other entry of the rank's output buffers stays exactly 0, so a sum
+    all-reduce over ranks reproduces the single-GPU arrays bit for bit."""
+    rows = list(range(info.resp_row_lo, info.resp_row_hi))
+    nw, nh = info.nw, info.nh
+    edge = list(range(info.lr_j_lo, info.lr_j_hi)) + [nh + j for j in range(info.lr_j_lo, info.lr_j_hi)]
+    for i in range(info.bnd_row_lo, info.bnd_row_hi):
+        edge += [2 * nh + (i - 1), 2 * nh + (nw - 2) + (i - 1)]
+    return rows, sorted(edge)
+
+
+def exchange(buf, group=None) -> None:
+    """Make a zero-padded rank slice replicated: one sum all-reduce (NCCL on GPUs, gloo in tests)."""
+    import torch.distributed as dist
+    dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=group)
+
+
 def efit_response(ctx, psi, resp, axbd=None, stream=None) -> None:
     _check(lib().efit_response(ctx, _ptr(psi), _ptr(resp), _ptr(axbd), _stream(stream)), ctx)
 
@@ -220,11 +247,11 @@ def efit_solve_update(ctx, pcurr, psib, psi_ext, psi, eps, stream=None) -> None:
                                    _stream(stream)), ctx)
 
 
-PROFILE_FIELDS = ("step", "normalize", "response", "lsq", "current", "bnd_tb", "bnd_lr", "bnd_reduce", "solve")
+PROFILE_FIELDS = ("step", "normalize", "response", "lsq_current", "bnd_tb", "bnd_lr", "tail")
 
 
-def efit_profile_begin(ctx, nsteps: int) -> None:
-    _check(lib().efit_profile_begin(ctx, nsteps), ctx)
+def efit_profile_begin(ctx, nsteps: int, every: int = 1) -> None:
+    _check(lib().efit_profile_begin(ctx, nsteps, every), ctx)
 
 
 def efit_profile_end(ctx):

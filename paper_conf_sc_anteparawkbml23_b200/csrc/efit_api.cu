@@ -292,24 +292,59 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
     }
     c.gexec = nullptr;
     c.prof_on = false;
+    c.prof_rec = false;
+    c.prof_every = 1;
+    c.prof_calls = 0;
+    c.prof_capture = false;
     c.prof_ev = nullptr;
     c.prof_slots = c.prof_next = 0;
+    c.pgraph = nullptr;
+    c.pexec = nullptr;
+    for (int id = 0; id < 16; ++id) c.prof_place[id] = nullptr;
+    for (int id = 0; id < efit::kNumMarks; ++id) {
+        if ((e = cudaEventCreate(&c.prof_place[id]))) {
+            for (int q = 0; q < id; ++q) cudaEventDestroy(c.prof_place[q]);
+            cudaStreamDestroy(c.side); cudaEventDestroy(c.ev_fork); cudaEventDestroy(c.ev_join);
+            delete h;
+            return cuda_fail(nullptr, e, "profile events");
+        }
+    }
     c.use_graph = getenv("EFIT_NO_GRAPH") == nullptr;
     c.err[0] = 0;
     *out = h;
     return EFIT_OK;
 }
 
-extern "C" int efit_info(const efit_ctx* h, efit_info_t* info) {
-    if (!h || !info) return fail(nullptr, EFIT_E_INVAL, "null argument");
-    const Ctx& c = h->c;
+static void fill_info(const Ctx& c, efit_info_t* info) {
     info->nw = c.nw; info->nh = c.nh; info->ndiag = c.ndiag; info->nbasis = c.nb; info->n_edge = c.n_edge;
     info->mode = c.mode; info->rank = c.rank; info->world = c.world;
     info->resp_row_lo = c.m_lo; info->resp_row_hi = c.m_hi;
     info->bnd_row_lo = c.i_lo; info->bnd_row_hi = c.i_hi;
     info->lr_blk_lo = c.jt_lo; info->lr_blk_hi = c.jt_hi;
+    const int tile = 32 * c.t.lr_jt;
+    info->lr_j_lo = c.jt_lo * tile < c.nh ? c.jt_lo * tile : c.nh;
+    info->lr_j_hi = c.jt_hi * tile < c.nh ? c.jt_hi * tile : c.nh;
     info->slab_stride = c.S;
     info->workspace_bytes = c.ws_bytes;
+}
+
+extern "C" int efit_plan_info(const efit_grid* grid, const efit_basis* basis, const efit_geometry* geom,
+                              const efit_dist* dist, int mode, efit_info_t* info) {
+    int st = validate(grid, basis, geom, dist, mode);
+    if (st) return st;
+    if (!info) return fail(nullptr, EFIT_E_INVAL, "info is null");
+    Ctx* c = new (std::nothrow) Ctx();
+    if (!c) return fail(nullptr, EFIT_E_NOMEM, "host allocation");
+    plan(*c, grid, basis, geom, dist, mode);
+    c->ws_bytes = carve(*c, nullptr);
+    fill_info(*c, info);
+    delete c;
+    return EFIT_OK;
+}
+
+extern "C" int efit_info(const efit_ctx* h, efit_info_t* info) {
+    if (!h || !info) return fail(nullptr, EFIT_E_INVAL, "null argument");
+    fill_info(h->c, info);
     return EFIT_OK;
 }
 
@@ -388,7 +423,11 @@ extern "C" int efit_lsq(efit_ctx* h, const double* d_resp, const double* d_meas,
 
 namespace efit {
 void mark(Ctx& c, cudaStream_t s, int id) {
-    if (!c.prof_on || c.prof_next >= c.prof_slots) return;
+    if (c.prof_capture) {  // building the profiled graph: external event-record node
+        cudaEventRecordWithFlags(c.prof_place[id], s, cudaEventRecordExternal);
+        return;
+    }
+    if (!c.prof_on || !c.prof_rec || c.prof_next >= c.prof_slots) return;
     cudaEvent_t ev = c.prof_ev[(size_t)c.prof_next * kNumMarks + id];
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     cudaStreamIsCapturing(s, &cs);
@@ -401,20 +440,20 @@ static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, 
                                     const double* sigma, double* coef, double* chi2, double* eps, cudaStream_t s) {
     using namespace efit;
     cudaError_t e;
+    c.prof_rec = c.prof_on && (c.prof_calls++ % c.prof_every == 0);
     mark(c, s, M_BEGIN);
     if ((e = launch_normalize(c, psi, s))) return e;
     mark(c, s, M_NORM);
     if ((e = launch_response(c, psi, c.resp, s))) return e;
     mark(c, s, M_RESP);
     if ((e = launch_lsq(c, c.resp, meas, sigma, coef, chi2, s))) return e;
-    mark(c, s, M_LSQ);
     if ((e = launch_current(c, psi, coef, c.pcurr, true, s))) return e;
     mark(c, s, M_CUR);
     if ((e = launch_boundary(c, c.pcurr, c.psib, s))) return e;  // marks M_TB, M_LR inside
-    mark(c, s, M_BRED);
     if ((e = launch_solve(c, c.pcurr, c.psib, nullptr, psi, psi_ext, eps, s))) return e;
     mark(c, s, M_SOLVE);
-    if (c.prof_on && c.prof_next < c.prof_slots) ++c.prof_next;
+    if (c.prof_on && c.prof_rec && !c.prof_capture && c.prof_next < c.prof_slots) ++c.prof_next;
+    c.prof_rec = false;
     return cudaSuccess;
 }
 
@@ -436,8 +475,8 @@ extern "C" int efit_fit_step(efit_ctx* h, double* d_psi, const double* d_psi_ext
     const void* key[8] = {d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, (const void*)s};
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     if (s != nullptr && (e = cudaStreamIsCapturing(s, &cs))) return cuda_fail(&c, e, "capture query");
-    // eager enqueue when profiling, when the caller is capturing the stream itself (the kernels
-    // then become nodes of the caller's graph), or on the legacy stream (not capturable)
+    // eager enqueue when the caller is capturing the stream itself (the kernels then become nodes
+    // of the caller's graph), when graphs are disabled, or on the legacy stream (not capturable)
     if (!c.use_graph || s == nullptr || c.prof_on || cs == cudaStreamCaptureStatusActive) {
         if ((e = enqueue_fit_step(c, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, s)))
             return cuda_fail(&c, e, "fit step");
@@ -474,8 +513,8 @@ extern "C" int efit_solve_update(efit_ctx* h, const double* d_pcurr, const doubl
     return EFIT_OK;
 }
 
-extern "C" int efit_profile_begin(efit_ctx* h, int32_t nsteps) {
-    if (!h || nsteps < 1) return fail(nullptr, EFIT_E_INVAL, "profile_begin: bad argument");
+extern "C" int efit_profile_begin(efit_ctx* h, int32_t nsteps, int32_t every) {
+    if (!h || nsteps < 1 || every < 1) return fail(nullptr, EFIT_E_INVAL, "profile_begin: bad argument");
     Ctx& c = h->c;
     if (c.prof_ev) return fail(&c, EFIT_E_STATE, "profiling already active");
     size_t n = (size_t)nsteps * efit::kNumMarks;
@@ -492,12 +531,14 @@ extern "C" int efit_profile_begin(efit_ctx* h, int32_t nsteps) {
     }
     c.prof_slots = nsteps;
     c.prof_next = 0;
+    c.prof_every = every;
+    c.prof_calls = 0;
     c.prof_on = true;
     return EFIT_OK;
 }
 
 extern "C" int efit_profile_end(efit_ctx* h, double* ms_out, int32_t nout, int32_t* nsteps_out) {
-    if (!h || !ms_out || nout < efit::kNumMarks) return fail(nullptr, EFIT_E_INVAL, "profile_end: bad argument");
+    if (!h || !ms_out || nout < efit::kNumProfileFields) return fail(nullptr, EFIT_E_INVAL, "profile_end: bad argument");
     Ctx& c = h->c;
     if (!c.prof_ev) return fail(&c, EFIT_E_STATE, "profiling not active");
     for (int k = 0; k < nout; ++k) ms_out[k] = 0.0;
@@ -508,11 +549,11 @@ extern "C" int efit_profile_end(efit_ctx* h, double* ms_out, int32_t nout, int32
         using namespace efit;
         // (from, to) mark pairs of the nine reported intervals; k_bnd_tb and k_bnd_lr both
         // start at the fork after the current kernel and run concurrently
-        static const int pairs[9][2] = {{M_BEGIN, M_SOLVE}, {M_BEGIN, M_NORM}, {M_NORM, M_RESP}, {M_RESP, M_LSQ},
-                                        {M_LSQ, M_CUR},     {M_CUR, M_TB},     {M_CUR, M_LR},   {M_TB, M_BRED},
-                                        {M_BRED, M_SOLVE}};
+        static const int pairs[kNumProfileFields][2] = {{M_BEGIN, M_SOLVE}, {M_BEGIN, M_NORM}, {M_NORM, M_RESP},
+                                                        {M_RESP, M_CUR},    {M_CUR, M_TB},     {M_CUR, M_LR},
+                                                        {M_TB, M_SOLVE}};
         float t;
-        for (int k = 0; k < 9; ++k)
+        for (int k = 0; k < kNumProfileFields; ++k)
             if (cudaEventElapsedTime(&t, ev[pairs[k][0]], ev[pairs[k][1]]) == cudaSuccess) ms_out[k] += t;
     }
     if (nsteps_out) *nsteps_out = c.prof_next;
@@ -556,6 +597,10 @@ extern "C" int efit_table(const efit_ctx* h, int which, const void** d_ptr) {
 extern "C" int efit_destroy(efit_ctx* h) {
     if (!h) return EFIT_OK;
     if (h->c.gexec) cudaGraphExecDestroy(h->c.gexec);
+    if (h->c.pexec) cudaGraphExecDestroy(h->c.pexec);
+    if (h->c.pgraph) cudaGraphDestroy(h->c.pgraph);
+    for (int id = 0; id < efit::kNumMarks; ++id)
+        if (h->c.prof_place[id]) cudaEventDestroy(h->c.prof_place[id]);
     if (h->c.side) cudaStreamDestroy(h->c.side);
     if (h->c.ev_fork) cudaEventDestroy(h->c.ev_fork);
     if (h->c.ev_join) cudaEventDestroy(h->c.ev_join);

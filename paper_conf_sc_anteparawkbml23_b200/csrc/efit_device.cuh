@@ -12,6 +12,11 @@ constexpr double kMu0 = 4.0e-7 * kPi;     // mu0 = 4 pi 1e-7 (reading 
 constexpr double kMu0Over2Pi = 2.0e-7;    // mu0 / (2 pi)
 constexpr int kAgmIters = 10;             // enough for m1 >= 1e-15 (quadratic convergence)
 
+// PDL: wait for the programmatic predecessor (no-op for a normal launch), then let dependents launch.
+__device__ __forceinline__ void griddep() {
+    asm volatile("griddepcontrol.wait;\n\tgriddepcontrol.launch_dependents;" ::: "memory");
+}
+
 // Grid coordinates without FMA contraction (R_i = rmin + i*dR rounded twice), so that
 // discrete decisions (limiter test, bilinear cell) are reproducible bit for bit.
 __device__ __forceinline__ double grid_coord(double lo, int i, double d) {

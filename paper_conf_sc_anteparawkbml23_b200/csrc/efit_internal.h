@@ -85,10 +85,19 @@ struct Ctx {
     double* eps_part;   // [red_blocks]
     double* scratch_meas;  // [ndiag] (unused placeholder)
 
-    // profiling: CUDA events recorded at marks inside the fit step (efit_profile_begin/end)
-    bool prof_on;
+    // profiling: CUDA events recorded at marks inside the fit step (efit_profile_begin/end).
+    // The profiled step is its own CUDA graph with external event-record nodes at the marks,
+    // retargeted to the step's events before every replay.
+    bool prof_on, prof_capture;
     int prof_slots, prof_next;
-    cudaEvent_t* prof_ev;  // [prof_slots][kNumMarks]
+    int prof_every, prof_calls;    // record marks on every prof_every-th fit step only
+    bool prof_rec;                 // this fit step records
+    cudaEvent_t* prof_ev;          // [prof_slots][kNumMarks]
+    cudaEvent_t prof_place[16];    // placeholder events used during capture
+    cudaGraph_t pgraph;
+    cudaGraphExec_t pexec;
+    cudaGraphNode_t pnode[16];
+    const void* pkey[8];
 
     // side stream + events: k_bnd_lr (FP64-bound) runs concurrently with k_bnd_tb (HBM-bound)
     cudaStream_t side;
@@ -104,7 +113,10 @@ struct Ctx {
 };
 
 // Marks recorded (as CUDA events) inside a profiled fit step, in stream order.
-enum Mark { M_BEGIN = 0, M_NORM, M_RESP, M_LSQ, M_CUR, M_TB, M_LR, M_BRED, M_SOLVE, kNumMarks };
+// Kept minimal: every mark between two kernels on the main stream costs one programmatic
+// (PDL) edge.  M_CUR sits where the k_bnd_lr fork already is; M_TB/M_LR precede the join.
+enum Mark { M_BEGIN = 0, M_NORM, M_RESP, M_CUR, M_TB, M_LR, M_SOLVE, kNumMarks };
+constexpr int kNumProfileFields = 7;  // step, normalize, response, lsq+current, bnd_tb, bnd_lr, tail
 void mark(Ctx& c, cudaStream_t s, int id);  // efit_api.cu; no-op unless profiling
 
 // ---- launchers (efit_kernels.cu) -------------------------------------------------

@@ -15,6 +15,7 @@
 #include <cfloat>
 #include <climits>
 #include <cstdio>
+#include <utility>
 
 #include "efit_device.cuh"
 #include "efit_internal.h"
@@ -22,6 +23,26 @@
 namespace efit {
 
 static int g_smem_optin = 227 * 1024;  // device opt-in shared memory per block (set in prepare_kernels)
+
+// Programmatic dependent launch: every per-iteration kernel is launched with programmatic stream
+// serialisation, so its CTAs are scheduled while the predecessor's last wave drains; the kernel
+// itself waits (griddepcontrol.wait) until the predecessor has completed and flushed before it
+// touches any of its outputs, then immediately allows its own dependents to launch.
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                              Args&&... args) {
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
 
 // Raise (never lower) a kernel's dynamic shared-memory limit to the device maximum minus its
 // static shared memory.  The limit is per function and process-wide.
@@ -278,6 +299,7 @@ __global__ void __launch_bounds__(256) k_normalize(const double* __restrict__ ps
                                                    int sgn, const double* __restrict__ lim, int n_lim,
                                                    double* __restrict__ part, unsigned* ticket,
                                                    double* __restrict__ axbd, int* status) {
+    griddep();
     __shared__ double sv[8];
     __shared__ long long si[8];
     __shared__ bool last;
@@ -349,7 +371,7 @@ __global__ void __launch_bounds__(256) k_normalize(const double* __restrict__ ps
 }
 
 cudaError_t launch_normalize(Ctx& c, const double* psi, cudaStream_t s) {
-    k_normalize<<<c.t.red_blocks, 256, 0, s>>>(psi, c.inlim, c.nw, c.nh, c.rmin, c.dr, c.zmin, c.dz,
+    launch_pdl(k_normalize, dim3(c.t.red_blocks), dim3(256), 0, s, psi, c.inlim, c.nw, c.nh, c.rmin, c.dr, c.zmin, c.dz,
                                                c.ip_sign, c.lim, c.n_lim, c.norm_part, c.tickets + 0,
                                                c.axbd, c.status);
     return cudaGetLastError();
@@ -380,6 +402,7 @@ __global__ void __launch_bounds__(1024) k_basis(const double* __restrict__ psi, 
                                                const double* __restrict__ axbd, int nw, int nh, double rmin,
                                                double dr, double cell, BasisParams bp, int gc, long long ldb,
                                                double* __restrict__ Bm, double* __restrict__ cnt_part) {
+    griddep();
     __shared__ int cnt_s[32];
     const int n = nw * nh;
     const int g0 = blockIdx.x * gc;
@@ -424,6 +447,7 @@ template <int NB, int MB>
 __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ Gd, long long S, int nrows, int n,
                                                      const double* __restrict__ Bm, long long ldb, int gc,
                                                      double* __restrict__ part) {
+    griddep();
     extern __shared__ __align__(16) double Bs[];  // [NB][gc] permuted
     const int c = blockIdx.x;
     const int g0 = c * gc;
@@ -485,6 +509,7 @@ __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ 
 // masked-node count decides EFIT_ST_NOPLASMA.
 __global__ void k_resp_reduce(const double* __restrict__ part, const double* __restrict__ cnt_part, int nchunk,
                               int total, double* __restrict__ out, int* status) {
+    griddep();
     const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
     if (w < total) {
         const double* p = part + (long long)w * nchunk;
@@ -508,7 +533,7 @@ static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t
     const long long ldb = (long long)c.t.resp_nchunk * gc;
     if (!prepare) {
         BasisParams bp = basis_params(c);
-        k_basis<NB><<<c.t.resp_nchunk, gc <= 1024 ? gc : 1024, 0, s>>>(psi, c.inlim, c.axbd, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp,
+        launch_pdl(k_basis<NB>, dim3(c.t.resp_nchunk), dim3(gc <= 1024 ? gc : 1024), 0, s, psi, c.inlim, c.axbd, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp,
                                                     gc, ldb, c.bmat, c.resp_cnt);
     }
     int mb = c.t.resp_mb;
@@ -517,7 +542,7 @@ static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t
         auto kern = k_response<NB, MBV>;                                                                   \
         if (prepare) { raise_smem_limit((const void*)kern, smem); break; }                               \
         dim3 grid(c.t.resp_nchunk, (nrows + 8 * MBV - 1) / (8 * MBV));                                    \
-        kern<<<grid, 256, smem, s>>>(c.Gd, c.S, nrows, c.nw * c.nh, c.bmat, ldb, gc, part);               \
+        launch_pdl(kern, dim3(grid), dim3(256), smem, s, c.Gd, c.S, nrows, c.nw * c.nh, c.bmat, ldb, gc, part);               \
     } while (0)
     if (mb >= 4) EFIT_RESP_LAUNCH(4);
     else if (mb == 3) EFIT_RESP_LAUNCH(3);
@@ -541,7 +566,7 @@ static cudaError_t response_impl(Ctx& c, const double* psi, double* resp_rows, c
     cudaError_t e = cudaGetLastError();
     if (e || prepare) return e;
     const int total = nrows * c.nb;
-    k_resp_reduce<<<(total + 7) / 8, 256, 0, s>>>(c.resp_part, c.resp_cnt, c.t.resp_nchunk, total, resp_rows,
+    launch_pdl(k_resp_reduce, dim3((total + 7) / 8), dim3(256), 0, s, c.resp_part, c.resp_cnt, c.t.resp_nchunk, total, resp_rows,
                                                   c.status);
     return cudaGetLastError();
 }
@@ -560,6 +585,7 @@ cudaError_t launch_response(Ctx& c, const double* psi, double* resp_rows, cudaSt
 __global__ void __launch_bounds__(128) k_lsq(const double* __restrict__ resp, const double* __restrict__ meas,
                                              const double* __restrict__ sigma, int nd, int nb,
                                              double* __restrict__ coef, double* __restrict__ chi2, int* status) {
+    griddep();
     extern __shared__ __align__(16) double sm[];
     double* A = sm;                   // [nb+1][nd] column-major (scaled); column nb = b
     double* isg = A + (size_t)(nb + 1) * nd;  // [nd] 1/sigma
@@ -657,7 +683,7 @@ static size_t lsq_smem(const Ctx& c) {
 cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const double* sigma, double* coef,
                        double* chi2, cudaStream_t s) {
     size_t smem = lsq_smem(c);
-    k_lsq<<<1, 128, smem, s>>>(resp, meas, sigma, c.ndiag, c.nb, coef, chi2, c.status);
+    launch_pdl(k_lsq, dim3(1), dim3(128), smem, s, resp, meas, sigma, c.ndiag, c.nb, coef, chi2, c.status);
     return cudaGetLastError();
 }
 
@@ -682,6 +708,7 @@ __global__ void k_current(const double* __restrict__ psi, const uint8_t* __restr
                           const double* __restrict__ axbd, const double* __restrict__ coef, int nw, int nh,
                           double rmin, double dr, double cell, BasisParams bp, double* __restrict__ pcurr,
                           double* __restrict__ pflip) {
+    griddep();
     const int n = nw * nh;
     const double pa = axbd[0], pb = axbd[1];
     double cf[NB];
@@ -702,6 +729,7 @@ __global__ void k_current(const double* __restrict__ psi, const uint8_t* __restr
 template <int NB>
 __global__ void k_current_from_basis(const double* __restrict__ Bm, long long ldb, const double* __restrict__ coef,
                                      int nw, int nh, double* __restrict__ pcurr, double* __restrict__ pflip) {
+    griddep();
     const int n = nw * nh;
     double cf[NB];
 #pragma unroll
@@ -724,7 +752,7 @@ cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double
         const long long ldb = (long long)c.t.resp_nchunk * c.t.resp_gc;
         switch (c.nb) {
 #define EFIT_NB_CASE(V) \
-    case V: k_current_from_basis<V><<<(n + 255) / 256, 256, 0, s>>>(c.bmat, ldb, coef, c.nw, c.nh, pcurr, c.pflip); break;
+    case V: launch_pdl(k_current_from_basis<V>, dim3((n + 255) / 256), dim3(256), 0, s, c.bmat, ldb, coef, c.nw, c.nh, pcurr, c.pflip); break;
             EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
             EFIT_NB_CASE(7) EFIT_NB_CASE(8) EFIT_NB_CASE(9) EFIT_NB_CASE(10) EFIT_NB_CASE(11) EFIT_NB_CASE(12)
             EFIT_NB_CASE(13) EFIT_NB_CASE(14) EFIT_NB_CASE(15) EFIT_NB_CASE(16) EFIT_NB_CASE(17) EFIT_NB_CASE(18)
@@ -739,7 +767,7 @@ cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double
     double* fl = pair ? c.pflip : nullptr;
     switch (c.nb) {
 #define EFIT_NB_CASE(V) \
-    case V: k_current<V><<<blocks, 256, 0, s>>>(psi, c.inlim, c.axbd, coef, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp, pcurr, fl); break;
+    case V: launch_pdl(k_current<V>, dim3(blocks), dim3(256), 0, s, psi, c.inlim, c.axbd, coef, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp, pcurr, fl); break;
         EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
         EFIT_NB_CASE(7) EFIT_NB_CASE(8) EFIT_NB_CASE(9) EFIT_NB_CASE(10) EFIT_NB_CASE(11) EFIT_NB_CASE(12)
         EFIT_NB_CASE(13) EFIT_NB_CASE(14) EFIT_NB_CASE(15) EFIT_NB_CASE(16) EFIT_NB_CASE(17) EFIT_NB_CASE(18)
@@ -764,6 +792,7 @@ __global__ void __launch_bounds__(256, 2) k_bnd_tb(const double* __restrict__ T,
                                                    int row_lo, int n, const double* __restrict__ Ib,
                                                    const double* __restrict__ Fb, int ch,
                                                    double* __restrict__ part) {
+    griddep();
     extern __shared__ __align__(16) double sm_tb[];
     double* sI = sm_tb;        // [ch]
     double* sF = sm_tb + ch;   // [ch]
@@ -838,6 +867,7 @@ template <int JT>
 __global__ void __launch_bounds__(256) k_bnd_lr(const double* __restrict__ Tedge, long long S,
                                                 const double* __restrict__ I, int nw, int nh, int JQ,
                                                 int jt_lo, double* __restrict__ part) {
+    griddep();
     extern __shared__ __align__(16) double sm_lr[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int TL = 32 * JT + JQ + 1;  // mirrored row window incl. one front pad
@@ -896,6 +926,7 @@ __global__ void __launch_bounds__(256) k_bnd_lr(const double* __restrict__ Tedge
 __global__ void k_bnd_reduce(const double* __restrict__ tb_part, int tb_nchunk, const double* __restrict__ lr_part,
                              int lr_nblk, int nw, int nh, int i_lo, int i_hi, int jlo, int jhi,
                              double* __restrict__ psib) {
+    griddep();
     const int n_edge = 2 * nh + 2 * (nw - 2);
     const int p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
     if (p >= n_edge) return;
@@ -929,6 +960,7 @@ __global__ void __launch_bounds__(256) k_bnd_tb_otf(int row_lo, int nslab, int n
                                                     double dz, const double* __restrict__ Ib,
                                                     const double* __restrict__ Fb, int ch,
                                                     double* __restrict__ part) {
+    griddep();
     extern __shared__ __align__(16) double sm_tb[];
     double* sI = sm_tb;
     double* sF = sm_tb + ch;
@@ -1014,7 +1046,7 @@ static cudaError_t launch_lr(Ctx& c, cudaStream_t s, bool prepare) {
     dim3 grid(ntile, c.t.lr_nblk, 2);
     switch (c.t.lr_jt) {
 #define EFIT_LR_CASE(V) \
-    case V: k_bnd_lr<V><<<grid, 256, smem, s>>>(c.Tedge, c.S, c.pcurr, c.nw, c.nh, c.t.lr_jj, c.jt_lo, c.lr_part); break;
+    case V: launch_pdl(k_bnd_lr<V>, dim3(grid), dim3(256), smem, s, c.Tedge, c.S, c.pcurr, c.nw, c.nh, c.t.lr_jj, c.jt_lo, c.lr_part); break;
         EFIT_LR_CASE(3) EFIT_LR_CASE(5) EFIT_LR_CASE(9) EFIT_LR_CASE(17)
 #undef EFIT_LR_CASE
     }
@@ -1034,10 +1066,10 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     if (nslab > 0) {
         dim3 grid(c.t.tb_nchunk, c.t.tb_ngroup);
         if (c.mode == EFIT_GREEN_TABLE) {
-            k_bnd_tb<kTbGI, kTbUnroll><<<grid, 256, smem_tb, s>>>(c.T, c.S, nslab, c.i_lo, c.nw * c.nh, c.pcurr,
+            launch_pdl(k_bnd_tb<kTbGI, kTbUnroll>, dim3(grid), dim3(256), smem_tb, s, c.T, c.S, nslab, c.i_lo, c.nw * c.nh, c.pcurr,
                                                                   c.pflip, c.t.tb_ch, c.tb_part);
         } else {
-            k_bnd_tb_otf<kTbGI><<<grid, 256, smem_tb, s>>>(c.i_lo, nslab, c.nw, c.nh, c.rmin, c.dr, c.dz, c.pcurr,
+            launch_pdl(k_bnd_tb_otf<kTbGI>, dim3(grid), dim3(256), smem_tb, s, c.i_lo, nslab, c.nw, c.nh, c.rmin, c.dr, c.dz, c.pcurr,
                                                            c.pflip, c.t.tb_ch, c.tb_part);
         }
         if ((e = cudaGetLastError())) return e;
@@ -1045,7 +1077,7 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     mark(c, s, M_TB);
     if ((e = cudaStreamWaitEvent(s, c.ev_join, 0))) return e;
     const int jlo = c.jt_lo * 32 * c.t.lr_jt, jhi = min(c.nh, c.jt_hi * 32 * c.t.lr_jt);
-    k_bnd_reduce<<<(c.n_edge + 7) / 8, 256, 0, s>>>(c.tb_part, c.t.tb_nchunk, c.lr_part, c.t.lr_nblk, c.nw, c.nh,
+    launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, c.tb_part, c.t.tb_nchunk, c.lr_part, c.t.lr_nblk, c.nw, c.nh,
                                                     c.i_lo, c.i_hi, jlo, jhi, psib);
     return cudaGetLastError();
 }
@@ -1089,7 +1121,8 @@ __global__ void __launch_bounds__(256) k_dst_fwd(const double* __restrict__ pcur
     const int r0 = 1 + 2 * blockIdx.x;  // first row of the pair
     const double idz2 = 1.0 / (dz * dz);
     const double cellinv = 1.0 / (dr * dz);
-    for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = __ldg(W + k);
+    for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = __ldg(W + k);  // init-time constants
+    griddep();
     for (int p = threadIdx.x; p < M; p += blockDim.x) {
         const int j = bitrev(p, log2m);  // a2[p] = z[bitrev(p)]: contiguous shared stores
         double v[2] = {0.0, 0.0};
@@ -1139,6 +1172,7 @@ __global__ void __launch_bounds__(256) k_dst_fwd(const double* __restrict__ pcur
 __global__ void __launch_bounds__(128) k_tridiag(double* __restrict__ fhat, const double* __restrict__ alpha,
                                                  const double* __restrict__ inv, const double* __restrict__ cp,
                                                  int ld, int nmode) {
+    griddep();
     const int mode = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (mode >= nmode) return;
@@ -1203,6 +1237,7 @@ __global__ void __launch_bounds__(256) k_dst_inv(const double* __restrict__ fhat
     extern __shared__ __align__(16) double2 a2[];  // [M] data, then [M/2] twiddles
     double2* Ws = a2 + M;
     __shared__ double wmax[8];
+    griddep();
     __shared__ bool last;
     const int n = nh - 2, ni = nw - 2;
     const int npairs = (ni + 1) / 2;
@@ -1290,14 +1325,14 @@ cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double
                          const double* psi_ext, double* eps, cudaStream_t s) {
     const int npairs = (c.ni + 1) / 2;
     const size_t smem = sizeof(double2) * (c.fft_m + c.fft_m / 2);
-    k_dst_fwd<<<npairs, 256, smem, s>>>(pcurr, psib, c.tri_a, c.nw, c.nh, c.rmin, c.dr, c.dz, c.twiddle, c.fft_m,
+    launch_pdl(k_dst_fwd, dim3(npairs), dim3(256), smem, s, pcurr, psib, c.tri_a, c.nw, c.nh, c.rmin, c.dr, c.dz, c.twiddle, c.fft_m,
                                         c.fft_log2, c.fhat, c.ni_pad);
     cudaError_t e = cudaGetLastError();
     if (e) return e;
-    k_tridiag<<<(c.nmode + 3) / 4, 128, 0, s>>>(c.fhat, c.tri_alpha, c.tri_inv, c.tri_cp, c.ni_pad, c.nmode);
+    launch_pdl(k_tridiag, dim3((c.nmode + 3) / 4), dim3(128), 0, s, c.fhat, c.tri_alpha, c.tri_inv, c.tri_cp, c.ni_pad, c.nmode);
     e = cudaGetLastError();
     if (e) return e;
-    k_dst_inv<<<npairs + 1, 256, smem, s>>>(c.fhat, c.ni_pad, psib, c.nw, c.nh, c.twiddle, c.fft_m, c.fft_log2, psi_out,
+    launch_pdl(k_dst_inv, dim3(npairs + 1), dim3(256), smem, s, c.fhat, c.ni_pad, psib, c.nw, c.nh, c.twiddle, c.fft_m, c.fft_log2, psi_out,
                                             psi_inout, psi_ext, c.eps_part, c.tickets + 1, c.axbd, eps);
     return cudaGetLastError();
 }
@@ -1306,6 +1341,7 @@ cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double
 // build the vertically mirrored copy used by the top targets.
 __global__ void k_make_pair(const double* __restrict__ I, double* __restrict__ pc, double* __restrict__ pf,
                             int nw, int nh) {
+    griddep();
     const int n = nw * nh;
     for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += gridDim.x * blockDim.x) {
         const int ii = g / nh, m = g - (g / nh) * nh;
@@ -1317,7 +1353,7 @@ __global__ void k_make_pair(const double* __restrict__ I, double* __restrict__ p
 
 cudaError_t launch_make_pair(Ctx& c, const double* pcurr, cudaStream_t s) {
     const int n = c.nw * c.nh;
-    k_make_pair<<<(n + 255) / 256, 256, 0, s>>>(pcurr, c.pcurr, c.pflip, c.nw, c.nh);
+    launch_pdl(k_make_pair, dim3((n + 255) / 256), dim3(256), 0, s, pcurr, c.pcurr, c.pflip, c.nw, c.nh);
     return cudaGetLastError();
 }
 
