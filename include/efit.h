@@ -51,7 +51,8 @@ extern "C" {
 typedef struct efit_ctx efit_ctx;
 typedef void* efit_stream_t; /* cudaStream_t */
 
-/* Uniform R-Z grid.  Requires 3 <= nw, nh <= 4097, 0 < rmin < rmax, zmin < zmax. */
+/* Uniform R-Z grid.  Requires 3 <= nw, nh <= 2049, nh - 1 a power of two (FFT-based interior
+ * solve), 0 < rmin < rmax, zmin < zmax. */
 typedef struct {
     int32_t nw, nh;
     double rmin, rmax, zmin, zmax;

@@ -119,7 +119,8 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     c.world = d ? d->world : 1;
     c.n_edge = 2 * c.nh + 2 * (c.nw - 2);
     c.ni = c.nw - 2;
-    c.ni_pad = 32 * ((c.ni + 31) / 32);  // segment-interleaved solve layout: 32 lanes x L rows
+    c.ni_pad = 32 * ((c.ni + 31) / 32);  // segment-interleaved factor layout: 32 lanes x L rows
+    c.fhat_ld = (c.ni + 3) / 4 * 4;
     c.nmode = c.nh - 2;
     c.fft_m = 2 * (c.nh - 1);
     c.fft_log2 = 0;
@@ -133,7 +134,10 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     t.tb_nchunk = (int)((n + t.tb_ch - 1) / t.tb_ch);
     t.tb_gi = 8;
     t.lr_jt = c.nh <= 96 ? 3 : (c.nh <= 160 ? 5 : (c.nh <= 288 ? 9 : 17));
-    t.lr_njt = (c.nh + 32 * t.lr_jt - 1) / (32 * t.lr_jt);
+    c.lr_direct = getenv("EFIT_LR_DIRECT") != nullptr;
+    c.lr_ldi = (c.nw + 3) / 4 * 4;
+    // the FFT path computes all left/right targets at once: a single "tile"
+    t.lr_njt = c.lr_direct ? (c.nh + 32 * t.lr_jt - 1) / (32 * t.lr_jt) : 1;
     t.lr_iib = 2;
     t.lr_nblk = (c.nw + t.lr_iib - 1) / t.lr_iib;
     {
@@ -203,10 +207,13 @@ static size_t carve(Ctx& c, char* base) {
     c.pflip = (double*)take(sizeof(double) * (size_t)round_up(n, c.t.tb_ch));
     c.tb_part = (double*)take(sizeof(double) * (size_t)c.t.tb_nchunk * c.nw * 2);
     c.lr_part = (double*)take(sizeof(double) * (size_t)c.t.lr_nblk * 2 * c.nh);
+    c.lr_spec = (double*)take(sizeof(double) * 2 * (size_t)c.nh * c.lr_ldi);
+    c.lr_xh = (double2*)take(sizeof(double2) * (size_t)c.nh * c.lr_ldi);
+    c.lr_y = (double2*)take(sizeof(double2) * 2 * (size_t)c.nh);
     c.psib = (double*)take(sizeof(double) * c.n_edge);
-    c.fhat = (double*)take(sizeof(double) * (size_t)c.ni_pad * c.nmode);
+    c.fhat = (double*)take(sizeof(double) * (size_t)c.fhat_ld * c.nmode);
     c.psip = (double*)take(sizeof(double) * (size_t)n);
-    c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 1));
+    c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 2));
     c.scratch_meas = (double*)take(sizeof(double) * c.ndiag);
     return (size_t)round_up((long long)off, 256);
 }
@@ -282,7 +289,9 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
         return cuda_fail(nullptr, e, "table build");
     }
     c.side = nullptr; c.ev_fork = nullptr; c.ev_join = nullptr;
-    if ((e = cudaStreamCreateWithFlags(&c.side, cudaStreamNonBlocking)) ||
+    int prio_lo = 0, prio_hi = 0;
+    cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+    if ((e = cudaStreamCreateWithPriority(&c.side, cudaStreamNonBlocking, prio_hi)) ||
         (e = cudaEventCreateWithFlags(&c.ev_fork, cudaEventDisableTiming)) ||
         (e = cudaEventCreateWithFlags(&c.ev_join, cudaEventDisableTiming))) {
         if (c.side) cudaStreamDestroy(c.side);

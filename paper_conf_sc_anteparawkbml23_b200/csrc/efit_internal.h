@@ -10,7 +10,7 @@ namespace efit {
 
 constexpr int kMaxBasis = 24;
 constexpr int kMaxKnots = 20;
-constexpr int kMaxN = 4097;
+constexpr int kMaxN = 2049;  // FFT working set 2.5*M*16 B of shared memory, M = 2(nh-1)
 constexpr int kLsqMaxRowsHost = 1024;
 
 // device status-word bits
@@ -40,7 +40,8 @@ struct Ctx {
     int n_fl, n_mp, n_int, ndiag, n_lim, ip_sign;
     int mode, rank, world;
     int n_edge, ni, nmode;       // ni = nw-2 interior rows, nmode = nh-2 sine modes
-    int ni_pad;                  // row stride of the mode-major solve arrays (even)
+    int ni_pad;                  // 32 * rows-per-lane: stride of the segment-interleaved Thomas factors
+    int fhat_ld;                 // row stride of the mode-major DST coefficients (multiple of 4)
     int fft_m, fft_log2;         // complex FFT length 2(nh-1) and its log2
     int m_lo, m_hi;              // response rows of this rank
     int i_lo, i_hi;              // top/bottom target rows of this rank (within [1, nw-1))
@@ -78,9 +79,14 @@ struct Ctx {
     double* pcurr;      // [roundup(nw*nh, tb_ch)]  current per cell, zero tail
     double* pflip;      // [roundup(nw*nh, tb_ch)]  I[ii][nh-1-m] (vertically mirrored), zero tail
     double* tb_part;    // [tb_nchunk][nw][2]
-    double* lr_part;    // [lr_nblk][2][nh]
+    double* lr_part;    // [2][nh][lr_nblk]  (direct left/right path)
+    double* lr_spec;    // [2][nh][lr_ldi]   real spectra of the circular left/right kernel rows
+    double2* lr_xh;     // [nh][lr_ldi]      half spectra of the source rows (per iteration)
+    double2* lr_y;      // [2][nh]           accumulated spectra of both sides
+    int lr_ldi;         // row stride of the spectral arrays (multiple of 4)
+    bool lr_direct;     // EFIT_LR_DIRECT=1: direct Toeplitz kernel instead of the FFT path
     double* psib;       // [n_edge]
-    double* fhat;       // [nmode][ld]  DST coefficients, mode-major (in place: tridiagonal solution)
+    double* fhat;       // [nmode][fhat_ld]  DST coefficients, mode-major (in place: tridiagonal solution)
     double* psip;       // [nw*nh]
     double* eps_part;   // [red_blocks]
     double* scratch_meas;  // [ndiag] (unused placeholder)

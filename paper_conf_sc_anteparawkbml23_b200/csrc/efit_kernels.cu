@@ -137,6 +137,10 @@ __device__ double bilinear(const double* psi, int nw, int nh, double rmin, doubl
     return s;
 }
 
+cudaError_t launch_lr_spectra(Ctx& c, cudaStream_t s);
+cudaError_t launch_lr_fft(Ctx& c, double* psib, cudaStream_t s);
+cudaError_t prepare_lr_fft(Ctx& c);
+
 // ================================================================================ init
 
 // Green's slabs: slab r is target row i = row_first + r*row_step;
@@ -282,6 +286,10 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
     k_tri_factors<<<(c.nmode + 63) / 64, 64, 0, s>>>(c.tri_a, c.tri_cp, c.tri_inv, c.tri_alpha, c.ni, c.ni_pad,
                                                      c.nmode, c.rmin, c.dr, c.dz);
     k_twiddles<<<(c.fft_m / 2 + 255) / 256, 256, 0, s>>>(c.twiddle, c.fft_m);
+    if (!c.lr_direct) {  // needs the edge slabs and the twiddles above
+        e = launch_lr_spectra(c, s);
+        if (e) return e;
+    }
     e = cudaMemsetAsync(c.status, 0, sizeof(int), s);
     if (e) return e;
     e = cudaMemsetAsync(c.tickets, 0, sizeof(unsigned) * 8, s);
@@ -1058,7 +1066,11 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     // fork: the FP64-bound left/right kernel runs on the side stream, concurrently with the
     // HBM-bound top/bottom stream (both only read pcurr / ipair); join before the reduce.
     if ((e = cudaEventRecord(c.ev_fork, s)) || (e = cudaStreamWaitEvent(c.side, c.ev_fork, 0))) return e;
-    if ((e = launch_lr(c, c.side, false))) return e;
+    if (c.lr_direct) {
+        if ((e = launch_lr(c, c.side, false))) return e;
+    } else {
+        if ((e = launch_lr_fft(c, psib, c.side))) return e;
+    }
     mark(c, c.side, M_LR);
     if ((e = cudaEventRecord(c.ev_join, c.side))) return e;
     const int nslab = c.i_hi - c.i_lo;
@@ -1076,7 +1088,9 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     }
     mark(c, s, M_TB);
     if ((e = cudaStreamWaitEvent(s, c.ev_join, 0))) return e;
-    const int jlo = c.jt_lo * 32 * c.t.lr_jt, jhi = min(c.nh, c.jt_hi * 32 * c.t.lr_jt);
+    // left/right entries come from the partials (direct path) or were written by k_lr_ifft
+    const int jlo = c.lr_direct ? c.jt_lo * 32 * c.t.lr_jt : 0;
+    const int jhi = c.lr_direct ? min(c.nh, c.jt_hi * 32 * c.t.lr_jt) : 0;
     launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, c.tb_part, c.t.tb_nchunk, c.lr_part, c.t.lr_nblk, c.nw, c.nh,
                                                     c.i_lo, c.i_hi, jlo, jhi, psib);
     return cudaGetLastError();
@@ -1084,47 +1098,91 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
 
 // ================================================================================ interior solve
 
-// In-place radix-2 complex FFT (forward, exp(-2 pi i jk/M)) of M = 2^log2m points in shared
-// memory; input must already be in bit-reversed order.  Twiddles W[k] = exp(-2 pi i k/M).
-__device__ void fft_smem(double2* a, int M, int log2m, const double2* W) {
-    for (int st = 1; st <= log2m; ++st) {
-        const int half = 1 << (st - 1);
-        const int tstride = M >> st;
-        for (int b = threadIdx.x; b < M / 2; b += blockDim.x) {
-            const int grp = b >> (st - 1);
-            const int pos = b & (half - 1);
-            const int i0 = (grp << st) + pos;
-            const int i1 = i0 + half;
-            const double2 w = W[pos * tstride];
-            const double2 u = a[i0], v = a[i1];
-            const double2 t = make_double2(w.x * v.x - w.y * v.y, w.x * v.y + w.y * v.x);
-            a[i0] = make_double2(u.x + t.x, u.y + t.y);
-            a[i1] = make_double2(u.x - t.x, u.y - t.y);
-        }
-        __syncthreads();
-    }
+// Forward complex FFT (exp(-2 pi i jk/M)) of M = 2^log2m points in shared memory, Stockham
+// auto-sort (natural order in and out, ping-pong between x and y), radix 4 while >= 2 bits remain,
+// one radix-2 stage otherwise.  At a stage with P sub-problems of length N_s = M/P the layout is
+// A[n P + b]; the radix-r DIF butterfly on inputs a_q = A[(n1 + q N_s/r) P + b] gives
+// y_k = sum_q a_q w_r^(q k) * w_M^(n1 k P), stored at B[n1 r P + b + k P].  W[e] = exp(-2 pi i e/M)
+// for e < M/2 (W[e + M/2] = -W[e]).  Returns the buffer holding the result.
+__device__ __forceinline__ double2 cmul(double2 a, double2 b) {
+    return make_double2(fma(a.x, b.x, -a.y * b.y), fma(a.x, b.y, a.y * b.x));
+}
+__device__ __forceinline__ double2 twid(const double2* W, int e, int M) {
+    const double2 w = W[e & ((M >> 1) - 1)];
+    return (e & (M >> 1)) ? make_double2(-w.x, -w.y) : w;
 }
 
-__device__ __forceinline__ int bitrev(int x, int log2m) { return (int)(__brev((unsigned)x) >> (32 - log2m)); }
+__device__ double2* fft_stockham(double2* x, double2* y, int M, int log2m, const double2* W, int tid, int nthr) {
+    double2* a = x;
+    double2* b = y;
+    int s = 0;  // log2 of the number of sub-problems P
+    while (s < log2m) {
+        const int P = 1 << s;
+        if (log2m - s >= 2) {
+            const int q = M >> (s + 2);  // N_s / 4
+            for (int t = tid; t < (M >> 2); t += nthr) {
+                const int bb = t & (P - 1), n1 = t >> s;
+                const double2 a0 = a[n1 * P + bb], a1 = a[(n1 + q) * P + bb];
+                const double2 a2 = a[(n1 + 2 * q) * P + bb], a3 = a[(n1 + 3 * q) * P + bb];
+                const double2 t0 = make_double2(a0.x + a2.x, a0.y + a2.y), t1 = make_double2(a0.x - a2.x, a0.y - a2.y);
+                const double2 t2 = make_double2(a1.x + a3.x, a1.y + a3.y);
+                const double2 t3 = make_double2(a1.y - a3.y, a3.x - a1.x);  // -i (a1 - a3)
+                const int e1 = (n1 * P) & (M - 1);
+                const double2 y1 = cmul(make_double2(t1.x + t3.x, t1.y + t3.y), twid(W, e1, M));
+                const double2 y2 = cmul(make_double2(t0.x - t2.x, t0.y - t2.y), twid(W, (2 * e1) & (M - 1), M));
+                const double2 y3 = cmul(make_double2(t1.x - t3.x, t1.y - t3.y), twid(W, (3 * e1) & (M - 1), M));
+                const int o = n1 * (P << 2) + bb;
+                b[o] = make_double2(t0.x + t2.x, t0.y + t2.y);
+                b[o + P] = y1;
+                b[o + 2 * P] = y2;
+                b[o + 3 * P] = y3;
+            }
+            s += 2;
+        } else {
+            const int q = M >> (s + 1);  // N_s / 2
+            for (int t = tid; t < (M >> 1); t += nthr) {
+                const int bb = t & (P - 1), n1 = t >> s;
+                const double2 a0 = a[n1 * P + bb], a1 = a[(n1 + q) * P + bb];
+                const int o = n1 * (P << 1) + bb;
+                b[o] = make_double2(a0.x + a1.x, a0.y + a1.y);
+                b[o + P] = cmul(make_double2(a0.x - a1.x, a0.y - a1.y), twid(W, (n1 * P) & (M - 1), M));
+            }
+            s += 1;
+        }
+        __syncthreads();
+        double2* tmp = a;
+        a = b;
+        b = tmp;
+    }
+    return a;
+}
 
-// Forward DST-I along Z of the right-hand side of two interior rows at once (packed as the real
-// and imaginary parts of one complex FFT of the odd extension, length M = 2(n+1)):
+// Number of Stockham stages for M = 2^log2m (radix 4, plus one radix 2 if log2m is odd): the
+// result is in the scratch buffer when it is odd.
+__host__ __device__ __forceinline__ int fft_stages(int log2m) { return (log2m >> 1) + (log2m & 1); }
+
+// Forward DST-I along Z of the right-hand side of 2*FPC interior rows per CTA (two rows packed as
+// the real and imaginary parts of one complex FFT of the odd extension, length M = 2(n+1); FPC
+// FFTs side by side, TPF threads each):
 //   f_ij = -mu0 R_i I_ij/(dR dZ) - (Dirichlet terms of the edge values psi_b).
-// DST_k(x) = -Im(Z_k)/2 for the real-part row, Re(Z_k)/2 for the imaginary-part row.
-__global__ void __launch_bounds__(256) k_dst_fwd(const double* __restrict__ pcurr, const double* __restrict__ psib,
+// DST_k(x) = -Im(Z_k)/2 for the real-part row, Re(Z_k)/2 for the imaginary-part row.  Output is
+// mode-major, fhat[k-1][r] (r = i-1), the CTA's 2*FPC rows contiguous (16/32-byte stores per mode).
+__global__ void __launch_bounds__(512) k_dst_fwd(const double* __restrict__ pcurr, const double* __restrict__ psib,
                                                  const double* __restrict__ tri_a, int nw, int nh, double rmin,
                                                  double dr, double dz, const double2* __restrict__ W, int M,
-                                                 int log2m, double* __restrict__ fhat, int ld) {
-    extern __shared__ __align__(16) double2 a2[];  // [M] data, then [M/2] twiddles
-    double2* Ws = a2 + M;
+                                                 int log2m, int FPC, double* __restrict__ fhat, int ld) {
+    extern __shared__ __align__(16) double2 a2[];  // FPC x ([M] data, [M] scratch), then [M/2] twiddles
+    double2* Ws = a2 + 2 * FPC * M;
     const int n = nh - 2, ni = nw - 2;
-    const int r0 = 1 + 2 * blockIdx.x;  // first row of the pair
+    const int TPF = blockDim.x / FPC;
+    const int f = threadIdx.x / TPF, lt = threadIdx.x - f * TPF;
+    const int rbase = 2 * FPC * blockIdx.x;  // first 0-based interior row of the CTA
+    double2* xf = a2 + 2 * f * M;
     const double idz2 = 1.0 / (dz * dz);
     const double cellinv = 1.0 / (dr * dz);
     for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = __ldg(W + k);  // init-time constants
     griddep();
-    for (int p = threadIdx.x; p < M; p += blockDim.x) {
-        const int j = bitrev(p, log2m);  // a2[p] = z[bitrev(p)]: contiguous shared stores
+    for (int j = lt; j < M; j += TPF) {
         double v[2] = {0.0, 0.0};
         int jj = 0;
         double sgn = 0.0;
@@ -1133,59 +1191,63 @@ __global__ void __launch_bounds__(256) k_dst_fwd(const double* __restrict__ pcur
         if (sgn != 0.0) {
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
-                const int i = r0 + h;
+                const int i = rbase + 2 * f + h + 1;  // grid row
                 if (i > ni) continue;
                 const double R = grid_coord(rmin, i, dr);
-                double f = -kMu0 * R * pcurr[(long long)i * nh + jj] * cellinv;
-                if (i == 1) f -= tri_a[0] * psib[jj];                                   // left edge
-                if (i == ni) f -= (2.0 / (dr * dr) - tri_a[ni - 1]) * psib[nh + jj];    // right edge (c_ni)
-                if (jj == 1) f -= psib[2 * nh + (i - 1)] * idz2;                        // bottom edge
-                if (jj == n) f -= psib[2 * nh + (nw - 2) + (i - 1)] * idz2;             // top edge
-                v[h] = sgn * f;
+                double fv = -kMu0 * R * pcurr[(long long)i * nh + jj] * cellinv;
+                if (i == 1) fv -= tri_a[0] * psib[jj];                                   // left edge
+                if (i == ni) fv -= (2.0 / (dr * dr) - tri_a[ni - 1]) * psib[nh + jj];    // right edge (c_ni)
+                if (jj == 1) fv -= psib[2 * nh + (i - 1)] * idz2;                        // bottom edge
+                if (jj == n) fv -= psib[2 * nh + (nw - 2) + (i - 1)] * idz2;             // top edge
+                v[h] = sgn * fv;
             }
         }
-        a2[p] = make_double2(v[0], v[1]);
+        xf[j] = make_double2(v[0], v[1]);
     }
     __syncthreads();
-    fft_smem(a2, M, log2m, Ws);
-    // mode-major, segment-interleaved output (see k_tridiag): row r at (r % L)*32 + r / L
-    const int L = ld >> 5;
-    const int ra = r0 - 1, rb = r0;
-    const long long pa = (long long)(ra % L) * 32 + ra / L, pb = (long long)(rb % L) * 32 + rb / L;
+    fft_stockham(xf, xf + M, M, log2m, Ws, lt, TPF);
+    const int ro = (fft_stages(log2m) & 1) ? M : 0;
     for (int k = 1 + threadIdx.x; k <= n; k += blockDim.x) {
-        const double2 z = a2[k];
-        double* dst = fhat + (long long)(k - 1) * ld;
-        dst[pa] = -0.5 * z.y;
-        if (r0 + 1 <= ni) dst[pb] = 0.5 * z.x;
+        double* dst = fhat + (long long)(k - 1) * ld + rbase;
+        for (int g = 0; g < FPC; ++g) {
+            const double2 z = a2[2 * g * M + ro + k];
+            *reinterpret_cast<double2*>(dst + 2 * g) = make_double2(-0.5 * z.y, 0.5 * z.x);
+        }
     }
 }
 
-// Radial tridiagonal solve per sine mode, one warp per mode, in place.  Row r of a mode lives at
-// (r % L)*32 + r / L (L = ld/32): lane l owns the contiguous rows [l L, (l+1) L) and element e of
-// every lane is one coalesced 256-byte line.  Both Thomas sweeps are first-order linear
-// recurrences,  forward d_r = inv_r f_r + alpha_r d_{r-1} (d_{-1} = 0),  backward
-// x_r = d_r - c'_r x_{r+1} (x_ni = 0): each lane composes the affine map of its segment, a 5-step
-// shuffle scan composes the maps of the preceding (following) lanes, and each lane replays its
-// segment from the exact incoming value.  Padding rows (r >= ni) have alpha = inv = c' = 0 and
-// only follow the real rows.  |alpha|, |c'| < 1 (diagonal dominance) keeps the reassociation as
-// accurate as the sequential sweep.
-__global__ void __launch_bounds__(128) k_tridiag(double* __restrict__ fhat, const double* __restrict__ alpha,
+// Radial tridiagonal solve per sine mode, one warp per mode, in place on the mode-major array.
+// The warp stages its mode column in shared memory with a skew (row r at r + r/L, L = rows per
+// lane) so both the global access and the lane-segment access are conflict-free.  Both Thomas
+// sweeps are first-order linear recurrences,  forward d_r = inv_r f_r + alpha_r d_{r-1}
+// (d_{-1} = 0),  backward x_r = d_r - c'_r x_{r+1} (x_ni = 0): each lane composes the affine map of
+// its segment of L rows, a 5-step shuffle scan composes the maps of the preceding (following)
+// lanes, and each lane replays its segment from the exact incoming value.  The factors are stored
+// segment-interleaved (row r at (r % L)*32 + r/L) so a lane's factor loads are coalesced across the
+// warp.  Padding rows (r >= ni) have alpha = inv = c' = 0 and only follow the real rows.
+// |alpha|, |c'| < 1 (diagonal dominance) keeps the reassociation as accurate as the sequential sweep.
+__global__ void __launch_bounds__(128) k_tridiag(double* __restrict__ fhat, int ld, const double* __restrict__ alpha,
                                                  const double* __restrict__ inv, const double* __restrict__ cp,
-                                                 int ld, int nmode) {
+                                                 int ni, int L, int nmode) {
+    extern __shared__ __align__(16) double sm_tri[];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int mode = blockIdx.x * 4 + warp;
+    double* sf = sm_tri + (size_t)warp * (32 * L + 32);  // skewed: row r at r + r/L < 32L + 32
     griddep();
-    const int mode = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int lane = threadIdx.x & 31;
     if (mode >= nmode) return;
-    const int L = ld >> 5;
-    double* f = fhat + (long long)mode * ld + lane;
-    const double* al = alpha + (long long)mode * ld + lane;
-    const double* iv = inv + (long long)mode * ld + lane;
-    const double* c = cp + (long long)mode * ld + lane;
+    double* fg = fhat + (long long)mode * ld;
+    for (int r = lane; r < 32 * L; r += 32) sf[r + r / L] = r < ni ? fg[r] : 0.0;
+    __syncwarp();
+    const long long fo = (long long)mode * 32 * L + lane;
+    const double* al = alpha + fo;
+    const double* iv = inv + fo;
+    const double* c = cp + fo;
+    double* f = sf + lane * (L + 1);  // this lane's segment rows lane*L .. lane*L + L - 1
     double A = 1.0, B = 0.0;
 #pragma unroll 4
     for (int e = 0; e < L; ++e) {
         const double a = al[32 * e];
-        B = fma(a, B, iv[32 * e] * f[32 * e]);
+        B = fma(a, B, iv[32 * e] * f[e]);
         A *= a;
     }
 #pragma unroll
@@ -1198,14 +1260,14 @@ __global__ void __launch_bounds__(128) k_tridiag(double* __restrict__ fhat, cons
     if (lane == 0) d = 0.0;
 #pragma unroll 4
     for (int e = 0; e < L; ++e) {
-        d = fma(al[32 * e], d, iv[32 * e] * f[32 * e]);
-        f[32 * e] = d;
+        d = fma(al[32 * e], d, iv[32 * e] * f[e]);
+        f[e] = d;
     }
     double C = 1.0, D = 0.0;
 #pragma unroll 4
     for (int e = L - 1; e >= 0; --e) {
         const double q = -c[32 * e];
-        D = fma(q, D, f[32 * e]);
+        D = fma(q, D, f[e]);
         C *= q;
     }
 #pragma unroll
@@ -1218,29 +1280,32 @@ __global__ void __launch_bounds__(128) k_tridiag(double* __restrict__ fhat, cons
     if (lane == 31) x = 0.0;
 #pragma unroll 4
     for (int e = L - 1; e >= 0; --e) {
-        x = fma(-c[32 * e], x, f[32 * e]);
-        f[32 * e] = x;
+        x = fma(-c[32 * e], x, f[e]);
+        f[e] = x;
     }
+    __syncwarp();
+    for (int r = lane; r < ni; r += 32) fg[r] = sf[r + r / L];
 }
 
-// Inverse DST-I (same transform, scale 2/(n+1)) of two rows, then either
+// Inverse DST-I (same transform, scale 2/(n+1)) of 2*FPC rows per CTA, then either
 //   psi_out = psi_p                                  (efit_interior_solve), or
 //   psi_inout <- psi_p + psi_ext, eps partial max     (efit_fit_step),
 // edges (j = 0, nh-1, and rows 0, nw-1 in the extra last block) take psi_b.
-__global__ void __launch_bounds__(256) k_dst_inv(const double* __restrict__ fhat, int ld,
+__global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat, int ld,
                                                  const double* __restrict__ psib,
                                                  int nw, int nh, const double2* __restrict__ W, int M, int log2m,
-                                                 double* __restrict__ psi_out, double* __restrict__ psi_inout,
+                                                 int FPC, double* __restrict__ psi_out, double* __restrict__ psi_inout,
                                                  const double* __restrict__ psi_ext, double* __restrict__ eps_part,
                                                  unsigned* ticket, const double* __restrict__ axbd,
                                                  double* __restrict__ eps) {
-    extern __shared__ __align__(16) double2 a2[];  // [M] data, then [M/2] twiddles
-    double2* Ws = a2 + M;
-    __shared__ double wmax[8];
-    griddep();
+    extern __shared__ __align__(16) double2 a2[];  // FPC x ([M] data, [M] scratch), then [M/2] twiddles
+    double2* Ws = a2 + 2 * FPC * M;
+    __shared__ double wmax[16];
     __shared__ bool last;
     const int n = nh - 2, ni = nw - 2;
-    const int npairs = (ni + 1) / 2;
+    const int nrb = (ni + 2 * FPC - 1) / (2 * FPC);  // row blocks; block nrb does the edge rows
+    const int TPF = blockDim.x / FPC;
+    const int f = threadIdx.x / TPF, lt = threadIdx.x - f * TPF;
     double dmax = 0.0;
     auto emit = [&](long long g, double pp) {
         if (psi_out) psi_out[g] = pp;
@@ -1250,43 +1315,49 @@ __global__ void __launch_bounds__(256) k_dst_inv(const double* __restrict__ fhat
             psi_inout[g] = nv;
         }
     };
-    if ((int)blockIdx.x < npairs) {
-        const int r0 = 1 + 2 * blockIdx.x;
+    if ((int)blockIdx.x < nrb) {
+        const int rbase = 2 * FPC * blockIdx.x;
         for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = __ldg(W + k);
-        for (int p = threadIdx.x; p < M; p += blockDim.x) {
-            const int j = bitrev(p, log2m);
-            double v[2] = {0.0, 0.0};
+        griddep();
+        // stage: for every mode the CTA's rows are contiguous in fhat
+        for (int j = threadIdx.x; j < M; j += blockDim.x) {
             int jj = 0;
             double sg = 0.0;
             if (j >= 1 && j <= n) { jj = j; sg = 1.0; }
             else if (j >= n + 2) { jj = M - j; sg = -1.0; }
-            if (sg != 0.0) {
-                const int L = ld >> 5;
-                const int ra = r0 - 1, rb = r0;
-                const double* src = fhat + (long long)(jj - 1) * ld;
-                v[0] = sg * src[(ra % L) * 32 + ra / L];
-                if (r0 + 1 <= ni) v[1] = sg * src[(rb % L) * 32 + rb / L];
+            const double* src = fhat + (long long)(jj > 0 ? jj - 1 : 0) * ld + rbase;
+            for (int g = 0; g < FPC; ++g) {
+                double2 v = make_double2(0.0, 0.0);
+                if (sg != 0.0) {
+                    const double2 w2 = *reinterpret_cast<const double2*>(src + 2 * g);
+                    v = make_double2(sg * w2.x, sg * w2.y);
+                }
+                a2[2 * g * M + j] = v;
             }
-            a2[p] = make_double2(v[0], v[1]);
         }
         __syncthreads();
-        fft_smem(a2, M, log2m, Ws);
+        fft_stockham(a2 + 2 * f * M, a2 + 2 * f * M + M, M, log2m, Ws, lt, TPF);
+        const int ro = (fft_stages(log2m) & 1) ? M : 0;
         const double sc = 2.0 / (double)(n + 1);
-        for (int h = 0; h < 2; ++h) {
-            const int i = r0 + h;
-            if (i > ni) break;
-            for (int j = threadIdx.x; j < nh; j += blockDim.x) {
-                double pp;
-                if (j == 0) pp = psib[2 * nh + (i - 1)];
-                else if (j == nh - 1) pp = psib[2 * nh + (nw - 2) + (i - 1)];
-                else {
-                    const double2 z = a2[j];
-                    pp = sc * (h == 0 ? -0.5 * z.y : 0.5 * z.x);
+        for (int g = 0; g < FPC; ++g) {
+            const double2* res = a2 + 2 * g * M + ro;
+            for (int h = 0; h < 2; ++h) {
+                const int i = rbase + 2 * g + h + 1;
+                if (i > ni) break;
+                for (int j = threadIdx.x; j < nh; j += blockDim.x) {
+                    double pp;
+                    if (j == 0) pp = psib[2 * nh + (i - 1)];
+                    else if (j == nh - 1) pp = psib[2 * nh + (nw - 2) + (i - 1)];
+                    else {
+                        const double2 z = res[j];
+                        pp = sc * (h == 0 ? -0.5 * z.y : 0.5 * z.x);
+                    }
+                    emit((long long)i * nh + j, pp);
                 }
-                emit((long long)i * nh + j, pp);
             }
         }
     } else {
+        griddep();
         // rows 0 and nw-1: left/right edge values
         for (int j = threadIdx.x; j < nh; j += blockDim.x) {
             emit((long long)j, psib[j]);
@@ -1321,20 +1392,213 @@ __global__ void __launch_bounds__(256) k_dst_inv(const double* __restrict__ fhat
     }
 }
 
+static void solve_shape(const Ctx& c, int& fpc, int& threads, size_t& smem) {
+    const int M = c.fft_m;
+    fpc = (sizeof(double2) * (size_t)(4 * M + M / 2) <= 160 * 1024) ? 2 : 1;
+    int tpf = M / 4;
+    if (tpf > 256) tpf = 256;
+    if (tpf < 32) tpf = 32;
+    threads = fpc * tpf;
+    smem = sizeof(double2) * (size_t)(2 * fpc * M + M / 2);
+}
+
 cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out, double* psi_inout,
                          const double* psi_ext, double* eps, cudaStream_t s) {
-    const int npairs = (c.ni + 1) / 2;
-    const size_t smem = sizeof(double2) * (c.fft_m + c.fft_m / 2);
-    launch_pdl(k_dst_fwd, dim3(npairs), dim3(256), smem, s, pcurr, psib, c.tri_a, c.nw, c.nh, c.rmin, c.dr, c.dz, c.twiddle, c.fft_m,
-                                        c.fft_log2, c.fhat, c.ni_pad);
-    cudaError_t e = cudaGetLastError();
+    int fpc, threads;
+    size_t smem;
+    solve_shape(c, fpc, threads, smem);
+    const int nrb = (c.ni + 2 * fpc - 1) / (2 * fpc);
+    cudaError_t e = launch_pdl(k_dst_fwd, dim3(nrb), dim3(threads), smem, s, pcurr, psib, c.tri_a, c.nw, c.nh, c.rmin,
+                               c.dr, c.dz, c.twiddle, c.fft_m, c.fft_log2, fpc, c.fhat, c.fhat_ld);
     if (e) return e;
-    launch_pdl(k_tridiag, dim3((c.nmode + 3) / 4), dim3(128), 0, s, c.fhat, c.tri_alpha, c.tri_inv, c.tri_cp, c.ni_pad, c.nmode);
-    e = cudaGetLastError();
+    const int L = c.ni_pad / 32;
+    e = launch_pdl(k_tridiag, dim3((c.nmode + 3) / 4), dim3(128), sizeof(double) * 4 * (32 * (size_t)L + 32), s, c.fhat,
+                   c.fhat_ld, c.tri_alpha, c.tri_inv, c.tri_cp, c.ni, L, c.nmode);
     if (e) return e;
-    launch_pdl(k_dst_inv, dim3(npairs + 1), dim3(256), smem, s, c.fhat, c.ni_pad, psib, c.nw, c.nh, c.twiddle, c.fft_m, c.fft_log2, psi_out,
-                                            psi_inout, psi_ext, c.eps_part, c.tickets + 1, c.axbd, eps);
+    return launch_pdl(k_dst_inv, dim3(nrb + 1), dim3(threads), smem, s, c.fhat, c.fhat_ld, psib, c.nw, c.nh,
+                      c.twiddle, c.fft_m, c.fft_log2, fpc, psi_out, psi_inout, psi_ext, c.eps_part, c.tickets + 1,
+                      c.axbd, eps);
+}
+
+// ================================================================================ left/right via FFT
+// The printed Fig. 2 nest is, for each side s, a sum over source rows of symmetric
+// Toeplitz products:  psi_b(s, j) = sum_ii sum_jj t_{s,ii}(|j - jj|) x_ii(jj).  With the even
+// circular extension c[d] = t(|d|) of length M = 2(nh-1) (d = +-(nh-1) share the same value, so the
+// wrap is exact for j, jj in [0, nh)) every row product is a circular convolution, and by linearity
+//   psi_b(s, .) = IFFT( sum_ii C_{s,ii} * FFT(x_ii) ),   C_{s,ii} = FFT(c_{s,ii})  (real: c is even).
+// C is table data (k_lr_spectra, once at init); per iteration: one FFT per source row pair,
+// a frequency-wise multiply-accumulate over rows (fixed order), and one inverse FFT for both sides.
+// O(N^2 log N) instead of the nest's 2 N^3 FMAs; same result to rounding (tested against the
+// oracle's direct sum at 1e-12).  EFIT_LR_DIRECT=1 selects the direct k_bnd_lr instead.
+
+// Spectra of the circular kernel rows: spec[(s*nh + f)*ldi + ii] = C_{s,ii}[f], f in [0, nh).
+__global__ void __launch_bounds__(512) k_lr_spectra(const double* __restrict__ Tedge, long long S, int nw, int nh,
+                                                    const double2* __restrict__ W, int M, int log2m, int FPC,
+                                                    double* __restrict__ spec, int ldi) {
+    extern __shared__ __align__(16) double2 a2[];
+    double2* Ws = a2 + 2 * FPC * M;
+    const int TPF = blockDim.x / FPC;
+    const int f = threadIdx.x / TPF, lt = threadIdx.x - f * TPF;
+    const int side = blockIdx.y;
+    const int ra = 2 * FPC * blockIdx.x + 2 * f, rb = ra + 1;
+    double2* xf = a2 + 2 * f * M;
+    for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = W[k];
+    const double* ta = Tedge + (long long)side * S + (long long)ra * nh;
+    const double* tb = Tedge + (long long)side * S + (long long)rb * nh;
+    for (int j = lt; j < M; j += TPF) {
+        const int d = j <= nh - 1 ? j : M - j;
+        xf[j] = make_double2(ra < nw ? ta[d] : 0.0, rb < nw ? tb[d] : 0.0);
+    }
+    __syncthreads();
+    fft_stockham(xf, xf + M, M, log2m, Ws, lt, TPF);
+    const int ro = (fft_stages(log2m) & 1) ? M : 0;
+    for (int g = 0; g < FPC; ++g) {
+        const int r0 = 2 * FPC * blockIdx.x + 2 * g;
+        const double2* res = a2 + 2 * g * M + ro;
+        for (int q = threadIdx.x; q < nh; q += blockDim.x) {
+            const double2 z = res[q];  // both spectra are real: Re -> row r0, Im -> row r0 + 1
+            if (r0 < nw) spec[((long long)side * nh + q) * ldi + r0] = z.x;
+            if (r0 + 1 < nw) spec[((long long)side * nh + q) * ldi + r0 + 1] = z.y;
+        }
+    }
+}
+
+// Per iteration: FFT of two source rows x_a + i x_b (zero-padded to M), unpacked to the two
+// half spectra X_a[f] = (Z[f] + conj Z[M-f])/2, X_b[f] = (Z[f] - conj Z[M-f])/(2i), f in [0, nh).
+__global__ void __launch_bounds__(512) k_lr_fft(const double* __restrict__ pcurr, int nw, int nh,
+                                                const double2* __restrict__ W, int M, int log2m, int FPC,
+                                                double2* __restrict__ Xh, int ldi) {
+    extern __shared__ __align__(16) double2 a2[];
+    double2* Ws = a2 + 2 * FPC * M;
+    const int TPF = blockDim.x / FPC;
+    const int f = threadIdx.x / TPF, lt = threadIdx.x - f * TPF;
+    const int ra = 2 * FPC * blockIdx.x + 2 * f, rb = ra + 1;
+    double2* xf = a2 + 2 * f * M;
+    for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = __ldg(W + k);
+    griddep();
+    const double* xa = pcurr + (long long)ra * nh;
+    const double* xb = pcurr + (long long)rb * nh;
+    for (int j = lt; j < M; j += TPF)
+        xf[j] = (j < nh) ? make_double2(ra < nw ? xa[j] : 0.0, rb < nw ? xb[j] : 0.0) : make_double2(0.0, 0.0);
+    __syncthreads();
+    fft_stockham(xf, xf + M, M, log2m, Ws, lt, TPF);
+    const int ro = (fft_stages(log2m) & 1) ? M : 0;
+    for (int g = 0; g < FPC; ++g) {
+        const int r0 = 2 * FPC * blockIdx.x + 2 * g;
+        const double2* res = a2 + 2 * g * M + ro;
+        for (int q = threadIdx.x; q < nh; q += blockDim.x) {
+            const double2 zf = res[q], zm = res[(M - q) & (M - 1)];
+            const double2 xa2 = make_double2(0.5 * (zf.x + zm.x), 0.5 * (zf.y - zm.y));
+            const double2 xb2 = make_double2(0.5 * (zf.y + zm.y), 0.5 * (zm.x - zf.x));
+            double2* dst = Xh + (long long)q * ldi + r0;
+            if (r0 + 1 < ldi) {
+                dst[0] = xa2;
+                dst[1] = xb2;
+            } else {
+                dst[0] = xa2;
+            }
+        }
+    }
+}
+
+// Y_s[f] = sum_ii C_{s,ii}[f] X_ii[f] for both sides; one warp per frequency, lanes over rows,
+// fixed butterfly => deterministic.
+__global__ void __launch_bounds__(256) k_lr_mac(const double* __restrict__ spec, const double2* __restrict__ Xh,
+                                                int nw, int nh, int ldi, double2* __restrict__ Y) {
+    griddep();
+    const int q = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+    if (q >= nh) return;
+    const double* c0 = spec + (long long)q * ldi;
+    const double* c1 = spec + ((long long)nh + q) * ldi;
+    const double2* x = Xh + (long long)q * ldi;
+    double a0r = 0.0, a0i = 0.0, a1r = 0.0, a1i = 0.0;
+    for (int ii = lane; ii < nw; ii += 32) {
+        const double2 xv = x[ii];
+        const double s0 = c0[ii], s1 = c1[ii];
+        a0r = fma(s0, xv.x, a0r);
+        a0i = fma(s0, xv.y, a0i);
+        a1r = fma(s1, xv.x, a1r);
+        a1i = fma(s1, xv.y, a1i);
+    }
+    a0r = warp_sum(a0r);
+    a0i = warp_sum(a0i);
+    a1r = warp_sum(a1r);
+    a1i = warp_sum(a1i);
+    if (lane == 0) {
+        Y[q] = make_double2(a0r, a0i);
+        Y[nh + q] = make_double2(a1r, a1i);
+    }
+}
+
+// Both real outputs with one inverse FFT: Q = Y_0 + i Y_1 on the full circle (Hermitian
+// extension Y_s[M-f] = conj Y_s[f]), q = IFFT(Q) = conj(FFT(conj Q))/M, psi_left = Re q,
+// psi_right = Im q.
+__global__ void __launch_bounds__(256) k_lr_ifft(const double2* __restrict__ Y, int nh, const double2* __restrict__ W,
+                                                 int M, int log2m, double* __restrict__ psib, int jlo, int jhi) {
+    extern __shared__ __align__(16) double2 a2[];
+    double2* Ws = a2 + 2 * M;
+    for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = __ldg(W + k);
+    griddep();
+    for (int f = threadIdx.x; f < M; f += blockDim.x) {
+        double2 y0, y1;
+        if (f <= M / 2) {
+            y0 = Y[f];
+            y1 = Y[nh + f];
+        } else {
+            const double2 u = Y[M - f], v = Y[nh + M - f];
+            y0 = make_double2(u.x, -u.y);
+            y1 = make_double2(v.x, -v.y);
+        }
+        const double2 qv = make_double2(y0.x - y1.y, y0.y + y1.x);  // Y_0 + i Y_1
+        a2[f] = make_double2(qv.x, -qv.y);                           // conj
+    }
+    __syncthreads();
+    fft_stockham(a2, a2 + M, M, log2m, Ws, threadIdx.x, blockDim.x);
+    const double2* res = a2 + ((fft_stages(log2m) & 1) ? M : 0);
+    const double im = 1.0 / (double)M;
+    for (int j = jlo + threadIdx.x; j < jhi; j += blockDim.x) {
+        const double2 p = res[j];
+        psib[j] = p.x * im;
+        psib[nh + j] = -p.y * im;
+    }
+}
+
+static size_t lr_fft_smem(const Ctx& c, int& fpc, int& threads) {
+    size_t smem;
+    solve_shape(c, fpc, threads, smem);
+    return smem;
+}
+
+cudaError_t launch_lr_spectra(Ctx& c, cudaStream_t s) {
+    int fpc, threads;
+    const size_t smem = lr_fft_smem(c, fpc, threads);
+    dim3 grid((c.nw + 2 * fpc - 1) / (2 * fpc), 2);
+    k_lr_spectra<<<grid, threads, smem, s>>>(c.Tedge, c.S, c.nw, c.nh, c.twiddle, c.fft_m, c.fft_log2, fpc, c.lr_spec,
+                                             c.lr_ldi);
     return cudaGetLastError();
+}
+
+cudaError_t launch_lr_fft(Ctx& c, double* psib, cudaStream_t s) {
+    if (c.jt_hi <= c.jt_lo) return cudaSuccess;  // left/right targets owned by another rank
+    int fpc, threads;
+    const size_t smem = lr_fft_smem(c, fpc, threads);
+    cudaError_t e = launch_pdl(k_lr_fft, dim3((c.nw + 2 * fpc - 1) / (2 * fpc)), dim3(threads), smem, s, c.pcurr,
+                               c.nw, c.nh, c.twiddle, c.fft_m, c.fft_log2, fpc, c.lr_xh, c.lr_ldi);
+    if (e) return e;
+    e = launch_pdl(k_lr_mac, dim3((c.nh + 7) / 8), dim3(256), 0, s, c.lr_spec, c.lr_xh, c.nw, c.nh, c.lr_ldi,
+                   c.lr_y);
+    if (e) return e;
+    return launch_pdl(k_lr_ifft, dim3(1), dim3(256), sizeof(double2) * (size_t)(2 * c.fft_m + c.fft_m / 2), s,
+                      c.lr_y, c.nh, c.twiddle, c.fft_m, c.fft_log2, psib, 0, c.nh);
+}
+
+cudaError_t prepare_lr_fft(Ctx& c) {
+    int fpc, threads;
+    const size_t smem = lr_fft_smem(c, fpc, threads);
+    cudaError_t e;
+    if ((e = raise_smem_limit((const void*)k_lr_spectra, smem))) return e;
+    if ((e = raise_smem_limit((const void*)k_lr_fft, smem))) return e;
+    return raise_smem_limit((const void*)k_lr_ifft, sizeof(double2) * (size_t)(2 * c.fft_m + c.fft_m / 2));
 }
 
 // Caller-supplied current (efit_boundary_flux): copy into the internal zero-padded buffer and
@@ -1371,10 +1635,17 @@ cudaError_t prepare_kernels(Ctx& c) {
     };
     if ((e = big((const void*)k_lsq, lsq_smem(c)))) return e;
     if ((e = launch_lr(c, nullptr, true))) return e;
+    if ((e = prepare_lr_fft(c))) return e;
     if ((e = big((const void*)k_bnd_tb<kTbGI, kTbUnroll>, 2 * sizeof(double) * c.t.tb_ch))) return e;
     if ((e = big((const void*)k_bnd_tb_otf<kTbGI>, 2 * sizeof(double) * c.t.tb_ch))) return e;
-    if ((e = big((const void*)k_dst_fwd, sizeof(double2) * (c.fft_m + c.fft_m / 2)))) return e;
-    if ((e = big((const void*)k_dst_inv, sizeof(double2) * (c.fft_m + c.fft_m / 2)))) return e;
+    {
+        int fpc, threads;
+        size_t smem;
+        solve_shape(c, fpc, threads, smem);
+        if ((e = big((const void*)k_dst_fwd, smem))) return e;
+        if ((e = big((const void*)k_dst_inv, smem))) return e;
+        if ((e = big((const void*)k_tridiag, sizeof(double) * 4 * ((size_t)c.ni_pad + 32)))) return e;
+    }
     return cudaSuccess;
 }
 
