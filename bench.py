@@ -245,8 +245,8 @@ def gpu_arm(args, rank, world, local):
             n = min(500, K - done)
             g = torch.cuda.CUDAGraph()
             with torch.cuda.graph(g, stream=cap):
-                for _ in range(n):
-                    step()
+                # n chained iterations: only the first normalises psi (efit_fit_steps)
+                ctx.fit_steps(n, psi, psi_ext, meas, sigma, coef, chi2, eps)
             graphs.append(g)
             done += n
         torch.cuda.synchronize()

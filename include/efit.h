@@ -173,6 +173,14 @@ int efit_fit_step(efit_ctx* ctx, double* d_psi, const double* d_psi_ext, const d
                   const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps,
                   efit_stream_t stream);
 
+/* nsteps chained Picard iterations in one call (one CUDA graph): the first normalises d_psi,
+ * later ones take psi_axis/psi_bdry from the previous iteration's update kernel (no separate
+ * normalisation pass).  d_coef/d_chi2/d_eps hold the last iteration's values; the caller checks
+ * eps < 1e-5 every nsteps iterations.  Same arguments and rules as efit_fit_step. */
+int efit_fit_steps(efit_ctx* ctx, int32_t nsteps, double* d_psi, const double* d_psi_ext,
+                   const double* d_meas, const double* d_sigma, double* d_coef, double* d_chi2,
+                   double* d_eps, efit_stream_t stream);
+
 /* Tail of a fit iteration for the sharded (world > 1) path, after the caller has exchanged the
  * boundary slices: interior solve of d_pcurr with edge values d_psib, then
  * psi <- psi_p + d_psi_ext (in place) and d_eps[0] = max|psi_new - psi_old| / |psi_bdry - psi_axis|,

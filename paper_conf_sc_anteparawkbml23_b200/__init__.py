@@ -19,7 +19,7 @@ import numpy as np
 __all__ = [
     "EfitError", "lib", "lib_path", "efit_workspace_bytes", "efit_green_init", "efit_info", "efit_response",
     "efit_current", "efit_boundary_flux", "efit_interior_solve", "efit_lsq", "efit_fit_step", "efit_status",
-    "efit_solve_update", "efit_profile_begin", "efit_profile_end",
+    "efit_solve_update", "efit_profile_begin", "efit_profile_end", "efit_fit_steps",
     "efit_table", "efit_shard", "efit_destroy", "efit_strerror", "efit_last_error", "efit_version",
     "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY", "efit_plan_info", "owned_targets", "exchange",
 ]
@@ -98,6 +98,7 @@ def lib() -> ctypes.CDLL:
             "efit_interior_solve": (I, [vp, vp, vp, vp, vp]),
             "efit_lsq": (I, [vp, vp, vp, vp, vp, vp, vp]),
             "efit_fit_step": (I, [vp, vp, vp, vp, vp, vp, vp, vp, vp]),
+            "efit_fit_steps": (I, [vp, ctypes.c_int32, vp, vp, vp, vp, vp, vp, vp, vp]),
             "efit_status": (I, [vp, vp]),
             "efit_solve_update": (I, [vp, vp, vp, vp, vp, vp, vp]),
             "efit_profile_begin": (I, [vp, ctypes.c_int32, ctypes.c_int32]),
@@ -262,6 +263,11 @@ def efit_profile_end(ctx):
     return dict(zip(PROFILE_FIELDS, list(out))), n.value
 
 
+def efit_fit_steps(ctx, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None) -> None:
+    _check(lib().efit_fit_steps(ctx, nsteps, _ptr(psi), _ptr(psi_ext), _ptr(meas), _ptr(sigma), _ptr(coef),
+                                _ptr(chi2), _ptr(eps), _stream(stream)), ctx)
+
+
 def efit_status(ctx, stream=None) -> int:
     return lib().efit_status(ctx, _stream(stream))
 
@@ -360,6 +366,9 @@ class EfitContext:
 
     def fit_step(self, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None):
         efit_fit_step(self.handle, psi, psi_ext, meas, sigma, coef, chi2, eps, stream)
+
+    def fit_steps(self, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None):
+        efit_fit_steps(self.handle, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream)
 
     def status(self, stream=None) -> int:
         return efit_status(self.handle, stream)

@@ -196,7 +196,7 @@ static size_t carve(Ctx& c, char* base) {
     c.axbd = (double*)take(sizeof(double) * 2);
     c.status = (int*)take(sizeof(int) * 4);
     c.tickets = (unsigned*)take(sizeof(unsigned) * 8);
-    c.norm_part = (double*)take(sizeof(double) * 2 * c.t.red_blocks);
+    c.norm_part = (double*)take(sizeof(double) * 2 * (size_t)(c.t.red_blocks > c.ni + 2 ? c.t.red_blocks : c.ni + 2));
     c.resp_part = (double*)take(sizeof(double) * (size_t)c.t.resp_nchunk * (nrows > 0 ? nrows : 1) * c.nb);
     c.resp_cnt = (double*)take(sizeof(double) * c.t.resp_nchunk);
     c.bmat = (double*)take(sizeof(double) * (size_t)c.nb * c.t.resp_nchunk * c.t.resp_gc);
@@ -445,13 +445,17 @@ void mark(Ctx& c, cudaStream_t s, int id) {
 }
 }  // namespace efit
 
+// One Picard iteration.  `normalize`: compute psi_axis/psi_bdry of psi first; otherwise they were
+// produced by the previous chained iteration's k_dst_inv.  Every iteration's k_dst_inv produces the
+// next axis/boundary (cheap: a per-block argmax over the nodes it writes + the last block).
 static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, const double* meas,
-                                    const double* sigma, double* coef, double* chi2, double* eps, cudaStream_t s) {
+                                    const double* sigma, double* coef, double* chi2, double* eps, cudaStream_t s,
+                                    bool normalize = true) {
     using namespace efit;
     cudaError_t e;
     c.prof_rec = c.prof_on && (c.prof_calls++ % c.prof_every == 0);
     mark(c, s, M_BEGIN);
-    if ((e = launch_normalize(c, psi, s))) return e;
+    if (normalize && (e = launch_normalize(c, psi, s))) return e;
     mark(c, s, M_NORM);
     if ((e = launch_response(c, psi, c.resp, s))) return e;
     mark(c, s, M_RESP);
@@ -459,19 +463,19 @@ static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, 
     if ((e = launch_current(c, psi, coef, c.pcurr, true, s))) return e;
     mark(c, s, M_CUR);
     if ((e = launch_boundary(c, c.pcurr, c.psib, s))) return e;  // marks M_TB, M_LR inside
-    if ((e = launch_solve(c, c.pcurr, c.psib, nullptr, psi, psi_ext, eps, s))) return e;
+    if ((e = launch_solve(c, c.pcurr, c.psib, nullptr, psi, psi_ext, eps, s, true))) return e;
     mark(c, s, M_SOLVE);
     if (c.prof_on && c.prof_rec && !c.prof_capture && c.prof_next < c.prof_slots) ++c.prof_next;
     c.prof_rec = false;
     return cudaSuccess;
 }
 
-extern "C" int efit_fit_step(efit_ctx* h, double* d_psi, const double* d_psi_ext, const double* d_meas,
-                             const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps,
-                             efit_stream_t stream) {
+static int fit_steps_impl(efit_ctx* h, int32_t nsteps, double* d_psi, const double* d_psi_ext, const double* d_meas,
+                          const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps, efit_stream_t stream) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
     Ctx& c = h->c;
-    if (c.world != 1) return fail(&c, EFIT_E_STATE, "efit_fit_step needs world == 1 (use the step calls)");
+    if (c.world != 1) return fail(&c, EFIT_E_STATE, "efit_fit_step(s) needs world == 1 (use the step calls)");
+    if (nsteps < 1) return fail(&c, EFIT_E_INVAL, "nsteps < 1");
     EFIT_CHECK_PTR(c, d_psi, "d_psi");
     EFIT_CHECK_PTR(c, d_psi_ext, "d_psi_ext");
     EFIT_CHECK_PTR(c, d_meas, "d_meas");
@@ -481,21 +485,28 @@ extern "C" int efit_fit_step(efit_ctx* h, double* d_psi, const double* d_psi_ext
     EFIT_CHECK_PTR(c, d_eps, "d_eps");
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e;
-    const void* key[8] = {d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, (const void*)s};
+    auto enqueue = [&]() -> cudaError_t {
+        for (int k = 0; k < nsteps; ++k) {
+            cudaError_t e1 = enqueue_fit_step(c, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, s, k == 0);
+            if (e1) return e1;
+        }
+        return cudaSuccess;
+    };
+    const void* key[9] = {d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, (const void*)s,
+                          (const void*)(intptr_t)nsteps};
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     if (s != nullptr && (e = cudaStreamIsCapturing(s, &cs))) return cuda_fail(&c, e, "capture query");
     // eager enqueue when the caller is capturing the stream itself (the kernels then become nodes
-    // of the caller's graph), when graphs are disabled, or on the legacy stream (not capturable)
+    // of the caller's graph), when profiling, when graphs are disabled, or on the legacy stream
     if (!c.use_graph || s == nullptr || c.prof_on || cs == cudaStreamCaptureStatusActive) {
-        if ((e = enqueue_fit_step(c, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, s)))
-            return cuda_fail(&c, e, "fit step");
+        if ((e = enqueue())) return cuda_fail(&c, e, "fit step");
         return EFIT_OK;
     }
     if (!c.gexec || std::memcmp(key, c.gkey, sizeof(key)) != 0) {
         if (c.gexec) { cudaGraphExecDestroy(c.gexec); c.gexec = nullptr; }
         cudaGraph_t graph = nullptr;
         if ((e = cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal))) return cuda_fail(&c, e, "begin capture");
-        cudaError_t e2 = enqueue_fit_step(c, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, s);
+        cudaError_t e2 = enqueue();
         e = cudaStreamEndCapture(s, &graph);
         if (e2) { if (graph) cudaGraphDestroy(graph); return cuda_fail(&c, e2, "fit step capture"); }
         if (e) return cuda_fail(&c, e, "end capture");
@@ -506,6 +517,18 @@ extern "C" int efit_fit_step(efit_ctx* h, double* d_psi, const double* d_psi_ext
     }
     if ((e = cudaGraphLaunch(c.gexec, s))) return cuda_fail(&c, e, "graph launch");
     return EFIT_OK;
+}
+
+extern "C" int efit_fit_step(efit_ctx* h, double* d_psi, const double* d_psi_ext, const double* d_meas,
+                             const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps,
+                             efit_stream_t stream) {
+    return fit_steps_impl(h, 1, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, stream);
+}
+
+extern "C" int efit_fit_steps(efit_ctx* h, int32_t nsteps, double* d_psi, const double* d_psi_ext,
+                              const double* d_meas, const double* d_sigma, double* d_coef, double* d_chi2,
+                              double* d_eps, efit_stream_t stream) {
+    return fit_steps_impl(h, nsteps, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, stream);
 }
 
 extern "C" int efit_solve_update(efit_ctx* h, const double* d_pcurr, const double* d_psib, const double* d_psi_ext,

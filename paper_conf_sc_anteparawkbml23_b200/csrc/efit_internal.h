@@ -111,7 +111,7 @@ struct Ctx {
 
     // CUDA graph cache for efit_fit_step
     cudaGraphExec_t gexec;
-    const void* gkey[8];
+    const void* gkey[9];
     cudaStream_t gstream;
     bool use_graph;
 
@@ -135,6 +135,7 @@ cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double
                            bool pair, cudaStream_t s);
 cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s);
 cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out,
-                         double* psi_inout, const double* psi_ext, double* eps, cudaStream_t s);
+                         double* psi_inout, const double* psi_ext, double* eps, cudaStream_t s,
+                         bool next_norm = false);
 
 }  // namespace efit

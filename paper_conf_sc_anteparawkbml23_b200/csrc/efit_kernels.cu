@@ -299,6 +299,53 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
 
 // ================================================================================ normalize
 
+// Last-block part of the normalisation (called by exactly one block after all `nparts` block
+// partials (value, index) are visible): psi_axis from the partials, psi_bdry from the limiter
+// vertices, status if there is no plasma.  Uses 256 threads.
+__device__ void normalize_finalize(const double* __restrict__ psi, int nw, int nh, double rmin, double dr,
+                                   double zmin, double dz, int sgn, const double* __restrict__ lim, int n_lim,
+                                   const double* part, int nparts, double* __restrict__ axbd, int* status) {
+    __shared__ double sv[32];
+    __shared__ long long si[32];
+    const double s = (double)sgn;
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31, nwarp = blockDim.x >> 5;
+    double best = -DBL_MAX;
+    long long bi = LLONG_MAX;
+    for (int b = threadIdx.x; b < nparts; b += blockDim.x) {
+        double v = __ldcg(part + 2 * b);
+        double ix = __ldcg(part + 2 * b + 1);
+        argmax_merge(best, bi, v, (long long)ix);
+    }
+    warp_argmax(best, bi);
+    if (l == 0) { sv[w] = best; si[w] = bi; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int q = 1; q < nwarp; ++q) argmax_merge(best, bi, sv[q], si[q]);
+        sv[0] = best; si[0] = bi;
+    }
+    __syncthreads();
+    const long long gax = si[0];
+    __syncthreads();
+    double vb = -DBL_MAX;
+    long long vi = LLONG_MAX;
+    for (int v = threadIdx.x; v < n_lim; v += blockDim.x) {
+        double pv = bilinear(psi, nw, nh, rmin, dr, zmin, dz, lim[v], lim[n_lim + v]);
+        argmax_merge(vb, vi, s * pv, (long long)v);
+    }
+    warp_argmax(vb, vi);
+    if (l == 0) { sv[w] = vb; si[w] = vi; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int q = 1; q < nwarp; ++q) argmax_merge(vb, vi, sv[q], si[q]);
+        const double pa = (gax == LLONG_MAX) ? 0.0 : __ldcg(psi + gax);
+        const double pb = (vi == LLONG_MAX) ? 0.0 : bilinear(psi, nw, nh, rmin, dr, zmin, dz, lim[vi], lim[n_lim + vi]);
+        axbd[0] = pa;
+        axbd[1] = pb;
+        if (gax == LLONG_MAX || !(s * (pa - pb) > 0.0)) atomicOr(status, EFIT_ST_NOPLASMA);
+    }
+    __syncthreads();
+}
+
 // psi_axis = s * max_{g in limiter} s psi_g (ties: lowest g);  psi_bdry = s * max over limiter
 // vertices of s * bilinear(psi) (ties: lowest vertex).  Last-block pattern: the final block
 // combines the per-block partials; `ticket` returns to 0 for the next launch.
@@ -340,42 +387,8 @@ __global__ void __launch_bounds__(256) k_normalize(const double* __restrict__ ps
     __syncthreads();
     if (!last) return;
     __threadfence();
-    best = -DBL_MAX;
-    bi = LLONG_MAX;
-    for (int b = threadIdx.x; b < (int)gridDim.x; b += blockDim.x) {
-        double v = __ldcg(part + 2 * b);
-        double ix = __ldcg(part + 2 * b + 1);
-        argmax_merge(best, bi, v, (long long)ix);
-    }
-    warp_argmax(best, bi);
-    if (l == 0) { sv[w] = best; si[w] = bi; }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        for (int q = 1; q < (int)(blockDim.x >> 5); ++q) argmax_merge(best, bi, sv[q], si[q]);
-        sv[0] = best; si[0] = bi;
-    }
-    __syncthreads();
-    long long gax = si[0];
-    __syncthreads();
-    // limiter vertices
-    double vb = -DBL_MAX;
-    long long vi = LLONG_MAX;
-    for (int v = threadIdx.x; v < n_lim; v += blockDim.x) {
-        double pv = bilinear(psi, nw, nh, rmin, dr, zmin, dz, lim[v], lim[n_lim + v]);
-        argmax_merge(vb, vi, s * pv, (long long)v);
-    }
-    warp_argmax(vb, vi);
-    if (l == 0) { sv[w] = vb; si[w] = vi; }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        for (int q = 1; q < (int)(blockDim.x >> 5); ++q) argmax_merge(vb, vi, sv[q], si[q]);
-        double pa = (gax == LLONG_MAX) ? 0.0 : psi[gax];
-        double pb = (vi == LLONG_MAX) ? 0.0 : bilinear(psi, nw, nh, rmin, dr, zmin, dz, lim[vi], lim[n_lim + vi]);
-        axbd[0] = pa;
-        axbd[1] = pb;
-        if (gax == LLONG_MAX || !(s * (pa - pb) > 0.0)) atomicOr(status, EFIT_ST_NOPLASMA);
-        *ticket = 0u;
-    }
+    normalize_finalize(psi, nw, nh, rmin, dr, zmin, dz, sgn, lim, n_lim, part, gridDim.x, axbd, status);
+    if (threadIdx.x == 0) *ticket = 0u;
 }
 
 cudaError_t launch_normalize(Ctx& c, const double* psi, cudaStream_t s) {
@@ -1157,6 +1170,16 @@ __device__ double2* fft_stockham(double2* x, double2* y, int M, int log2m, const
     return a;
 }
 
+// What k_dst_inv needs to produce the next iteration's psi_axis/psi_bdry (chained fit steps).
+struct NextNorm {
+    int on, sgn, n_lim;
+    const uint8_t* inlim;
+    const double* lim;
+    double rmin, dr, zmin, dz;
+    double* part;
+    int* status;
+};
+
 // Number of Stockham stages for M = 2^log2m (radix 4, plus one radix 2 if log2m is odd): the
 // result is in the scratch buffer when it is odd.
 __host__ __device__ __forceinline__ int fft_stages(int log2m) { return (log2m >> 1) + (log2m & 1); }
@@ -1296,8 +1319,8 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
                                                  int nw, int nh, const double2* __restrict__ W, int M, int log2m,
                                                  int FPC, double* __restrict__ psi_out, double* __restrict__ psi_inout,
                                                  const double* __restrict__ psi_ext, double* __restrict__ eps_part,
-                                                 unsigned* ticket, const double* __restrict__ axbd,
-                                                 double* __restrict__ eps) {
+                                                 unsigned* ticket, double* __restrict__ axbd,
+                                                 double* __restrict__ eps, NextNorm nn) {
     extern __shared__ __align__(16) double2 a2[];  // FPC x ([M] data, [M] scratch), then [M/2] twiddles
     double2* Ws = a2 + 2 * FPC * M;
     __shared__ double wmax[16];
@@ -1307,12 +1330,20 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
     const int TPF = blockDim.x / FPC;
     const int f = threadIdx.x / TPF, lt = threadIdx.x - f * TPF;
     double dmax = 0.0;
+    double best = -DBL_MAX;  // next iteration's axis partial (nn.on)
+    long long bi = LLONG_MAX;
+    bool bad = false;
+    const double sg = (double)nn.sgn;
     auto emit = [&](long long g, double pp) {
         if (psi_out) psi_out[g] = pp;
         if (psi_inout) {
             const double nv = pp + psi_ext[g];
             dmax = fmax(dmax, fabs(nv - psi_inout[g]));
             psi_inout[g] = nv;
+            if (nn.on) {
+                if (!isfinite(nv)) bad = true;
+                if (nn.inlim[g]) argmax_merge(best, bi, sg * nv, g);
+            }
         }
     };
     if ((int)blockIdx.x < nrb) {
@@ -1368,11 +1399,23 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
     dmax = warp_max(dmax);
     const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
     if (l == 0) wmax[w] = dmax;
+    __shared__ double av[16];
+    __shared__ long long ai[16];
+    if (nn.on) {
+        if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(nn.status, EFIT_ST_NONFINITE);
+        warp_argmax(best, bi);
+        if (l == 0) { av[w] = best; ai[w] = bi; }
+    }
     __syncthreads();
     if (threadIdx.x == 0) {
         double m = 0.0;
         for (int q = 0; q < (int)(blockDim.x >> 5); ++q) m = fmax(m, wmax[q]);
         eps_part[blockIdx.x] = m;
+        if (nn.on) {
+            for (int q = 1; q < (int)(blockDim.x >> 5); ++q) argmax_merge(best, bi, av[q], ai[q]);
+            nn.part[2 * blockIdx.x] = best;
+            nn.part[2 * blockIdx.x + 1] = (double)bi;
+        }
         __threadfence();
         last = (atomicAdd(ticket, 1u) == gridDim.x - 1);
     }
@@ -1390,6 +1433,11 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
         *eps = mm / fabs(axbd[1] - axbd[0]);
         *ticket = 0u;
     }
+    __syncthreads();
+    // the new psi's axis/boundary for the next chained iteration (replaces its k_normalize)
+    if (nn.on)
+        normalize_finalize(psi_inout, nw, nh, nn.rmin, nn.dr, nn.zmin, nn.dz, nn.sgn, nn.lim, nn.n_lim, nn.part,
+                           gridDim.x, axbd, nn.status);
 }
 
 static void solve_shape(const Ctx& c, int& fpc, int& threads, size_t& smem) {
@@ -1403,7 +1451,7 @@ static void solve_shape(const Ctx& c, int& fpc, int& threads, size_t& smem) {
 }
 
 cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out, double* psi_inout,
-                         const double* psi_ext, double* eps, cudaStream_t s) {
+                         const double* psi_ext, double* eps, cudaStream_t s, bool next_norm) {
     int fpc, threads;
     size_t smem;
     solve_shape(c, fpc, threads, smem);
@@ -1415,9 +1463,18 @@ cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double
     e = launch_pdl(k_tridiag, dim3((c.nmode + 3) / 4), dim3(128), sizeof(double) * 4 * (32 * (size_t)L + 32), s, c.fhat,
                    c.fhat_ld, c.tri_alpha, c.tri_inv, c.tri_cp, c.ni, L, c.nmode);
     if (e) return e;
+    NextNorm nn;
+    nn.on = (next_norm && psi_inout) ? 1 : 0;
+    nn.sgn = c.ip_sign;
+    nn.n_lim = c.n_lim;
+    nn.inlim = c.inlim;
+    nn.lim = c.lim;
+    nn.rmin = c.rmin; nn.dr = c.dr; nn.zmin = c.zmin; nn.dz = c.dz;
+    nn.part = c.norm_part;
+    nn.status = c.status;
     return launch_pdl(k_dst_inv, dim3(nrb + 1), dim3(threads), smem, s, c.fhat, c.fhat_ld, psib, c.nw, c.nh,
                       c.twiddle, c.fft_m, c.fft_log2, fpc, psi_out, psi_inout, psi_ext, c.eps_part, c.tickets + 1,
-                      c.axbd, eps);
+                      c.axbd, eps, nn);
 }
 
 // ================================================================================ left/right via FFT

@@ -402,3 +402,26 @@ def test_c4_solve_and_current(torch_mod, c4):
     ref = c4.orc.interior_solve(Iref, psib)
     out = c4.ctx.interior_solve(T(torch, Iref), T(torch, psib)).cpu().numpy()
     assert rel(out, ref) < TOL
+
+
+def test_fit_steps_chained_equals_repeated(torch_mod, efit, orc_mod):
+    """efit_fit_steps(n) (axis/boundary of iterations 2..n taken from the previous update kernel)
+    is bitwise identical to n separate efit_fit_step calls (each normalising from scratch)."""
+    torch = torch_mod
+    c = case("C2", efit, orc_mod)
+    psi_s, ct, tw = _twin(c, noise_seed=1)
+    ext, y, s = T(torch, tw["psi_ext"]), T(torch, tw["y"]), T(torch, tw["sigma"])
+    psi0 = synth.perturbed_psi(c.cfg.grid, seed=5, rel=1e-3)
+    outs = []
+    for chained in (False, True):
+        psi = T(torch, psi0)
+        coef, chi2, eps = c.ctx._t(c.ctx.nbasis), c.ctx._t(1), c.ctx._t(1)
+        if chained:
+            c.ctx.fit_steps(5, psi, ext, y, s, coef, chi2, eps)
+        else:
+            for _ in range(5):
+                c.ctx.fit_step(psi, ext, y, s, coef, chi2, eps)
+        assert c.ctx.status() == 0
+        outs.append((psi.clone(), coef.clone(), eps.clone()))
+    for a, b in zip(*outs):
+        assert torch.equal(a, b)
