@@ -128,7 +128,7 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     const long long n = (long long)c.nw * c.nh;
     c.S = round_up(n, 64);
     efit::Tiling& t = c.t;
-    t.resp_gc = c.nb <= 8 ? 1024 : (c.nb <= 16 ? 512 : 256);
+    t.resp_gc = c.nb <= 8 ? 1152 : (c.nb <= 16 ? 768 : 512);  // multiples of NP x 128-node positions
     t.resp_nchunk = (int)((n + t.resp_gc - 1) / t.resp_gc);
     t.tb_ch = 2048;
     t.tb_nchunk = (int)((n + t.tb_ch - 1) / t.tb_ch);
@@ -160,10 +160,11 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     // a CTA covers 8*MB rows (one MB-row block per warp); pick MB (<= 5, MB*NB <= 40 registers'
     // worth of accumulators) minimising padded rows, then preferring more rows per warp
     int best_mb = 1, best_cost = 1 << 30;
-    for (int mb = 1; mb <= 4; ++mb) {
-        if (16 * mb + 2 * mb * c.nb > 90 && mb > 1) continue;  // loads + accumulators under 128 regs
-        int groups = (nrows + 8 * mb - 1) / (8 * mb);
-        int cost = groups * 8 * mb + 4 * groups;  // padded rows + per-CTA basis work
+    for (int mb = 4; mb >= 1; --mb) {  // ties -> more rows per warp (more reuse of each basis value)
+        const int np = efit::resp_np(c.nb, mb);                // 256-bit positions per step (k_response)
+        if (8 * np * mb + 2 * mb * c.nb > 112 && mb > 1) continue;  // loads + accumulators under 128 regs
+        const int nmb = (nrows + mb - 1) / mb;        // row blocks, dealt round-robin to 8 warps
+        int cost = ((nmb + 7) / 8) * mb;               // rows on the busiest warp
         if (cost < best_cost) { best_cost = cost; best_mb = mb; }
     }
     t.resp_mb = best_mb;

@@ -12,9 +12,11 @@ constexpr double kMu0 = 4.0e-7 * kPi;     // mu0 = 4 pi 1e-7 (reading 
 constexpr double kMu0Over2Pi = 2.0e-7;    // mu0 / (2 pi)
 constexpr int kAgmIters = 10;             // enough for m1 >= 1e-15 (quadratic convergence)
 
-// PDL: wait for the programmatic predecessor (no-op for a normal launch), then let dependents launch.
+// PDL: wait for the programmatic predecessor (no-op for a normal launch).  Dependents are not
+// triggered early (implicit trigger at completion): early-launched dependent CTAs would hold SM
+// slots while this kernel still has waves to run (measured slower on the C4 step).
 __device__ __forceinline__ void griddep() {
-    asm volatile("griddepcontrol.wait;\n\tgriddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
 // Grid coordinates without FMA contraction (R_i = rmin + i*dR rounded twice), so that
@@ -24,12 +26,16 @@ __device__ __forceinline__ double grid_coord(double lo, int i, double d) {
 }
 
 // Complete elliptic integrals by the arithmetic-geometric mean (Gauss; A&S 17.6):
-//   a0 = 1, b0 = sqrt(m1), c0^2 = m;  a' = (a+b)/2, b' = sqrt(ab), c' = c^2/(4a')
+//   a0 = 1, b0 = sqrt(m1), c0^2 = m;  a' = (a+b)/2, b' = sqrt(ab), c' = (a-b)/2
 //   K = pi/(2 a_inf),  E = K (1 - sum_{n>=0} 2^(n-1) c_n^2).
 // Returns K and S1 = sum_{n>=1} 2^(n-1) c_n^2, so that
 //   (1 - m/2) K - E = K * S1        (no cancellation; all terms positive)
 //   E = K (1 - m/2 - S1).
-// c1 = (1 - sqrt(m1))/2 is formed as m / (2 (1 + sqrt(m1))) (cancellation-free).
+// c1 = (1 - sqrt(m1))/2 is formed as m / (2 (1 + sqrt(m1))) (cancellation-free: it carries the
+// far-field O(m) information); later c_n = (a_{n-1} - b_{n-1})/2, whose absolute rounding error
+// (~ulp(a)) moves S1 by < 1e-16 relative because c_n^2 <= c_1^4/16.  The loop stops once the
+// increment 2^(n-1) c_n^2 no longer changes S1 (quadratic convergence: <= 6 iterations for
+// m1 >= 1e-9, the cap covers m1 >= 1e-15).
 __device__ __forceinline__ void agm_ks1(double m, double m1, double& K, double& S1) {
     double b = sqrt(m1);
     double c = m / (2.0 * (1.0 + b));  // c1
@@ -37,15 +43,17 @@ __device__ __forceinline__ void agm_ks1(double m, double m1, double& K, double& 
     b = sqrt(b);                       // b1 = sqrt(a0 b0) = sqrt(sqrt(m1))
     double s = c * c;                  // 2^0 c1^2
     double p = 1.0;
-#pragma unroll
+#pragma unroll 1
     for (int n = 1; n < kAgmIters; ++n) {
-        double an = 0.5 * (a + b);
-        double bn = sqrt(a * b);
-        c = c * c / (4.0 * an);
-        p *= 2.0;
-        s += p * c * c;
+        c = 0.5 * (a - b);             // c_{n+1}
+        const double an = 0.5 * (a + b);
+        b = sqrt(a * b);
         a = an;
-        b = bn;
+        p *= 2.0;
+        const double t = p * c * c;
+        const double s2 = s + t;
+        if (s2 == s) break;            // converged (also covers c == 0)
+        s = s2;
     }
     K = kPi / (2.0 * a);
     S1 = s;

@@ -11,7 +11,13 @@ namespace efit {
 constexpr int kMaxBasis = 24;
 constexpr int kMaxKnots = 20;
 constexpr int kMaxN = 2049;  // FFT working set 2.5*M*16 B of shared memory, M = 2(nh-1)
-constexpr int kLsqMaxRowsHost = 1024;
+constexpr int kLsqMaxRowsHost = 960;  // k_lsq shared memory: (nb|1 + 2)*nd doubles
+
+// k_response: 256-bit positions per step for NB basis functions and MB rows per warp, keeping
+// loads (8*NP*MB regs) + accumulators (2*MB*NB regs) <= 112 of the 128-register budget.
+__host__ __device__ constexpr int resp_np(int nb, int mb) {
+    return (112 - 2 * mb * nb) / (8 * mb) >= 3 ? 3 : ((112 - 2 * mb * nb) / (8 * mb) >= 1 ? (112 - 2 * mb * nb) / (8 * mb) : 1);
+}
 
 // device status-word bits
 #define EFIT_ST_NOPLASMA 1

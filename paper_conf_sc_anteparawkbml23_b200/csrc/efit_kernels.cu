@@ -15,6 +15,7 @@
 #include <cfloat>
 #include <climits>
 #include <cstdio>
+#include <cstdlib>
 #include <utility>
 
 #include "efit_device.cuh"
@@ -28,12 +29,14 @@ static int g_smem_optin = 227 * 1024;  // device opt-in shared memory per block 
 // serialisation, so its CTAs are scheduled while the predecessor's last wave drains; the kernel
 // itself waits (griddepcontrol.wait) until the predecessor has completed and flushed before it
 // touches any of its outputs, then immediately allows its own dependents to launch.
+static const bool g_no_pdl = getenv("EFIT_NO_PDL") != nullptr;  // A/B switch for profiling
+
 template <typename... KArgs, typename... Args>
 static cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
                               Args&&... args) {
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    attr[0].val.programmaticStreamSerializationAllowed = g_no_pdl ? 0 : 1;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = grid;
     cfg.blockDim = block;
@@ -464,63 +467,64 @@ __device__ __forceinline__ int bperm(int q) {  // node q of a chunk -> permuted 
     return (blk << 7) + (h << 6) + (lane << 1) + w;
 }
 
-template <int NB, int MB>
+template <int NB, int MB, int NP>
 __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ Gd, long long S, int nrows, int n,
                                                      const double* __restrict__ Bm, long long ldb, int gc,
                                                      double* __restrict__ part) {
-    griddep();
     extern __shared__ __align__(16) double Bs[];  // [NB][gc] permuted
+    griddep();
     const int c = blockIdx.x;
     const int g0 = c * gc;
-    for (int e = 2 * threadIdx.x; e < NB * gc; e += 2 * blockDim.x) {
-        const int k = e / gc, q = e - (e / gc) * gc;
-        const double2 v = __ldg(reinterpret_cast<const double2*>(Bm + k * ldb + g0 + q));
-        *reinterpret_cast<double2*>(Bs + k * gc + bperm(q)) = v;
-    }
+#pragma unroll
+    for (int k = 0; k < NB; ++k)
+        for (int q = 2 * threadIdx.x; q < gc; q += 2 * blockDim.x) {
+            const double2 v = __ldg(reinterpret_cast<const double2*>(Bm + k * ldb + g0 + q));
+            *reinterpret_cast<double2*>(Bs + k * gc + bperm(q)) = v;
+        }
     __syncthreads();
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int row0 = (blockIdx.y * 8 + warp) * MB;
-    if (row0 >= nrows) return;
     const int qend = min(gc, n - g0);  // valid nodes; a 4-wide load may read up to 3 zero pads
-    double acc[MB][NB];
+    const int nmb = (nrows + MB - 1) / MB;
+    for (int mb = warp; mb < nmb; mb += (int)(blockDim.x >> 5)) {  // every row block of the chunk
+        const int row0 = mb * MB;
+        double acc[MB][NB];
 #pragma unroll
-    for (int r = 0; r < MB; ++r)
+        for (int r = 0; r < MB; ++r)
 #pragma unroll
-        for (int k = 0; k < NB; ++k) acc[r][k] = 0.0;
-    const double* rowp[MB];
+            for (int k = 0; k < NB; ++k) acc[r][k] = 0.0;
+        const double* rowp[MB];
 #pragma unroll
-    for (int r = 0; r < MB; ++r) rowp[r] = Gd + (long long)min(row0 + r, nrows - 1) * S + g0;
-    for (int q0 = 0; q0 < qend; q0 += 256) {
-        const int qa = q0 + 4 * lane, qb = qa + 128;
-        const bool va = qa < qend, vb = qb < qend;
-        d4 ga[MB], gb[MB];
+        for (int r = 0; r < MB; ++r) rowp[r] = Gd + (long long)min(row0 + r, nrows - 1) * S + g0;
+        for (int q0 = 0; q0 < qend; q0 += 128 * NP) {
+            d4 gv[NP][MB];
 #pragma unroll
-        for (int r = 0; r < MB; ++r) {
-            ga[r] = va ? ld256_stream(rowp[r] + qa) : d4{0.0, 0.0, 0.0, 0.0};
-            gb[r] = vb ? ld256_stream(rowp[r] + qb) : d4{0.0, 0.0, 0.0, 0.0};
-        }
+            for (int p = 0; p < NP; ++p) {
+                const int q = q0 + 128 * p + 4 * lane;
+                const bool ok = q < qend;
 #pragma unroll
-        for (int k = 0; k < NB; ++k) {
-            const double* bk = Bs + k * gc + q0 + 2 * lane;
-            const double2 a0 = *reinterpret_cast<const double2*>(bk);
-            const double2 a1 = *reinterpret_cast<const double2*>(bk + 64);
-            const double2 b0 = *reinterpret_cast<const double2*>(bk + 128);
-            const double2 b1 = *reinterpret_cast<const double2*>(bk + 192);
-            const d4 ba{a0.x, a0.y, a1.x, a1.y}, bb{b0.x, b0.y, b1.x, b1.y};
+                for (int r = 0; r < MB; ++r) gv[p][r] = ok ? ld256_stream(rowp[r] + q) : d4{0.0, 0.0, 0.0, 0.0};
+            }
 #pragma unroll
-            for (int r = 0; r < MB; ++r) {
-                acc[r][k] = dot4(ga[r], ba, acc[r][k]);
-                acc[r][k] = dot4(gb[r], bb, acc[r][k]);
+            for (int k = 0; k < NB; ++k) {
+#pragma unroll
+                for (int p = 0; p < NP; ++p) {
+                    const double* bk = Bs + k * gc + q0 + 128 * p + 2 * lane;
+                    const double2 b0 = *reinterpret_cast<const double2*>(bk);
+                    const double2 b1 = *reinterpret_cast<const double2*>(bk + 64);
+                    const d4 bb{b0.x, b0.y, b1.x, b1.y};
+#pragma unroll
+                    for (int r = 0; r < MB; ++r) acc[r][k] = dot4(gv[p][r], bb, acc[r][k]);
+                }
             }
         }
-    }
 #pragma unroll
-    for (int r = 0; r < MB; ++r) {
-        const int row = row0 + r;
+        for (int r = 0; r < MB; ++r) {
+            const int row = row0 + r;
 #pragma unroll
-        for (int k = 0; k < NB; ++k) {
-            double v = warp_sum(acc[r][k]);
-            if (lane == 0 && row < nrows) part[((long long)row * NB + k) * gridDim.x + c] = v;
+            for (int k = 0; k < NB; ++k) {
+                double v = warp_sum(acc[r][k]);
+                if (lane == 0 && row < nrows) part[((long long)row * NB + k) * gridDim.x + c] = v;
+            }
         }
     }
 }
@@ -549,6 +553,7 @@ __global__ void k_resp_reduce(const double* __restrict__ part, const double* __r
 
 template <int NB>
 static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t s, int nrows, bool prepare) {
+    static_assert(resp_np(NB, 1) >= 1, "positions per step");
     const int gc = c.t.resp_gc;
     const size_t smem = sizeof(double) * NB * gc;
     const long long ldb = (long long)c.t.resp_nchunk * gc;
@@ -560,9 +565,9 @@ static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t
     int mb = c.t.resp_mb;
 #define EFIT_RESP_LAUNCH(MBV)                                                                              \
     do {                                                                                                   \
-        auto kern = k_response<NB, MBV>;                                                                   \
+        auto kern = k_response<NB, MBV, resp_np(NB, MBV)>;                                                \
         if (prepare) { raise_smem_limit((const void*)kern, smem); break; }                               \
-        dim3 grid(c.t.resp_nchunk, (nrows + 8 * MBV - 1) / (8 * MBV));                                    \
+        dim3 grid(c.t.resp_nchunk);                                                                        \
         launch_pdl(kern, dim3(grid), dim3(256), smem, s, c.Gd, c.S, nrows, c.nw * c.nh, c.bmat, ldb, gc, part);               \
     } while (0)
     if (mb >= 4) EFIT_RESP_LAUNCH(4);
@@ -598,89 +603,155 @@ cudaError_t launch_response(Ctx& c, const double* psi, double* resp_rows, cudaSt
 
 // ================================================================================ least squares
 
-// One CTA of 4 warps: rows scaled by 1/sigma, columns to unit 2-norm, Householder QR (reflectors
-// v = x - alpha e_k, alpha = -sign(x_k)|x|, H = I - v v^T/(|x|(|x| + |x_k|))), back substitution,
-// unscale; chi2 = sum((meas - A c)/sigma)^2.  Per reflection: warp 0 forms alpha and v, then the
-// remaining columns (and b) are updated by different warps in parallel -- two barriers per
-// reflection.  Lane-strided sums + fixed butterflies => deterministic.
-__global__ void __launch_bounds__(128) k_lsq(const double* __restrict__ resp, const double* __restrict__ meas,
+// Weighted least squares by CholeskyQR2 (Yamamoto, Nakatsukasa, Yanagisawa & Fukaya,
+// ETNA 2015): rows scaled by 1/sigma, columns to unit 2-norm (A), then
+//   G1 = A^T A = R1^T R1,  Q1 = A R1^-1,  G2 = Q1^T Q1 = R2^T R2  (so A = (Q1 R2^-1)(R2 R1)),
+//   c_hat = R1^-1 R2^-1 R2^-T (Q1^T b),  c = c_hat / column scale,
+// chi2 = sum((meas - resp c)/sigma)^2 from the unscaled system.  Backward stable for
+// cond(A) << eps^-1/2 ~ 1e8 (the synthetic bases: 3.6e3 .. 1.4e7).  Unlike Householder's chain of
+// nb reflections, both Gram matrices are formed with all entries in parallel and the Q1 rows are
+// independent; only the two nb x nb Cholesky factorisations and the triangular solves are serial
+// (one warp).  Fixed summation orders => deterministic.  Singular if a Cholesky pivot is not
+// positive or |R_kk| < 1e-13 max |R_jj|.
+__device__ __forceinline__ void lsq_gram(const double* __restrict__ A, int ld, int nd, int nb, double* G) {
+    // G[i*nb + j] for i <= j, one thread per entry, rows in order
+    const int ne = nb * (nb + 1) / 2;
+    for (int e = threadIdx.x; e < ne; e += blockDim.x) {
+        int i = 0, rem = e;
+        while (rem >= nb - i) { rem -= nb - i; ++i; }
+        const int j = i + rem;
+        double s = 0.0;
+        for (int m = 0; m < nd; ++m) s = fma(A[m * ld + i], A[m * ld + j], s);
+        G[i * nb + j] = s;
+        G[j * nb + i] = s;
+    }
+}
+
+// Upper Cholesky factor R (row-major, R[k*nb + j], j >= k) of G (overwritten), one warp.
+// Returns false on a non-positive pivot.  Also stores 1/R_kk in rinv[k].
+__device__ __forceinline__ bool lsq_chol(double* G, double* R, double* rinv, int nb) {
+    const int lane = threadIdx.x & 31;
+    for (int k = 0; k < nb; ++k) {
+        const double d = G[k * nb + k];
+        if (!(d > 0.0)) return false;
+        const double r = sqrt(d), ir = 1.0 / r;
+        for (int j = k + lane; j < nb; j += 32) R[k * nb + j] = (j == k) ? r : G[k * nb + j] * ir;
+        if (lane == 0) rinv[k] = ir;
+        __syncwarp();
+        const int w = nb - k - 1;
+        for (int e = lane; e < w * w; e += 32) {
+            const int i = k + 1 + e / w, j = k + 1 + e % w;
+            if (j >= i) {
+                const double v = G[i * nb + j] - R[k * nb + i] * R[k * nb + j];
+                G[i * nb + j] = v;
+                G[j * nb + i] = v;
+            }
+        }
+        __syncwarp();
+    }
+    return true;
+}
+
+// row m of A (in place): a <- a R^-1  (forward substitution with the upper factor)
+__device__ __forceinline__ void lsq_rsolve_rows(double* A, int ld, int nd, int nb, const double* R, const double* rinv) {
+    for (int m = threadIdx.x; m < nd; m += blockDim.x) {
+        double* a = A + m * ld;
+        for (int j = 0; j < nb; ++j) {
+            double s = a[j];
+            for (int i = 0; i < j; ++i) s = fma(-a[i], R[i * nb + j], s);
+            a[j] = s * rinv[j];
+        }
+    }
+}
+
+__global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, const double* __restrict__ meas,
                                              const double* __restrict__ sigma, int nd, int nb,
                                              double* __restrict__ coef, double* __restrict__ chi2, int* status) {
-    griddep();
     extern __shared__ __align__(16) double sm[];
-    double* A = sm;                   // [nb+1][nd] column-major (scaled); column nb = b
-    double* isg = A + (size_t)(nb + 1) * nd;  // [nd] 1/sigma
-    double* sc = isg + nd;            // [32] column scales
-    double* x = sc + 32;              // [32] solution
-    double* red = x + 32;             // [8]
-    __shared__ double s_alpha, s_vtv2;
+    const int ld = nb | 1;                         // odd row stride: conflict-free column walks
+    double* A = sm;                                // [nd][ld] scaled rows
+    double* b = A + (size_t)nd * ld;               // [nd]
+    double* isg = b + nd;                          // [nd] 1/sigma
+    double* G = isg + nd;                          // [nb][nb]
+    double* R1 = G + nb * nb;                      // [nb][nb]
+    double* R2 = R1 + nb * nb;                     // [nb][nb]
+    double* r1i = R2 + nb * nb;                    // [32]
+    double* r2i = r1i + 32;                        // [32]
+    double* sc = r2i + 32;                         // [32] column scales
+    double* z = sc + 32;                           // [32]
+    double* red = z + 32;                          // [16] chi2 partials
+    __shared__ int s_sing;
+    griddep();
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarp = blockDim.x >> 5;
+    if (tid == 0) s_sing = 0;
     for (int m = tid; m < nd; m += blockDim.x) {
         const double is = 1.0 / sigma[m];
         isg[m] = is;
-        for (int k = 0; k < nb; ++k) A[(size_t)k * nd + m] = resp[(size_t)m * nb + k] * is;
-        A[(size_t)nb * nd + m] = meas[m] * is;
+        for (int k = 0; k < nb; ++k) A[m * ld + k] = resp[(size_t)m * nb + k] * is;
+        b[m] = meas[m] * is;
     }
     __syncthreads();
-    for (int k = warp; k < nb; k += nwarp) {
-        double* col = A + (size_t)k * nd;
+    for (int k = warp; k < nb; k += nwarp) {  // column 2-norms
         double s = 0.0;
-        for (int m = lane; m < nd; m += 32) s = fma(col[m], col[m], s);
+        for (int m = lane; m < nd; m += 32) s = fma(A[m * ld + k], A[m * ld + k], s);
         s = sqrt(warp_sum(s));
-        const double is = s > 0.0 ? 1.0 / s : 0.0;
-        for (int m = lane; m < nd; m += 32) col[m] *= is;
         if (lane == 0) sc[k] = s;
     }
     __syncthreads();
-    for (int k = 0; k < nb; ++k) {
-        double* ck = A + (size_t)k * nd;
-        if (warp == 0) {
-            double s = 0.0;
-            for (int m = k + lane; m < nd; m += 32) s = fma(ck[m], ck[m], s);
-            const double nx = sqrt(warp_sum(s));
-            if (lane == 0) {
-                const double x0 = ck[k];
-                const double alpha = x0 >= 0.0 ? -nx : nx;
-                s_alpha = alpha;
-                s_vtv2 = nx * (nx + fabs(x0));
-                ck[k] = x0 - alpha;  // ck[k..nd) now holds v
-            }
-        }
-        __syncthreads();
-        const double vtv2 = s_vtv2;
-        for (int j = k + 1 + warp; j <= nb; j += nwarp) {
-            double* cj = A + (size_t)j * nd;
-            double d = 0.0;
-            for (int m = k + lane; m < nd; m += 32) d = fma(ck[m], cj[m], d);
-            d = warp_sum(d);
-            const double f = vtv2 > 0.0 ? d / vtv2 : 0.0;
-            for (int m = k + lane; m < nd; m += 32) cj[m] = fma(-f, ck[m], cj[m]);
-        }
-        __syncthreads();
-        if (tid == 0) ck[k] = s_alpha;  // R_kk (rows below k of column k are no longer read)
+    for (int e = tid; e < nd * nb; e += blockDim.x) {
+        const int m = e / nb, k = e - (e / nb) * nb;
+        const double s = sc[k];
+        A[m * ld + k] = s > 0.0 ? A[m * ld + k] / s : 0.0;
     }
     __syncthreads();
-    if (tid == 0) {
-        double rmax = 0.0;
-        for (int k = 0; k < nb; ++k) rmax = fmax(rmax, fabs(A[(size_t)k * nd + k]));
-        bool sing = false;
-        for (int k = 0; k < nb; ++k)
-            if (!(fabs(A[(size_t)k * nd + k]) >= 1e-13 * rmax) || !(sc[k] > 0.0)) sing = true;
-        const double* bq = A + (size_t)nb * nd;
-        for (int k = nb - 1; k >= 0; --k) {
-            double s = bq[k];
-            for (int j = k + 1; j < nb; ++j) s -= A[(size_t)j * nd + k] * x[j];
-            x[k] = s / A[(size_t)k * nd + k];
+    // pass 1: G1 = A^T A, R1, Q1 = A R1^-1
+    lsq_gram(A, ld, nd, nb, G);
+    __syncthreads();
+    if (warp == 0 && !lsq_chol(G, R1, r1i, nb) && lane == 0) s_sing = 1;
+    __syncthreads();
+    if (!s_sing) lsq_rsolve_rows(A, ld, nd, nb, R1, r1i);
+    __syncthreads();
+    // pass 2: G2 = Q1^T Q1, R2, z = Q1^T b
+    if (!s_sing) lsq_gram(A, ld, nd, nb, G);
+    for (int k = warp; k < nb; k += nwarp) {
+        double s = 0.0;
+        for (int m = lane; m < nd; m += 32) s = fma(A[m * ld + k], b[m], s);
+        s = warp_sum(s);
+        if (lane == 0) z[k] = s;
+    }
+    __syncthreads();
+    if (warp == 0 && !s_sing && !lsq_chol(G, R2, r2i, nb) && lane == 0) s_sing = 1;
+    __syncthreads();
+    if (tid == 0 && !s_sing) {
+        // z <- R2^-T z (forward), z <- R2^-1 z (back), z <- R1^-1 z (back), c = z / scale
+        for (int j = 0; j < nb; ++j) {
+            double s = z[j];
+            for (int i = 0; i < j; ++i) s = fma(-R2[i * nb + j], z[i], s);
+            z[j] = s * r2i[j];
         }
-        for (int k = 0; k < nb; ++k) x[k] = x[k] / sc[k];
-        if (sing) atomicOr(status, EFIT_ST_SINGULAR);
-        red[7] = sing ? 1.0 : 0.0;
+        const double* Rs[2] = {R2, R1};
+        const double* Ri[2] = {r2i, r1i};
+        for (int t = 0; t < 2; ++t)
+            for (int k = nb - 1; k >= 0; --k) {
+                double s = z[k];
+                for (int j = k + 1; j < nb; ++j) s = fma(-Rs[t][k * nb + j], z[j], s);
+                z[k] = s * Ri[t][k];
+            }
+        double rmax = 0.0, rmin = DBL_MAX;
+        for (int k = 0; k < nb; ++k) {
+            const double d = fabs(R1[k * nb + k] * R2[k * nb + k]);
+            rmax = fmax(rmax, d);
+            rmin = fmin(rmin, d);
+            if (!(sc[k] > 0.0)) s_sing = 1;
+        }
+        if (!(rmin >= 1e-13 * rmax)) s_sing = 1;
+        for (int k = 0; k < nb; ++k) z[k] = z[k] / sc[k];
     }
     __syncthreads();
     double s = 0.0;
     for (int m = tid; m < nd; m += blockDim.x) {
         double r = meas[m];
-        for (int k = 0; k < nb; ++k) r = fma(-resp[(size_t)m * nb + k], x[k], r);
+        for (int k = 0; k < nb; ++k) r = fma(-resp[(size_t)m * nb + k], z[k], r);
         r *= isg[m];
         s = fma(r, r, s);
     }
@@ -690,21 +761,209 @@ __global__ void __launch_bounds__(128) k_lsq(const double* __restrict__ resp, co
     if (tid == 0) {
         double t = 0.0;
         for (int q = 0; q < nwarp; ++q) t += red[q];
-        const bool bad = (*status & (EFIT_ST_NOPLASMA | EFIT_ST_NONFINITE)) != 0 || red[7] != 0.0;
+        if (s_sing) atomicOr(status, EFIT_ST_SINGULAR);
+        const bool bad = (*status & (EFIT_ST_NOPLASMA | EFIT_ST_NONFINITE)) != 0 || s_sing;
         const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
         *chi2 = bad ? nanv : t;
-        for (int k = 0; k < nb; ++k) coef[k] = bad ? nanv : x[k];
+        for (int k = 0; k < nb; ++k) coef[k] = bad ? nanv : z[k];
     }
 }
 
+// Single-warp CholeskyQR2 for small bases (NB <= 8, nd <= 32*RPL): each lane keeps its RPL rows
+// in registers, the NB(NB+1)/2 Gram entries are independent warp butterflies (interleaved), and the
+// tiny Cholesky factorisations and triangular solves run redundantly in every lane (registers, no
+// barriers).  Same arithmetic definition as k_lsq.
+template <int NB>
+__device__ __forceinline__ void lsq_chol_reg(const double (&G)[NB][NB], double (&R)[NB][NB], double (&ri)[NB],
+                                             bool& ok) {
+#pragma unroll
+    for (int i = 0; i < NB; ++i)
+#pragma unroll
+        for (int j = 0; j < NB; ++j) R[i][j] = (j >= i) ? G[i][j] : 0.0;
+#pragma unroll
+    for (int k = 0; k < NB; ++k) {
+        const double d = R[k][k];
+        ok = ok && (d > 0.0);
+        const double r = sqrt(d), ir = 1.0 / r;
+        ri[k] = ir;
+        R[k][k] = r;
+#pragma unroll
+        for (int j = k + 1; j < NB; ++j) R[k][j] *= ir;
+#pragma unroll
+        for (int i = k + 1; i < NB; ++i)
+#pragma unroll
+            for (int j = i; j < NB; ++j) R[i][j] = fma(-R[k][i], R[k][j], R[i][j]);
+    }
+}
+
+template <int NB, int RPL>
+__device__ __forceinline__ void lsq_gram_reg(const double (&a)[RPL][NB], double (&G)[NB][NB]) {
+#pragma unroll
+    for (int i = 0; i < NB; ++i)
+#pragma unroll
+        for (int j = i; j < NB; ++j) {
+            double s = 0.0;
+#pragma unroll
+            for (int r = 0; r < RPL; ++r) s = fma(a[r][i], a[r][j], s);
+            G[i][j] = s;
+        }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+        for (int i = 0; i < NB; ++i)
+#pragma unroll
+            for (int j = i; j < NB; ++j) G[i][j] += __shfl_xor_sync(0xffffffffu, G[i][j], o);
+#pragma unroll
+    for (int i = 0; i < NB; ++i)
+#pragma unroll
+        for (int j = 0; j < i; ++j) G[i][j] = G[j][i];
+}
+
+template <int NB, int RPL>
+__global__ void __launch_bounds__(32) k_lsq_warp(const double* __restrict__ resp, const double* __restrict__ meas,
+                                                 const double* __restrict__ sigma, int nd,
+                                                 double* __restrict__ coef, double* __restrict__ chi2, int* status) {
+    griddep();
+    const int lane = threadIdx.x;
+    double a[RPL][NB], bb[RPL], is[RPL];
+#pragma unroll
+    for (int r = 0; r < RPL; ++r) {
+        const int m = lane + 32 * r;
+        const bool ok = m < nd;
+        is[r] = ok ? 1.0 / sigma[m] : 0.0;
+#pragma unroll
+        for (int k = 0; k < NB; ++k) a[r][k] = ok ? resp[(size_t)m * NB + k] * is[r] : 0.0;
+        bb[r] = ok ? meas[m] * is[r] : 0.0;
+    }
+    double sc[NB];
+#pragma unroll
+    for (int k = 0; k < NB; ++k) {
+        double s = 0.0;
+#pragma unroll
+        for (int r = 0; r < RPL; ++r) s = fma(a[r][k], a[r][k], s);
+        sc[k] = s;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+        for (int k = 0; k < NB; ++k) sc[k] += __shfl_xor_sync(0xffffffffu, sc[k], o);
+    bool ok = true;
+#pragma unroll
+    for (int k = 0; k < NB; ++k) {
+        sc[k] = sqrt(sc[k]);
+        ok = ok && (sc[k] > 0.0);
+        const double isc = sc[k] > 0.0 ? 1.0 / sc[k] : 0.0;
+#pragma unroll
+        for (int r = 0; r < RPL; ++r) a[r][k] *= isc;
+    }
+    double G[NB][NB], R1[NB][NB], R2[NB][NB], r1i[NB], r2i[NB];
+    lsq_gram_reg<NB, RPL>(a, G);
+    lsq_chol_reg<NB>(G, R1, r1i, ok);
+#pragma unroll
+    for (int r = 0; r < RPL; ++r)  // rows <- rows R1^-1
+#pragma unroll
+        for (int j = 0; j < NB; ++j) {
+            double s = a[r][j];
+#pragma unroll
+            for (int i = 0; i < j; ++i) s = fma(-a[r][i], R1[i][j], s);
+            a[r][j] = s * r1i[j];
+        }
+    lsq_gram_reg<NB, RPL>(a, G);
+    lsq_chol_reg<NB>(G, R2, r2i, ok);
+    double z[NB];
+#pragma unroll
+    for (int k = 0; k < NB; ++k) {
+        double s = 0.0;
+#pragma unroll
+        for (int r = 0; r < RPL; ++r) s = fma(a[r][k], bb[r], s);
+        z[k] = s;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+        for (int k = 0; k < NB; ++k) z[k] += __shfl_xor_sync(0xffffffffu, z[k], o);
+#pragma unroll
+    for (int j = 0; j < NB; ++j) {  // R2^-T
+        double s = z[j];
+#pragma unroll
+        for (int i = 0; i < j; ++i) s = fma(-R2[i][j], z[i], s);
+        z[j] = s * r2i[j];
+    }
+#pragma unroll
+    for (int k = NB - 1; k >= 0; --k) {  // R2^-1
+        double s = z[k];
+#pragma unroll
+        for (int j = k + 1; j < NB; ++j) s = fma(-R2[k][j], z[j], s);
+        z[k] = s * r2i[k];
+    }
+#pragma unroll
+    for (int k = NB - 1; k >= 0; --k) {  // R1^-1
+        double s = z[k];
+#pragma unroll
+        for (int j = k + 1; j < NB; ++j) s = fma(-R1[k][j], z[j], s);
+        z[k] = s * r1i[k];
+    }
+    double rmax = 0.0, rmin = DBL_MAX;
+#pragma unroll
+    for (int k = 0; k < NB; ++k) {
+        const double d = fabs(R1[k][k] * R2[k][k]);
+        rmax = fmax(rmax, d);
+        rmin = fmin(rmin, d);
+        z[k] = z[k] / sc[k];
+    }
+    ok = ok && (rmin >= 1e-13 * rmax);
+    double cs = 0.0;
+#pragma unroll
+    for (int r = 0; r < RPL; ++r) {
+        const int m = lane + 32 * r;
+        if (m < nd) {
+            double res = meas[m];
+#pragma unroll
+            for (int k = 0; k < NB; ++k) res = fma(-resp[(size_t)m * NB + k], z[k], res);
+            res *= is[r];
+            cs = fma(res, res, cs);
+        }
+    }
+    cs = warp_sum(cs);
+    if (lane == 0) {
+        if (!ok) atomicOr(status, EFIT_ST_SINGULAR);
+        const bool bad = (*status & (EFIT_ST_NOPLASMA | EFIT_ST_NONFINITE)) != 0 || !ok;
+        const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
+        *chi2 = bad ? nanv : cs;
+#pragma unroll
+        for (int k = 0; k < NB; ++k) coef[k] = bad ? nanv : z[k];
+    }
+}
+
+template <int NB>
+static bool launch_lsq_warp(int nd, const double* resp, const double* meas, const double* sigma, double* coef,
+                            double* chi2, int* status, cudaStream_t s) {
+    if (nd <= 64) launch_pdl(k_lsq_warp<NB, 2>, dim3(1), dim3(32), 0, s, resp, meas, sigma, nd, coef, chi2, status);
+    else if (nd <= 128) launch_pdl(k_lsq_warp<NB, 4>, dim3(1), dim3(32), 0, s, resp, meas, sigma, nd, coef, chi2, status);
+    else if (nd <= 192) launch_pdl(k_lsq_warp<NB, 6>, dim3(1), dim3(32), 0, s, resp, meas, sigma, nd, coef, chi2, status);
+    else return false;
+    return true;
+}
+
 static size_t lsq_smem(const Ctx& c) {
-    return sizeof(double) * ((size_t)(c.nb + 2) * c.ndiag + 72);
+    return sizeof(double) * ((size_t)((c.nb | 1) + 2) * c.ndiag + 3 * (size_t)c.nb * c.nb + 5 * 32);
 }
 
 cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const double* sigma, double* coef,
                        double* chi2, cudaStream_t s) {
     size_t smem = lsq_smem(c);
-    launch_pdl(k_lsq, dim3(1), dim3(128), smem, s, resp, meas, sigma, c.ndiag, c.nb, coef, chi2, c.status);
+    bool done = false;
+    switch (c.nb) {
+        case 1: done = launch_lsq_warp<1>(c.ndiag, resp, meas, sigma, coef, chi2, c.status, s); break;
+        case 2: done = launch_lsq_warp<2>(c.ndiag, resp, meas, sigma, coef, chi2, c.status, s); break;
+        case 3: done = launch_lsq_warp<3>(c.ndiag, resp, meas, sigma, coef, chi2, c.status, s); break;
+        case 4: done = launch_lsq_warp<4>(c.ndiag, resp, meas, sigma, coef, chi2, c.status, s); break;
+        case 5: done = launch_lsq_warp<5>(c.ndiag, resp, meas, sigma, coef, chi2, c.status, s); break;
+        case 6: done = launch_lsq_warp<6>(c.ndiag, resp, meas, sigma, coef, chi2, c.status, s); break;
+        default: break;
+    }
+    if (done) return cudaGetLastError();
+    launch_pdl(k_lsq, dim3(1), dim3(256), smem, s, resp, meas, sigma, c.ndiag, c.nb, coef, chi2, c.status);
     return cudaGetLastError();
 }
 
