@@ -194,6 +194,7 @@ static size_t carve(Ctx& c, char* base) {
     c.tri_inv = (double*)take(sizeof(double) * (size_t)c.ni_pad * c.nmode);
     c.tri_alpha = (double*)take(sizeof(double) * (size_t)c.ni_pad * c.nmode);
     c.twiddle = (double2*)take(sizeof(double2) * (size_t)(c.fft_m / 2));
+    c.sin_tab = (double*)take(sizeof(double) * (size_t)c.nmode);
     c.axbd = (double*)take(sizeof(double) * 2);
     c.status = (int*)take(sizeof(int) * 4);
     c.tickets = (unsigned*)take(sizeof(unsigned) * 8);
@@ -331,7 +332,7 @@ static void fill_info(const Ctx& c, efit_info_t* info) {
     info->resp_row_lo = c.m_lo; info->resp_row_hi = c.m_hi;
     info->bnd_row_lo = c.i_lo; info->bnd_row_hi = c.i_hi;
     info->lr_blk_lo = c.jt_lo; info->lr_blk_hi = c.jt_hi;
-    const int tile = 32 * c.t.lr_jt;
+    const int tile = c.lr_direct ? 32 * c.t.lr_jt : c.nh;  // FFT mode: one tile holds every j
     info->lr_j_lo = c.jt_lo * tile < c.nh ? c.jt_lo * tile : c.nh;
     info->lr_j_hi = c.jt_hi * tile < c.nh ? c.jt_hi * tile : c.nh;
     info->slab_stride = c.S;
@@ -463,8 +464,12 @@ static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, 
     if ((e = launch_lsq(c, c.resp, meas, sigma, coef, chi2, s))) return e;
     if ((e = launch_current(c, psi, coef, c.pcurr, true, s))) return e;
     mark(c, s, M_CUR);
-    if ((e = launch_boundary(c, c.pcurr, c.psib, s))) return e;  // marks M_TB, M_LR inside
-    if ((e = launch_solve(c, c.pcurr, c.psib, nullptr, psi, psi_ext, eps, s, true))) return e;
+    // boundary flux (marks M_TB, M_LR inside); in FFT mode the forward DST (without the bottom/top
+    // edge terms) runs on the side stream under k_bnd_tb and the tridiagonal solve adds those terms
+    const bool overlap = !c.lr_direct;
+    if ((e = launch_boundary(c, c.pcurr, c.psib, s, overlap))) return e;
+    if (!overlap && (e = launch_solve_fwd(c, c.pcurr, c.psib, s, 1))) return e;
+    if ((e = launch_solve_rest(c, c.psib, nullptr, psi, psi_ext, eps, s, true, overlap))) return e;
     mark(c, s, M_SOLVE);
     if (c.prof_on && c.prof_rec && !c.prof_capture && c.prof_next < c.prof_slots) ++c.prof_next;
     c.prof_rec = false;

@@ -70,6 +70,7 @@ struct Ctx {
     double* tri_inv;    // [nmode][ld]      1/den_i per mode
     double* tri_alpha;  // [nmode][ld]      -a_i/den_i (forward-sweep recurrence coefficient)
     double2* twiddle;   // [fft_m/2]        exp(-2 pi i k/M)
+    double* sin_tab;    // [nmode]          sin(pi k/(n+1)), k = 1..n
 
     // per-iteration scratch
     double* axbd;       // [2] psi_axis, psi_bdry
@@ -139,7 +140,11 @@ cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const dou
                        double* coef, double* chi2, cudaStream_t s);
 cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double* pcurr,
                            bool pair, cudaStream_t s);
-cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s);
+cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s,
+                            bool overlap_solve = false);
+cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cudaStream_t s, int with_bnd);
+cudaError_t launch_solve_rest(Ctx& c, const double* psib, double* psi_out, double* psi_inout, const double* psi_ext,
+                              double* eps, cudaStream_t s, bool next_norm, bool tb_fix);
 cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out,
                          double* psi_inout, const double* psi_ext, double* eps, cudaStream_t s,
                          bool next_norm = false);

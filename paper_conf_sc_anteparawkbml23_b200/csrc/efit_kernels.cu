@@ -249,6 +249,11 @@ __global__ void k_tri_factors(double* __restrict__ tri_a, double* __restrict__ c
     }
 }
 
+__global__ void k_sin_table(double* __restrict__ sk, int n) {  // sin(pi k/(n+1)), k = 1..n
+    const int k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k < n) sk[k] = sinpi((double)(k + 1) / (double)(n + 1));
+}
+
 __global__ void k_twiddles(double2* __restrict__ w, int M) {
     int k = blockIdx.x * blockDim.x + threadIdx.x;
     if (k >= M / 2) return;
@@ -289,6 +294,7 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
     k_tri_factors<<<(c.nmode + 63) / 64, 64, 0, s>>>(c.tri_a, c.tri_cp, c.tri_inv, c.tri_alpha, c.ni, c.ni_pad,
                                                      c.nmode, c.rmin, c.dr, c.dz);
     k_twiddles<<<(c.fft_m / 2 + 255) / 256, 256, 0, s>>>(c.twiddle, c.fft_m);
+    k_sin_table<<<(c.nmode + 255) / 256, 256, 0, s>>>(c.sin_tab, c.nmode);
     if (!c.lr_direct) {  // needs the edge slabs and the twiddles above
         e = launch_lr_spectra(c, s);
         if (e) return e;
@@ -1333,7 +1339,9 @@ static cudaError_t launch_lr(Ctx& c, cudaStream_t s, bool prepare) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s) {
+cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cudaStream_t s, int with_bnd);
+
+cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s, bool overlap_solve) {
     cudaError_t e;
     // fork: the FP64-bound left/right kernel runs on the side stream, concurrently with the
     // HBM-bound top/bottom stream (both only read pcurr / ipair); join before the reduce.
@@ -1343,6 +1351,10 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     } else {
         if ((e = launch_lr_fft(c, psib, c.side))) return e;
     }
+    // superposition: apart from the bottom/top edge terms the GS right-hand side is known once the
+    // left/right FFT chain has written psi_b(left/right), so its forward DST also runs under the
+    // HBM-bound stream; k_tridiag adds the bottom/top terms in the sine domain afterwards
+    if (overlap_solve && (e = launch_solve_fwd(c, pcurr, psib, c.side, 2))) return e;
     mark(c, c.side, M_LR);
     if ((e = cudaEventRecord(c.ev_join, c.side))) return e;
     const int nslab = c.i_hi - c.i_lo;
@@ -1452,7 +1464,7 @@ __host__ __device__ __forceinline__ int fft_stages(int log2m) { return (log2m >>
 __global__ void __launch_bounds__(512) k_dst_fwd(const double* __restrict__ pcurr, const double* __restrict__ psib,
                                                  const double* __restrict__ tri_a, int nw, int nh, double rmin,
                                                  double dr, double dz, const double2* __restrict__ W, int M,
-                                                 int log2m, int FPC, double* __restrict__ fhat, int ld) {
+                                                 int log2m, int FPC, double* __restrict__ fhat, int ld, int with_bnd) {
     extern __shared__ __align__(16) double2 a2[];  // FPC x ([M] data, [M] scratch), then [M/2] twiddles
     double2* Ws = a2 + 2 * FPC * M;
     const int n = nh - 2, ni = nw - 2;
@@ -1477,10 +1489,14 @@ __global__ void __launch_bounds__(512) k_dst_fwd(const double* __restrict__ pcur
                 if (i > ni) continue;
                 const double R = grid_coord(rmin, i, dr);
                 double fv = -kMu0 * R * pcurr[(long long)i * nh + jj] * cellinv;
-                if (i == 1) fv -= tri_a[0] * psib[jj];                                   // left edge
-                if (i == ni) fv -= (2.0 / (dr * dr) - tri_a[ni - 1]) * psib[nh + jj];    // right edge (c_ni)
-                if (jj == 1) fv -= psib[2 * nh + (i - 1)] * idz2;                        // bottom edge
-                if (jj == n) fv -= psib[2 * nh + (nw - 2) + (i - 1)] * idz2;             // top edge
+                if (with_bnd) {
+                    if (i == 1) fv -= tri_a[0] * psib[jj];                                   // left edge
+                    if (i == ni) fv -= (2.0 / (dr * dr) - tri_a[ni - 1]) * psib[nh + jj];    // right edge (c_ni)
+                }
+                if (with_bnd == 1) {  // with_bnd == 2: k_tridiag adds these in the sine domain
+                    if (jj == 1) fv -= psib[2 * nh + (i - 1)] * idz2;                        // bottom edge
+                    if (jj == n) fv -= psib[2 * nh + (nw - 2) + (i - 1)] * idz2;             // top edge
+                }
                 v[h] = sgn * fv;
             }
         }
@@ -1498,6 +1514,21 @@ __global__ void __launch_bounds__(512) k_dst_fwd(const double* __restrict__ pcur
     }
 }
 
+// Bottom/top edge terms of the right-hand side in the sine domain (superposition, see
+// launch_boundary): f_{j=1} -= psi_bot/dz^2 and f_{j=n} -= psi_top/dz^2 transform to
+//   fhat[k][r] -= (psi_bot(r) + (-1)^(k+1) psi_top(r)) sin(pi k/(n+1)) / dz^2,
+// added by the tridiagonal kernel as it loads its mode column (bot == nullptr: nothing to add).
+struct TbFix {
+    const double* bot;   // psi_b bottom edge, rows i = 1..ni (ABI edge order offset 2 nh)
+    const double* top;   // psi_b top edge
+    const double* sink;  // sin(pi k/(n+1)), k = 1..n
+    double idz2;
+};
+__device__ __forceinline__ double tb_fix(const TbFix& fx, int mode, int r) {
+    const double sgn = (mode & 1) ? -1.0 : 1.0;  // k = mode + 1: (-1)^(k+1)
+    return -(fx.bot[r] + sgn * fx.top[r]) * (fx.sink[mode] * fx.idz2);
+}
+
 // Radial tridiagonal solve per sine mode, one warp per mode, in place on the mode-major array.
 // The warp stages its mode column in shared memory with a skew (row r at r + r/L, L = rows per
 // lane) so both the global access and the lane-segment access are conflict-free.  Both Thomas
@@ -1510,7 +1541,7 @@ __global__ void __launch_bounds__(512) k_dst_fwd(const double* __restrict__ pcur
 // |alpha|, |c'| < 1 (diagonal dominance) keeps the reassociation as accurate as the sequential sweep.
 __global__ void __launch_bounds__(128) k_tridiag(double* __restrict__ fhat, int ld, const double* __restrict__ alpha,
                                                  const double* __restrict__ inv, const double* __restrict__ cp,
-                                                 int ni, int L, int nmode) {
+                                                 int ni, int L, int nmode, TbFix fx) {
     extern __shared__ __align__(16) double sm_tri[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int mode = blockIdx.x * 4 + warp;
@@ -1518,7 +1549,8 @@ __global__ void __launch_bounds__(128) k_tridiag(double* __restrict__ fhat, int 
     griddep();
     if (mode >= nmode) return;
     double* fg = fhat + (long long)mode * ld;
-    for (int r = lane; r < 32 * L; r += 32) sf[r + r / L] = r < ni ? fg[r] : 0.0;
+    for (int r = lane; r < 32 * L; r += 32)
+        sf[r + r / L] = r < ni ? (fx.bot ? fg[r] + tb_fix(fx, mode, r) : fg[r]) : 0.0;
     __syncwarp();
     const long long fo = (long long)mode * 32 * L + lane;
     const double* al = alpha + fo;
@@ -1567,6 +1599,74 @@ __global__ void __launch_bounds__(128) k_tridiag(double* __restrict__ fhat, int 
     }
     __syncwarp();
     for (int r = lane; r < ni; r += 32) fg[r] = sf[r + r / L];
+}
+
+// Register variant of k_tridiag for L <= 16 rows per lane: every lane loads its whole segment
+// (data, alpha, inv, c') with independent loads first, so the two sweeps run from registers after a
+// single memory latency.  Same recurrences and scan as k_tridiag (bitwise-identical results).
+template <int L>
+__global__ void __launch_bounds__(128) k_tridiag_reg(double* __restrict__ fhat, int ld,
+                                                     const double* __restrict__ alpha,
+                                                     const double* __restrict__ inv, const double* __restrict__ cp,
+                                                     int ni, int nmode, TbFix fx) {
+    griddep();
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int mode = blockIdx.x * 4 + warp;
+    if (mode >= nmode) return;
+    double* fg = fhat + (long long)mode * ld;
+    const long long fo = (long long)mode * 32 * L + lane;
+    double f[L], al[L], iv[L], c[L];
+#pragma unroll
+    for (int e = 0; e < L; ++e) {
+        const int r = lane * L + e;
+        f[e] = r < ni ? (fx.bot ? fg[r] + tb_fix(fx, mode, r) : fg[r]) : 0.0;
+        al[e] = alpha[fo + 32 * e];
+        iv[e] = inv[fo + 32 * e];
+        c[e] = cp[fo + 32 * e];
+    }
+    double A = 1.0, B = 0.0;
+#pragma unroll
+    for (int e = 0; e < L; ++e) {
+        B = fma(al[e], B, iv[e] * f[e]);
+        A *= al[e];
+    }
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        const double Ap = __shfl_up_sync(0xffffffffu, A, off);
+        const double Bp = __shfl_up_sync(0xffffffffu, B, off);
+        if (lane >= off) { B = fma(A, Bp, B); A *= Ap; }
+    }
+    double d = __shfl_up_sync(0xffffffffu, B, 1);
+    if (lane == 0) d = 0.0;
+#pragma unroll
+    for (int e = 0; e < L; ++e) {
+        d = fma(al[e], d, iv[e] * f[e]);
+        f[e] = d;
+    }
+    double C = 1.0, D = 0.0;
+#pragma unroll
+    for (int e = L - 1; e >= 0; --e) {
+        D = fma(-c[e], D, f[e]);
+        C *= -c[e];
+    }
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        const double Cn = __shfl_down_sync(0xffffffffu, C, off);
+        const double Dn = __shfl_down_sync(0xffffffffu, D, off);
+        if (lane + off < 32) { D = fma(C, Dn, D); C *= Cn; }
+    }
+    double x = __shfl_down_sync(0xffffffffu, D, 1);
+    if (lane == 31) x = 0.0;
+#pragma unroll
+    for (int e = L - 1; e >= 0; --e) {
+        x = fma(-c[e], x, f[e]);
+        f[e] = x;
+    }
+#pragma unroll
+    for (int e = 0; e < L; ++e) {
+        const int r = lane * L + e;
+        if (r < ni) fg[r] = f[e];
+    }
 }
 
 // Inverse DST-I (same transform, scale 2/(n+1)) of 2*FPC rows per CTA, then either
@@ -1709,18 +1809,41 @@ static void solve_shape(const Ctx& c, int& fpc, int& threads, size_t& smem) {
     smem = sizeof(double2) * (size_t)(2 * fpc * M + M / 2);
 }
 
-cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out, double* psi_inout,
-                         const double* psi_ext, double* eps, cudaStream_t s, bool next_norm) {
+// forward DST of the interior right-hand side; with_bnd: 1 = all edge terms, 2 = left/right only
+cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cudaStream_t s, int with_bnd) {
     int fpc, threads;
     size_t smem;
     solve_shape(c, fpc, threads, smem);
     const int nrb = (c.ni + 2 * fpc - 1) / (2 * fpc);
-    cudaError_t e = launch_pdl(k_dst_fwd, dim3(nrb), dim3(threads), smem, s, pcurr, psib, c.tri_a, c.nw, c.nh, c.rmin,
-                               c.dr, c.dz, c.twiddle, c.fft_m, c.fft_log2, fpc, c.fhat, c.fhat_ld);
-    if (e) return e;
+    return launch_pdl(k_dst_fwd, dim3(nrb), dim3(threads), smem, s, pcurr, psib, c.tri_a, c.nw, c.nh, c.rmin, c.dr,
+                      c.dz, c.twiddle, c.fft_m, c.fft_log2, fpc, c.fhat, c.fhat_ld, with_bnd);
+}
+
+// tridiagonal solve + inverse DST + update (after the forward coefficients are complete)
+// tb_fix: the forward coefficients lack the bottom/top edge terms (superposed fit step)
+cudaError_t launch_solve_rest(Ctx& c, const double* psib, double* psi_out, double* psi_inout, const double* psi_ext,
+                              double* eps, cudaStream_t s, bool next_norm, bool tb_fix) {
+    TbFix fx;
+    fx.bot = tb_fix ? psib + 2 * c.nh : nullptr;
+    fx.top = psib + 2 * c.nh + (c.nw - 2);
+    fx.sink = c.sin_tab;
+    fx.idz2 = 1.0 / (c.dz * c.dz);
+    int fpc, threads;
+    size_t smem;
+    solve_shape(c, fpc, threads, smem);
+    const int nrb = (c.ni + 2 * fpc - 1) / (2 * fpc);
+    cudaError_t e;
     const int L = c.ni_pad / 32;
-    e = launch_pdl(k_tridiag, dim3((c.nmode + 3) / 4), dim3(128), sizeof(double) * 4 * (32 * (size_t)L + 32), s, c.fhat,
-                   c.fhat_ld, c.tri_alpha, c.tri_inv, c.tri_cp, c.ni, L, c.nmode);
+    const dim3 tg((c.nmode + 3) / 4), tb(128);
+    switch (L) {
+#define EFIT_TRI(V) case V: e = launch_pdl(k_tridiag_reg<V>, tg, tb, 0, s, c.fhat, c.fhat_ld, c.tri_alpha, c.tri_inv, \
+                                           c.tri_cp, c.ni, c.nmode, fx); break;
+        EFIT_TRI(1) EFIT_TRI(2) EFIT_TRI(4) EFIT_TRI(8) EFIT_TRI(16)
+#undef EFIT_TRI
+        default:
+            e = launch_pdl(k_tridiag, tg, tb, sizeof(double) * 4 * (32 * (size_t)L + 32), s, c.fhat, c.fhat_ld,
+                           c.tri_alpha, c.tri_inv, c.tri_cp, c.ni, L, c.nmode, fx);
+    }
     if (e) return e;
     NextNorm nn;
     nn.on = (next_norm && psi_inout) ? 1 : 0;
@@ -1734,6 +1857,13 @@ cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double
     return launch_pdl(k_dst_inv, dim3(nrb + 1), dim3(threads), smem, s, c.fhat, c.fhat_ld, psib, c.nw, c.nh,
                       c.twiddle, c.fft_m, c.fft_log2, fpc, psi_out, psi_inout, psi_ext, c.eps_part, c.tickets + 1,
                       c.axbd, eps, nn);
+}
+
+cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out, double* psi_inout,
+                         const double* psi_ext, double* eps, cudaStream_t s, bool next_norm) {
+    cudaError_t e = launch_solve_fwd(c, pcurr, psib, s, 1);
+    if (e) return e;
+    return launch_solve_rest(c, psib, psi_out, psi_inout, psi_ext, eps, s, next_norm, false);
 }
 
 // ================================================================================ left/right via FFT
