@@ -32,6 +32,7 @@ import numpy as np  # noqa: E402
 import synth  # noqa: E402
 
 METRIC = "fit iterations/s and response+boundary GB/s vs B200 HBM peak at 1/2/4/8 GPUs"
+MODES = {"table": 0, "otf": 1, "sym": 2, "otf-sym": 3}  # EFIT_GREEN_* (include/efit.h)
 UNIT = "fit iterations/s"
 
 
@@ -44,7 +45,9 @@ def parse():
     ap.add_argument("--impl", default="efit", choices=["efit", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--mode", default="table", choices=["table", "otf"])
+    ap.add_argument("--mode", default="table", choices=list(MODES),
+                    help="Green's mode of the top/bottom nest (include/efit.h): table = full table "
+                         "(the paper's gridpc), sym = half table by reciprocity, otf / otf-sym = recomputed")
     ap.add_argument("--no-profile", action="store_true",
                     help="time graph replays without per-kernel events (no roofline breakdown)")
     return ap.parse_args()
@@ -203,7 +206,7 @@ def gpu_arm(args, rank, world, local):
         dist.init_process_group("nccl", device_id=dev)
     cfg = synth.config(args.config)
     N, ndiag = cfg.grid.nw, cfg.geometry.ndiag
-    mode = efit.EFIT_GREEN_TABLE if args.mode == "table" else efit.EFIT_GREEN_ONTHEFLY
+    mode = MODES[args.mode]
     t0 = time.time()
     ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=mode, rank=rank, world=world, device=dev)
     torch.cuda.synchronize()
@@ -291,8 +294,17 @@ def gpu_arm(args, rank, world, local):
 
     # ---------------- roofline of the dominant kernel (k_bnd_tb) and response+boundary GB/s
     peak, peak_kind = measured_peaks()
-    nslab = ctx.info.bnd_row_hi - ctx.info.bnd_row_lo
-    tb_bytes = 8.0 * nslab * N * N + 16.0 * N * N  # T slabs once + (I, I_flipped) pair array
+    if args.mode in ("sym", "otf-sym"):
+        # half table: this rank's 8 x 8 row-pair tiles of 64*nh doubles, streamed once, + (I, I_flipped)
+        ntile = ctx.info.sym_tile_hi - ctx.info.sym_tile_lo
+        tb_bytes = 8.0 * 64 * N * ntile + 16.0 * N * N
+        tb_kernel = "k_bnd_sym"
+    else:
+        nslab = ctx.info.bnd_row_hi - ctx.info.bnd_row_lo
+        tb_bytes = 8.0 * nslab * N * N + 16.0 * N * N  # T slabs once + (I, I_flipped) pair array
+        tb_kernel = "k_bnd_tb"
+    if args.mode in ("otf", "otf-sym"):
+        tb_bytes = 16.0 * N * N  # no table: only the current pair is read
     gd_bytes = 8.0 * (ctx.info.resp_row_hi - ctx.info.resp_row_lo) * N * N
     if prof is None:
         tb_ms, rb_ms, breakdown = float("nan"), None, {}
@@ -311,10 +323,10 @@ def gpu_arm(args, rank, world, local):
         try:
             d = json.load(open(ncu_sum))
             if d.get("config") == args.config and d.get("world", 1) == world:
-                traffic = d.get("k_bnd_tb", {}).get("dram_bytes_per_launch")
+                traffic = d.get(tb_kernel, {}).get("dram_bytes_per_launch")
         except Exception:
             traffic = None
-    roof = {"kernel": "k_bnd_tb" if sharded is None else "boundary_flux (k_bnd_tb+k_bnd_lr+reduce)",
+    roof = {"kernel": tb_kernel if sharded is None else f"boundary_flux ({tb_kernel}+lr+reduce)",
             "bound": "hbm", "achieved": round(tb_gbs, 1), "peak": peak, "unit": "GB/s",
             "frac": round(tb_gbs / peak, 4), "traffic": traffic, "peak_source": peak_kind,
             "algorithmic_bytes_per_launch": tb_bytes}

@@ -96,10 +96,25 @@ typedef struct {
     int32_t lr_blk_lo, lr_blk_hi;       /* this rank's left/right target tiles           */
     int32_t lr_j_lo, lr_j_hi;           /* this rank's left/right targets j [lo, hi)     */
     int64_t slab_stride;                /* doubles between Green's-table slabs           */
+    int32_t sym_nblk;                   /* SYM modes: 8-row blocks of the nw-2 interior rows */
+    int32_t sym_tile_lo, sym_tile_hi;   /* SYM modes: this rank's row-pair tiles [lo, hi)   */
     size_t workspace_bytes;
 } efit_info_t;
 
-enum { EFIT_GREEN_TABLE = 0, EFIT_GREEN_ONTHEFLY = 1 };
+/* Green's-function modes of the top/bottom boundary nest (the dominant O(N^3) stream):
+ *   EFIT_GREEN_TABLE         full table T[i][ii][m], one slab per target row (the paper's gridpc
+ *                            use); targets sharded by row.
+ *   EFIT_GREEN_ONTHEFLY      same decomposition, G recomputed from (R_i, R_ii, m dZ); bitwise
+ *                            equal to EFIT_GREEN_TABLE.
+ *   EFIT_GREEN_TABLE_SYM     half table by reciprocity G(a; b) = G(b; a): only the
+ *                            interior row pairs i <= ii are stored, in 8 x 8 row-pair tiles, and each
+ *                            stored entry serves both targets i and ii -> half the bytes of TABLE.
+ *                            Results equal TABLE to rounding (<= 1e-14 relative), not bit for bit.
+ *   EFIT_GREEN_ONTHEFLY_SYM  the SYM decomposition with G recomputed (half the Green's evaluations
+ *                            of ONTHEFLY); bitwise equal to EFIT_GREEN_TABLE_SYM.
+ * SYM modes with world > 1: the row-pair tiles are sharded, so every rank writes a partial sum for
+ * every top/bottom target; the caller SUMS the zero-initialised d_psib over ranks (all-reduce). */
+enum { EFIT_GREEN_TABLE = 0, EFIT_GREEN_ONTHEFLY = 1, EFIT_GREEN_TABLE_SYM = 2, EFIT_GREEN_ONTHEFLY_SYM = 3 };
 
 enum {
     EFIT_OK = 0,
@@ -208,7 +223,10 @@ int efit_status(efit_ctx* ctx, efit_stream_t stream);
 /* Test/inspection access: device pointers into the workspace.  which = 0: top/bottom Green's
  * slabs (slab of target row i at T + (i - bnd_row_lo)*slab_stride, entry ii*nh + m),
  * 1: Gd (row m at Gd + (m - resp_row_lo)*slab_stride, entry g), 2: in-limiter flags
- * (uint8[nw*nh]), 3: the two edge slabs i = 0 and i = nw-1 (at 0 and slab_stride).
+ * (uint8[nw*nh]), 3: the two edge slabs i = 0 and i = nw-1 (at 0 and slab_stride),
+ * 4: the SYM half table: tile t (global index t = Q(Q+1)/2 + P, P <= Q, this rank's tiles
+ * [sym_tile_lo, sym_tile_hi) stored contiguously) at (t - sym_tile_lo)*64*nh doubles, entry
+ * [p][m][q] (q fastest) = G(R_i, m dZ; R_ii, 0), i = 1 + 8P + p, ii = 1 + 8Q + q (0 if i or ii > nw-2).
  * Returns EFIT_E_STATE if the table is not built in this mode. */
 int efit_table(const efit_ctx* ctx, int which, const void** d_ptr);
 

@@ -21,14 +21,18 @@ __all__ = [
     "efit_current", "efit_boundary_flux", "efit_interior_solve", "efit_lsq", "efit_fit_step", "efit_status",
     "efit_solve_update", "efit_profile_begin", "efit_profile_end", "efit_fit_steps",
     "efit_table", "efit_shard", "efit_destroy", "efit_strerror", "efit_last_error", "efit_version",
-    "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY", "efit_plan_info", "owned_targets", "exchange",
+    "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY", "EFIT_GREEN_TABLE_SYM",
+    "EFIT_GREEN_ONTHEFLY_SYM", "efit_plan_info", "owned_targets", "exchange",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-lib_path = os.path.join(_HERE, "libefit_b200.so")
+# EFIT_B200_LIB: load an in-tree build variant instead (kernel tuning sweeps, scripts/tune_sym.sh)
+lib_path = os.environ.get("EFIT_B200_LIB") or os.path.join(_HERE, "libefit_b200.so")
 
 EFIT_GREEN_TABLE = 0
 EFIT_GREEN_ONTHEFLY = 1
+EFIT_GREEN_TABLE_SYM = 2       # half table by reciprocity (include/efit.h)
+EFIT_GREEN_ONTHEFLY_SYM = 3
 EFIT_OK, EFIT_E_INVAL, EFIT_E_NOMEM, EFIT_E_CUDA, EFIT_E_NCCL = 0, -1, -2, -3, -4
 EFIT_E_SINGULAR, EFIT_E_NOPLASMA, EFIT_E_NONFINITE, EFIT_E_STATE = -5, -6, -7, -8
 
@@ -65,7 +69,9 @@ class efit_info_t(ctypes.Structure):
                 ("bnd_row_lo", ctypes.c_int32), ("bnd_row_hi", ctypes.c_int32),
                 ("lr_blk_lo", ctypes.c_int32), ("lr_blk_hi", ctypes.c_int32),
                 ("lr_j_lo", ctypes.c_int32), ("lr_j_hi", ctypes.c_int32),
-                ("slab_stride", ctypes.c_int64), ("workspace_bytes", ctypes.c_size_t)]
+                ("slab_stride", ctypes.c_int64), ("sym_nblk", ctypes.c_int32),
+                ("sym_tile_lo", ctypes.c_int32), ("sym_tile_hi", ctypes.c_int32),
+                ("workspace_bytes", ctypes.c_size_t)]
 
 
 class EfitError(RuntimeError):

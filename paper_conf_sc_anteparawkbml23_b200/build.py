@@ -23,32 +23,36 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, defines=(), out: str = LIB) -> str:
+    """Compile both sources and link `out`.  `defines` (e.g. ["EFIT_SYM_UNR=3"]) build a tuning
+    variant into another file (the default library is always the untuned default build)."""
+    if not force and not defines and out == LIB and not _stale():
         return LIB
     objs = []
     log = []
     for src in SOURCES:
-        obj = os.path.join(CSRC, src.replace(".cu", ".o"))
-        cmd = ["nvcc", *NVCC_FLAGS, "-c", os.path.join(CSRC, src), "-o", obj]
+        tag = "" if out == LIB else "." + os.path.basename(out).replace(".so", "")
+        obj = os.path.join(CSRC, src.replace(".cu", tag + ".o"))
+        cmd = ["nvcc", *NVCC_FLAGS, *["-D" + d for d in defines], "-c", os.path.join(CSRC, src), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         log.append(r.stdout + r.stderr)
         if r.returncode != 0:
             sys.stderr.write(r.stdout + r.stderr)
             raise RuntimeError(f"nvcc failed on {src}")
         objs.append(obj)
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = out + f".tmp{os.getpid()}"
     cmd = ["nvcc", "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", tmp, *objs, "-lcudart"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
         raise RuntimeError("nvcc link failed")
-    os.replace(tmp, LIB)
-    with open(os.path.join(CSRC, "ptxas.log"), "w") as f:
-        f.write("\n".join(log))
+    os.replace(tmp, out)
+    if out == LIB:
+        with open(os.path.join(CSRC, "ptxas.log"), "w") as f:
+            f.write("\n".join(log))
     if verbose:
         print("\n".join(log))
-    return LIB
+    return out
 
 
 if __name__ == "__main__":

@@ -95,7 +95,9 @@ static int validate(const efit_grid* g, const efit_basis* b, const efit_geometry
     for (int m = 0; m < geo->n_mp; ++m) if (!(geo->mp_r[m] > 0)) return fail(nullptr, EFIT_E_INVAL, "probe R <= 0");
     for (int m = 0; m < geo->n_int; ++m) if (!(geo->int_r[m] > 0)) return fail(nullptr, EFIT_E_INVAL, "internal point R <= 0");
     if (geo->ip_sign != 1 && geo->ip_sign != -1) return fail(nullptr, EFIT_E_INVAL, "ip_sign must be +1 or -1");
-    if (mode != EFIT_GREEN_TABLE && mode != EFIT_GREEN_ONTHEFLY) return fail(nullptr, EFIT_E_INVAL, "mode %d", mode);
+    if (mode != EFIT_GREEN_TABLE && mode != EFIT_GREEN_ONTHEFLY && mode != EFIT_GREEN_TABLE_SYM &&
+        mode != EFIT_GREEN_ONTHEFLY_SYM)
+        return fail(nullptr, EFIT_E_INVAL, "mode %d", mode);
     if (d && (d->world < 1 || d->rank < 0 || d->rank >= d->world))
         return fail(nullptr, EFIT_E_INVAL, "rank %d / world %d", d->rank, d->world);
     return EFIT_OK;
@@ -115,6 +117,8 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     c.ndiag = geo->n_fl + geo->n_mp + geo->n_int;
     c.n_lim = geo->n_lim; c.ip_sign = geo->ip_sign;
     c.mode = mode;
+    c.sym = mode == EFIT_GREEN_TABLE_SYM || mode == EFIT_GREEN_ONTHEFLY_SYM;
+    c.otf = mode == EFIT_GREEN_ONTHEFLY || mode == EFIT_GREEN_ONTHEFLY_SYM;
     c.rank = d ? d->rank : 0;
     c.world = d ? d->world : 1;
     c.n_edge = 2 * c.nh + 2 * (c.nw - 2);
@@ -128,7 +132,19 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     const long long n = (long long)c.nw * c.nh;
     c.S = round_up(n, 64);
     efit::Tiling& t = c.t;
-    t.resp_gc = c.nb <= 8 ? 1152 : (c.nb <= 16 ? 768 : 512);  // multiples of NP x 128-node positions
+    {
+        // response chunk: a multiple of 128 nodes (the permuted shared layout), at most the size
+        // whose NB x gc basis slice keeps 2 CTAs per SM, chosen to minimise the busiest CTA slot's
+        // nodes (ceil(chunks / 296 slots) x gc): one CTA wave without a partial tail where possible
+        const int gc_max = c.nb <= 8 ? 1152 : (c.nb <= 16 ? 768 : 512);
+        const long long slots = 2LL * efit::kNumSMs;
+        long long best = -1;
+        for (int gc = 256; gc <= gc_max; gc += 128) {
+            const long long nch = (n + gc - 1) / gc;
+            const long long cost = (nch + slots - 1) / slots * gc;
+            if (best < 0 || cost <= best) { best = cost; t.resp_gc = gc; }  // ties -> larger chunks
+        }
+    }
     t.resp_nchunk = (int)((n + t.resp_gc - 1) / t.resp_gc);
     t.tb_ch = 2048;
     t.tb_nchunk = (int)((n + t.tb_ch - 1) / t.tb_ch);
@@ -153,6 +169,19 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     c.i_lo = 1 + lo; c.i_hi = 1 + hi;
     efit_shard(t.lr_njt, c.rank, c.world, &lo, &hi);
     c.jt_lo = lo; c.jt_hi = hi;
+    // SYM modes: row-pair tiles of 8 x 8 interior rows; the tiles (not the targets) are sharded
+    c.sym_nblk = (c.ni + 7) / 8;
+    c.sym_ntile = (long long)c.sym_nblk * (c.sym_nblk + 1) / 2;
+    {
+        const long long base = c.sym_ntile / c.world, rem = c.sym_ntile % c.world;
+        c.sym_tile_lo = c.rank * base + (c.rank < rem ? c.rank : rem);
+        c.sym_tile_hi = c.sym_tile_lo + base + (c.rank < rem ? 1 : 0);
+    }
+    // one chunk (F read mirrored from the staged I: 128 nh B of staging) up to nh = 576, else
+    // chunks of <= 440 values with I and F staged (256 mc B): 3 CTAs per SM either way
+    t.sym_nmc = c.nh <= 576 ? 1 : (c.nh + 439) / 440;
+    t.sym_mc = ((c.nh + t.sym_nmc - 1) / t.sym_nmc + 1) / 2 * 2;  // even: 16-byte chunk starts
+    c.nhp = (c.nh + 1) / 2 * 2;
     t.tb_ngroup = (c.i_hi - c.i_lo + t.tb_gi - 1) / t.tb_gi;
     if (t.tb_ngroup < 1) t.tb_ngroup = 1;
     // response rows per warp block: fewest rows on the busiest warp, registers MB*NB <= 40
@@ -183,6 +212,13 @@ static size_t carve(Ctx& c, char* base) {
     const int nrows = c.m_hi - c.m_lo;
     const int nslab = c.i_hi - c.i_lo;
     c.T = (c.mode == EFIT_GREEN_TABLE && nslab > 0) ? (double*)take(sizeof(double) * (size_t)nslab * c.S) : nullptr;
+    const long long ntile_rank = c.sym_tile_hi - c.sym_tile_lo;
+    c.U = (c.mode == EFIT_GREEN_TABLE_SYM && ntile_rank > 0)
+              ? (double*)take(sizeof(double) * 64 * (size_t)c.nh * (size_t)ntile_rank) : nullptr;
+    c.symq = c.sym ? (double*)take(sizeof(double) * 16 * (size_t)c.sym_nblk * c.nh) : nullptr;
+    c.symp = c.sym ? (double*)take(sizeof(double) * 16 * (size_t)c.sym_nblk * c.nhp) : nullptr;
+    c.sym_part = c.sym ? (double*)take(sizeof(double) * 2 * (size_t)(c.ni > 0 ? c.ni : 1) * c.sym_nblk * c.t.sym_nmc)
+                       : nullptr;
     c.Tedge = (double*)take(sizeof(double) * 2 * (size_t)c.S);
     c.Gd = (double*)take(sizeof(double) * (size_t)(nrows > 0 ? nrows : 1) * c.S);
     c.inlim = (uint8_t*)take((size_t)n);
@@ -336,6 +372,9 @@ static void fill_info(const Ctx& c, efit_info_t* info) {
     info->lr_j_lo = c.jt_lo * tile < c.nh ? c.jt_lo * tile : c.nh;
     info->lr_j_hi = c.jt_hi * tile < c.nh ? c.jt_hi * tile : c.nh;
     info->slab_stride = c.S;
+    info->sym_nblk = c.sym_nblk;
+    info->sym_tile_lo = (int32_t)c.sym_tile_lo;
+    info->sym_tile_hi = (int32_t)c.sym_tile_hi;
     info->workspace_bytes = c.ws_bytes;
 }
 
@@ -626,6 +665,7 @@ extern "C" int efit_table(const efit_ctx* h, int which, const void** d_ptr) {
         case 1: *d_ptr = c.Gd; break;
         case 2: *d_ptr = c.inlim; break;
         case 3: *d_ptr = c.Tedge; break;
+        case 4: *d_ptr = c.U; break;
         default: return fail(nullptr, EFIT_E_INVAL, "which = %d", which);
     }
     if (!*d_ptr) return fail(nullptr, EFIT_E_STATE, "table %d not built in this mode", which);

@@ -36,51 +36,58 @@ __device__ __forceinline__ double grid_coord(double lo, int i, double d) {
 // (~ulp(a)) moves S1 by < 1e-16 relative because c_n^2 <= c_1^4/16.  The loop stops once the
 // increment 2^(n-1) c_n^2 no longer changes S1 (quadratic convergence: <= 6 iterations for
 // m1 >= 1e-9, the cap covers m1 >= 1e-15).
+// Every operation below is an explicit IEEE intrinsic (no FMA contraction left to the compiler),
+// so a Green's value is the same bits in every kernel that evaluates it: the table builds and the
+// on-the-fly kernels agree bit for bit by construction.
 __device__ __forceinline__ void agm_ks1(double m, double m1, double& K, double& S1) {
-    double b = sqrt(m1);
-    double c = m / (2.0 * (1.0 + b));  // c1
-    double a = 0.5 * (1.0 + b);        // a1
-    b = sqrt(b);                       // b1 = sqrt(a0 b0) = sqrt(sqrt(m1))
-    double s = c * c;                  // 2^0 c1^2
+    double b = __dsqrt_rn(m1);
+    double c = __ddiv_rn(m, __dmul_rn(2.0, __dadd_rn(1.0, b)));  // c1
+    double a = __dmul_rn(0.5, __dadd_rn(1.0, b));                // a1
+    b = __dsqrt_rn(b);                                           // b1 = sqrt(a0 b0) = sqrt(sqrt(m1))
+    double s = __dmul_rn(c, c);                                  // 2^0 c1^2
     double p = 1.0;
 #pragma unroll 1
     for (int n = 1; n < kAgmIters; ++n) {
-        c = 0.5 * (a - b);             // c_{n+1}
-        const double an = 0.5 * (a + b);
-        b = sqrt(a * b);
+        c = __dmul_rn(0.5, __dsub_rn(a, b));                     // c_{n+1}
+        const double an = __dmul_rn(0.5, __dadd_rn(a, b));
+        b = __dsqrt_rn(__dmul_rn(a, b));
         a = an;
-        p *= 2.0;
-        const double t = p * c * c;
-        const double s2 = s + t;
-        if (s2 == s) break;            // converged (also covers c == 0)
+        p = __dmul_rn(p, 2.0);
+        const double t = __dmul_rn(__dmul_rn(p, c), c);
+        const double s2 = __dadd_rn(s, t);
+        if (s2 == s) break;                                      // converged (also covers c == 0)
         s = s2;
     }
-    K = kPi / (2.0 * a);
+    K = __ddiv_rn(kPi, __dmul_rn(2.0, a));
     S1 = s;
 }
 
 // Flux per radian at (R, Z) from a 1 A filament at (Rs, Zs):
 //   G = (mu0/2pi) sqrt((R+Rs)^2 + dz^2) [(1 - m/2) K(m) - E(m)],  m = 4 R Rs / den.
 __device__ __forceinline__ double green_psi(double R, double Z, double Rs, double Zs) {
-    double dz = Z - Zs;
-    double dz2 = dz * dz;
-    double sp = R + Rs, sm = R - Rs;
-    double den = sp * sp + dz2;
-    double inv = 1.0 / den;
-    double m = 4.0 * R * Rs * inv;
-    double m1 = (sm * sm + dz2) * inv;
+    const double dz = __dsub_rn(Z, Zs);
+    const double dz2 = __dmul_rn(dz, dz);
+    const double sp = __dadd_rn(R, Rs), sm = __dsub_rn(R, Rs);
+    const double den = __fma_rn(sp, sp, dz2);
+    const double inv = __ddiv_rn(1.0, den);
+    const double m = __dmul_rn(__dmul_rn(__dmul_rn(4.0, R), Rs), inv);
+    const double m1 = __dmul_rn(__fma_rn(sm, sm, dz2), inv);
     double K, S1;
     agm_ks1(m, m1, K, S1);
-    return kMu0Over2Pi * sqrt(den) * K * S1;
+    return __dmul_rn(__dmul_rn(__dmul_rn(kMu0Over2Pi, __dsqrt_rn(den)), K), S1);
 }
 
 // Self term: point-to-cell average of (mu0/2pi) R (ln(8R/rho) - 2) over a dR x dZ cell
 // (reading Q5).
 __device__ __forceinline__ double green_self(double R, double dR, double dZ) {
-    double p = 0.5 * dR, q = 0.5 * dZ;
-    double lnrho = (p * q * log(p * p + q * q) - 3.0 * p * q + p * p * atan(q / p) + q * q * atan(p / q))
-                   / (2.0 * p * q);
-    return kMu0Over2Pi * R * (log(8.0 * R) - lnrho - 2.0);
+    const double p = __dmul_rn(0.5, dR), q = __dmul_rn(0.5, dZ);
+    const double pq = __dmul_rn(p, q), p2 = __dmul_rn(p, p), q2 = __dmul_rn(q, q);
+    double num = __dmul_rn(pq, log(__dadd_rn(p2, q2)));
+    num = __dsub_rn(num, __dmul_rn(3.0, pq));
+    num = __dadd_rn(num, __dmul_rn(p2, atan(__ddiv_rn(q, p))));
+    num = __dadd_rn(num, __dmul_rn(q2, atan(__ddiv_rn(p, q))));
+    const double lnrho = __ddiv_rn(num, __dmul_rn(2.0, pq));
+    return __dmul_rn(__dmul_rn(kMu0Over2Pi, R), __dsub_rn(__dsub_rn(log(__dmul_rn(8.0, R)), lnrho), 2.0));
 }
 
 // Field of a 1 A filament at (Rs, Zs) measured at (R, Z) (Smythe; a = Rs, z = Z - Zs):

@@ -9,6 +9,7 @@
 namespace efit {
 
 constexpr int kMaxBasis = 24;
+constexpr int kNumSMs = 148;  // B200 (sm_100a): grid sizing in multiples of the SM count
 constexpr int kMaxKnots = 20;
 constexpr int kMaxN = 2049;  // FFT working set 2.5*M*16 B of shared memory, M = 2(nh-1)
 constexpr int kLsqMaxRowsHost = 960;  // k_lsq shared memory: (nb|1 + 2)*nd doubles
@@ -33,6 +34,9 @@ struct Tiling {
     // left/right boundary: lr_jt targets per lane (odd), j-tiles of 32*lr_jt targets, 4 source
     // rows per CTA (lr_nblk blocks), source loop padded to lr_jj = roundup(nh, lr_jt)
     int lr_jt, lr_njt, lr_iib, lr_nblk, lr_jj;
+    // symmetric (SYM-mode) top/bottom: 8 x 8 row-pair tiles, m split into sym_nmc chunks of
+    // <= sym_mc values (the staged source columns and target rows fit 2 CTAs per SM)
+    int sym_nmc, sym_mc;
     // normalisation / eps reductions
     int red_blocks;
 };
@@ -45,6 +49,10 @@ struct Ctx {
     double knots[kMaxKnots];
     int n_fl, n_mp, n_int, ndiag, n_lim, ip_sign;
     int mode, rank, world;
+    bool sym, otf;               // SYM modes (half table by reciprocity); on-the-fly Green's
+    int sym_nblk;                // 8-row blocks of the ni interior rows
+    long long sym_ntile;         // sym_nblk (sym_nblk + 1) / 2 row-pair tiles (P <= Q)
+    long long sym_tile_lo, sym_tile_hi;  // this rank's tiles
     int n_edge, ni, nmode;       // ni = nw-2 interior rows, nmode = nh-2 sine modes
     int ni_pad;                  // 32 * rows-per-lane: stride of the segment-interleaved Thomas factors
     int fhat_ld;                 // row stride of the mode-major DST coefficients (multiple of 4)
@@ -59,6 +67,11 @@ struct Ctx {
 
     // device pointers carved from the workspace
     double* T;          // [i_hi-i_lo][S]   top/bottom Green's slabs (table mode)
+    double* U;          // [sym_tile_hi-sym_tile_lo][8][nh][8]  SYM half table (table mode)
+    double* sym_part;   // [ni][2][sym_nblk*sym_nmc]  SYM top/bottom partials (slot = block, chunk)
+    double* symq;       // [sym_nblk][2 (I,F)][2 h][nh][2 qh][2]  per-iteration source columns, staged layout
+    double* symp;       // [sym_nblk][2 (I,F)][8][nhp]             per-iteration block rows, 16-B aligned rows
+    int nhp;            // nh rounded up to even (16-byte rows)
     double* Tedge;      // [2][S]           slabs i = 0 and i = nw-1 (left/right)
     double* Gd;         // [m_hi-m_lo][S]   diagnostic Green's rows
     uint8_t* inlim;     // [nw*nh]

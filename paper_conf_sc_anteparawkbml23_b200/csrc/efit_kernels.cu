@@ -82,6 +82,39 @@ __device__ __forceinline__ d4 ld256_stream(const double* p) {
     return v;
 }
 
+// Asynchronous global -> shared copy of one double (cp.async.ca, 8 bytes); ok == false writes 0.
+__device__ __forceinline__ void cp_async8(double* dst, const double* src, bool ok) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(d), "l"(src), "r"(ok ? 8 : 0) : "memory");
+}
+
+// mbarrier + bulk (TMA 1-D) copies global -> shared, completing on the barrier's transaction count.
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n\tfence.mbarrier_init.release.cluster;" ::"r"(smem_u32(bar)),
+                 "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes, unsigned long long* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned phase) {
+    asm volatile("{\n\t.reg .pred p;\n\tWAIT%=:\n\t"
+                 "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+                 "@!p bra WAIT%=;\n\t}" ::"r"(smem_u32(bar)), "r"(phase) : "memory");
+}
+
+__device__ __forceinline__ void cp_async_wait_all() {
+    asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+}
+
 __device__ __forceinline__ d4 lds256(const double* p) {  // two 128-bit shared loads
     const double2 a = reinterpret_cast<const double2*>(p)[0];
     const double2 b = reinterpret_cast<const double2*>(p)[1];
@@ -193,6 +226,42 @@ __global__ void k_green_diag(double* __restrict__ Gd, long long S, int nrows, in
     }
 }
 
+// SYM-mode half table (see the SYM section of the boundary flux below).
+__device__ __forceinline__ void sym_tile_pq(long long t, int& P, int& Q) {
+    int q = (int)((sqrt(8.0 * (double)t + 1.0) - 1.0) * 0.5);
+    while ((long long)(q + 1) * (q + 2) / 2 <= t) ++q;
+    while ((long long)q * (q + 1) / 2 > t) --q;
+    Q = q;
+    P = (int)(t - (long long)q * (q + 1) / 2);
+}
+
+// The one expression both the SYM table build and the SYM on-the-fly kernel evaluate (bitwise
+// identical modes): same arguments as the full table's k_green_slabs entry for target row i.
+__device__ __forceinline__ double sym_entry(int rp, int rq, int m, int ni, double rmin, double dr, double dz) {
+    if (rp >= ni || rq >= ni) return 0.0;
+    const int i = 1 + rp, ii = 1 + rq;
+    const double Ri = grid_coord(rmin, i, dr);
+    return (i == ii && m == 0) ? green_self(Ri, dr, dz)
+                               : green_psi(Ri, __dmul_rn((double)m, dz), grid_coord(rmin, ii, dr), 0.0);
+}
+
+__global__ void k_green_sym(double* __restrict__ U, long long ntile, long long tile_lo, int ni, int nh, double rmin,
+                            double dr, double dz) {
+    const long long tsz = 64LL * nh;
+    const long long total = ntile * tsz;
+    for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < total;
+         e += (long long)gridDim.x * blockDim.x) {
+        const long long tl = e / tsz;
+        const long long rem = e - tl * tsz;
+        const int p = (int)(rem / (8LL * nh));
+        const int rem2 = (int)(rem - (long long)p * 8 * nh);
+        const int m = rem2 >> 3, q = rem2 & 7;
+        int P, Q;
+        sym_tile_pq(tile_lo + tl, P, Q);
+        U[e] = sym_entry(8 * P + p, 8 * Q + q, m, ni, rmin, dr, dz);
+    }
+}
+
 // In-limiter flags: even-odd crossing rule with the fixed formula
 // x = ((r1 - r0) * (Z - z0)) / (z1 - z0) + r0 (reading Q9).
 __global__ void k_inlim(uint8_t* __restrict__ inlim, const double* __restrict__ lim, int n_lim,
@@ -287,6 +356,13 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
     k_green_slabs<<<sms * 8, bs, 0, s>>>(c.Tedge, c.S, 2, 0, nw - 1, nw, nh, c.rmin, c.dr, c.dz);
     if (c.T && c.i_hi > c.i_lo)
         k_green_slabs<<<sms * 16, bs, 0, s>>>(c.T, c.S, c.i_hi - c.i_lo, c.i_lo, 1, nw, nh, c.rmin, c.dr, c.dz);
+    if (c.U) {
+        const long long ntl = c.sym_tile_hi - c.sym_tile_lo;
+        k_green_sym<<<sms * 16, bs, 0, s>>>(c.U, ntl, c.sym_tile_lo, c.ni, nh, c.rmin, c.dr, c.dz);
+    }
+    if (c.sym_part &&
+        (e = cudaMemsetAsync(c.sym_part, 0, sizeof(double) * 2 * (size_t)(c.ni > 0 ? c.ni : 1) * c.sym_nblk * c.t.sym_nmc, s)))
+        return e;
     if (c.m_hi > c.m_lo)
         k_green_diag<<<sms * 16, bs, 0, s>>>(c.Gd, c.S, c.m_hi - c.m_lo, c.m_lo, c.dgeo, c.dkind, nw, nh,
                                               c.rmin, c.dr, c.zmin, c.dz);
@@ -514,7 +590,9 @@ __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ 
             for (int k = 0; k < NB; ++k) {
 #pragma unroll
                 for (int p = 0; p < NP; ++p) {
-                    const double* bk = Bs + k * gc + q0 + 128 * p + 2 * lane;
+                    // gc is a multiple of 128 but not necessarily of 128*NP: positions past the
+                    // chunk read a valid (clamped) slot of Bs and multiply a zero gv
+                    const double* bk = Bs + k * gc + min(q0 + 128 * p, gc - 128) + 2 * lane;
                     const double2 b0 = *reinterpret_cast<const double2*>(bk);
                     const double2 b1 = *reinterpret_cast<const double2*>(bk + 64);
                     const d4 bb{b0.x, b0.y, b1.x, b1.y};
@@ -1209,15 +1287,28 @@ __global__ void __launch_bounds__(256) k_bnd_lr(const double* __restrict__ Tedge
 
 // psi_b in edge order from the partials: one warp per edge target, chunk-fastest partials,
 // fixed lane assignment + butterfly => deterministic and independent of the rank count.
+// SYM mode: top/bottom partials per (target, side, slot) from k_bnd_sym, plus the edge-row sources
+// ii = 0, nw-1 through the edge slabs (reciprocity: T[i][0][m] = Tedge[0][i][m]) for the rank's
+// own target rows [i_lo, i_hi) only, so that a sum over ranks counts them once.
+struct SymReduce {
+    const double* part;   // nullptr: full-table mode
+    int nslot;
+    const double* Tedge;
+    long long S;
+    const double* pc;     // I  (zero-padded pcurr)
+    const double* pf;     // F  (vertically mirrored)
+};
+
 __global__ void k_bnd_reduce(const double* __restrict__ tb_part, int tb_nchunk, const double* __restrict__ lr_part,
                              int lr_nblk, int nw, int nh, int i_lo, int i_hi, int jlo, int jhi,
-                             double* __restrict__ psib) {
+                             double* __restrict__ psib, SymReduce sy) {
     griddep();
     const int n_edge = 2 * nh + 2 * (nw - 2);
     const int p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
     if (p >= n_edge) return;
     const double* src;
     int cnt;
+    double s = 0.0;
     if (p < 2 * nh) {
         const int side = p < nh ? 0 : 1;
         const int j = p - side * nh;
@@ -1228,11 +1319,22 @@ __global__ void k_bnd_reduce(const double* __restrict__ tb_part, int tb_nchunk, 
         const int q = p - 2 * nh;
         const int side = q < nw - 2 ? 0 : 1;
         const int i = q - side * (nw - 2) + 1;
-        if (i < i_lo || i >= i_hi) return;
-        src = tb_part + ((long long)i * 2 + side) * tb_nchunk;
-        cnt = tb_nchunk;
+        if (sy.part) {
+            src = sy.part + ((long long)(i - 1) * 2 + side) * sy.nslot;
+            cnt = sy.nslot;
+            if (i >= i_lo && i < i_hi) {
+                const double* x0 = (side ? sy.pf : sy.pc);
+                const double* x1 = x0 + (long long)(nw - 1) * nh;
+                const double* t0 = sy.Tedge + (long long)i * nh;
+                const double* t1 = t0 + sy.S;
+                for (int m = lane; m < nh; m += 32) s = fma(t0[m], x0[m], fma(t1[m], x1[m], s));
+            }
+        } else {
+            if (i < i_lo || i >= i_hi) return;
+            src = tb_part + ((long long)i * 2 + side) * tb_nchunk;
+            cnt = tb_nchunk;
+        }
     }
-    double s = 0.0;
     for (int c = lane; c < cnt; c += 32) s += src[c];
     s = warp_sum(s);
     if (lane == 0) psib[p] = s;
@@ -1308,6 +1410,278 @@ __global__ void __launch_bounds__(256) k_bnd_tb_otf(int row_lo, int nslab, int n
     }
 }
 
+// ------------------------------------------------------------ symmetric (SYM-mode) top/bottom
+//
+// Reciprocity G(R_i, z; R_ii, 0) = G(R_ii, z; R_i, 0) (pinned in the oracle tests)
+// makes the top/bottom table symmetric in the row pair: T[i][ii][m] = T[ii][i][m].  Only the
+// interior pairs with i <= ii are stored, blocked into 8 x 8 row-pair tiles (P <= Q of the 8-row
+// blocks of the interior index r = i - 1), tile t = Q(Q+1)/2 + P, entry [p][m][q] (q fastest):
+//   U_t[p][m][q] = G(R_i, m dZ; R_ii, 0),  i = 1 + 8P + p,  ii = 1 + 8Q + q  (0 outside).
+// One streamed entry serves both directions of the pair:
+//   row   target i  (bottom, top) += U I[ii][m],  U F[ii][m]     (sources ii of block Q)
+//   col   target ii (bottom, top) += U I[i][m],   U F[i][m]      (sources i of block P; P < Q only)
+// so every top/bottom Green's byte crosses HBM half as often as in the full-table nest.  The
+// edge-row sources ii = 0, nw-1 come from the (replicated) edge slabs in the reduce kernel.
+
+// CTA (4 warps) = one tile x one m-chunk.  Warp w streams rows p = w and w + 4 of the tile ([m][q],
+// 2 x 32-byte vectors per m: lane l takes vector v = l + 32k of each row, i.e. m = m0 + (v >> 1) and
+// q = 4 (l & 1) .. +3, fixed per lane), so every staged source-column value it reads serves two
+// table rows.  Shared memory holds the chunk's source columns I^T (and F^T) of block Q as two
+// planes of 16-byte pairs (q = 4qh + {0,1} | 4qh + {2,3}; a warp's 128-bit reads are contiguous
+// and conflict-free) and the tile's own rows I[i][m] (and F[i][m]) of block P (col direction; lane
+// pairs read the same word).  MIRROR (one chunk = the whole column): F[ii][m] = I[ii][nh-1-m] is
+// read from the staged I at the mirrored m, halving the staging (65.7 KB at nh = 513 -> 3 CTAs
+// per SM).  The table stream is double-buffered in registers: round k+1's UNR vectors per row and
+// lane are requested before round k is consumed, the first round before the staging (the table is
+// constant, so also before the wait on the predecessor kernel); the staging is asynchronous
+// 8-byte copies, all in flight at once.  Reductions: row direction = warp butterfly; col direction
+// = 16-lane butterfly (lanes with the same q set) + fixed-order sum over the 4 warps.  Partials go
+// to slot (block, chunk) of each target: row direction slot Q, col direction slot P, so every slot
+// of every target is written by exactly one CTA.
+constexpr int kSymThreads = 128;
+
+
+template <bool OTF, bool MIRROR, int UNR, int NBUF>
+__global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __restrict__ U, long long tile_lo, int ni,
+                                                            int nh, int nmc, int mc, const double* __restrict__ symq,
+                                                            const double* __restrict__ symp, int nhp, int nslot,
+                                                            double* __restrict__ part, double rmin, double dr,
+                                                            double dz) {
+    extern __shared__ __align__(16) double xs[];
+    __shared__ double red[4][16];
+    __shared__ __align__(8) unsigned long long bar;
+    if (threadIdx.x == 0) mbar_init(&bar, 1);
+    __syncthreads();
+    const int tl = blockIdx.x / nmc, mch = blockIdx.x - tl * nmc;
+    int P, Q;
+    sym_tile_pq(tile_lo + tl, P, Q);
+    const bool diag = P == Q;  // diagonal tile: stored in full, row direction only
+    const int m0 = mch * mc, mlen = min(mc, nh - m0);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, qh = lane & 1;
+    const int rp0 = 8 * P + warp, rp1 = rp0 + 4;
+    const int nvec = 2 * mlen;
+    const double* tp0 = OTF ? nullptr : U + ((long long)tl * 64 + (long long)warp * 8) * nh + 8LL * m0;
+    const double* tp1 = OTF ? nullptr : tp0 + 32LL * nh;
+    // Lane addressing: vector v = k0 + 32u + lane of a row sits at tp + 4v; its staged plane
+    // pair index is v itself (m = v >> 1, qh = v & 1); the mirrored plane index is
+    // 2 (nh - 1 - m) + qh = 2 (nh - 1) + 2 qh - v.  Full rounds run without bounds checks.
+    auto load = [&](d4 (&x0)[UNR], d4 (&x1)[UNR], int k0, bool tail) {
+#pragma unroll
+        for (int u = 0; u < UNR; ++u) {
+            const int v = k0 + 32 * u + lane;
+            const bool ok = !tail || v < nvec;
+            if (OTF) {
+                double a4[4], b4[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const int rq = 8 * Q + 4 * qh + j, m = m0 + (v >> 1);
+                    a4[j] = ok ? sym_entry(rp0, rq, m, ni, rmin, dr, dz) : 0.0;
+                    b4[j] = ok ? sym_entry(rp1, rq, m, ni, rmin, dr, dz) : 0.0;
+                }
+                x0[u] = d4{a4[0], a4[1], a4[2], a4[3]};
+                x1[u] = d4{b4[0], b4[1], b4[2], b4[3]};
+            } else if (!tail) {
+                x0[u] = ld256_stream(tp0 + 4 * (k0 + lane) + 128 * u);
+                x1[u] = ld256_stream(tp1 + 4 * (k0 + lane) + 128 * u);
+            } else {
+                x0[u] = ok ? ld256_stream(tp0 + 4 * v) : d4{0.0, 0.0, 0.0, 0.0};
+                x1[u] = ok ? ld256_stream(tp1 + 4 * v) : d4{0.0, 0.0, 0.0, 0.0};
+            }
+        }
+    };
+    constexpr int kStep = 32 * UNR;
+    const int nfull = nvec / kStep;          // rounds without a bounds check
+    const int nround = (nvec + kStep - 1) / kStep;
+    d4 tv[NBUF][2][UNR];  // ring of NBUF rounds: NBUF - 1 rounds stay in flight while one is consumed
+#pragma unroll
+    for (int b = 0; b + 1 < NBUF; ++b)
+        if (b < nround) load(tv[b][0], tv[b][1], b * kStep, b >= nfull);
+    griddep();
+    // staged layout: xqi planes [2][mc][2][2] | (xqf planes) | xpi rows [8][ms] | (xpf rows [8][ms]),
+    // copied from the per-iteration packed arrays (k_sym_pack) by bulk (TMA 1-D) copies issued by
+    // one thread and completing on an mbarrier: no per-element staging instructions
+    const int ms = MIRROR ? nhp : mc;  // staged row stride of the block-P rows
+    const int ps = MIRROR ? nh : mc;   // staged plane length (m values)
+    double* xqi = xs;
+    double* xqf = MIRROR ? xs : xs + 8 * mc;
+    double* xpi = xs + 8 * ps * (MIRROR ? 1 : 2);
+    double* xpf = MIRROR ? xpi : xpi + 8 * ms;
+    if (threadIdx.x == 0) {
+        const double* q0 = symq + (size_t)Q * 16 * nh;   // [arr][h][nh][2][2]
+        const double* p0 = symp + (size_t)P * 16 * nhp;  // [arr][8][nhp]
+        if (MIRROR) {
+            mbar_expect_tx(&bar, (unsigned)(sizeof(double) * (8 * nh + 8 * nhp)));
+            bulk_g2s(xqi, q0, (unsigned)(sizeof(double) * 8 * nh), &bar);
+            bulk_g2s(xpi, p0, (unsigned)(sizeof(double) * 8 * nhp), &bar);
+        } else {
+            const int ml2 = (mlen + 1) & ~1;  // rows are zero-padded to nhp
+            mbar_expect_tx(&bar, (unsigned)(sizeof(double) * (2 * 2 * 4 * mlen + 2 * 8 * ml2)));
+#pragma unroll 1
+            for (int arr = 0; arr < 2; ++arr) {
+                double* dq = arr ? xqf : xqi;
+                double* dp = arr ? xpf : xpi;
+                for (int h = 0; h < 2; ++h)
+                    bulk_g2s(dq + h * 4 * mc, q0 + (size_t)arr * 8 * nh + (size_t)h * 4 * nh + 4 * m0,
+                             (unsigned)(sizeof(double) * 4 * mlen), &bar);
+                for (int r8 = 0; r8 < 8; ++r8)
+                    bulk_g2s(dp + r8 * ms, p0 + (size_t)arr * 8 * nhp + (size_t)r8 * nhp + m0,
+                             (unsigned)(sizeof(double) * ml2), &bar);
+            }
+        }
+    }
+    mbar_wait(&bar, 0);
+    const double* xpi0 = xpi + warp * ms;
+    const double* xpf0 = xpf + warp * ms;
+    const double* xpi1 = xpi0 + 4 * ms;
+    const double* xpf1 = xpf0 + 4 * ms;
+    const double2* pi0 = reinterpret_cast<const double2*>(xqi);           // q pairs 4qh + {0,1}
+    const double2* pi1 = reinterpret_cast<const double2*>(xqi + 4 * ps);  // q pairs 4qh + {2,3}
+    const double2* pf0 = reinterpret_cast<const double2*>(xqf);
+    const double2* pf1 = reinterpret_cast<const double2*>(xqf + 4 * ps);
+    const int wfb = MIRROR ? 2 * (nh - 1) + 2 * qh : 0;   // mirrored plane index = wfb - v
+    double arI0 = 0.0, arF0 = 0.0, arI1 = 0.0, arF1 = 0.0, acI[4], acF[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) { acI[j] = 0.0; acF[j] = 0.0; }
+    auto compute = [&](const d4 (&x0)[UNR], const d4 (&x1)[UNR], int k0, bool tail) {
+        // round base pointers; the u-th vector is at a compile-time offset from them
+        const int kl = k0 + lane;
+        const double2* ai = pi0 + kl;
+        const double2* bi = pi1 + kl;
+        const double2* cf = pf0 + (MIRROR ? wfb - kl : kl);
+        const double2* df = pf1 + (MIRROR ? wfb - kl : kl);
+        const int ml = kl >> 1;
+        const double* pI0 = xpi0 + ml;
+        const double* pI1 = xpi1 + ml;
+        const double* pF0 = xpf0 + (MIRROR ? nh - 1 - ml : ml);
+        const double* pF1 = xpf1 + (MIRROR ? nh - 1 - ml : ml);
+        constexpr int sgn = MIRROR ? -1 : 1;
+#pragma unroll
+        for (int u = 0; u < UNR; ++u) {
+            double2 a, b, c, d;
+            double i0, i1, f0, f1;
+            if (!tail) {
+                a = ai[32 * u]; b = bi[32 * u]; c = cf[sgn * 32 * u]; d = df[sgn * 32 * u];
+                i0 = pI0[16 * u]; i1 = pI1[16 * u]; f0 = pF0[sgn * 16 * u]; f1 = pF1[sgn * 16 * u];
+            } else {  // x = 0 past the end: read any valid slot
+                const int v = min(k0 + 32 * u + lane, nvec - 2 + qh);  // keeps the parity (= qh)
+                const int mm = v >> 1, wf = MIRROR ? wfb - v : v, mf = MIRROR ? nh - 1 - mm : mm;
+                a = pi0[v]; b = pi1[v]; c = pf0[wf]; d = pf1[wf];
+                i0 = xpi0[mm]; i1 = xpi1[mm]; f0 = xpf0[mf]; f1 = xpf1[mf];
+            }
+            const d4 xi{a.x, a.y, b.x, b.y}, xf{c.x, c.y, d.x, d.y};
+            arI0 = dot4(x0[u], xi, arI0);
+            arF0 = dot4(x0[u], xf, arF0);
+            arI1 = dot4(x1[u], xi, arI1);
+            arF1 = dot4(x1[u], xf, arF1);
+            acI[0] = fma(x1[u].x, i1, fma(x0[u].x, i0, acI[0]));
+            acI[1] = fma(x1[u].y, i1, fma(x0[u].y, i0, acI[1]));
+            acI[2] = fma(x1[u].z, i1, fma(x0[u].z, i0, acI[2]));
+            acI[3] = fma(x1[u].w, i1, fma(x0[u].w, i0, acI[3]));
+            acF[0] = fma(x1[u].x, f1, fma(x0[u].x, f0, acF[0]));
+            acF[1] = fma(x1[u].y, f1, fma(x0[u].y, f0, acF[1]));
+            acF[2] = fma(x1[u].z, f1, fma(x0[u].z, f0, acF[2]));
+            acF[3] = fma(x1[u].w, f1, fma(x0[u].w, f0, acF[3]));
+        }
+    };
+    // round r is consumed from buffer r % NBUF after round r + NBUF - 1 has been requested into the
+    // buffer freed by round r - 1
+#pragma unroll 1
+    for (int r0 = 0; r0 < nround; r0 += NBUF) {
+#pragma unroll
+        for (int b = 0; b < NBUF; ++b) {
+            const int r = r0 + b;
+            if (r >= nround) break;
+            const int rn = r + NBUF - 1;
+            if (rn < nround) load(tv[(b + NBUF - 1) % NBUF][0], tv[(b + NBUF - 1) % NBUF][1], rn * kStep, rn >= nfull);
+            compute(tv[b][0], tv[b][1], r * kStep, r >= nfull);
+        }
+    }
+    arI0 = warp_sum(arI0);
+    arF0 = warp_sum(arF0);
+    arI1 = warp_sum(arI1);
+    arF1 = warp_sum(arF1);
+    if (lane == 0) {
+        const int slot = Q * nmc + mch;
+        if (rp0 < ni) {
+            part[((long long)rp0 * 2 + 0) * nslot + slot] = arI0;
+            part[((long long)rp0 * 2 + 1) * nslot + slot] = arF0;
+        }
+        if (rp1 < ni) {
+            part[((long long)rp1 * 2 + 0) * nslot + slot] = arI1;
+            part[((long long)rp1 * 2 + 1) * nslot + slot] = arF1;
+        }
+    }
+    if (!diag) {  // CTA-uniform
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            double a = acI[j], b = acF[j];
+#pragma unroll
+            for (int o = 2; o < 32; o <<= 1) {
+                a += __shfl_xor_sync(0xffffffffu, a, o);
+                b += __shfl_xor_sync(0xffffffffu, b, o);
+            }
+            if (lane < 2) {
+                const int q = 4 * lane + j;
+                red[warp][2 * q] = a;
+                red[warp][2 * q + 1] = b;
+            }
+        }
+        __syncthreads();
+        if (threadIdx.x < 16) {
+            const int q = threadIdx.x >> 1, side = threadIdx.x & 1, rq = 8 * Q + q;
+            double s = 0.0;
+#pragma unroll
+            for (int w = 0; w < 4; ++w) s += red[w][threadIdx.x];
+            if (rq < ni) part[((long long)rq * 2 + side) * nslot + P * nmc + mch] = s;
+        }
+    }
+}
+
+static size_t sym_smem(const Ctx& c) {
+    return sizeof(double) * (c.t.sym_nmc == 1 ? 8 * (size_t)c.nh + 8 * (size_t)c.nhp : 32 * (size_t)c.t.sym_mc);
+}
+
+// Per-iteration packing of the current pair into the layouts k_bnd_sym stages with bulk copies:
+//   symq[B][arr][h][m][qh][w] = X_arr[1 + 8B + q][m],  q = 4 qh + 2 h + w  (0 past the interior)
+//   symp[B][arr][p][m]        = X_arr[1 + 8B + p][m]   (rows padded to nhp, 0 past the interior)
+// X_0 = I (pcurr), X_1 = F (pflip); narr = 1 when F is read mirrored from I.
+__global__ void k_sym_pack(const double* __restrict__ I, const double* __restrict__ F, int nh, int nhp, int ni,
+                           int nblk, int narr, double* __restrict__ symq, double* __restrict__ symp) {
+    griddep();
+    const long long nq = 16LL * nh, np = 16LL * nhp;  // per block, both arrays
+    const long long total = (long long)nblk * (nq + np);
+    for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < total;
+         e += (long long)gridDim.x * blockDim.x) {
+        if (e < (long long)nblk * nq) {
+            const int B = (int)(e / nq);
+            const int rem = (int)(e - (long long)B * nq);
+            const int arr = rem / (8 * nh);
+            if (arr >= narr) continue;
+            const int r2 = rem - arr * 8 * nh, h = r2 / (4 * nh), r3 = r2 - h * 4 * nh;
+            const int m = r3 >> 2, qh = (r3 >> 1) & 1, w = r3 & 1, q = 4 * qh + 2 * h + w, r = 8 * B + q;
+            symq[e] = r < ni ? (arr ? F : I)[(long long)(1 + r) * nh + m] : 0.0;
+        } else {
+            const long long e2 = e - (long long)nblk * nq;
+            const int B = (int)(e2 / np);
+            const int rem = (int)(e2 - (long long)B * np);
+            const int arr = rem / (8 * nhp);
+            if (arr >= narr) continue;
+            const int r2 = rem - arr * 8 * nhp, p = r2 / nhp, m = r2 - p * nhp, r = 8 * B + p;
+            symp[e2] = (r < ni && m < nh) ? (arr ? F : I)[(long long)(1 + r) * nh + m] : 0.0;
+        }
+    }
+}
+
+// table vectors per row and lane per round, rounds in the register ring (EFIT_SYM_UNR/BUF
+// override at build time for tuning)
+#ifndef EFIT_SYM_UNR
+#define EFIT_SYM_UNR 2
+#endif
+#ifndef EFIT_SYM_BUF
+#define EFIT_SYM_BUF 3
+#endif
+constexpr int kSymUnr = EFIT_SYM_UNR, kSymBuf = EFIT_SYM_BUF;
+
 constexpr int kTbGI = 8;
 constexpr int kTbUnroll = 4;
 
@@ -1359,9 +1733,36 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     if ((e = cudaEventRecord(c.ev_join, c.side))) return e;
     const int nslab = c.i_hi - c.i_lo;
     const size_t smem_tb = 2 * sizeof(double) * c.t.tb_ch;
-    if (nslab > 0) {
+    SymReduce sy{nullptr, 0, c.Tedge, c.S, c.pcurr, c.pflip};
+    if (c.sym) {
+        sy.part = c.sym_part;
+        sy.nslot = c.sym_nblk * c.t.sym_nmc;
+        const long long ntl = c.sym_tile_hi - c.sym_tile_lo;
+        if (ntl > 0) {
+            const int narr = c.t.sym_nmc == 1 ? 1 : 2;
+            launch_pdl(k_sym_pack, dim3(4 * kNumSMs), dim3(256), 0, s, (const double*)c.pcurr, (const double*)c.pflip,
+                       c.nh, c.nhp, c.ni, c.sym_nblk, narr, c.symq, c.symp);
+            if ((e = cudaGetLastError())) return e;
+            const size_t smem = sym_smem(c);
+            const bool mir = c.t.sym_nmc == 1;
+            const dim3 grid((unsigned)(ntl * c.t.sym_nmc));
+#define EFIT_SYM_LAUNCH(OTFV, MIRV, UNRV, NBV)                                                                      \
+    launch_pdl(k_bnd_sym<OTFV, MIRV, UNRV, NBV>, grid, dim3(kSymThreads), smem, s, (const double*)c.U, c.sym_tile_lo,  \
+               c.ni, c.nh, c.t.sym_nmc, c.t.sym_mc, (const double*)c.symq, (const double*)c.symp, c.nhp, sy.nslot, \
+               c.sym_part, c.rmin, c.dr, c.dz)
+            if (c.otf) {  // FP64-bound: a short unroll keeps the inlined AGM in registers
+                if (mir) EFIT_SYM_LAUNCH(true, true, 1, 2); else EFIT_SYM_LAUNCH(true, false, 1, 2);
+            } else if (mir) {
+                EFIT_SYM_LAUNCH(false, true, kSymUnr, kSymBuf);
+            } else {
+                EFIT_SYM_LAUNCH(false, false, kSymUnr, kSymBuf);
+            }
+#undef EFIT_SYM_LAUNCH
+            if ((e = cudaGetLastError())) return e;
+        }
+    } else if (nslab > 0) {
         dim3 grid(c.t.tb_nchunk, c.t.tb_ngroup);
-        if (c.mode == EFIT_GREEN_TABLE) {
+        if (!c.otf) {
             launch_pdl(k_bnd_tb<kTbGI, kTbUnroll>, dim3(grid), dim3(256), smem_tb, s, c.T, c.S, nslab, c.i_lo, c.nw * c.nh, c.pcurr,
                                                                   c.pflip, c.t.tb_ch, c.tb_part);
         } else {
@@ -1376,7 +1777,7 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     const int jlo = c.lr_direct ? c.jt_lo * 32 * c.t.lr_jt : 0;
     const int jhi = c.lr_direct ? min(c.nh, c.jt_hi * 32 * c.t.lr_jt) : 0;
     launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, c.tb_part, c.t.tb_nchunk, c.lr_part, c.t.lr_nblk, c.nw, c.nh,
-                                                    c.i_lo, c.i_hi, jlo, jhi, psib);
+                                                    c.i_lo, c.i_hi, jlo, jhi, psib, sy);
     return cudaGetLastError();
 }
 
@@ -2084,6 +2485,14 @@ cudaError_t prepare_kernels(Ctx& c) {
     if ((e = prepare_lr_fft(c))) return e;
     if ((e = big((const void*)k_bnd_tb<kTbGI, kTbUnroll>, 2 * sizeof(double) * c.t.tb_ch))) return e;
     if ((e = big((const void*)k_bnd_tb_otf<kTbGI>, 2 * sizeof(double) * c.t.tb_ch))) return e;
+    {
+        const size_t sm = sym_smem(c);
+        const void* ks[4] = {(const void*)k_bnd_sym<false, true, kSymUnr, kSymBuf>,
+                             (const void*)k_bnd_sym<false, false, kSymUnr, kSymBuf>,
+                             (const void*)k_bnd_sym<true, true, 1, 2>, (const void*)k_bnd_sym<true, false, 1, 2>};
+        for (const void* f : ks)
+            if ((e = big(f, sm))) return e;
+    }
     {
         int fpc, threads;
         size_t smem;

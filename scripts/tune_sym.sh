@@ -1,0 +1,5 @@
+# time the sym-mode fit step with each tuning variant in tune/
+mkdir -p gpurun_out
+for L in tune/libefit_*.so; do
+  EFIT_B200_LIB=$PWD/$L timeout 300 python bench.py --steps 1000 --warmup 20 --no-cpu-baseline --no-e2e --mode sym 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('$L', d['value'], d['config']['step_breakdown_us']['bnd_tb'], d['roofline']['achieved'])" || echo "$L failed"
+done

@@ -233,12 +233,14 @@ def perturbed_psi(grid: Grid, seed: int = 5, rel: float = 1e-3) -> np.ndarray:
     return ps + rel * span * smooth_modes(grid, seed) / 3.0
 
 
-def random_current(grid: Grid, seed: int = 2, signed: bool = False) -> np.ndarray:
-    """I ~ U(0,1) (or U(-1,1) if signed) on interior nodes, 0 on the edge ring."""
+def random_current(grid: Grid, seed: int = 2, signed: bool = False, edge: bool = False) -> np.ndarray:
+    """I ~ U(0,1) (or U(-1,1) if signed) on interior nodes, 0 on the edge ring (edge=True:
+    on every node, the edge ring included -- exercises the edge-row sources)."""
     rng = np.random.default_rng(seed)
     lo = -1.0 if signed else 0.0
     I = rng.uniform(lo, 1.0, size=(grid.nw, grid.nh))
-    I[0, :] = 0.0; I[-1, :] = 0.0; I[:, 0] = 0.0; I[:, -1] = 0.0
+    if not edge:
+        I[0, :] = 0.0; I[-1, :] = 0.0; I[:, 0] = 0.0; I[:, -1] = 0.0
     return I.reshape(-1)
 
 

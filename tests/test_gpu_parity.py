@@ -165,15 +165,102 @@ def test_current(torch_mod, efit, orc_mod, name):
 
 # ------------------------------------------------------------------ a6: boundary flux
 
-@pytest.mark.parametrize("name", ["9x9", "33x33", "40x33", "65x65", "C2"])
+@pytest.mark.parametrize("name", ["9x9", "33x33", "40x33", "65x65", "C2", "21x1025"])
 @pytest.mark.parametrize("signed", [False, True])
-def test_boundary_flux(torch_mod, efit, orc_mod, name, signed):
+@pytest.mark.parametrize("mode", [0, 2])  # EFIT_GREEN_TABLE, EFIT_GREEN_TABLE_SYM (21x1025: m-chunked path)
+def test_boundary_flux(torch_mod, efit, orc_mod, name, signed, mode):
     torch = torch_mod
-    c = case(name, efit, orc_mod)
+    c = case(name, efit, orc_mod, mode=mode)
     I = synth.random_current(c.cfg.grid, seed=3 if signed else 2, signed=signed)
     ref = c.orc.boundary(I)
     out = c.ctx.boundary_flux(T(torch, I)).cpu().numpy()
     assert rel(out, ref) < TOL, rel(out, ref)
+
+
+@pytest.mark.parametrize("name", ["9x9", "33x33", "40x33", "21x1025"])
+@pytest.mark.parametrize("mode", [0, 2, 3])
+def test_boundary_flux_edge_sources(torch_mod, efit, orc_mod, name, mode):
+    """Current on every node, the edge ring included: the edge-row sources (ii = 0, nw-1; in SYM
+    mode taken from the edge slabs by reciprocity) and the self terms of edge targets."""
+    torch = torch_mod
+    c = case(name, efit, orc_mod, mode=mode)
+    I = synth.random_current(c.cfg.grid, seed=6, signed=True, edge=True)
+    ref = c.orc.boundary(I)
+    out = c.ctx.boundary_flux(T(torch, I)).cpu().numpy()
+    assert rel(out, ref) < TOL, rel(out, ref)
+
+
+@pytest.mark.parametrize("name", ["9x9", "33x33", "40x33", "65x65"])
+def test_green_sym_table(torch_mod, efit, orc_mod, name):
+    """SYM half table (include/efit.h, efit_table which = 4): tile t = Q(Q+1)/2 + P, entry
+    [p][m][q] = T[1+8P+p][1+8Q+q][m] of the oracle's table, 0 outside the interior rows."""
+    torch = torch_mod
+    c = case(name, efit, orc_mod, mode=efit.EFIT_GREEN_TABLE_SYM)
+    nw, nh = c.cfg.grid.nw, c.cfg.grid.nh
+    ni = nw - 2
+    nblk = c.ctx.info.sym_nblk
+    assert nblk == (ni + 7) // 8
+    ntile = nblk * (nblk + 1) // 2
+    assert (c.ctx.info.sym_tile_lo, c.ctx.info.sym_tile_hi) == (0, ntile)
+    U = _device_view(torch, c.ctx.table_ptr(4), ntile * 64 * nh).view(ntile, 8, nh, 8).cpu().numpy()
+    Tref = c.orc.table_T()
+    ref = np.zeros_like(U)
+    t = 0
+    for Q in range(nblk):
+        for P in range(Q + 1):
+            for p in range(8):
+                for q in range(8):
+                    rp, rq = 8 * P + p, 8 * Q + q
+                    if rp < ni and rq < ni:
+                        ref[t, p, :, q] = Tref[1 + rp, 1 + rq, :]
+            t += 1
+    nz = ref != 0
+    assert np.array_equal(U != 0, nz)
+    assert np.max(np.abs(U[nz] - ref[nz]) / np.abs(ref[nz])) < 1e-12
+
+
+def test_boundary_sym_onthefly_bitwise(torch_mod, efit, orc_mod):
+    torch = torch_mod
+    a = case("65x65", efit, orc_mod, mode=efit.EFIT_GREEN_TABLE_SYM)
+    b = case("65x65", efit, orc_mod, mode=efit.EFIT_GREEN_ONTHEFLY_SYM)
+    I = T(torch, synth.random_current(a.cfg.grid, seed=3, signed=True, edge=True))
+    assert torch.equal(a.ctx.boundary_flux(I), b.ctx.boundary_flux(I))
+
+
+def test_boundary_sym_matches_full_table(torch_mod, efit, orc_mod):
+    """Reciprocity: the half-table nest equals the full-table nest to rounding."""
+    torch = torch_mod
+    a = case("C2", efit, orc_mod)
+    b = case("C2", efit, orc_mod, mode=efit.EFIT_GREEN_TABLE_SYM)
+    I = T(torch, synth.random_current(a.cfg.grid, seed=2))
+    x, y = a.ctx.boundary_flux(I).cpu().numpy(), b.ctx.boundary_flux(I).cpu().numpy()
+    assert rel(y, x) < 1e-14
+
+
+def test_sym_sharded_sum_matches_single(torch_mod, efit, orc_mod):
+    """SYM mode, world = 3 emulated on one GPU: each rank streams its share of the row-pair tiles
+    and writes partial sums for every top/bottom target (and its own left/right targets); the
+    sum over ranks (the caller's all-reduce) equals world = 1 to rounding."""
+    torch = torch_mod
+    c1 = case("65x65", efit, orc_mod, mode=efit.EFIT_GREEN_TABLE_SYM)
+    cfg = c1.cfg
+    I = T(torch, synth.random_current(cfg.grid, seed=3, signed=True, edge=True))
+    psib1 = c1.ctx.boundary_flux(I)
+    acc = torch.zeros_like(psib1)
+    world = 3
+    tiles = []
+    for r in range(world):
+        ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=efit.EFIT_GREEN_TABLE_SYM, rank=r, world=world)
+        tiles.append((ctx.info.sym_tile_lo, ctx.info.sym_tile_hi))
+        part = torch.zeros_like(psib1)
+        efit.efit_boundary_flux(ctx.handle, I, part)
+        torch.cuda.synchronize()
+        acc += part
+        ctx.close()
+    nblk = c1.ctx.info.sym_nblk
+    assert tiles[0][0] == 0 and tiles[-1][1] == nblk * (nblk + 1) // 2
+    assert all(a[1] == b[0] for a, b in zip(tiles, tiles[1:]))
+    assert rel(acc.cpu().numpy(), psib1.cpu().numpy()) < 1e-14
 
 
 def test_boundary_literal_fig2(torch_mod, efit, orc_mod):
@@ -285,9 +372,10 @@ def _twin(c, noise_seed=1):
 
 
 @pytest.mark.parametrize("name", ["33x33", "C1", "C2"])
-def test_fit_step(torch_mod, efit, orc_mod, name):
+@pytest.mark.parametrize("mode", [0, 2])
+def test_fit_step(torch_mod, efit, orc_mod, name, mode):
     torch = torch_mod
-    c = case(name, efit, orc_mod)
+    c = case(name, efit, orc_mod, mode=mode)
     psi_s, ct, tw = _twin(c)
     psi0 = synth.perturbed_psi(c.cfg.grid, seed=5, rel=1e-3)
     st, psi_ref, cref, chi2ref, epsref = c.orc.fit_step(psi0, tw["psi_ext"], tw["y"], tw["sigma"])
@@ -370,12 +458,14 @@ def c4(efit, orc_mod):
     return case("C4", efit, orc_mod)
 
 
-def test_c4_boundary_sampled(torch_mod, c4):
+@pytest.mark.parametrize("mode", [0, 2])
+def test_c4_boundary_sampled(torch_mod, efit, orc_mod, c4, mode):
     torch = torch_mod
-    I = synth.random_current(c4.cfg.grid, seed=2)
-    out = c4.ctx.boundary_flux(T(torch, I)).cpu().numpy()
+    c = c4 if mode == 0 else case("C4", efit, orc_mod, mode=mode)
+    I = synth.random_current(c.cfg.grid, seed=2)
+    out = c.ctx.boundary_flux(T(torch, I)).cpu().numpy()
     rng = np.random.default_rng(0)
-    tg = np.unique(np.concatenate([[0, 512, 513, 1025, 1026, 1536, 2043], rng.integers(0, c4.ctx.n_edge, 40)]))
+    tg = np.unique(np.concatenate([[0, 512, 513, 1025, 1026, 1536, 2043], rng.integers(0, c.ctx.n_edge, 40)]))
     ref = c4.orc.boundary_targets(I, tg)
     assert rel(out[tg], ref) < TOL
 
