@@ -190,8 +190,8 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     // worth of accumulators) minimising padded rows, then preferring more rows per warp
     int best_mb = 1, best_cost = 1 << 30;
     for (int mb = 4; mb >= 1; --mb) {  // ties -> more rows per warp (more reuse of each basis value)
-        const int np = efit::resp_np(c.nb, mb);                // 256-bit positions per step (k_response)
-        if (8 * np * mb + 2 * mb * c.nb > 112 && mb > 1) continue;  // loads + accumulators under 128 regs
+        const int np = efit::resp_np(c.nb, mb);                // register-ring depth (k_response)
+        if (4 * np * mb + mb * c.nb > 56 && mb > 1) continue;  // ring + accumulators (no spills)
         const int nmb = (nrows + mb - 1) / mb;        // row blocks, dealt round-robin to 8 warps
         int cost = ((nmb + 7) / 8) * mb;               // rows on the busiest warp
         if (cost < best_cost) { best_cost = cost; best_mb = mb; }

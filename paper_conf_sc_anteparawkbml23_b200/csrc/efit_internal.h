@@ -14,10 +14,11 @@ constexpr int kMaxKnots = 20;
 constexpr int kMaxN = 2049;  // FFT working set 2.5*M*16 B of shared memory, M = 2(nh-1)
 constexpr int kLsqMaxRowsHost = 960;  // k_lsq shared memory: (nb|1 + 2)*nd doubles
 
-// k_response: 256-bit positions per step for NB basis functions and MB rows per warp, keeping
-// loads (8*NP*MB regs) + accumulators (2*MB*NB regs) <= 112 of the 128-register budget.
+// k_response: depth of the register ring of MB-row load steps (4 registers per 256-bit load),
+// keeping ring (4 NP MB) + accumulators (MB NB) <= 56 registers (the rest of the 128-register
+// budget goes to addressing and the staged basis vector; larger rings spill), 2 <= NP <= 4.
 __host__ __device__ constexpr int resp_np(int nb, int mb) {
-    return (112 - 2 * mb * nb) / (8 * mb) >= 3 ? 3 : ((112 - 2 * mb * nb) / (8 * mb) >= 1 ? (112 - 2 * mb * nb) / (8 * mb) : 1);
+    return (56 - mb * nb) / (4 * mb) >= 4 ? 4 : ((56 - mb * nb) / (4 * mb) >= 2 ? (56 - mb * nb) / (4 * mb) : 2);
 }
 
 // device status-word bits

@@ -553,10 +553,38 @@ template <int NB, int MB, int NP>
 __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ Gd, long long S, int nrows, int n,
                                                      const double* __restrict__ Bm, long long ldb, int gc,
                                                      double* __restrict__ part) {
+    // NP = rounds of MB row loads kept in a register ring: the warp's (row block, position) steps
+    // form one flat sequence, and step s + NP - 1 is requested before step s is consumed, across
+    // row-block boundaries (the first steps before the basis staging and the predecessor wait:
+    // Gd is constant).
     extern __shared__ __align__(16) double Bs[];  // [NB][gc] permuted
-    griddep();
     const int c = blockIdx.x;
     const int g0 = c * gc;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int qend = min(gc, n - g0);  // valid nodes; a 4-wide load may read up to 3 zero pads
+    const int npos = (qend + 127) >> 7;  // 128-node positions of this chunk
+    const int nmb = (nrows + MB - 1) / MB;
+    const int nwarps = (int)(blockDim.x >> 5);
+    const int nmb_w = warp < nmb ? (nmb - warp + nwarps - 1) / nwarps : 0;  // row blocks warp, warp+8, ...
+    const int nsteps = nmb_w * npos;
+    // the prefetch cursor (row block lj, position lp) runs NP - 1 steps ahead of the consumer
+    int lj = 0, lp = 0;
+    auto load_step = [&](d4 (&x)[MB]) {
+        const int row0 = (warp + lj * nwarps) * MB;
+        const int q = lp * 128 + 4 * lane;
+        if (++lp == npos) { lp = 0; ++lj; }
+        const bool ok = q < qend;
+#pragma unroll
+        for (int r = 0; r < MB; ++r) {
+            const double* rp = Gd + (long long)min(row0 + r, nrows - 1) * S + g0 + q;
+            x[r] = ok ? ld256_stream(rp) : d4{0.0, 0.0, 0.0, 0.0};
+        }
+    };
+    d4 ring[NP][MB];
+#pragma unroll
+    for (int b = 0; b + 1 < NP; ++b)
+        if (b < nsteps) load_step(ring[b]);
+    griddep();
 #pragma unroll
     for (int k = 0; k < NB; ++k)
         for (int q = 2 * threadIdx.x; q < gc; q += 2 * blockDim.x) {
@@ -564,50 +592,41 @@ __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ 
             *reinterpret_cast<double2*>(Bs + k * gc + bperm(q)) = v;
         }
     __syncthreads();
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int qend = min(gc, n - g0);  // valid nodes; a 4-wide load may read up to 3 zero pads
-    const int nmb = (nrows + MB - 1) / MB;
-    for (int mb = warp; mb < nmb; mb += (int)(blockDim.x >> 5)) {  // every row block of the chunk
-        const int row0 = mb * MB;
-        double acc[MB][NB];
+    double acc[MB][NB];
 #pragma unroll
-        for (int r = 0; r < MB; ++r)
+    for (int r = 0; r < MB; ++r)
 #pragma unroll
-            for (int k = 0; k < NB; ++k) acc[r][k] = 0.0;
-        const double* rowp[MB];
+        for (int k = 0; k < NB; ++k) acc[r][k] = 0.0;
+    int pos = 0, j = 0;
+#pragma unroll 1
+    for (int s0 = 0; s0 < nsteps; s0 += NP) {
 #pragma unroll
-        for (int r = 0; r < MB; ++r) rowp[r] = Gd + (long long)min(row0 + r, nrows - 1) * S + g0;
-        for (int q0 = 0; q0 < qend; q0 += 128 * NP) {
-            d4 gv[NP][MB];
-#pragma unroll
-            for (int p = 0; p < NP; ++p) {
-                const int q = q0 + 128 * p + 4 * lane;
-                const bool ok = q < qend;
-#pragma unroll
-                for (int r = 0; r < MB; ++r) gv[p][r] = ok ? ld256_stream(rowp[r] + q) : d4{0.0, 0.0, 0.0, 0.0};
-            }
+        for (int b = 0; b < NP; ++b) {
+            const int st = s0 + b;
+            if (st >= nsteps) break;
+            if (st + NP - 1 < nsteps) load_step(ring[(b + NP - 1) % NP]);
 #pragma unroll
             for (int k = 0; k < NB; ++k) {
+                const double* bk = Bs + k * gc + pos * 128 + 2 * lane;
+                const double2 b0 = *reinterpret_cast<const double2*>(bk);
+                const double2 b1 = *reinterpret_cast<const double2*>(bk + 64);
+                const d4 bb{b0.x, b0.y, b1.x, b1.y};
 #pragma unroll
-                for (int p = 0; p < NP; ++p) {
-                    // gc is a multiple of 128 but not necessarily of 128*NP: positions past the
-                    // chunk read a valid (clamped) slot of Bs and multiply a zero gv
-                    const double* bk = Bs + k * gc + min(q0 + 128 * p, gc - 128) + 2 * lane;
-                    const double2 b0 = *reinterpret_cast<const double2*>(bk);
-                    const double2 b1 = *reinterpret_cast<const double2*>(bk + 64);
-                    const d4 bb{b0.x, b0.y, b1.x, b1.y};
+                for (int r = 0; r < MB; ++r) acc[r][k] = dot4(ring[b][r], bb, acc[r][k]);
+            }
+            if (++pos == npos) {  // row block done: reduce and store its MB x NB partials
+                const int row0 = (warp + j * nwarps) * MB;
 #pragma unroll
-                    for (int r = 0; r < MB; ++r) acc[r][k] = dot4(gv[p][r], bb, acc[r][k]);
+                for (int r = 0; r < MB; ++r) {
+#pragma unroll
+                    for (int k = 0; k < NB; ++k) {
+                        const double v = warp_sum(acc[r][k]);
+                        acc[r][k] = 0.0;
+                        if (lane == 0 && row0 + r < nrows) part[((long long)(row0 + r) * NB + k) * gridDim.x + c] = v;
+                    }
                 }
-            }
-        }
-#pragma unroll
-        for (int r = 0; r < MB; ++r) {
-            const int row = row0 + r;
-#pragma unroll
-            for (int k = 0; k < NB; ++k) {
-                double v = warp_sum(acc[r][k]);
-                if (lane == 0 && row < nrows) part[((long long)row * NB + k) * gridDim.x + c] = v;
+                pos = 0;
+                ++j;
             }
         }
     }
@@ -1423,32 +1442,34 @@ __global__ void __launch_bounds__(256) k_bnd_tb_otf(int row_lo, int nslab, int n
 // so every top/bottom Green's byte crosses HBM half as often as in the full-table nest.  The
 // edge-row sources ii = 0, nw-1 come from the (replicated) edge slabs in the reduce kernel.
 
-// CTA (4 warps) = one tile x one m-chunk.  Warp w streams rows p = w and w + 4 of the tile ([m][q],
-// 2 x 32-byte vectors per m: lane l takes vector v = l + 32k of each row, i.e. m = m0 + (v >> 1) and
-// q = 4 (l & 1) .. +3, fixed per lane), so every staged source-column value it reads serves two
-// table rows.  Shared memory holds the chunk's source columns I^T (and F^T) of block Q as two
-// planes of 16-byte pairs (q = 4qh + {0,1} | 4qh + {2,3}; a warp's 128-bit reads are contiguous
-// and conflict-free) and the tile's own rows I[i][m] (and F[i][m]) of block P (col direction; lane
-// pairs read the same word).  MIRROR (one chunk = the whole column): F[ii][m] = I[ii][nh-1-m] is
-// read from the staged I at the mirrored m, halving the staging (65.7 KB at nh = 513 -> 3 CTAs
-// per SM).  The table stream is double-buffered in registers: round k+1's UNR vectors per row and
-// lane are requested before round k is consumed, the first round before the staging (the table is
-// constant, so also before the wait on the predecessor kernel); the staging is asynchronous
-// 8-byte copies, all in flight at once.  Reductions: row direction = warp butterfly; col direction
-// = 16-lane butterfly (lanes with the same q set) + fixed-order sum over the 4 warps.  Partials go
-// to slot (block, chunk) of each target: row direction slot Q, col direction slot P, so every slot
-// of every target is written by exactly one CTA.
-constexpr int kSymThreads = 128;
-
-
-template <bool OTF, bool MIRROR, int UNR, int NBUF>
-__global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __restrict__ U, long long tile_lo, int ni,
-                                                            int nh, int nmc, int mc, const double* __restrict__ symq,
-                                                            const double* __restrict__ symp, int nhp, int nslot,
-                                                            double* __restrict__ part, double rmin, double dr,
-                                                            double dz) {
+// CTA = one tile x one m-chunk, WG groups of 4 warps.  Warp w of a group streams rows p = w and
+// w + 4 of the tile ([m][q], 2 x 32-byte vectors per m: lane l takes vector v = l + 32k of each row,
+// i.e. m = m0 + (v >> 1) and q = 4 (l & 1) .. +3, fixed per lane), so every staged source-column
+// value it reads serves two table rows; the WG groups split each row's vector range (WG = 2: 16
+// warps per SM at the 128-register budget -- measured best on B200; more loads in flight per warp
+// spill).  Shared memory holds the chunk's source columns I^T (and F^T) of block Q as two planes
+// of 16-byte pairs (q = 4qh + {0,1} | 4qh + {2,3}; a warp's 128-bit reads are contiguous and
+// conflict-free) and the tile's own rows I[i][m] (and F[i][m]) of block P (col direction; lane
+// pairs read the same word), both bulk-copied (TMA 1-D, one mbarrier) from the per-iteration
+// packed arrays of k_sym_pack.  MIRROR (one chunk = the whole column): F[ii][m] = I[ii][nh-1-m] is
+// read from the staged I at the mirrored m, halving the staging (65.7 KB at nh = 513).  The table
+// stream runs through a register ring of NBUF rounds of UNR vectors per row and lane: round r+NBUF-1
+// is requested before round r is consumed, the first rounds before the staging (the table is
+// constant, so also before the wait on the predecessor kernel).  Reductions: row direction = warp
+// butterfly + fixed-order group sum; col direction = 16-lane butterfly (lanes with the same q set)
+// + fixed-order sum over the warps.  Partials go to slot (block, chunk) of each target: row
+// direction slot Q, col direction slot P, so every slot of every target is written by exactly one CTA.
+#ifndef EFIT_SYM_MINB
+#define EFIT_SYM_MINB 0
+#endif
+template <bool OTF, bool MIRROR, int UNR, int NBUF, int WG>
+__global__ void __launch_bounds__(128 * WG, EFIT_SYM_MINB ? EFIT_SYM_MINB : (WG == 1 ? 3 : (WG == 2 ? 2 : 1)))
+    k_bnd_sym(const double* __restrict__ U, long long tile_lo, int ni, int nh, int nmc, int mc,
+              const double* __restrict__ symq, const double* __restrict__ symp, int nhp, int nslot,
+              double* __restrict__ part, double rmin, double dr, double dz) {
     extern __shared__ __align__(16) double xs[];
-    __shared__ double red[4][16];
+    __shared__ double red[4 * WG][16];
+    __shared__ double rrow[4 * WG][4];
     __shared__ __align__(8) unsigned long long bar;
     if (threadIdx.x == 0) mbar_init(&bar, 1);
     __syncthreads();
@@ -1458,9 +1479,12 @@ __global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __rest
     const bool diag = P == Q;  // diagonal tile: stored in full, row direction only
     const int m0 = mch * mc, mlen = min(mc, nh - m0);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, qh = lane & 1;
-    const int rp0 = 8 * P + warp, rp1 = rp0 + 4;
+    const int wr = warp & 3, grp = warp >> 2;
+    const int rp0 = 8 * P + wr, rp1 = rp0 + 4;
     const int nvec = 2 * mlen;
-    const double* tp0 = OTF ? nullptr : U + ((long long)tl * 64 + (long long)warp * 8) * nh + 8LL * m0;
+    const int seg = WG == 1 ? nvec : (nvec / (32 * WG)) * 32;  // group g: [g seg, (g+1) seg), last to nvec
+    const int vb = grp * seg, ve = grp == WG - 1 ? nvec : vb + seg;
+    const double* tp0 = OTF ? nullptr : U + ((long long)tl * 64 + (long long)wr * 8) * nh + 8LL * m0;
     const double* tp1 = OTF ? nullptr : tp0 + 32LL * nh;
     // Lane addressing: vector v = k0 + 32u + lane of a row sits at tp + 4v; its staged plane
     // pair index is v itself (m = v >> 1, qh = v & 1); the mirrored plane index is
@@ -1469,7 +1493,7 @@ __global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __rest
 #pragma unroll
         for (int u = 0; u < UNR; ++u) {
             const int v = k0 + 32 * u + lane;
-            const bool ok = !tail || v < nvec;
+            const bool ok = !tail || v < ve;
             if (OTF) {
                 double a4[4], b4[4];
 #pragma unroll
@@ -1490,12 +1514,12 @@ __global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __rest
         }
     };
     constexpr int kStep = 32 * UNR;
-    const int nfull = nvec / kStep;          // rounds without a bounds check
-    const int nround = (nvec + kStep - 1) / kStep;
+    const int nfull = (ve - vb) / kStep;          // rounds without a bounds check
+    const int nround = (ve - vb + kStep - 1) / kStep;
     d4 tv[NBUF][2][UNR];  // ring of NBUF rounds: NBUF - 1 rounds stay in flight while one is consumed
 #pragma unroll
     for (int b = 0; b + 1 < NBUF; ++b)
-        if (b < nround) load(tv[b][0], tv[b][1], b * kStep, b >= nfull);
+        if (b < nround) load(tv[b][0], tv[b][1], vb + b * kStep, b >= nfull);
     griddep();
     // staged layout: xqi planes [2][mc][2][2] | (xqf planes) | xpi rows [8][ms] | (xpf rows [8][ms]),
     // copied from the per-iteration packed arrays (k_sym_pack) by bulk (TMA 1-D) copies issued by
@@ -1530,8 +1554,8 @@ __global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __rest
         }
     }
     mbar_wait(&bar, 0);
-    const double* xpi0 = xpi + warp * ms;
-    const double* xpf0 = xpf + warp * ms;
+    const double* xpi0 = xpi + wr * ms;
+    const double* xpf0 = xpf + wr * ms;
     const double* xpi1 = xpi0 + 4 * ms;
     const double* xpf1 = xpf0 + 4 * ms;
     const double2* pi0 = reinterpret_cast<const double2*>(xqi);           // q pairs 4qh + {0,1}
@@ -1563,7 +1587,7 @@ __global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __rest
                 a = ai[32 * u]; b = bi[32 * u]; c = cf[sgn * 32 * u]; d = df[sgn * 32 * u];
                 i0 = pI0[16 * u]; i1 = pI1[16 * u]; f0 = pF0[sgn * 16 * u]; f1 = pF1[sgn * 16 * u];
             } else {  // x = 0 past the end: read any valid slot
-                const int v = min(k0 + 32 * u + lane, nvec - 2 + qh);  // keeps the parity (= qh)
+                const int v = min(k0 + 32 * u + lane, ve - 2 + qh);  // keeps the parity (= qh)
                 const int mm = v >> 1, wf = MIRROR ? wfb - v : v, mf = MIRROR ? nh - 1 - mm : mm;
                 a = pi0[v]; b = pi1[v]; c = pf0[wf]; d = pf1[wf];
                 i0 = xpi0[mm]; i1 = xpi1[mm]; f0 = xpf0[mf]; f1 = xpf1[mf];
@@ -1592,8 +1616,9 @@ __global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __rest
             const int r = r0 + b;
             if (r >= nround) break;
             const int rn = r + NBUF - 1;
-            if (rn < nround) load(tv[(b + NBUF - 1) % NBUF][0], tv[(b + NBUF - 1) % NBUF][1], rn * kStep, rn >= nfull);
-            compute(tv[b][0], tv[b][1], r * kStep, r >= nfull);
+            if (rn < nround)
+                load(tv[(b + NBUF - 1) % NBUF][0], tv[(b + NBUF - 1) % NBUF][1], vb + rn * kStep, rn >= nfull);
+            compute(tv[b][0], tv[b][1], vb + r * kStep, r >= nfull);
         }
     }
     arI0 = warp_sum(arI0);
@@ -1601,15 +1626,7 @@ __global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __rest
     arI1 = warp_sum(arI1);
     arF1 = warp_sum(arF1);
     if (lane == 0) {
-        const int slot = Q * nmc + mch;
-        if (rp0 < ni) {
-            part[((long long)rp0 * 2 + 0) * nslot + slot] = arI0;
-            part[((long long)rp0 * 2 + 1) * nslot + slot] = arF0;
-        }
-        if (rp1 < ni) {
-            part[((long long)rp1 * 2 + 0) * nslot + slot] = arI1;
-            part[((long long)rp1 * 2 + 1) * nslot + slot] = arF1;
-        }
+        rrow[warp][0] = arI0; rrow[warp][1] = arF0; rrow[warp][2] = arI1; rrow[warp][3] = arF1;
     }
     if (!diag) {  // CTA-uniform
 #pragma unroll
@@ -1626,14 +1643,21 @@ __global__ void __launch_bounds__(kSymThreads, 3) k_bnd_sym(const double* __rest
                 red[warp][2 * q + 1] = b;
             }
         }
-        __syncthreads();
-        if (threadIdx.x < 16) {
-            const int q = threadIdx.x >> 1, side = threadIdx.x & 1, rq = 8 * Q + q;
-            double s = 0.0;
+    }
+    __syncthreads();
+    const int t = threadIdx.x;
+    if (t < 16) {  // row direction: targets 8P + wr (+4), slot Q; groups summed in order
+        const int w4 = t >> 2, k = t & 3, rp = 8 * P + w4 + (k >> 1) * 4, side = k & 1;
+        double v = 0.0;
 #pragma unroll
-            for (int w = 0; w < 4; ++w) s += red[w][threadIdx.x];
-            if (rq < ni) part[((long long)rq * 2 + side) * nslot + P * nmc + mch] = s;
-        }
+        for (int g = 0; g < WG; ++g) v += rrow[4 * g + w4][k];
+        if (rp < ni) part[((long long)rp * 2 + side) * nslot + Q * nmc + mch] = v;
+    } else if (t < 32 && !diag) {  // col direction: targets 8Q + q, slot P
+        const int i = t - 16, q = i >> 1, side = i & 1, rq = 8 * Q + q;
+        double v = 0.0;
+#pragma unroll
+        for (int w = 0; w < 4 * WG; ++w) v += red[w][i];
+        if (rq < ni) part[((long long)rq * 2 + side) * nslot + P * nmc + mch] = v;
     }
 }
 
@@ -1678,9 +1702,12 @@ __global__ void k_sym_pack(const double* __restrict__ I, const double* __restric
 #define EFIT_SYM_UNR 2
 #endif
 #ifndef EFIT_SYM_BUF
-#define EFIT_SYM_BUF 3
+#define EFIT_SYM_BUF 2
 #endif
-constexpr int kSymUnr = EFIT_SYM_UNR, kSymBuf = EFIT_SYM_BUF;
+#ifndef EFIT_SYM_WG
+#define EFIT_SYM_WG 2
+#endif
+constexpr int kSymUnr = EFIT_SYM_UNR, kSymBuf = EFIT_SYM_BUF, kSymWg = EFIT_SYM_WG;
 
 constexpr int kTbGI = 8;
 constexpr int kTbUnroll = 4;
@@ -1746,16 +1773,16 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
             const size_t smem = sym_smem(c);
             const bool mir = c.t.sym_nmc == 1;
             const dim3 grid((unsigned)(ntl * c.t.sym_nmc));
-#define EFIT_SYM_LAUNCH(OTFV, MIRV, UNRV, NBV)                                                                      \
-    launch_pdl(k_bnd_sym<OTFV, MIRV, UNRV, NBV>, grid, dim3(kSymThreads), smem, s, (const double*)c.U, c.sym_tile_lo,  \
+#define EFIT_SYM_LAUNCH(OTFV, MIRV, UNRV, NBV, WGV)                                                                      \
+    launch_pdl(k_bnd_sym<OTFV, MIRV, UNRV, NBV, WGV>, grid, dim3(128 * WGV), smem, s, (const double*)c.U, c.sym_tile_lo,  \
                c.ni, c.nh, c.t.sym_nmc, c.t.sym_mc, (const double*)c.symq, (const double*)c.symp, c.nhp, sy.nslot, \
                c.sym_part, c.rmin, c.dr, c.dz)
             if (c.otf) {  // FP64-bound: a short unroll keeps the inlined AGM in registers
-                if (mir) EFIT_SYM_LAUNCH(true, true, 1, 2); else EFIT_SYM_LAUNCH(true, false, 1, 2);
+                if (mir) EFIT_SYM_LAUNCH(true, true, 1, 2, kSymWg); else EFIT_SYM_LAUNCH(true, false, 1, 2, kSymWg);
             } else if (mir) {
-                EFIT_SYM_LAUNCH(false, true, kSymUnr, kSymBuf);
+                EFIT_SYM_LAUNCH(false, true, kSymUnr, kSymBuf, kSymWg);
             } else {
-                EFIT_SYM_LAUNCH(false, false, kSymUnr, kSymBuf);
+                EFIT_SYM_LAUNCH(false, false, kSymUnr, kSymBuf, kSymWg);
             }
 #undef EFIT_SYM_LAUNCH
             if ((e = cudaGetLastError())) return e;
@@ -2487,9 +2514,9 @@ cudaError_t prepare_kernels(Ctx& c) {
     if ((e = big((const void*)k_bnd_tb_otf<kTbGI>, 2 * sizeof(double) * c.t.tb_ch))) return e;
     {
         const size_t sm = sym_smem(c);
-        const void* ks[4] = {(const void*)k_bnd_sym<false, true, kSymUnr, kSymBuf>,
-                             (const void*)k_bnd_sym<false, false, kSymUnr, kSymBuf>,
-                             (const void*)k_bnd_sym<true, true, 1, 2>, (const void*)k_bnd_sym<true, false, 1, 2>};
+        const void* ks[4] = {(const void*)k_bnd_sym<false, true, kSymUnr, kSymBuf, kSymWg>,
+                             (const void*)k_bnd_sym<false, false, kSymUnr, kSymBuf, kSymWg>,
+                             (const void*)k_bnd_sym<true, true, 1, 2, kSymWg>, (const void*)k_bnd_sym<true, false, 1, 2, kSymWg>};
         for (const void* f : ks)
             if ((e = big(f, sm))) return e;
     }
