@@ -203,6 +203,41 @@ int efit_fit_steps(efit_ctx* ctx, int32_t nsteps, double* d_psi, const double* d
 int efit_solve_update(efit_ctx* ctx, const double* d_pcurr, const double* d_psib, const double* d_psi_ext,
                       double* d_psi, double* d_eps, efit_stream_t stream);
 
+/* ---- multi-time-slice batch ------------------------------------------------
+ * EFIT reconstructs many time slices of one discharge with the same machine and grid (P:L161:
+ * slices are independent fits).  A batch of S <= 8 slices shares one pass over the top/bottom
+ * Green's table: the O(N^3) nest of P:L187 / Fig. 2-3 becomes a product of the slab matrix with 2S
+ * right-hand sides (each slice's current and its mirror), computed on the FP64 tensor cores
+ * (mma.sync m8n8k4), while every slice's O(N^2) steps run concurrently on a stream of their own.
+ * Each slice's results equal those of efit_fit_step on that slice alone to rounding (the table
+ * pass sums in another order; not bit for bit).  Requires mode EFIT_GREEN_TABLE, world == 1.
+ *
+ * efit_batch_workspace_bytes: device bytes of per-slice scratch for nslice slices.
+ * efit_batch_attach: carve that scratch from caller-owned device memory d_workspace (256-byte
+ *   aligned, kept alive until efit_destroy or the next attach; cleared here, synchronising the
+ *   device) and create one stream per slice.  Re-attaching replaces the previous batch.
+ *   EFIT_E_INVAL: nslice outside [1, 8] / bad workspace; EFIT_E_NOMEM: too small;
+ *   EFIT_E_STATE: mode != EFIT_GREEN_TABLE, world > 1 or EFIT_LR_DIRECT set. */
+int efit_batch_workspace_bytes(const efit_ctx* ctx, int32_t nslice, size_t* bytes_out);
+int efit_batch_attach(efit_ctx* ctx, int32_t nslice, void* d_workspace, size_t ws_bytes);
+
+/* One fit iteration of every attached slice (efit_fit_step semantics per slice k):
+ *   d_psi[S][nw*nh] (in/out), d_psi_ext[S][nw*nh], d_meas[S][ndiag], d_sigma[S][ndiag],
+ *   d_coef[S][nbasis], d_chi2[S], d_eps[S]; slices contiguous without padding (base pointers
+ *   16-byte aligned; the per-slice sub-arrays need only 8-byte alignment).  stream must not be NULL (the
+ *   slice streams fork from and join back into it).  Captured as one CUDA graph per pointer set.
+ *   EFIT_E_STATE if no batch is attached. */
+int efit_fit_step_batch(efit_ctx* ctx, double* d_psi, const double* d_psi_ext, const double* d_meas,
+                        const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps,
+                        efit_stream_t stream);
+/* nsteps chained iterations per slice (efit_fit_steps semantics). */
+int efit_fit_steps_batch(efit_ctx* ctx, int32_t nsteps, double* d_psi, const double* d_psi_ext,
+                         const double* d_meas, const double* d_sigma, double* d_coef, double* d_chi2,
+                         double* d_eps, efit_stream_t stream);
+/* Boundary flux of S currents at once: d_pcurr[S][nw*nh] -> d_psib[S][n_edge] (efit_boundary_flux
+ * semantics per slice). */
+int efit_boundary_flux_batch(efit_ctx* ctx, const double* d_pcurr, double* d_psib, efit_stream_t stream);
+
 /* Per-step kernel timing (the measurement hook used by bench.py).  After
  * efit_profile_begin(ctx, n, every), every `every`-th efit_fit_step call (the 1st, (every+1)-th, ...)
  * records CUDA events at seven marks, on the streams the kernels run on, until n steps are recorded.  The calls enqueue eagerly, or -- when the caller is capturing the stream into its own CUDA

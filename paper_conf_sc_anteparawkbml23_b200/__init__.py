@@ -23,6 +23,8 @@ __all__ = [
     "efit_table", "efit_shard", "efit_destroy", "efit_strerror", "efit_last_error", "efit_version",
     "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY", "EFIT_GREEN_TABLE_SYM",
     "EFIT_GREEN_ONTHEFLY_SYM", "efit_plan_info", "owned_targets", "exchange",
+    "efit_batch_workspace_bytes", "efit_batch_attach", "efit_fit_step_batch", "efit_fit_steps_batch",
+    "efit_boundary_flux_batch",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -110,6 +112,11 @@ def lib() -> ctypes.CDLL:
             "efit_profile_begin": (I, [vp, ctypes.c_int32, ctypes.c_int32]),
             "efit_profile_end": (I, [vp, P(ctypes.c_double), ctypes.c_int32, P(ctypes.c_int32)]),
             "efit_table": (I, [vp, I, P(vp)]),
+            "efit_batch_workspace_bytes": (I, [vp, ctypes.c_int32, P(ctypes.c_size_t)]),
+            "efit_batch_attach": (I, [vp, ctypes.c_int32, vp, ctypes.c_size_t]),
+            "efit_fit_step_batch": (I, [vp, vp, vp, vp, vp, vp, vp, vp, vp]),
+            "efit_fit_steps_batch": (I, [vp, ctypes.c_int32, vp, vp, vp, vp, vp, vp, vp, vp]),
+            "efit_boundary_flux_batch": (I, [vp, vp, vp, vp]),
             "efit_shard": (None, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int32),
                                   P(ctypes.c_int32)]),
             "efit_destroy": (I, [vp]),
@@ -274,6 +281,30 @@ def efit_fit_steps(ctx, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stre
                                 _ptr(chi2), _ptr(eps), _stream(stream)), ctx)
 
 
+def efit_batch_workspace_bytes(ctx, nslice: int) -> int:
+    n = ctypes.c_size_t()
+    _check(lib().efit_batch_workspace_bytes(ctx, nslice, ctypes.byref(n)), ctx)
+    return n.value
+
+
+def efit_batch_attach(ctx, nslice: int, workspace) -> None:
+    _check(lib().efit_batch_attach(ctx, nslice, _ptr(workspace), workspace.numel()), ctx)
+
+
+def efit_fit_step_batch(ctx, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None) -> None:
+    _check(lib().efit_fit_step_batch(ctx, _ptr(psi), _ptr(psi_ext), _ptr(meas), _ptr(sigma), _ptr(coef),
+                                     _ptr(chi2), _ptr(eps), _stream(stream)), ctx)
+
+
+def efit_fit_steps_batch(ctx, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None) -> None:
+    _check(lib().efit_fit_steps_batch(ctx, nsteps, _ptr(psi), _ptr(psi_ext), _ptr(meas), _ptr(sigma),
+                                      _ptr(coef), _ptr(chi2), _ptr(eps), _stream(stream)), ctx)
+
+
+def efit_boundary_flux_batch(ctx, pcurr, psib, stream=None) -> None:
+    _check(lib().efit_boundary_flux_batch(ctx, _ptr(pcurr), _ptr(psib), _stream(stream)), ctx)
+
+
 def efit_status(ctx, stream=None) -> int:
     return lib().efit_status(ctx, _stream(stream))
 
@@ -378,6 +409,28 @@ class EfitContext:
 
     def status(self, stream=None) -> int:
         return efit_status(self.handle, stream)
+
+    # multi-time-slice batch (include/efit.h: efit_batch_attach)
+    def batch_attach(self, nslice: int) -> None:
+        import torch
+        nbytes = efit_batch_workspace_bytes(self.handle, nslice)
+        raw = torch.empty(nbytes + 256, dtype=torch.uint8, device=self.device)
+        off = (-raw.data_ptr()) % 256
+        self._batch_raw = raw
+        self.batch_workspace = raw[off:off + nbytes]
+        efit_batch_attach(self.handle, nslice, self.batch_workspace)
+        self.nslice = nslice
+
+    def fit_step_batch(self, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None):
+        efit_fit_step_batch(self.handle, psi, psi_ext, meas, sigma, coef, chi2, eps, stream)
+
+    def fit_steps_batch(self, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None):
+        efit_fit_steps_batch(self.handle, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream)
+
+    def boundary_flux_batch(self, pcurr, stream=None):
+        out = self._t(self.nslice * self.n_edge)
+        efit_boundary_flux_batch(self.handle, pcurr, out, stream)
+        return out.view(self.nslice, self.n_edge)
 
     def table_ptr(self, which: int) -> int:
         return efit_table(self.handle, which)

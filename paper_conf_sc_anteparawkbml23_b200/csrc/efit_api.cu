@@ -146,6 +146,9 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
         }
     }
     t.resp_nchunk = (int)((n + t.resp_gc - 1) / t.resp_gc);
+    c.tbb_nchunk = (int)((n + efit::kBatchCh - 1) / efit::kBatchCh);
+    c.respb_nchunk = (int)((n + efit::kRespBatchGc - 1) / efit::kRespBatchGc);
+    c.respb = false;
     t.tb_ch = 2048;
     t.tb_nchunk = (int)((n + t.tb_ch - 1) / t.tb_ch);
     t.tb_gi = 8;
@@ -199,6 +202,37 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     t.resp_mb = best_mb;
 }
 
+// Per-iteration scratch (also the whole of a batch slice context).  batch: tb_part sized for the
+// k_bnd_tb_mma chunks.
+template <typename Take>
+static size_t carve_scratch(Ctx& c, Take& take, size_t& off, bool batch) {
+    const long long n = (long long)c.nw * c.nh;
+    const int nrows = c.m_hi - c.m_lo;
+    c.axbd = (double*)take(sizeof(double) * 2);
+    c.status = (int*)take(sizeof(int) * 4);
+    c.tickets = (unsigned*)take(sizeof(unsigned) * 8);
+    c.norm_part = (double*)take(sizeof(double) * 2 * (size_t)(c.t.red_blocks > c.ni + 2 ? c.t.red_blocks : c.ni + 2));
+    const int rchunk = batch && c.respb_nchunk > c.t.resp_nchunk ? c.respb_nchunk : c.t.resp_nchunk;
+    c.resp_part = (double*)take(sizeof(double) * (size_t)rchunk * (nrows > 0 ? nrows : 1) * c.nb);
+    c.resp_cnt = (double*)take(sizeof(double) * c.t.resp_nchunk);
+    c.bmat = (double*)take(sizeof(double) * (size_t)c.nb * c.t.resp_nchunk * c.t.resp_gc);
+    c.resp = (double*)take(sizeof(double) * (size_t)c.ndiag * c.nb);
+    c.coef = (double*)take(sizeof(double) * 32);
+    c.chi2 = (double*)take(sizeof(double) * 4);
+    c.pcurr = (double*)take(sizeof(double) * (size_t)round_up(n, c.t.tb_ch));
+    c.pflip = (double*)take(sizeof(double) * (size_t)round_up(n, c.t.tb_ch));
+    c.tb_part = (double*)take(sizeof(double) * (size_t)(batch ? c.tbb_nchunk : c.t.tb_nchunk) * c.nw * 2);
+    c.lr_part = (double*)take(sizeof(double) * (size_t)c.t.lr_nblk * 2 * c.nh);
+    c.lr_xh = (double2*)take(sizeof(double2) * (size_t)c.nh * c.lr_ldi);
+    c.lr_y = (double2*)take(sizeof(double2) * 2 * (size_t)c.nh);
+    c.psib = (double*)take(sizeof(double) * c.n_edge);
+    c.fhat = (double*)take(sizeof(double) * (size_t)c.fhat_ld * c.nmode);
+    c.psip = (double*)take(sizeof(double) * (size_t)n);
+    c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 2));
+    c.scratch_meas = (double*)take(sizeof(double) * c.ndiag);
+    return (size_t)round_up((long long)off, 256);
+}
+
 // Carve the workspace (base == nullptr: sizing only).  Returns total bytes.
 static size_t carve(Ctx& c, char* base) {
     size_t off = 0;
@@ -231,29 +265,8 @@ static size_t carve(Ctx& c, char* base) {
     c.tri_alpha = (double*)take(sizeof(double) * (size_t)c.ni_pad * c.nmode);
     c.twiddle = (double2*)take(sizeof(double2) * (size_t)(c.fft_m / 2));
     c.sin_tab = (double*)take(sizeof(double) * (size_t)c.nmode);
-    c.axbd = (double*)take(sizeof(double) * 2);
-    c.status = (int*)take(sizeof(int) * 4);
-    c.tickets = (unsigned*)take(sizeof(unsigned) * 8);
-    c.norm_part = (double*)take(sizeof(double) * 2 * (size_t)(c.t.red_blocks > c.ni + 2 ? c.t.red_blocks : c.ni + 2));
-    c.resp_part = (double*)take(sizeof(double) * (size_t)c.t.resp_nchunk * (nrows > 0 ? nrows : 1) * c.nb);
-    c.resp_cnt = (double*)take(sizeof(double) * c.t.resp_nchunk);
-    c.bmat = (double*)take(sizeof(double) * (size_t)c.nb * c.t.resp_nchunk * c.t.resp_gc);
-    c.resp = (double*)take(sizeof(double) * (size_t)c.ndiag * c.nb);
-    c.coef = (double*)take(sizeof(double) * 32);
-    c.chi2 = (double*)take(sizeof(double) * 4);
-    c.pcurr = (double*)take(sizeof(double) * (size_t)round_up(n, c.t.tb_ch));
-    c.pflip = (double*)take(sizeof(double) * (size_t)round_up(n, c.t.tb_ch));
-    c.tb_part = (double*)take(sizeof(double) * (size_t)c.t.tb_nchunk * c.nw * 2);
-    c.lr_part = (double*)take(sizeof(double) * (size_t)c.t.lr_nblk * 2 * c.nh);
     c.lr_spec = (double*)take(sizeof(double) * 2 * (size_t)c.nh * c.lr_ldi);
-    c.lr_xh = (double2*)take(sizeof(double2) * (size_t)c.nh * c.lr_ldi);
-    c.lr_y = (double2*)take(sizeof(double2) * 2 * (size_t)c.nh);
-    c.psib = (double*)take(sizeof(double) * c.n_edge);
-    c.fhat = (double*)take(sizeof(double) * (size_t)c.fhat_ld * c.nmode);
-    c.psip = (double*)take(sizeof(double) * (size_t)n);
-    c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 2));
-    c.scratch_meas = (double*)take(sizeof(double) * c.ndiag);
-    return (size_t)round_up((long long)off, 256);
+    return carve_scratch(c, take, off, false);
 }
 
 static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
@@ -357,6 +370,11 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
         }
     }
     c.use_graph = getenv("EFIT_NO_GRAPH") == nullptr;
+    c.nslice = 0;
+    for (int k = 0; k < efit::kMaxSlices; ++k) c.slice[k] = nullptr;
+    c.shadow = false;
+    c.bev_fork = c.bev_tb = c.bev_resp = nullptr;
+    c.bexec = nullptr;
     c.err[0] = 0;
     *out = h;
     return EFIT_OK;
@@ -576,6 +594,260 @@ extern "C" int efit_fit_steps(efit_ctx* h, int32_t nsteps, double* d_psi, const 
     return fit_steps_impl(h, nsteps, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, stream);
 }
 
+// ------------------------------------------------------------------ multi-time-slice batch
+// (EFIT reconstructs many time slices of a discharge with the same machine, P:L161;
+// S slices share one pass over the top/bottom Green's table.)
+
+static void release_slices(Ctx& c);
+
+static size_t slice_bytes(const Ctx& c) {
+    Ctx* tmp = new (std::nothrow) Ctx(c);
+    if (!tmp) return 0;
+    size_t off = 0;
+    auto take = [&](size_t bytes) -> char* {
+        off = (size_t)round_up((long long)off, 256);
+        off += bytes;
+        return nullptr;
+    };
+    size_t b = carve_scratch(*tmp, take, off, true);
+    delete tmp;
+    return b;
+}
+
+static int batch_check(Ctx& c, int32_t nslice) {
+    if (c.shadow) return fail(&c, EFIT_E_STATE, "not a primary context");
+    if (nslice < 1 || nslice > efit::kMaxSlices)
+        return fail(&c, EFIT_E_INVAL, "nslice %d outside [1, %d]", nslice, efit::kMaxSlices);
+    if (c.mode != EFIT_GREEN_TABLE) return fail(&c, EFIT_E_STATE, "batching needs mode EFIT_GREEN_TABLE");
+    if (c.world != 1) return fail(&c, EFIT_E_STATE, "batching needs world == 1");
+    if (c.lr_direct) return fail(&c, EFIT_E_STATE, "batching needs the FFT left/right path");
+    return EFIT_OK;
+}
+
+extern "C" int efit_batch_workspace_bytes(const efit_ctx* h, int32_t nslice, size_t* bytes_out) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = const_cast<efit_ctx*>(h)->c;
+    int st = batch_check(c, nslice);
+    if (st) return st;
+    if (!bytes_out) return fail(&c, EFIT_E_INVAL, "bytes_out is null");
+    *bytes_out = (size_t)nslice * slice_bytes(c);
+    return EFIT_OK;
+}
+
+extern "C" int efit_batch_attach(efit_ctx* h, int32_t nslice, void* d_workspace, size_t ws_bytes) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    int st = batch_check(c, nslice);
+    if (st) return st;
+    const size_t per = slice_bytes(c);
+    if (!d_workspace || ((uintptr_t)d_workspace & 255u))
+        return fail(&c, EFIT_E_INVAL, "batch workspace must be non-null and 256-byte aligned");
+    if (ws_bytes < per * (size_t)nslice)
+        return fail(&c, EFIT_E_NOMEM, "batch workspace %zu bytes < required %zu", ws_bytes, per * (size_t)nslice);
+    cudaError_t e;
+    if ((e = cudaDeviceSynchronize())) return cuda_fail(&c, e, "batch attach sync");
+    release_slices(c);
+    if ((e = cudaMemset(d_workspace, 0, per * (size_t)nslice))) return cuda_fail(&c, e, "batch workspace clear");
+    if (!c.bev_fork && (e = cudaEventCreateWithFlags(&c.bev_fork, cudaEventDisableTiming))) return cuda_fail(&c, e, "event");
+    if (!c.bev_tb && (e = cudaEventCreateWithFlags(&c.bev_tb, cudaEventDisableTiming))) return cuda_fail(&c, e, "event");
+    if (!c.bev_resp && (e = cudaEventCreateWithFlags(&c.bev_resp, cudaEventDisableTiming))) return cuda_fail(&c, e, "event");
+    int prio_lo = 0, prio_hi = 0;
+    cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+    for (int k = 0; k < nslice; ++k) {
+        Ctx* q = new (std::nothrow) Ctx(c);  // tables, tiling and constants shared with the primary
+        if (!q) { release_slices(c); return fail(&c, EFIT_E_NOMEM, "host allocation"); }
+        q->shadow = true;
+        q->nslice = 0;
+        for (int j = 0; j < efit::kMaxSlices; ++j) q->slice[j] = nullptr;
+        q->gexec = nullptr; q->bexec = nullptr; q->pexec = nullptr; q->pgraph = nullptr;
+        q->prof_on = q->prof_rec = q->prof_capture = false;
+        q->prof_ev = nullptr;
+        for (int j = 0; j < 16; ++j) q->prof_place[j] = nullptr;
+        q->side = nullptr; q->ev_fork = q->ev_join = nullptr;
+        c.slice[k] = q;
+        char* base = (char*)d_workspace + per * (size_t)k;
+        size_t off = 0;
+        auto take = [&](size_t bytes) -> char* {
+            off = (size_t)round_up((long long)off, 256);
+            char* p = base + off;
+            off += bytes;
+            return p;
+        };
+        carve_scratch(*q, take, off, true);
+        q->status = c.status;  // one sticky status word for the whole batch
+        if ((e = cudaStreamCreateWithPriority(&q->side, cudaStreamNonBlocking, prio_hi)) ||
+            (e = cudaEventCreateWithFlags(&q->ev_fork, cudaEventDisableTiming)) ||
+            (e = cudaEventCreateWithFlags(&q->ev_join, cudaEventDisableTiming))) {
+            release_slices(c);
+            return cuda_fail(&c, e, "slice stream");
+        }
+    }
+    c.nslice = nslice;
+    c.respb = efit::response_batch_ok(c, nslice) && getenv("EFIT_NO_RESP_BATCH") == nullptr;
+    return EFIT_OK;
+}
+
+// One Picard iteration of every slice.  Slice k runs its own chain on its stream (normalise,
+// response, LSQ, current, left/right FFT chain + forward DST); the shared table pass (k_bnd_tb_mma)
+// joins all slices' currents; then each slice reduces its boundary and finishes its solve.
+static cudaError_t enqueue_fit_step_batch(Ctx& c, double* psi, const double* psi_ext, const double* meas,
+                                          const double* sigma, double* coef, double* chi2, double* eps,
+                                          cudaStream_t s, bool normalize) {
+    using namespace efit;
+    cudaError_t e;
+    const size_t n = (size_t)c.nw * c.nh;
+    if ((e = cudaEventRecord(c.bev_fork, s))) return e;
+    if (c.respb) {  // every slice's basis matrix, then one pass over Gd for all slices
+        for (int k = 0; k < c.nslice; ++k) {
+            Ctx& q = *c.slice[k];
+            cudaStream_t sk = q.side;
+            double* pk = psi + k * n;
+            if ((e = cudaStreamWaitEvent(sk, c.bev_fork, 0))) return e;
+            if (normalize && (e = launch_normalize(q, pk, sk))) return e;
+            if ((e = launch_basis(q, pk, sk))) return e;
+            if ((e = cudaEventRecord(q.ev_join, sk))) return e;
+        }
+        for (int k = 0; k < c.nslice; ++k)
+            if ((e = cudaStreamWaitEvent(s, c.slice[k]->ev_join, 0))) return e;
+        if ((e = launch_response_batch(c, c.nslice, c.slice, s))) return e;
+        if ((e = cudaEventRecord(c.bev_resp, s))) return e;
+    }
+    for (int k = 0; k < c.nslice; ++k) {
+        Ctx& q = *c.slice[k];
+        cudaStream_t sk = q.side;
+        double* pk = psi + k * n;
+        if (c.respb) {
+            if ((e = cudaStreamWaitEvent(sk, c.bev_resp, 0))) return e;
+            if ((e = launch_resp_reduce_batch(q, c.respb_nchunk, q.resp, sk))) return e;
+        } else {
+            if ((e = cudaStreamWaitEvent(sk, c.bev_fork, 0))) return e;
+            if (normalize && (e = launch_normalize(q, pk, sk))) return e;
+            if ((e = launch_response(q, pk, q.resp, sk))) return e;
+        }
+        if ((e = launch_lsq(q, q.resp, meas + (size_t)k * c.ndiag, sigma + (size_t)k * c.ndiag, coef + (size_t)k * c.nb,
+                            chi2 + k, sk)))
+            return e;
+        if ((e = launch_current(q, pk, coef + (size_t)k * c.nb, q.pcurr, true, sk))) return e;
+        if ((e = cudaEventRecord(q.ev_fork, sk))) return e;  // this slice's current pair is ready
+        if ((e = launch_lr_fft(q, q.psib, sk))) return e;
+        if ((e = launch_solve_fwd(q, q.pcurr, q.psib, sk, 2))) return e;
+    }
+    for (int k = 0; k < c.nslice; ++k)
+        if ((e = cudaStreamWaitEvent(s, c.slice[k]->ev_fork, 0))) return e;
+    if ((e = launch_boundary_batch(c, c.nslice, c.slice, s))) return e;
+    if ((e = cudaEventRecord(c.bev_tb, s))) return e;
+    for (int k = 0; k < c.nslice; ++k) {
+        Ctx& q = *c.slice[k];
+        cudaStream_t sk = q.side;
+        if ((e = cudaStreamWaitEvent(sk, c.bev_tb, 0))) return e;
+        if ((e = launch_bnd_reduce(q, q.tb_part, c.tbb_nchunk, q.psib, sk))) return e;
+        if ((e = launch_solve_rest(q, q.psib, nullptr, psi + k * n, psi_ext + k * n, eps + k, sk, true, true))) return e;
+        if ((e = cudaEventRecord(q.ev_join, sk))) return e;
+    }
+    for (int k = 0; k < c.nslice; ++k)
+        if ((e = cudaStreamWaitEvent(s, c.slice[k]->ev_join, 0))) return e;
+    return cudaSuccess;
+}
+
+static int fit_steps_batch_impl(efit_ctx* h, int32_t nsteps, double* d_psi, const double* d_psi_ext,
+                                const double* d_meas, const double* d_sigma, double* d_coef, double* d_chi2,
+                                double* d_eps, efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    if (c.nslice < 1) return fail(&c, EFIT_E_STATE, "no batch attached (efit_batch_attach)");
+    if (nsteps < 1) return fail(&c, EFIT_E_INVAL, "nsteps < 1");
+    EFIT_CHECK_PTR(c, d_psi, "d_psi");
+    EFIT_CHECK_PTR(c, d_psi_ext, "d_psi_ext");
+    EFIT_CHECK_PTR(c, d_meas, "d_meas");
+    EFIT_CHECK_PTR(c, d_sigma, "d_sigma");
+    EFIT_CHECK_PTR(c, d_coef, "d_coef");
+    EFIT_CHECK_PTR(c, d_chi2, "d_chi2");
+    EFIT_CHECK_PTR(c, d_eps, "d_eps");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (s == nullptr) return fail(&c, EFIT_E_INVAL, "batched calls need a non-default stream");
+    cudaError_t e;
+    auto enqueue = [&]() -> cudaError_t {
+        for (int k = 0; k < nsteps; ++k) {
+            cudaError_t e1 = enqueue_fit_step_batch(c, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, s, k == 0);
+            if (e1) return e1;
+        }
+        return cudaSuccess;
+    };
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if ((e = cudaStreamIsCapturing(s, &cs))) return cuda_fail(&c, e, "capture query");
+    if (!c.use_graph || cs == cudaStreamCaptureStatusActive) {
+        if ((e = enqueue())) return cuda_fail(&c, e, "batched fit step");
+        return EFIT_OK;
+    }
+    const void* key[10] = {d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, (const void*)s,
+                           (const void*)(intptr_t)nsteps, (const void*)(intptr_t)c.nslice};
+    if (!c.bexec || std::memcmp(key, c.bkey, sizeof(key)) != 0) {
+        if (c.bexec) { cudaGraphExecDestroy(c.bexec); c.bexec = nullptr; }
+        cudaGraph_t graph = nullptr;
+        if ((e = cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal))) return cuda_fail(&c, e, "begin capture");
+        cudaError_t e2 = enqueue();
+        e = cudaStreamEndCapture(s, &graph);
+        if (e2) { if (graph) cudaGraphDestroy(graph); return cuda_fail(&c, e2, "batched fit step capture"); }
+        if (e) return cuda_fail(&c, e, "end capture");
+        e = cudaGraphInstantiateWithFlags(&c.bexec, graph, 0);
+        cudaGraphDestroy(graph);
+        if (e) { c.bexec = nullptr; return cuda_fail(&c, e, "graph instantiate"); }
+        std::memcpy(c.bkey, key, sizeof(key));
+    }
+    if ((e = cudaGraphLaunch(c.bexec, s))) return cuda_fail(&c, e, "graph launch");
+    return EFIT_OK;
+}
+
+extern "C" int efit_fit_step_batch(efit_ctx* h, double* d_psi, const double* d_psi_ext, const double* d_meas,
+                                   const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps,
+                                   efit_stream_t stream) {
+    return fit_steps_batch_impl(h, 1, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, stream);
+}
+
+extern "C" int efit_fit_steps_batch(efit_ctx* h, int32_t nsteps, double* d_psi, const double* d_psi_ext,
+                                    const double* d_meas, const double* d_sigma, double* d_coef, double* d_chi2,
+                                    double* d_eps, efit_stream_t stream) {
+    return fit_steps_batch_impl(h, nsteps, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, stream);
+}
+
+extern "C" int efit_boundary_flux_batch(efit_ctx* h, const double* d_pcurr, double* d_psib, efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    if (c.nslice < 1) return fail(&c, EFIT_E_STATE, "no batch attached (efit_batch_attach)");
+    EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
+    EFIT_CHECK_PTR(c, d_psib, "d_psib");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (s == nullptr) return fail(&c, EFIT_E_INVAL, "batched calls need a non-default stream");
+    const size_t n = (size_t)c.nw * c.nh;
+    cudaError_t e;
+    auto run = [&]() -> cudaError_t {
+        cudaError_t e1;
+        if ((e1 = cudaEventRecord(c.bev_fork, s))) return e1;
+        for (int k = 0; k < c.nslice; ++k) {
+            Ctx& q = *c.slice[k];
+            if ((e1 = cudaStreamWaitEvent(q.side, c.bev_fork, 0))) return e1;
+            if ((e1 = efit::launch_make_pair(q, d_pcurr + k * n, q.side))) return e1;
+            if ((e1 = cudaEventRecord(q.ev_fork, q.side))) return e1;
+            if ((e1 = efit::launch_lr_fft(q, d_psib + (size_t)k * c.n_edge, q.side))) return e1;
+        }
+        for (int k = 0; k < c.nslice; ++k)
+            if ((e1 = cudaStreamWaitEvent(s, c.slice[k]->ev_fork, 0))) return e1;
+        if ((e1 = efit::launch_boundary_batch(c, c.nslice, c.slice, s))) return e1;
+        if ((e1 = cudaEventRecord(c.bev_tb, s))) return e1;
+        for (int k = 0; k < c.nslice; ++k) {
+            Ctx& q = *c.slice[k];
+            if ((e1 = cudaStreamWaitEvent(q.side, c.bev_tb, 0))) return e1;
+            if ((e1 = efit::launch_bnd_reduce(q, q.tb_part, c.tbb_nchunk, d_psib + (size_t)k * c.n_edge, q.side))) return e1;
+            if ((e1 = cudaEventRecord(q.ev_join, q.side))) return e1;
+        }
+        for (int k = 0; k < c.nslice; ++k)
+            if ((e1 = cudaStreamWaitEvent(s, c.slice[k]->ev_join, 0))) return e1;
+        return cudaSuccess;
+    };
+    if ((e = run())) return cuda_fail(&c, e, "batched boundary flux");
+    return EFIT_OK;
+}
+
 extern "C" int efit_solve_update(efit_ctx* h, const double* d_pcurr, const double* d_psib, const double* d_psi_ext,
                                  double* d_psi, double* d_eps, efit_stream_t stream) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
@@ -672,8 +944,26 @@ extern "C" int efit_table(const efit_ctx* h, int which, const void** d_ptr) {
     return EFIT_OK;
 }
 
+static void release_slices(Ctx& c) {
+    for (int k = 0; k < efit::kMaxSlices; ++k) {
+        Ctx* q = c.slice[k];
+        if (!q) continue;
+        if (q->side) cudaStreamDestroy(q->side);
+        if (q->ev_fork) cudaEventDestroy(q->ev_fork);
+        if (q->ev_join) cudaEventDestroy(q->ev_join);
+        delete q;
+        c.slice[k] = nullptr;
+    }
+    c.nslice = 0;
+    if (c.bexec) { cudaGraphExecDestroy(c.bexec); c.bexec = nullptr; }
+}
+
 extern "C" int efit_destroy(efit_ctx* h) {
     if (!h) return EFIT_OK;
+    release_slices(h->c);
+    if (h->c.bev_fork) cudaEventDestroy(h->c.bev_fork);
+    if (h->c.bev_tb) cudaEventDestroy(h->c.bev_tb);
+    if (h->c.bev_resp) cudaEventDestroy(h->c.bev_resp);
     if (h->c.gexec) cudaGraphExecDestroy(h->c.gexec);
     if (h->c.pexec) cudaGraphExecDestroy(h->c.pexec);
     if (h->c.pgraph) cudaGraphDestroy(h->c.pgraph);

@@ -12,7 +12,11 @@ constexpr int kMaxBasis = 24;
 constexpr int kNumSMs = 148;  // B200 (sm_100a): grid sizing in multiples of the SM count
 constexpr int kMaxKnots = 20;
 constexpr int kMaxN = 2049;  // FFT working set 2.5*M*16 B of shared memory, M = 2(nh-1)
-constexpr int kLsqMaxRowsHost = 960;  // k_lsq shared memory: (nb|1 + 2)*nd doubles
+constexpr int kLsqMaxRowsHost = 960;
+constexpr int kMaxSlices = 8;   // multi-time-slice batch (efit_batch_attach): slices per pass
+constexpr int kBatchCh = 512;   // k_bnd_tb_mma: table elements per chunk (16 per mma k-step quad)
+constexpr int kRespBatchGc = 256;   // k_response_mma: grid nodes per chunk
+constexpr int kRespBatchMaxBlk = 4; // k_response_mma: <= 32 basis columns (slices x nbasis) per pass  // k_lsq shared memory: (nb|1 + 2)*nd doubles
 
 // k_response: depth of the register ring of MB-row load steps (4 registers per 256-bit load),
 // keeping ring (4 NP MB) + accumulators (MB NB) <= 56 registers (the rest of the 128-register
@@ -136,6 +140,19 @@ struct Ctx {
     cudaStream_t gstream;
     bool use_graph;
 
+    // multi-time-slice batch: shadow contexts share this context's tables and own
+    // their per-iteration scratch (carved from the caller's batch workspace) and a stream each
+    int nslice;
+    Ctx* slice[kMaxSlices];
+    bool shadow;                   // a slice context (tables not owned)
+    int tbb_nchunk;                // k_bnd_tb_mma chunks (kBatchCh elements)
+    int respb_nchunk;              // k_response_mma chunks (kRespBatchGc nodes)
+    bool respb;                    // this batch contracts Gd once for all slices (k_response_mma)
+    cudaEvent_t bev_fork, bev_tb;  // batch: fork of the slice streams, end of the shared table pass
+    cudaEvent_t bev_resp;          // batch: end of the shared Gd pass
+    cudaGraphExec_t bexec;
+    const void* bkey[10];
+
     char err[256];
 };
 
@@ -159,6 +176,14 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
 cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cudaStream_t s, int with_bnd);
 cudaError_t launch_solve_rest(Ctx& c, const double* psib, double* psi_out, double* psi_inout, const double* psi_ext,
                               double* eps, cudaStream_t s, bool next_norm, bool tb_fix);
+cudaError_t launch_basis(Ctx& c, const double* psi, cudaStream_t s);
+bool response_batch_ok(const Ctx& c, int nslice);
+cudaError_t launch_response_batch(Ctx& c, int nslice, Ctx* const* slices, cudaStream_t s);
+cudaError_t launch_resp_reduce_batch(Ctx& q, int nchunk, double* resp_rows, cudaStream_t s);
+cudaError_t launch_bnd_reduce(Ctx& c, const double* tb_part, int tb_nchunk, double* psib, cudaStream_t s);
+cudaError_t launch_lr_fft(Ctx& c, double* psib, cudaStream_t s);
+// multi-slice top/bottom nest: one pass over this rank's slabs for the slices' (pcurr, pflip) pairs
+cudaError_t launch_boundary_batch(Ctx& c, int nslice, Ctx* const* slices, cudaStream_t s);
 cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out,
                          double* psi_inout, const double* psi_ext, double* eps, cudaStream_t s,
                          bool next_norm = false);

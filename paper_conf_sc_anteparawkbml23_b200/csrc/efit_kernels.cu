@@ -121,6 +121,13 @@ __device__ __forceinline__ d4 lds256(const double* p) {  // two 128-bit shared l
     return d4{a.x, a.y, b.x, b.y};
 }
 
+// FP64 tensor-core MMA (DMMA.8x8x4): D[8x8] += A[8x4] B[4x8]; lane (g = lane/4, k4 = lane%4) holds
+// A[g][k4], B[k4][g] and D[g][2k4 .. 2k4+1].
+__device__ __forceinline__ void dmma884(double& d0, double& d1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
+                 : "+d"(d0), "+d"(d1) : "d"(a), "d"(b));
+}
+
 __device__ __forceinline__ double dot4(const d4& a, const d4& b, double acc) {
     acc = fma(a.x, b.x, acc);
     acc = fma(a.y, b.y, acc);
@@ -636,7 +643,7 @@ __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ 
 // chunks lane, lane+32, ... and a fixed butterfly combines them => deterministic.  The total
 // masked-node count decides EFIT_ST_NOPLASMA.
 __global__ void k_resp_reduce(const double* __restrict__ part, const double* __restrict__ cnt_part, int nchunk,
-                              int total, double* __restrict__ out, int* status) {
+                              int ncnt, int total, double* __restrict__ out, int* status) {
     griddep();
     const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
     if (w < total) {
@@ -648,7 +655,7 @@ __global__ void k_resp_reduce(const double* __restrict__ part, const double* __r
     }
     if (blockIdx.x == 0 && threadIdx.x < 32) {
         double cnt = 0.0;
-        for (int c = lane; c < nchunk; c += 32) cnt += cnt_part[c];
+        for (int c = lane; c < ncnt; c += 32) cnt += cnt_part[c];
         cnt = warp_sum(cnt);
         if (lane == 0 && cnt == 0.0) atomicOr(status, EFIT_ST_NOPLASMA);
     }
@@ -695,13 +702,154 @@ static cudaError_t response_impl(Ctx& c, const double* psi, double* resp_rows, c
     cudaError_t e = cudaGetLastError();
     if (e || prepare) return e;
     const int total = nrows * c.nb;
-    launch_pdl(k_resp_reduce, dim3((total + 7) / 8), dim3(256), 0, s, c.resp_part, c.resp_cnt, c.t.resp_nchunk, total, resp_rows,
+    launch_pdl(k_resp_reduce, dim3((total + 7) / 8), dim3(256), 0, s, c.resp_part, c.resp_cnt, c.t.resp_nchunk,
+               c.t.resp_nchunk, total, resp_rows,
                                                   c.status);
     return cudaGetLastError();
 }
 
 cudaError_t launch_response(Ctx& c, const double* psi, double* resp_rows, cudaStream_t s) {
     return response_impl(c, psi, resp_rows, s, false);
+}
+
+// ------------------------------------------------------------ multi-slice response (tensor cores)
+//
+// S time slices' response matrices in one pass over Gd:
+//   R_s[m][k] = sum_g Gd[m][g] B_s[k][g],
+// a product of Gd (rows m x N^2 nodes) with the S*NB basis columns of all slices -> DMMA m8n8k4
+// exactly as k_bnd_tb_mma: lane (g, k4) streams Gd[8o + g][g0 + 16j + 4k4 .. +3] (one 256-bit
+// streaming load; warp octet o = blockIdx.y * 8 + warp) and takes its B values from the staged
+// basis columns (column 8bl + g = slice-major s*NB + k, zero past S*NB), 256-bit shared loads with
+// rows padded by 2 doubles.  C stays in registers for the whole chunk; lane writes
+// (row 8o + g, columns 8bl + 2k4, +1) to the partials of the owning slices.
+struct RespBatchIO {
+    const double* B[kMaxSlices];  // slice basis matrices [NB][ldb] (k_basis)
+    double* part[kMaxSlices];     // slice partials [row][k][chunk]
+};
+
+template <int NBLK, int NP>
+__global__ void __launch_bounds__(256, 2) k_response_mma(const double* __restrict__ Gd, long long S, int nrows, int n,
+                                                        int nb, int ncol, long long ldb, RespBatchIO io, int nchunk) {
+    constexpr int gc = kRespBatchGc, ldx = kRespBatchGc + 2, nstep = kRespBatchGc / 16;
+    static_assert(nstep % NP == 0, "ring depth divides the steps");
+    extern __shared__ __align__(16) double bsm[];  // [8 NBLK columns][ldx]
+    const int c = blockIdx.x;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, k4 = lane & 3;
+    const long long g0 = (long long)c * gc;
+    const int row = (blockIdx.y * 8 + warp) * 8 + g;
+    const bool okr = row < nrows;
+    const double* tp = Gd + (long long)min(row, nrows - 1) * S + g0 + 4 * k4;
+    auto load = [&](d4& a, int j) {
+        const bool ok = okr && g0 + 16 * j + 4 * k4 < n;
+        a = ok ? ld256_stream(tp + 16 * j) : d4{0.0, 0.0, 0.0, 0.0};
+    };
+    d4 ring[NP];
+#pragma unroll
+    for (int b = 0; b + 1 < NP; ++b) load(ring[b], b);  // Gd is constant: before the wait
+    // staging: one bulk (TMA 1-D) copy per basis column, all in flight at once on one mbarrier;
+    // padding columns and nodes past ldb (basis matrices are zero-padded to ldb) are zeroed
+    __shared__ __align__(8) unsigned long long bar;
+    const int nvalid = (int)min((long long)gc, ldb - g0);
+    if (threadIdx.x == 0) mbar_init(&bar, 1);
+    __syncthreads();
+    griddep();
+    if (threadIdx.x == 0) {
+        mbar_expect_tx(&bar, (unsigned)(sizeof(double) * ncol * nvalid));
+        for (int col = 0; col < ncol; ++col) {
+            const int sl = col / nb, k = col - sl * nb;
+            bulk_g2s(bsm + col * ldx, io.B[sl] + (long long)k * ldb + g0, (unsigned)(sizeof(double) * nvalid), &bar);
+        }
+    }
+    for (int q = threadIdx.x; q < 8 * NBLK * gc; q += blockDim.x) {
+        const int col = q / gc, e = q - col * gc;
+        if (col >= ncol || e >= nvalid) bsm[col * ldx + e] = 0.0;
+    }
+    mbar_wait(&bar, 0);
+    __syncthreads();
+    double acc[NBLK][2];
+#pragma unroll
+    for (int b = 0; b < NBLK; ++b) { acc[b][0] = 0.0; acc[b][1] = 0.0; }
+#pragma unroll 1
+    for (int j0 = 0; j0 < nstep; j0 += NP) {
+#pragma unroll
+        for (int b = 0; b < NP; ++b) {
+            const int j = j0 + b;
+            if (j + NP - 1 < nstep) load(ring[(b + NP - 1) % NP], j + NP - 1);
+#pragma unroll
+            for (int bl = 0; bl < NBLK; ++bl) {
+                const d4 xb = lds256(bsm + (8 * bl + g) * ldx + 16 * j + 4 * k4);
+                dmma884(acc[bl][0], acc[bl][1], ring[b].x, xb.x);
+                dmma884(acc[bl][0], acc[bl][1], ring[b].y, xb.y);
+                dmma884(acc[bl][0], acc[bl][1], ring[b].z, xb.z);
+                dmma884(acc[bl][0], acc[bl][1], ring[b].w, xb.w);
+            }
+        }
+    }
+    if (!okr) return;
+#pragma unroll
+    for (int bl = 0; bl < NBLK; ++bl)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int col = 8 * bl + 2 * k4 + h;
+            if (col < ncol) {
+                const int sl = col / nb, k = col - sl * nb;
+                io.part[sl][((long long)row * nb + k) * nchunk + c] = acc[bl][h];
+            }
+        }
+}
+
+// k_basis of one slice (basis matrix + masked-node counts for this iteration's psi)
+cudaError_t launch_basis(Ctx& c, const double* psi, cudaStream_t s) {
+    const int gc = c.t.resp_gc;
+    const long long ldb = (long long)c.t.resp_nchunk * gc;
+    BasisParams bp = basis_params(c);
+    switch (c.nb) {
+#define EFIT_NB_CASE(V)                                                                                              \
+    case V:                                                                                                          \
+        return launch_pdl(k_basis<V>, dim3(c.t.resp_nchunk), dim3(gc <= 1024 ? gc : 1024), 0, s, psi, c.inlim, c.axbd, \
+                          c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp, gc, ldb, c.bmat, c.resp_cnt);
+        EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
+        EFIT_NB_CASE(7) EFIT_NB_CASE(8) EFIT_NB_CASE(9) EFIT_NB_CASE(10) EFIT_NB_CASE(11) EFIT_NB_CASE(12)
+        EFIT_NB_CASE(13) EFIT_NB_CASE(14) EFIT_NB_CASE(15) EFIT_NB_CASE(16) EFIT_NB_CASE(17) EFIT_NB_CASE(18)
+        EFIT_NB_CASE(19) EFIT_NB_CASE(20) EFIT_NB_CASE(21) EFIT_NB_CASE(22) EFIT_NB_CASE(23) EFIT_NB_CASE(24)
+#undef EFIT_NB_CASE
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+bool response_batch_ok(const Ctx& c, int nslice) { return nslice * c.nb <= 8 * kRespBatchMaxBlk; }
+
+constexpr int kRespMmaNP = 8;
+
+// one pass over Gd for all slices (after every slice's k_basis)
+cudaError_t launch_response_batch(Ctx& c, int nslice, Ctx* const* slices, cudaStream_t s) {
+    const int nrows = c.m_hi - c.m_lo;
+    if (nrows <= 0) return cudaSuccess;
+    RespBatchIO io;
+    for (int k = 0; k < kMaxSlices; ++k) { io.B[k] = nullptr; io.part[k] = nullptr; }
+    for (int k = 0; k < nslice; ++k) { io.B[k] = slices[k]->bmat; io.part[k] = slices[k]->resp_part; }
+    const int ncol = nslice * c.nb;
+    const long long ldb = (long long)c.t.resp_nchunk * c.t.resp_gc;
+    const dim3 grid((unsigned)c.respb_nchunk, (unsigned)((nrows + 63) / 64));
+    const int n = c.nw * c.nh;
+    const int nblk = (ncol + 7) / 8;
+    switch (nblk) {
+#define EFIT_RB(V)                                                                                                 \
+    case V:                                                                                                        \
+        return launch_pdl(k_response_mma<V, kRespMmaNP>, grid, dim3(256), sizeof(double) * 8 * V * (kRespBatchGc + 2), s, \
+                          (const double*)c.Gd, c.S, nrows, n, c.nb, ncol, ldb, io, c.respb_nchunk);
+        EFIT_RB(1) EFIT_RB(2) EFIT_RB(3) EFIT_RB(4)
+#undef EFIT_RB
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+// per-slice chunk sums of the batched partials -> the slice's response rows (+ its NOPLASMA check)
+cudaError_t launch_resp_reduce_batch(Ctx& q, int nchunk, double* resp_rows, cudaStream_t s) {
+    const int total = (q.m_hi - q.m_lo) * q.nb;
+    if (total <= 0) return cudaSuccess;
+    return launch_pdl(k_resp_reduce, dim3((total + 7) / 8), dim3(256), 0, s, q.resp_part, q.resp_cnt, nchunk,
+                      q.t.resp_nchunk, total, resp_rows, q.status);
 }
 
 // ================================================================================ least squares
@@ -1808,6 +1956,140 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     return cudaGetLastError();
 }
 
+// ------------------------------------------------------------ multi-slice top/bottom (tensor cores)
+//
+// S time slices share one pass over the top/bottom slabs: the nest becomes the
+// product  Psi[i][c] = sum_e T[i][e] X_c[e]  of the slab matrix (target rows i x N^2 sources) with
+// 2S right-hand sides X_{2s} = I_s, X_{2s+1} = F_s (F = vertically mirrored I), i.e. a dense
+// contraction with 2S-fold reuse of every table element -> DMMA (mma.sync m8n8k4 fp64): A = 8 slabs
+// x 4 sources, B = 4 sources x 8 columns (NBLK blocks of 8 columns), C = 8 x 8 accumulators in 2
+// registers per lane.  Lane (g = lane/4, k4 = lane%4) loads T[slab 8o + g][e0 + 16j + 4k4 .. +3]
+// with one 256-bit streaming load (4 lanes = 128 contiguous bytes of a slab) and uses its 4 values
+// in 4 consecutive mma k-steps; its B values are X_{8b+g}[same 4 sources], one 256-bit shared load
+// (columns padded by 2 doubles: conflict-free).  C needs no cross-lane reduction: lane holds
+// (I, F) of slice 4b + k4 for slab 8o + g.  A CTA = one chunk of kBatchCh sources x 8 warps x NOCT
+// octets of slabs; a ring of NP steps keeps NP*NOCT*32 B per lane of table loads in flight.
+struct BatchIO {
+    const double* X[2 * kMaxSlices];  // column c: I_{c/2} (even c) or F_{c/2} (odd), zero past nw*nh
+    double* part[kMaxSlices];         // slice partials [row i][side][chunk]
+};
+
+template <int NBLK, int NOCT, int NP>
+__global__ void __launch_bounds__(256, 2) k_bnd_tb_mma(const double* __restrict__ T, long long S, int nslab,
+                                                      int row_lo, int n, int ncol, BatchIO io, int nchunk) {
+    constexpr int ch = kBatchCh, ldx = kBatchCh + 2, nstep = kBatchCh / 16;
+    static_assert(nstep % NP == 0, "ring depth divides the steps");
+    extern __shared__ __align__(16) double xsm[];  // [8 NBLK columns][ldx]
+    const int c = blockIdx.x;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, k4 = lane & 3;
+    const long long e0 = (long long)c * ch;
+    const int s0 = (blockIdx.y * 8 + warp) * 8 * NOCT;  // first slab of this warp
+    const double* tp[NOCT];
+    bool okr[NOCT];
+#pragma unroll
+    for (int o = 0; o < NOCT; ++o) {
+        const int sl = s0 + 8 * o + g;
+        okr[o] = sl < nslab;
+        tp[o] = T + (long long)min(sl, nslab - 1) * S + e0 + 4 * k4;
+    }
+    auto load = [&](d4 (&a)[NOCT], int j) {
+        const bool ok = e0 + 16 * j + 4 * k4 < n;
+#pragma unroll
+        for (int o = 0; o < NOCT; ++o) a[o] = (ok && okr[o]) ? ld256_stream(tp[o] + 16 * j) : d4{0.0, 0.0, 0.0, 0.0};
+    };
+    d4 ring[NP][NOCT];
+#pragma unroll
+    for (int b = 0; b + 1 < NP; ++b) load(ring[b], b);  // the table is constant: before the wait
+    // staging: one bulk (TMA 1-D) copy per column (the pairs are zero-padded to whole chunks),
+    // all in flight at once on one mbarrier; padding columns are zeroed
+    __shared__ __align__(8) unsigned long long bar;
+    if (threadIdx.x == 0) mbar_init(&bar, 1);
+    __syncthreads();
+    griddep();
+    if (threadIdx.x == 0) {
+        mbar_expect_tx(&bar, (unsigned)(sizeof(double) * ncol * ch));
+        for (int col = 0; col < ncol; ++col)
+            bulk_g2s(xsm + col * ldx, io.X[col] + e0, (unsigned)(sizeof(double) * ch), &bar);
+    }
+    for (int q = ncol * ch + threadIdx.x; q < 8 * NBLK * ch; q += blockDim.x) {
+        const int col = q / ch, e = q - col * ch;
+        xsm[col * ldx + e] = 0.0;
+    }
+    mbar_wait(&bar, 0);
+    __syncthreads();
+    double acc[NOCT][NBLK][2];
+#pragma unroll
+    for (int o = 0; o < NOCT; ++o)
+#pragma unroll
+        for (int b = 0; b < NBLK; ++b) { acc[o][b][0] = 0.0; acc[o][b][1] = 0.0; }
+#pragma unroll 1
+    for (int j0 = 0; j0 < nstep; j0 += NP) {
+#pragma unroll
+        for (int b = 0; b < NP; ++b) {
+            const int j = j0 + b;
+            if (j + NP - 1 < nstep) load(ring[(b + NP - 1) % NP], j + NP - 1);
+            d4 xb[NBLK];
+#pragma unroll
+            for (int bl = 0; bl < NBLK; ++bl) xb[bl] = lds256(xsm + (8 * bl + g) * ldx + 16 * j + 4 * k4);
+#pragma unroll
+            for (int o = 0; o < NOCT; ++o)
+#pragma unroll
+                for (int bl = 0; bl < NBLK; ++bl) {
+                    dmma884(acc[o][bl][0], acc[o][bl][1], ring[b][o].x, xb[bl].x);
+                    dmma884(acc[o][bl][0], acc[o][bl][1], ring[b][o].y, xb[bl].y);
+                    dmma884(acc[o][bl][0], acc[o][bl][1], ring[b][o].z, xb[bl].z);
+                    dmma884(acc[o][bl][0], acc[o][bl][1], ring[b][o].w, xb[bl].w);
+                }
+        }
+    }
+    // lane holds C[slab 8o + g][columns 8bl + 2k4, +1] = (I, F) sums of slice 4bl + k4
+#pragma unroll
+    for (int o = 0; o < NOCT; ++o) {
+        if (!okr[o]) continue;
+        const int row = row_lo + s0 + 8 * o + g;
+#pragma unroll
+        for (int bl = 0; bl < NBLK; ++bl) {
+            const int sl = 4 * bl + k4;
+            if (2 * sl < ncol) {
+                double* pp = io.part[sl];
+                pp[((long long)row * 2 + 0) * nchunk + c] = acc[o][bl][0];
+                pp[((long long)row * 2 + 1) * nchunk + c] = acc[o][bl][1];
+            }
+        }
+    }
+}
+
+constexpr int kMmaOct = 2, kMmaNP = 4;
+
+cudaError_t launch_boundary_batch(Ctx& c, int nslice, Ctx* const* slices, cudaStream_t s) {
+    const int nslab = c.i_hi - c.i_lo;
+    if (nslab <= 0) return cudaSuccess;
+    BatchIO io;
+    for (int k = 0; k < 2 * kMaxSlices; ++k) io.X[k] = nullptr;
+    for (int k = 0; k < kMaxSlices; ++k) io.part[k] = nullptr;
+    for (int k = 0; k < nslice; ++k) {
+        io.X[2 * k] = slices[k]->pcurr;
+        io.X[2 * k + 1] = slices[k]->pflip;
+        io.part[k] = slices[k]->tb_part;
+    }
+    const int spc = 8 * 8 * kMmaOct;  // slabs per CTA
+    const dim3 grid((unsigned)c.tbb_nchunk, (unsigned)((nslab + spc - 1) / spc));
+    const int n = c.nw * c.nh;
+    if (nslice <= 4)
+        return launch_pdl(k_bnd_tb_mma<1, kMmaOct, kMmaNP>, grid, dim3(256), sizeof(double) * 8 * (kBatchCh + 2), s,
+                          (const double*)c.T, c.S, nslab, c.i_lo, n, 2 * nslice, io, c.tbb_nchunk);
+    return launch_pdl(k_bnd_tb_mma<2, kMmaOct, kMmaNP>, grid, dim3(256), sizeof(double) * 16 * (kBatchCh + 2), s,
+                      (const double*)c.T, c.S, nslab, c.i_lo, n, 2 * nslice, io, c.tbb_nchunk);
+}
+
+// Top/bottom entries of psib from k_bnd_tb_mma partials (full-table mode, FFT left/right path: the
+// left/right entries were written by k_lr_ifft).
+cudaError_t launch_bnd_reduce(Ctx& c, const double* tb_part, int tb_nchunk, double* psib, cudaStream_t s) {
+    SymReduce sy{nullptr, 0, c.Tedge, c.S, c.pcurr, c.pflip};
+    return launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, tb_part, tb_nchunk, c.lr_part,
+                      c.t.lr_nblk, c.nw, c.nh, c.i_lo, c.i_hi, 0, 0, psib, sy);
+}
+
 // ================================================================================ interior solve
 
 // Forward complex FFT (exp(-2 pi i jk/M)) of M = 2^log2m points in shared memory, Stockham
@@ -2512,6 +2794,9 @@ cudaError_t prepare_kernels(Ctx& c) {
     if ((e = prepare_lr_fft(c))) return e;
     if ((e = big((const void*)k_bnd_tb<kTbGI, kTbUnroll>, 2 * sizeof(double) * c.t.tb_ch))) return e;
     if ((e = big((const void*)k_bnd_tb_otf<kTbGI>, 2 * sizeof(double) * c.t.tb_ch))) return e;
+    if ((e = big((const void*)k_bnd_tb_mma<2, kMmaOct, kMmaNP>, sizeof(double) * 16 * (kBatchCh + 2)))) return e;
+    if ((e = big((const void*)k_response_mma<3, kRespMmaNP>, sizeof(double) * 24 * (kRespBatchGc + 2)))) return e;
+    if ((e = big((const void*)k_response_mma<4, kRespMmaNP>, sizeof(double) * 32 * (kRespBatchGc + 2)))) return e;
     {
         const size_t sm = sym_smem(c);
         const void* ks[4] = {(const void*)k_bnd_sym<false, true, kSymUnr, kSymBuf, kSymWg>,

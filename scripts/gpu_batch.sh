@@ -1,0 +1,10 @@
+# multi-slice batch bring-up: GPU tests (batch first), then bench at S = 2, 4, 8
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests/test_gpu_batch.py -x -q 2>&1 | tail -25 | cut -c1-300
+timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
+for S in 2 4 8; do
+  timeout 300 python bench.py --steps 400 --warmup 10 --slices $S > gpurun_out/bench_s$S.log 2>&1
+  tail -1 gpurun_out/bench_s$S.log | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('S=$S', d['value'], d['ms_per_step'], d['roofline']['achieved'], d['roofline']['frac'], d['e2e']['value'])" || tail -5 gpurun_out/bench_s$S.log
+done
+timeout 600 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -s 100 -c 80 --csv --log-file gpurun_out/r01_launches_s4.csv python bench.py --steps 10 --warmup 10 --slices 4 > gpurun_out/ncu_s4.log 2>&1
+python scripts/ncu_summarize.py gpurun_out/r01_launches_s4.csv
