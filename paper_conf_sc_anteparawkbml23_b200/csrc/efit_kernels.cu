@@ -727,8 +727,11 @@ struct RespBatchIO {
     double* part[kMaxSlices];     // slice partials [row][k][chunk]
 };
 
+#ifndef EFIT_RESPB_MINB
+#define EFIT_RESPB_MINB 2
+#endif
 template <int NBLK, int NP>
-__global__ void __launch_bounds__(256, 2) k_response_mma(const double* __restrict__ Gd, long long S, int nrows, int n,
+__global__ void __launch_bounds__(256, EFIT_RESPB_MINB) k_response_mma(const double* __restrict__ Gd, long long S, int nrows, int n,
                                                         int nb, int ncol, long long ldb, RespBatchIO io, int nchunk) {
     constexpr int gc = kRespBatchGc, ldx = kRespBatchGc + 2, nstep = kRespBatchGc / 16;
     static_assert(nstep % NP == 0, "ring depth divides the steps");
@@ -766,9 +769,12 @@ __global__ void __launch_bounds__(256, 2) k_response_mma(const double* __restric
     }
     mbar_wait(&bar, 0);
     __syncthreads();
-    double acc[NBLK][2];
+    if ((blockIdx.y * 8 + warp) * 8 >= nrows) return;  // octet past the last row (warp-uniform)
+    // two accumulator sets per column block (k-substeps x, y | z, w): twice the independent DMMA
+    // chains per warp; summed once at the end
+    double acc[NBLK][2][2];
 #pragma unroll
-    for (int b = 0; b < NBLK; ++b) { acc[b][0] = 0.0; acc[b][1] = 0.0; }
+    for (int b = 0; b < NBLK; ++b) { acc[b][0][0] = acc[b][0][1] = acc[b][1][0] = acc[b][1][1] = 0.0; }
 #pragma unroll 1
     for (int j0 = 0; j0 < nstep; j0 += NP) {
 #pragma unroll
@@ -778,10 +784,10 @@ __global__ void __launch_bounds__(256, 2) k_response_mma(const double* __restric
 #pragma unroll
             for (int bl = 0; bl < NBLK; ++bl) {
                 const d4 xb = lds256(bsm + (8 * bl + g) * ldx + 16 * j + 4 * k4);
-                dmma884(acc[bl][0], acc[bl][1], ring[b].x, xb.x);
-                dmma884(acc[bl][0], acc[bl][1], ring[b].y, xb.y);
-                dmma884(acc[bl][0], acc[bl][1], ring[b].z, xb.z);
-                dmma884(acc[bl][0], acc[bl][1], ring[b].w, xb.w);
+                dmma884(acc[bl][0][0], acc[bl][0][1], ring[b].x, xb.x);
+                dmma884(acc[bl][1][0], acc[bl][1][1], ring[b].z, xb.z);
+                dmma884(acc[bl][0][0], acc[bl][0][1], ring[b].y, xb.y);
+                dmma884(acc[bl][1][0], acc[bl][1][1], ring[b].w, xb.w);
             }
         }
     }
@@ -793,7 +799,7 @@ __global__ void __launch_bounds__(256, 2) k_response_mma(const double* __restric
             const int col = 8 * bl + 2 * k4 + h;
             if (col < ncol) {
                 const int sl = col / nb, k = col - sl * nb;
-                io.part[sl][((long long)row * nb + k) * nchunk + c] = acc[bl][h];
+                io.part[sl][((long long)row * nb + k) * nchunk + c] = acc[bl][0][h] + acc[bl][1][h];
             }
         }
 }
@@ -819,7 +825,10 @@ cudaError_t launch_basis(Ctx& c, const double* psi, cudaStream_t s) {
 
 bool response_batch_ok(const Ctx& c, int nslice) { return nslice * c.nb <= 8 * kRespBatchMaxBlk; }
 
-constexpr int kRespMmaNP = 8;
+#ifndef EFIT_RESPB_NP
+#define EFIT_RESPB_NP 8
+#endif
+constexpr int kRespMmaNP = EFIT_RESPB_NP;
 
 // one pass over Gd for all slices (after every slice's k_basis)
 cudaError_t launch_response_batch(Ctx& c, int nslice, Ctx* const* slices, cudaStream_t s) {
