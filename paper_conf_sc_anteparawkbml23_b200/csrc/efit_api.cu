@@ -149,6 +149,8 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     c.tbb_nchunk = (int)((n + efit::kBatchCh - 1) / efit::kBatchCh);
     c.respb_nchunk = (int)((n + efit::kRespBatchGc - 1) / efit::kRespBatchGc);
     c.respb = false;
+    c.resp_mma = c.nb <= 8 * efit::kRespBatchMaxBlk && getenv("EFIT_RESP_MMA") != nullptr;
+    c.resp_fuse = getenv("EFIT_RESP_NOFUSE") == nullptr;
     t.tb_ch = 2048;
     t.tb_nchunk = (int)((n + t.tb_ch - 1) / t.tb_ch);
     t.tb_gi = 8;
@@ -212,7 +214,7 @@ static size_t carve_scratch(Ctx& c, Take& take, size_t& off, bool batch) {
     c.status = (int*)take(sizeof(int) * 4);
     c.tickets = (unsigned*)take(sizeof(unsigned) * 8);
     c.norm_part = (double*)take(sizeof(double) * 2 * (size_t)(c.t.red_blocks > c.ni + 2 ? c.t.red_blocks : c.ni + 2));
-    const int rchunk = batch && c.respb_nchunk > c.t.resp_nchunk ? c.respb_nchunk : c.t.resp_nchunk;
+    const int rchunk = (batch || c.resp_mma) && c.respb_nchunk > c.t.resp_nchunk ? c.respb_nchunk : c.t.resp_nchunk;
     c.resp_part = (double*)take(sizeof(double) * (size_t)rchunk * (nrows > 0 ? nrows : 1) * c.nb);
     c.resp_cnt = (double*)take(sizeof(double) * c.t.resp_nchunk);
     c.bmat = (double*)take(sizeof(double) * (size_t)c.nb * c.t.resp_nchunk * c.t.resp_gc);

@@ -556,10 +556,26 @@ __device__ __forceinline__ int bperm(int q) {  // node q of a chunk -> permuted 
     return (blk << 7) + (h << 6) + (lane << 1) + w;
 }
 
+// Fused basis (fb.on): instead of staging Bm written by a separate k_basis launch, each CTA evaluates
+// the basis of its own chunk from psi (after the wait on the predecessor that produced psi_axis /
+// psi_bdry), stores it in the staged layout and writes Bm for the current kernel, plus the chunk's
+// masked-node count: one launch less per iteration on the critical path.
+struct FusedBasis {
+    int on;
+    const double* psi;
+    const uint8_t* inlim;
+    const double* axbd;
+    int nh;
+    double rmin, dr, cell;
+    BasisParams bp;
+    double* Bm;        // written: [NB][ldb]
+    double* cnt_part;  // written: [nchunk]
+};
+
 template <int NB, int MB, int NP>
 __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ Gd, long long S, int nrows, int n,
                                                      const double* __restrict__ Bm, long long ldb, int gc,
-                                                     double* __restrict__ part) {
+                                                     double* __restrict__ part, FusedBasis fb) {
     // NP = rounds of MB row loads kept in a register ring: the warp's (row block, position) steps
     // form one flat sequence, and step s + NP - 1 is requested before step s is consumed, across
     // row-block boundaries (the first steps before the basis staging and the predecessor wait:
@@ -592,13 +608,42 @@ __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ 
     for (int b = 0; b + 1 < NP; ++b)
         if (b < nsteps) load_step(ring[b]);
     griddep();
+    if (fb.on) {
+        __shared__ int cnt_s;
+        if (threadIdx.x == 0) cnt_s = 0;
+        __syncthreads();
+        const double pa = fb.axbd[0], pb = fb.axbd[1];
+        int cnt = 0;
+        for (int q = threadIdx.x; q < gc; q += blockDim.x) {
+            const int g = g0 + q;
+            double f[NB];
 #pragma unroll
-    for (int k = 0; k < NB; ++k)
-        for (int q = 2 * threadIdx.x; q < gc; q += 2 * blockDim.x) {
-            const double2 v = __ldg(reinterpret_cast<const double2*>(Bm + k * ldb + g0 + q));
-            *reinterpret_cast<double2*>(Bs + k * gc + bperm(q)) = v;
+            for (int k = 0; k < NB; ++k) f[k] = 0.0;
+            double h;
+            if (g < n && node_psihat(fb.psi, fb.inlim, g, pa, pb, h)) {
+                basis_eval<NB>(fb.bp, h, grid_coord(fb.rmin, g / fb.nh, fb.dr), f);
+                ++cnt;
+            }
+#pragma unroll
+            for (int k = 0; k < NB; ++k) {
+                const double v = fb.cell * f[k];
+                Bs[k * gc + bperm(q)] = v;
+                fb.Bm[k * ldb + g] = v;
+            }
         }
-    __syncthreads();
+        cnt = __reduce_add_sync(0xffffffffu, cnt);
+        if ((threadIdx.x & 31) == 0) atomicAdd(&cnt_s, cnt);
+        __syncthreads();
+        if (threadIdx.x == 0) fb.cnt_part[c] = (double)cnt_s;
+    } else {
+#pragma unroll
+        for (int k = 0; k < NB; ++k)
+            for (int q = 2 * threadIdx.x; q < gc; q += 2 * blockDim.x) {
+                const double2 v = __ldg(reinterpret_cast<const double2*>(Bm + k * ldb + g0 + q));
+                *reinterpret_cast<double2*>(Bs + k * gc + bperm(q)) = v;
+            }
+        __syncthreads();
+    }
     double acc[MB][NB];
 #pragma unroll
     for (int r = 0; r < MB; ++r)
@@ -667,7 +712,9 @@ static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t
     const int gc = c.t.resp_gc;
     const size_t smem = sizeof(double) * NB * gc;
     const long long ldb = (long long)c.t.resp_nchunk * gc;
-    if (!prepare) {
+    FusedBasis fb{c.resp_fuse ? 1 : 0, psi, c.inlim, c.axbd, c.nh, c.rmin, c.dr, c.dr * c.dz, basis_params(c),
+                  c.bmat, c.resp_cnt};
+    if (!prepare && !c.resp_fuse) {
         BasisParams bp = basis_params(c);
         launch_pdl(k_basis<NB>, dim3(c.t.resp_nchunk), dim3(gc <= 1024 ? gc : 1024), 0, s, psi, c.inlim, c.axbd, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp,
                                                     gc, ldb, c.bmat, c.resp_cnt);
@@ -678,7 +725,7 @@ static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t
         auto kern = k_response<NB, MBV, resp_np(NB, MBV)>;                                                \
         if (prepare) { raise_smem_limit((const void*)kern, smem); break; }                               \
         dim3 grid(c.t.resp_nchunk);                                                                        \
-        launch_pdl(kern, dim3(grid), dim3(256), smem, s, c.Gd, c.S, nrows, c.nw * c.nh, c.bmat, ldb, gc, part);               \
+        launch_pdl(kern, dim3(grid), dim3(256), smem, s, c.Gd, c.S, nrows, c.nw * c.nh, c.bmat, ldb, gc, part, fb);           \
     } while (0)
     if (mb >= 4) EFIT_RESP_LAUNCH(4);
     else if (mb == 3) EFIT_RESP_LAUNCH(3);
@@ -690,6 +737,13 @@ static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t
 static cudaError_t response_impl(Ctx& c, const double* psi, double* resp_rows, cudaStream_t s, bool prepare) {
     const int nrows = c.m_hi - c.m_lo;
     if (nrows <= 0) return cudaSuccess;
+    if (c.resp_mma && !prepare) {  // the tensor-core contraction with a batch of one slice
+        cudaError_t e = launch_basis(c, psi, s);
+        if (e) return e;
+        Ctx* self = &c;
+        if ((e = launch_response_batch(c, 1, &self, s))) return e;
+        return launch_resp_reduce_batch(c, c.respb_nchunk, resp_rows, s);
+    }
     switch (c.nb) {
 #define EFIT_NB_CASE(V) case V: launch_resp_nb<V>(c, psi, c.resp_part, s, nrows, prepare); break;
         EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
