@@ -232,6 +232,7 @@ static size_t carve_scratch(Ctx& c, Take& take, size_t& off, bool batch) {
     c.psip = (double*)take(sizeof(double) * (size_t)n);
     c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 2));
     c.scratch_meas = (double*)take(sizeof(double) * c.ndiag);
+    c.sym_edge = c.sym ? (double*)take(sizeof(double) * 2 * (size_t)(c.nw > 2 ? c.nw - 2 : 1)) : nullptr;
     return (size_t)round_up((long long)off, 256);
 }
 

@@ -77,6 +77,7 @@ struct Ctx {
     double* symq;       // [sym_nblk][2 (I,F)][2 h][nh][2 qh][2]  per-iteration source columns, staged layout
     double* symp;       // [sym_nblk][2 (I,F)][8][nhp]             per-iteration block rows, 16-B aligned rows
     int nhp;            // nh rounded up to even (16-byte rows)
+    double* sym_edge;   // [2][nw-2] SYM: edge-row source sums of the top/bottom targets (per iteration)
     double* Tedge;      // [2][S]           slabs i = 0 and i = nw-1 (left/right)
     double* Gd;         // [m_hi-m_lo][S]   diagnostic Green's rows
     uint8_t* inlim;     // [nw*nh]

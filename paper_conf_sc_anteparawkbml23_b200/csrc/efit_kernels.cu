@@ -1527,7 +1527,32 @@ struct SymReduce {
     long long S;
     const double* pc;     // I  (zero-padded pcurr)
     const double* pf;     // F  (vertically mirrored)
+    const double* edge;   // SYM: edge-row source sums per top/bottom target (k_sym_edge_src), or nullptr
 };
+
+// SYM modes: the top/bottom targets' sums over the edge-row sources ii = 0, nw-1 (not in the half
+// table), from the replicated edge slabs: out[side*(nw-2) + i-1] = sum_m T0[i][m] X[0][m] + T1[i][m] X[nw-1][m],
+// X = I (bottom) or F (top).  One warp per target; runs on the side stream under the table stream.
+__global__ void k_sym_edge_src(const double* __restrict__ Tedge, long long S, const double* __restrict__ pc,
+                               const double* __restrict__ pf, int nw, int nh, int i_lo, int i_hi,
+                               double* __restrict__ out) {
+    griddep();
+    const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+    const int q = w;  // 0 .. 2(nw-2)-1
+    if (q >= 2 * (nw - 2)) return;
+    const int side = q < nw - 2 ? 0 : 1;
+    const int i = q - side * (nw - 2) + 1;
+    double s = 0.0;
+    if (i >= i_lo && i < i_hi) {
+        const double* x0 = (side ? pf : pc);
+        const double* x1 = x0 + (long long)(nw - 1) * nh;
+        const double* t0 = Tedge + (long long)i * nh;
+        const double* t1 = t0 + S;
+        for (int m = lane; m < nh; m += 32) s = fma(t0[m], x0[m], fma(t1[m], x1[m], s));
+    }
+    s = warp_sum(s);
+    if (lane == 0) out[q] = s;
+}
 
 __global__ void k_bnd_reduce(const double* __restrict__ tb_part, int tb_nchunk, const double* __restrict__ lr_part,
                              int lr_nblk, int nw, int nh, int i_lo, int i_hi, int jlo, int jhi,
@@ -1553,11 +1578,15 @@ __global__ void k_bnd_reduce(const double* __restrict__ tb_part, int tb_nchunk, 
             src = sy.part + ((long long)(i - 1) * 2 + side) * sy.nslot;
             cnt = sy.nslot;
             if (i >= i_lo && i < i_hi) {
-                const double* x0 = (side ? sy.pf : sy.pc);
-                const double* x1 = x0 + (long long)(nw - 1) * nh;
-                const double* t0 = sy.Tedge + (long long)i * nh;
-                const double* t1 = t0 + sy.S;
-                for (int m = lane; m < nh; m += 32) s = fma(t0[m], x0[m], fma(t1[m], x1[m], s));
+                if (sy.edge) {
+                    if (lane == 0) s = sy.edge[q];
+                } else {
+                    const double* x0 = (side ? sy.pf : sy.pc);
+                    const double* x1 = x0 + (long long)(nw - 1) * nh;
+                    const double* t0 = sy.Tedge + (long long)i * nh;
+                    const double* t1 = t0 + sy.S;
+                    for (int m = lane; m < nh; m += 32) s = fma(t0[m], x0[m], fma(t1[m], x1[m], s));
+                }
             }
         } else {
             if (i < i_lo || i >= i_hi) return;
@@ -1967,13 +1996,18 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     // left/right FFT chain has written psi_b(left/right), so its forward DST also runs under the
     // HBM-bound stream; k_tridiag adds the bottom/top terms in the sine domain afterwards
     if (overlap_solve && (e = launch_solve_fwd(c, pcurr, psib, c.side, 2))) return e;
+    if (c.sym && c.sym_edge &&
+        (e = launch_pdl(k_sym_edge_src, dim3((2 * (c.nw - 2) + 7) / 8), dim3(256), 0, c.side, (const double*)c.Tedge, c.S,
+                        (const double*)c.pcurr, (const double*)c.pflip, c.nw, c.nh, c.i_lo, c.i_hi, c.sym_edge)))
+        return e;
     mark(c, c.side, M_LR);
     if ((e = cudaEventRecord(c.ev_join, c.side))) return e;
     const int nslab = c.i_hi - c.i_lo;
     const size_t smem_tb = 2 * sizeof(double) * c.t.tb_ch;
-    SymReduce sy{nullptr, 0, c.Tedge, c.S, c.pcurr, c.pflip};
+    SymReduce sy{nullptr, 0, c.Tedge, c.S, c.pcurr, c.pflip, nullptr};
     if (c.sym) {
         sy.part = c.sym_part;
+        sy.edge = c.sym_edge;
         sy.nslot = c.sym_nblk * c.t.sym_nmc;
         const long long ntl = c.sym_tile_hi - c.sym_tile_lo;
         if (ntl > 0) {
@@ -2148,7 +2182,7 @@ cudaError_t launch_boundary_batch(Ctx& c, int nslice, Ctx* const* slices, cudaSt
 // Top/bottom entries of psib from k_bnd_tb_mma partials (full-table mode, FFT left/right path: the
 // left/right entries were written by k_lr_ifft).
 cudaError_t launch_bnd_reduce(Ctx& c, const double* tb_part, int tb_nchunk, double* psib, cudaStream_t s) {
-    SymReduce sy{nullptr, 0, c.Tedge, c.S, c.pcurr, c.pflip};
+    SymReduce sy{nullptr, 0, c.Tedge, c.S, c.pcurr, c.pflip, nullptr};
     return launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, tb_part, tb_nchunk, c.lr_part,
                       c.t.lr_nblk, c.nw, c.nh, c.i_lo, c.i_hi, 0, 0, psib, sy);
 }
