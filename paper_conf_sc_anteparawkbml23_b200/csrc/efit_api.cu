@@ -527,7 +527,7 @@ static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, 
     // boundary flux (marks M_TB, M_LR inside); in FFT mode the forward DST (without the bottom/top
     // edge terms) runs on the side stream under k_bnd_tb and the tridiagonal solve adds those terms
     const bool overlap = !c.lr_direct;
-    if ((e = launch_boundary(c, c.pcurr, c.psib, s, overlap))) return e;
+    if ((e = launch_boundary(c, c.pcurr, c.psib, s, overlap, c.sym))) return e;
     if (!overlap && (e = launch_solve_fwd(c, c.pcurr, c.psib, s, 1))) return e;
     if ((e = launch_solve_rest(c, c.psib, nullptr, psi, psi_ext, eps, s, true, overlap))) return e;
     mark(c, s, M_SOLVE);

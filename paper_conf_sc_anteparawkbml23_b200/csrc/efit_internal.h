@@ -174,8 +174,9 @@ cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const dou
                        double* coef, double* chi2, cudaStream_t s);
 cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double* pcurr,
                            bool pair, cudaStream_t s);
+// prepacked: the SYM staged layouts were written by this iteration's current kernel (fit step)
 cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s,
-                            bool overlap_solve = false);
+                            bool overlap_solve = false, bool prepacked = false);
 cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cudaStream_t s, int with_bnd);
 cudaError_t launch_solve_rest(Ctx& c, const double* psib, double* psi_out, double* psi_inout, const double* psi_ext,
                               double* eps, cudaStream_t s, bool next_norm, bool tb_fix);

@@ -367,6 +367,8 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
         const long long ntl = c.sym_tile_hi - c.sym_tile_lo;
         k_green_sym<<<sms * 16, bs, 0, s>>>(c.U, ntl, c.sym_tile_lo, c.ni, nh, c.rmin, c.dr, c.dz);
     }
+    if (c.symq && (e = cudaMemsetAsync(c.symq, 0, sizeof(double) * 16 * (size_t)c.sym_nblk * c.nh, s))) return e;
+    if (c.symp && (e = cudaMemsetAsync(c.symp, 0, sizeof(double) * 16 * (size_t)c.sym_nblk * c.nhp, s))) return e;
     if (c.sym_part &&
         (e = cudaMemsetAsync(c.sym_part, 0, sizeof(double) * 2 * (size_t)(c.ni > 0 ? c.ni : 1) * c.sym_nblk * c.t.sym_nmc, s)))
         return e;
@@ -1320,9 +1322,18 @@ __global__ void k_current(const double* __restrict__ psi, const uint8_t* __restr
 
 // Fit-step current from this iteration's basis matrix (already masked and scaled by dR dZ):
 // I_g = sum_k c_k Bm[k][g]  -- no second basis evaluation.
+// SYM modes: the current kernel also writes the staged layouts of k_sym_pack (interior rows only;
+// the zero padding of the last 8-row block is set once at init), so the fit step needs no pack launch.
+struct SymPackOut {
+    double* q;  // symq (nullptr: no packing)
+    double* p;  // symp
+    int narr, nhp, ni;
+};
+
 template <int NB>
 __global__ void k_current_from_basis(const double* __restrict__ Bm, long long ldb, const double* __restrict__ coef,
-                                     int nw, int nh, double* __restrict__ pcurr, double* __restrict__ pflip) {
+                                     int nw, int nh, double* __restrict__ pcurr, double* __restrict__ pflip,
+                                     SymPackOut sp) {
     griddep();
     const int n = nw * nh;
     double cf[NB];
@@ -1335,6 +1346,19 @@ __global__ void k_current_from_basis(const double* __restrict__ Bm, long long ld
         pcurr[g] = I;
         const int ii = g / nh, m = g - (g / nh) * nh;
         pflip[ii * nh + (nh - 1 - m)] = I;
+        const int r = ii - 1;
+        if (sp.q && r >= 0 && r < sp.ni) {  // symq[B][arr][h][m][qh][w], symp[B][arr][p][m] (k_sym_pack)
+            const int B = r >> 3, q = r & 7, qh = q >> 2, h = (q >> 1) & 1, w = q & 1;
+            const long long qb = (long long)B * 16 * nh + (long long)h * 4 * nh + 2 * qh + w;
+            const long long pb = (long long)B * 16 * sp.nhp + (long long)q * sp.nhp;
+            sp.q[qb + 4LL * m] = I;
+            sp.p[pb + m] = I;
+            if (sp.narr == 2) {  // F[ii][nh-1-m] = I
+                const int mf = nh - 1 - m;
+                sp.q[qb + 8LL * nh + 4LL * mf] = I;
+                sp.p[pb + 8LL * sp.nhp + mf] = I;
+            }
+        }
     }
 }
 
@@ -1343,10 +1367,16 @@ cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double
     BasisParams bp = basis_params(c);
     if (pair) {  // fit step: the basis matrix of this iteration is in c.bmat (k_basis ran in response)
         const int n = c.nw * c.nh;
+        SymPackOut sp{nullptr, nullptr, 0, c.nhp, c.ni};
+        if (c.sym && c.sym_tile_hi > c.sym_tile_lo && c.ni > 0) {
+            sp.q = c.symq;
+            sp.p = c.symp;
+            sp.narr = c.t.sym_nmc == 1 ? 1 : 2;
+        }
         const long long ldb = (long long)c.t.resp_nchunk * c.t.resp_gc;
         switch (c.nb) {
 #define EFIT_NB_CASE(V) \
-    case V: launch_pdl(k_current_from_basis<V>, dim3((n + 255) / 256), dim3(256), 0, s, c.bmat, ldb, coef, c.nw, c.nh, pcurr, c.pflip); break;
+    case V: launch_pdl(k_current_from_basis<V>, dim3((n + 255) / 256), dim3(256), 0, s, c.bmat, ldb, coef, c.nw, c.nh, pcurr, c.pflip, sp); break;
             EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
             EFIT_NB_CASE(7) EFIT_NB_CASE(8) EFIT_NB_CASE(9) EFIT_NB_CASE(10) EFIT_NB_CASE(11) EFIT_NB_CASE(12)
             EFIT_NB_CASE(13) EFIT_NB_CASE(14) EFIT_NB_CASE(15) EFIT_NB_CASE(16) EFIT_NB_CASE(17) EFIT_NB_CASE(18)
@@ -1982,7 +2012,8 @@ static cudaError_t launch_lr(Ctx& c, cudaStream_t s, bool prepare) {
 
 cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cudaStream_t s, int with_bnd);
 
-cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s, bool overlap_solve) {
+cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s, bool overlap_solve,
+                            bool prepacked) {
     cudaError_t e;
     // fork: the FP64-bound left/right kernel runs on the side stream, concurrently with the
     // HBM-bound top/bottom stream (both only read pcurr / ipair); join before the reduce.
@@ -2012,8 +2043,9 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
         const long long ntl = c.sym_tile_hi - c.sym_tile_lo;
         if (ntl > 0) {
             const int narr = c.t.sym_nmc == 1 ? 1 : 2;
-            launch_pdl(k_sym_pack, dim3(4 * kNumSMs), dim3(256), 0, s, (const double*)c.pcurr, (const double*)c.pflip,
-                       c.nh, c.nhp, c.ni, c.sym_nblk, narr, c.symq, c.symp);
+            if (!prepacked)
+                launch_pdl(k_sym_pack, dim3(4 * kNumSMs), dim3(256), 0, s, (const double*)c.pcurr, (const double*)c.pflip,
+                           c.nh, c.nhp, c.ni, c.sym_nblk, narr, c.symq, c.symp);
             if ((e = cudaGetLastError())) return e;
             const size_t smem = sym_smem(c);
             const bool mir = c.t.sym_nmc == 1;
