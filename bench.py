@@ -456,6 +456,26 @@ def gpu_arm(args, rank, world, local):
             "bound": "hbm", "achieved": round(tb_gbs, 1), "peak": peak, "unit": "GB/s",
             "frac": round(tb_gbs / peak, 4), "traffic": traffic, "peak_source": peak_kind,
             "algorithmic_bytes_per_launch": tb_bytes}
+    if args.mode in ("otf", "otf-sym"):
+        # recomputed Green's functions: FP64-ALU bound.  FLOPs per launch = the kernel's executed
+        # dadd + dmul + 2 dfma (ncu, profiles/ncu_summary.json) for this config; peak derived from the
+        # unit counts: 148 SMs x 64 FP64 FMA/clk x 2 x 1.965 GHz
+        key = "k_bnd_tb_otf" if args.mode == "otf" else "k_bnd_sym_otf"
+        flops = None
+        if os.path.exists(ncu_sum):
+            try:
+                d = json.load(open(ncu_sum))
+                if d.get("config") == args.config and world == 1:
+                    flops = d.get(key, {}).get("fp64_flops_per_launch")
+            except Exception:
+                flops = None
+        fp64_peak = 148 * 64 * 2 * 1.965e9 / 1e12
+        tf = flops / (tb_ms * 1e-3) / 1e12 if flops else None
+        roof = {"kernel": key.replace("_otf", "") + " (on-the-fly)", "bound": "alu",
+                "achieved": round(tf, 2) if tf else None, "peak": round(fp64_peak, 2), "unit": "TFLOP/s",
+                "frac": round(tf / fp64_peak, 4) if tf else None, "traffic": None,
+                "peak_source": "derived from unit counts (no measured FP64 peak)",
+                "fp64_flops_per_launch": flops}
     rb = None
     if rb_ms is not None:
         rb_gbs = (tb_bytes + gd_bytes) / (rb_ms * 1e-3) / 1e9
