@@ -16,7 +16,7 @@ constexpr int kLsqMaxRowsHost = 960;
 constexpr int kMaxSlices = 8;   // multi-time-slice batch (efit_batch_attach): slices per pass
 constexpr int kBatchCh = 512;   // k_bnd_tb_mma: table elements per chunk (16 per mma k-step quad)
 constexpr int kRespBatchGc = 256;   // k_response_mma: grid nodes per chunk
-constexpr int kRespBatchMaxBlk = 4; // k_response_mma: <= 32 basis columns (slices x nbasis) per pass  // k_lsq shared memory: (nb|1 + 2)*nd doubles
+constexpr int kRespBatchMaxBlk = 5; // k_response_mma: <= 40 basis columns (slices x nbasis) per pass  // k_lsq shared memory: (nb|1 + 2)*nd doubles
 
 // k_response: depth of the register ring of MB-row load steps (4 registers per 256-bit load),
 // keeping ring (4 NP MB) + accumulators (MB NB) <= 56 registers (the rest of the 128-register

@@ -885,6 +885,8 @@ bool response_batch_ok(const Ctx& c, int nslice) { return nslice * c.nb <= 8 * k
 #define EFIT_RESPB_NP 8
 #endif
 constexpr int kRespMmaNP = EFIT_RESPB_NP;
+// ring depth: the accumulators of 5 column blocks (20 doubles) leave room for 4 steps in flight
+constexpr int resp_mma_np(int nblk) { return nblk >= 5 ? 4 : kRespMmaNP; }
 
 // one pass over Gd for all slices (after every slice's k_basis)
 cudaError_t launch_response_batch(Ctx& c, int nslice, Ctx* const* slices, cudaStream_t s) {
@@ -901,9 +903,9 @@ cudaError_t launch_response_batch(Ctx& c, int nslice, Ctx* const* slices, cudaSt
     switch (nblk) {
 #define EFIT_RB(V)                                                                                                 \
     case V:                                                                                                        \
-        return launch_pdl(k_response_mma<V, kRespMmaNP>, grid, dim3(256), sizeof(double) * 8 * V * (kRespBatchGc + 2), s, \
+        return launch_pdl(k_response_mma<V, resp_mma_np(V)>, grid, dim3(256), sizeof(double) * 8 * V * (kRespBatchGc + 2), s, \
                           (const double*)c.Gd, c.S, nrows, n, c.nb, ncol, ldb, io, c.respb_nchunk);
-        EFIT_RB(1) EFIT_RB(2) EFIT_RB(3) EFIT_RB(4)
+        EFIT_RB(1) EFIT_RB(2) EFIT_RB(3) EFIT_RB(4) EFIT_RB(5)
 #undef EFIT_RB
         default: return cudaErrorInvalidValue;
     }
@@ -2924,8 +2926,9 @@ cudaError_t prepare_kernels(Ctx& c) {
     if ((e = big((const void*)k_bnd_tb<kTbGI, kTbUnroll>, 2 * sizeof(double) * c.t.tb_ch))) return e;
     if ((e = big((const void*)k_bnd_tb_otf<kTbGI>, 2 * sizeof(double) * c.t.tb_ch))) return e;
     if ((e = big((const void*)k_bnd_tb_mma<2, kMmaOct, kMmaNP>, sizeof(double) * 16 * (kBatchCh + 2)))) return e;
-    if ((e = big((const void*)k_response_mma<3, kRespMmaNP>, sizeof(double) * 24 * (kRespBatchGc + 2)))) return e;
-    if ((e = big((const void*)k_response_mma<4, kRespMmaNP>, sizeof(double) * 32 * (kRespBatchGc + 2)))) return e;
+    if ((e = big((const void*)k_response_mma<3, resp_mma_np(3)>, sizeof(double) * 24 * (kRespBatchGc + 2)))) return e;
+    if ((e = big((const void*)k_response_mma<4, resp_mma_np(4)>, sizeof(double) * 32 * (kRespBatchGc + 2)))) return e;
+    if ((e = big((const void*)k_response_mma<5, resp_mma_np(5)>, sizeof(double) * 40 * (kRespBatchGc + 2)))) return e;
     {
         const size_t sm = sym_smem(c);
         const void* ks[4] = {(const void*)k_bnd_sym<false, true, kSymUnr, kSymBuf, kSymWg>,

@@ -104,7 +104,7 @@ def _slices(orc, cfg, S):
 
 
 @pytest.mark.parametrize("name", ["33x33", "C1", "C2"])
-@pytest.mark.parametrize("S", [1, 3, 4])
+@pytest.mark.parametrize("S", [1, 3, 4, 8])
 def test_batch_fit_step(torch_mod, efit, orc_mod, name, S):
     torch = torch_mod
     cfg, orc, ctx = setup(name, efit, orc_mod)
