@@ -515,3 +515,37 @@ def test_fit_steps_chained_equals_repeated(torch_mod, efit, orc_mod):
         outs.append((psi.clone(), coef.clone(), eps.clone()))
     for a, b in zip(*outs):
         assert torch.equal(a, b)
+
+
+# ------------------------------------------------------------------ stress size (C5 1025^2): sampled
+
+@pytest.mark.parametrize("mode", [0, 2])  # full table (8.6 GB) and half table: the m-chunked SYM path
+def test_c5_boundary_sampled(torch_mod, efit, orc_mod, mode):
+    """configs[4] (1025^2, the largest grid the ABI is quoted on): sampled edge targets, including
+    the corners and both ends of every side, against the oracle's per-target sums."""
+    torch = torch_mod
+    c = case("C5", efit, orc_mod, mode=mode)
+    I = synth.random_current(c.cfg.grid, seed=3, signed=True)
+    out = c.ctx.boundary_flux(T(torch, I)).cpu().numpy()
+    nh, nw = c.cfg.grid.nh, c.cfg.grid.nw
+    fixed = [0, nh - 1, nh, 2 * nh - 1, 2 * nh, 2 * nh + nw - 3, 2 * nh + nw - 2, c.ctx.n_edge - 1]
+    rng = np.random.default_rng(1)
+    tg = np.unique(np.concatenate([fixed, rng.integers(0, c.ctx.n_edge, 24)]))
+    ref = c.orc.boundary_targets(I, tg)
+    assert rel(out[tg], ref) < TOL
+    c.ctx.close()
+    _cases.pop(("C5", mode, None, 0), None)
+
+
+def test_c5_response_sampled(torch_mod, efit, orc_mod):
+    torch = torch_mod
+    c = case("C5", efit, orc_mod, mode=efit.EFIT_GREEN_TABLE_SYM)
+    psi = synth.perturbed_psi(c.cfg.grid, seed=5, rel=1e-3)
+    resp, axbd = c.ctx.response(T(torch, psi))
+    rows = [0, 43, 44, 119]
+    ref = c.orc.response_rows(psi, rows)
+    r = resp.cpu().numpy()[rows]
+    for k in range(c.ctx.nbasis):
+        assert rel(r[:, k], ref[:, k]) < TOL
+    c.ctx.close()
+    _cases.pop(("C5", efit.EFIT_GREEN_TABLE_SYM, None, 0), None)
