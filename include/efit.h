@@ -238,6 +238,17 @@ int efit_fit_steps_batch(efit_ctx* ctx, int32_t nsteps, double* d_psi, const dou
  * semantics per slice). */
 int efit_boundary_flux_batch(efit_ctx* ctx, const double* d_pcurr, double* d_psib, efit_stream_t stream);
 
+/* Fused single-pass variant: the boundary flux of every basis current instead of
+ * the fitted one.  d_rb[k*n_edge + p] = sum_g G(x_p; x_g) I_k[g], with I_k[g] = dR dZ mask_g w_k(R_g)
+ * phi_k(psihat_g) the current of basis function k alone (Eq. 2 with c = e_k, mask and psihat of
+ * d_psi), edge order as efit_boundary_flux.  By linearity psi_b = sum_k c_k d_rb[k] for any
+ * coefficients, so the O(N^3) table pass no longer waits for the least squares (it depends on psi
+ * only, like efit_response) at nbasis right-hand-side pairs per table element (the shared
+ * tensor-core pass of the batch).  Needs a batch of >= nbasis slices attached (their scratch holds
+ * the basis currents); d_axbd[2] (may be NULL) receives {psi_axis, psi_bdry}.  EFIT_E_STATE
+ * otherwise. */
+int efit_boundary_basis(efit_ctx* ctx, const double* d_psi, double* d_rb, double* d_axbd, efit_stream_t stream);
+
 /* Per-step kernel timing (the measurement hook used by bench.py).  After
  * efit_profile_begin(ctx, n, every), every `every`-th efit_fit_step call (the 1st, (every+1)-th, ...)
  * records CUDA events at seven marks, on the streams the kernels run on, until n steps are recorded.  The calls enqueue eagerly, or -- when the caller is capturing the stream into its own CUDA

@@ -24,7 +24,7 @@ __all__ = [
     "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY", "EFIT_GREEN_TABLE_SYM",
     "EFIT_GREEN_ONTHEFLY_SYM", "efit_plan_info", "owned_targets", "exchange",
     "efit_batch_workspace_bytes", "efit_batch_attach", "efit_fit_step_batch", "efit_fit_steps_batch",
-    "efit_boundary_flux_batch",
+    "efit_boundary_flux_batch", "efit_boundary_basis",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -117,6 +117,7 @@ def lib() -> ctypes.CDLL:
             "efit_fit_step_batch": (I, [vp, vp, vp, vp, vp, vp, vp, vp, vp]),
             "efit_fit_steps_batch": (I, [vp, ctypes.c_int32, vp, vp, vp, vp, vp, vp, vp, vp]),
             "efit_boundary_flux_batch": (I, [vp, vp, vp, vp]),
+            "efit_boundary_basis": (I, [vp, vp, vp, vp, vp]),
             "efit_shard": (None, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int32),
                                   P(ctypes.c_int32)]),
             "efit_destroy": (I, [vp]),
@@ -305,6 +306,10 @@ def efit_boundary_flux_batch(ctx, pcurr, psib, stream=None) -> None:
     _check(lib().efit_boundary_flux_batch(ctx, _ptr(pcurr), _ptr(psib), _stream(stream)), ctx)
 
 
+def efit_boundary_basis(ctx, psi, rb, axbd=None, stream=None) -> None:
+    _check(lib().efit_boundary_basis(ctx, _ptr(psi), _ptr(rb), _ptr(axbd), _stream(stream)), ctx)
+
+
 def efit_status(ctx, stream=None) -> int:
     return lib().efit_status(ctx, _stream(stream))
 
@@ -426,6 +431,12 @@ class EfitContext:
 
     def fit_steps_batch(self, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None):
         efit_fit_steps_batch(self.handle, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream)
+
+    def boundary_basis(self, psi, stream=None):
+        """[nbasis, n_edge]: boundary flux of every basis current of psi (efit_boundary_basis)."""
+        out = self._t(self.nbasis * self.n_edge)
+        efit_boundary_basis(self.handle, psi, out, None, stream)
+        return out.view(self.nbasis, self.n_edge)
 
     def boundary_flux_batch(self, pcurr, stream=None):
         out = self._t(self.nslice * self.n_edge)

@@ -813,6 +813,34 @@ extern "C" int efit_fit_steps_batch(efit_ctx* h, int32_t nsteps, double* d_psi, 
     return fit_steps_batch_impl(h, nsteps, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, stream);
 }
 
+// Shared table pass for ns current pairs: slice k's current is src + k * src_ld (n nodes); its
+// boundary flux goes to d_psib + k * n_edge.  Slice streams fork from / join into s.
+static cudaError_t enqueue_boundary_batch(Ctx& c, int ns, const double* src, size_t src_ld, double* d_psib,
+                                          cudaStream_t s) {
+    cudaError_t e1;
+    if ((e1 = cudaEventRecord(c.bev_fork, s))) return e1;
+    for (int k = 0; k < ns; ++k) {
+        Ctx& q = *c.slice[k];
+        if ((e1 = cudaStreamWaitEvent(q.side, c.bev_fork, 0))) return e1;
+        if ((e1 = efit::launch_make_pair(q, src + k * src_ld, q.side))) return e1;
+        if ((e1 = cudaEventRecord(q.ev_fork, q.side))) return e1;
+        if ((e1 = efit::launch_lr_fft(q, d_psib + (size_t)k * c.n_edge, q.side))) return e1;
+    }
+    for (int k = 0; k < ns; ++k)
+        if ((e1 = cudaStreamWaitEvent(s, c.slice[k]->ev_fork, 0))) return e1;
+    if ((e1 = efit::launch_boundary_batch(c, ns, c.slice, s))) return e1;
+    if ((e1 = cudaEventRecord(c.bev_tb, s))) return e1;
+    for (int k = 0; k < ns; ++k) {
+        Ctx& q = *c.slice[k];
+        if ((e1 = cudaStreamWaitEvent(q.side, c.bev_tb, 0))) return e1;
+        if ((e1 = efit::launch_bnd_reduce(q, q.tb_part, c.tbb_nchunk, d_psib + (size_t)k * c.n_edge, q.side))) return e1;
+        if ((e1 = cudaEventRecord(q.ev_join, q.side))) return e1;
+    }
+    for (int k = 0; k < ns; ++k)
+        if ((e1 = cudaStreamWaitEvent(s, c.slice[k]->ev_join, 0))) return e1;
+    return cudaSuccess;
+}
+
 extern "C" int efit_boundary_flux_batch(efit_ctx* h, const double* d_pcurr, double* d_psib, efit_stream_t stream) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
     Ctx& c = h->c;
@@ -821,33 +849,28 @@ extern "C" int efit_boundary_flux_batch(efit_ctx* h, const double* d_pcurr, doub
     EFIT_CHECK_PTR(c, d_psib, "d_psib");
     cudaStream_t s = (cudaStream_t)stream;
     if (s == nullptr) return fail(&c, EFIT_E_INVAL, "batched calls need a non-default stream");
-    const size_t n = (size_t)c.nw * c.nh;
+    cudaError_t e = enqueue_boundary_batch(c, c.nslice, d_pcurr, (size_t)c.nw * c.nh, d_psib, s);
+    if (e) return cuda_fail(&c, e, "batched boundary flux");
+    return EFIT_OK;
+}
+
+extern "C" int efit_boundary_basis(efit_ctx* h, const double* d_psi, double* d_rb, double* d_axbd,
+                                   efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    if (c.nslice < c.nb)
+        return fail(&c, EFIT_E_STATE, "efit_boundary_basis needs a batch of >= nbasis (%d) slices", c.nb);
+    EFIT_CHECK_PTR(c, d_psi, "d_psi");
+    EFIT_CHECK_PTR(c, d_rb, "d_rb");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (s == nullptr) return fail(&c, EFIT_E_INVAL, "batched calls need a non-default stream");
     cudaError_t e;
-    auto run = [&]() -> cudaError_t {
-        cudaError_t e1;
-        if ((e1 = cudaEventRecord(c.bev_fork, s))) return e1;
-        for (int k = 0; k < c.nslice; ++k) {
-            Ctx& q = *c.slice[k];
-            if ((e1 = cudaStreamWaitEvent(q.side, c.bev_fork, 0))) return e1;
-            if ((e1 = efit::launch_make_pair(q, d_pcurr + k * n, q.side))) return e1;
-            if ((e1 = cudaEventRecord(q.ev_fork, q.side))) return e1;
-            if ((e1 = efit::launch_lr_fft(q, d_psib + (size_t)k * c.n_edge, q.side))) return e1;
-        }
-        for (int k = 0; k < c.nslice; ++k)
-            if ((e1 = cudaStreamWaitEvent(s, c.slice[k]->ev_fork, 0))) return e1;
-        if ((e1 = efit::launch_boundary_batch(c, c.nslice, c.slice, s))) return e1;
-        if ((e1 = cudaEventRecord(c.bev_tb, s))) return e1;
-        for (int k = 0; k < c.nslice; ++k) {
-            Ctx& q = *c.slice[k];
-            if ((e1 = cudaStreamWaitEvent(q.side, c.bev_tb, 0))) return e1;
-            if ((e1 = efit::launch_bnd_reduce(q, q.tb_part, c.tbb_nchunk, d_psib + (size_t)k * c.n_edge, q.side))) return e1;
-            if ((e1 = cudaEventRecord(q.ev_join, q.side))) return e1;
-        }
-        for (int k = 0; k < c.nslice; ++k)
-            if ((e1 = cudaStreamWaitEvent(s, c.slice[k]->ev_join, 0))) return e1;
-        return cudaSuccess;
-    };
-    if ((e = run())) return cuda_fail(&c, e, "batched boundary flux");
+    if ((e = efit::launch_normalize(c, d_psi, s))) return cuda_fail(&c, e, "normalize");
+    if ((e = efit::launch_basis(c, d_psi, s))) return cuda_fail(&c, e, "basis");
+    const size_t ldb = (size_t)c.t.resp_nchunk * c.t.resp_gc;  // basis matrix row stride
+    if ((e = enqueue_boundary_batch(c, c.nb, c.bmat, ldb, d_rb, s))) return cuda_fail(&c, e, "boundary basis");
+    if (d_axbd && (e = cudaMemcpyAsync(d_axbd, c.axbd, 2 * sizeof(double), cudaMemcpyDeviceToDevice, s)))
+        return cuda_fail(&c, e, "axbd copy");
     return EFIT_OK;
 }
 

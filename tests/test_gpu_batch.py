@@ -225,3 +225,38 @@ def test_c4_batch_boundary_sampled(torch_mod, efit, orc_mod):
     for k in range(S):
         ref = orc.boundary_targets(Is[k], tg)
         assert rel(out[k][tg], ref) < TOL, (k, rel(out[k][tg], ref))
+
+
+@pytest.mark.parametrize("name", ["33x33", "40x33", "C1", "C2"])
+def test_boundary_basis(torch_mod, efit, orc_mod, name):
+    """the boundary flux of every basis current (efit_boundary_basis) equals the
+    oracle's boundary flux of the current with c = e_k, and sum_k c_k R_b[k] equals the paper-order
+    path boundary_flux(current(psi, c)) (linearity)."""
+    torch = torch_mod
+    cfg, orc, ctx = setup(name, efit, orc_mod)
+    nb = ctx.nbasis
+    ctx.batch_attach(nb)
+    psi0 = synth.perturbed_psi(cfg.grid, seed=5, rel=1e-3)
+    st = torch.cuda.Stream()
+    with torch.cuda.stream(st):
+        rb = ctx.boundary_basis(T(torch, psi0), stream=st)
+    st.synchronize()
+    assert ctx.status() == 0
+    rb = rb.cpu().numpy()
+    for k in range(nb):
+        e = np.zeros(nb)
+        e[k] = 1.0
+        ref = orc.boundary(orc.current(psi0, e))
+        assert rel(rb[k], ref) < TOL, (k, rel(rb[k], ref))
+    c = synth.c_true(cfg.basis)
+    direct = ctx.boundary_flux(ctx.current(T(torch, psi0), T(torch, c))).cpu().numpy()
+    assert rel(c @ rb, direct) < TOL
+
+
+def test_boundary_basis_needs_batch(torch_mod, efit, orc_mod):
+    torch = torch_mod
+    cfg, orc, ctx = setup("9x9", efit, orc_mod)
+    ctx.batch_attach(1)
+    with pytest.raises(efit.EfitError) as ei:
+        ctx.boundary_basis(T(torch, synth.perturbed_psi(cfg.grid, seed=5, rel=1e-3)), stream=torch.cuda.Stream())
+    assert ei.value.code == efit.EFIT_E_STATE
