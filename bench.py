@@ -540,11 +540,13 @@ def gpu_arm(args, rank, world, local):
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(args.config)
 
-    # our kernels per step (ncu launch list, profiles/): basis, response, resp_reduce, lsq, current,
-    # lr_fft, lr_mac, lr_ifft, dst_fwd, bnd_tb | (sym_pack + bnd_sym), bnd_reduce, tridiag, dst_inv;
-    # + k_normalize at the start of every captured graph; sharded: + make-pair, normalize, solve fwd
-    per_step = 13 + (1 if args.mode in ("sym", "otf-sym") else 0)
-    launches = per_step * K + len(graphs) if sharded is None else (per_step + 2) * K
+    # our kernels per step (ncu launch list, profiles/r01_launches_final.csv): response (basis fused),
+    # resp_reduce, lsq, current, lr_fft, lr_mac, lr_ifft, dst_fwd, bnd_tb | (bnd_sym + sym_edge_src),
+    # bnd_reduce, tridiag, dst_inv; + k_normalize at the start of every captured graph.
+    # sharded (step API): + normalize, make_pair (+ sym_pack in the SYM modes) every step
+    sym_mode = args.mode in ("sym", "otf-sym")
+    per_step = 12 + (1 if sym_mode else 0)
+    launches = per_step * K + len(graphs) if sharded is None else (per_step + 2 + (1 if sym_mode else 0)) * K
     if rank == 0:
         out = {
             "metric": METRIC, "value": round(1000.0 / ms_step, 2), "unit": UNIT,
