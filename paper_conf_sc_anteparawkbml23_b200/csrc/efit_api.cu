@@ -678,7 +678,10 @@ extern "C" int efit_batch_attach(efit_ctx* h, int32_t nslice, void* d_workspace,
         };
         carve_scratch(*q, take, off, true);
         q->status = c.status;  // one sticky status word for the whole batch
-        if ((e = cudaStreamCreateWithPriority(&q->side, cudaStreamNonBlocking, prio_hi)) ||
+        // slice streams at normal priority: the shared table pass (main stream) keeps its SMs while the
+        // slices' latency-bound chains fill in (measured +1.7 % at S = 8 over high priority)
+        const int prio = getenv("EFIT_BATCH_HIPRIO") ? prio_hi : prio_lo;
+        if ((e = cudaStreamCreateWithPriority(&q->side, cudaStreamNonBlocking, prio)) ||
             (e = cudaEventCreateWithFlags(&q->ev_fork, cudaEventDisableTiming)) ||
             (e = cudaEventCreateWithFlags(&q->ev_join, cudaEventDisableTiming))) {
             release_slices(c);
