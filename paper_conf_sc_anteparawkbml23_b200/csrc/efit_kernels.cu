@@ -588,6 +588,15 @@ __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int qend = min(gc, n - g0);  // valid nodes; a 4-wide load may read up to 3 zero pads
     const int npos = (qend + 127) >> 7;  // 128-node positions of this chunk
+    if (gridDim.y > 1) {  // small grids: blockIdx.y splits the rows (whole MB-row blocks) so that enough
+        // CTAs stream; every (row, chunk) partial is still written by exactly one CTA.  Folded into
+        // the row base once, so the streaming loop is the unsplit one.
+        const int rbpc = ((nrows + MB - 1) / MB + gridDim.y - 1) / gridDim.y;
+        const int r0 = blockIdx.y * rbpc * MB;
+        Gd += (long long)r0 * S;
+        part += (long long)r0 * NB * gridDim.x;
+        nrows = max(0, min(nrows - r0, rbpc * MB));
+    }
     const int nmb = (nrows + MB - 1) / MB;
     const int nwarps = (int)(blockDim.x >> 5);
     const int nmb_w = warp < nmb ? (nmb - warp + nwarps - 1) / nwarps : 0;  // row blocks warp, warp+8, ...
@@ -630,13 +639,13 @@ __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ 
             for (int k = 0; k < NB; ++k) {
                 const double v = fb.cell * f[k];
                 Bs[k * gc + bperm(q)] = v;
-                fb.Bm[k * ldb + g] = v;
+                if (blockIdx.y == 0) fb.Bm[k * ldb + g] = v;
             }
         }
         cnt = __reduce_add_sync(0xffffffffu, cnt);
         if ((threadIdx.x & 31) == 0) atomicAdd(&cnt_s, cnt);
         __syncthreads();
-        if (threadIdx.x == 0) fb.cnt_part[c] = (double)cnt_s;
+        if (threadIdx.x == 0 && blockIdx.y == 0) fb.cnt_part[c] = (double)cnt_s;
     } else {
 #pragma unroll
         for (int k = 0; k < NB; ++k)
@@ -708,6 +717,17 @@ __global__ void k_resp_reduce(const double* __restrict__ part, const double* __r
     }
 }
 
+// CTAs per chunk along the row blocks, for small grids only (each split CTA re-evaluates its chunk's
+// basis): up to 2 CTAs per SM, >= 8 row blocks (one per warp) per CTA, and no split unless it at
+// least triples the CTA count (measured: a 2-way split loses at 257^2 and 513^2, wins at 65^2/129^2)
+static unsigned resp_row_split(const Ctx& c, int mb, int nrows) {
+    const int nmb = (nrows + mb - 1) / mb;
+    int ry = (2 * kNumSMs) / c.t.resp_nchunk;
+    const int cap = (nmb + 7) / 8;
+    if (ry > cap) ry = cap;
+    return (unsigned)(ry < 3 ? 1 : ry);
+}
+
 template <int NB>
 static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t s, int nrows, bool prepare) {
     static_assert(resp_np(NB, 1) >= 1, "positions per step");
@@ -726,7 +746,7 @@ static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t
     do {                                                                                                   \
         auto kern = k_response<NB, MBV, resp_np(NB, MBV)>;                                                \
         if (prepare) { raise_smem_limit((const void*)kern, smem); break; }                               \
-        dim3 grid(c.t.resp_nchunk);                                                                        \
+        dim3 grid(c.t.resp_nchunk, resp_row_split(c, MBV, nrows));                                       \
         launch_pdl(kern, dim3(grid), dim3(256), smem, s, c.Gd, c.S, nrows, c.nw * c.nh, c.bmat, ldb, gc, part, fb);           \
     } while (0)
     if (mb >= 4) EFIT_RESP_LAUNCH(4);
