@@ -217,7 +217,7 @@ int efit_solve_update(efit_ctx* ctx, const double* d_pcurr, const double* d_psib
  *   aligned, kept alive until efit_destroy or the next attach; cleared here, synchronising the
  *   device) and create one stream per slice.  Re-attaching replaces the previous batch.
  *   EFIT_E_INVAL: nslice outside [1, 8] / bad workspace; EFIT_E_NOMEM: too small;
- *   EFIT_E_STATE: mode != EFIT_GREEN_TABLE, world > 1 or EFIT_LR_DIRECT set. */
+ *   EFIT_E_STATE: mode != EFIT_GREEN_TABLE or world > 1. */
 int efit_batch_workspace_bytes(const efit_ctx* ctx, int32_t nslice, size_t* bytes_out);
 int efit_batch_attach(efit_ctx* ctx, int32_t nslice, void* d_workspace, size_t ws_bytes);
 

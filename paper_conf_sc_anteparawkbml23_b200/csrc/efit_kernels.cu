@@ -380,7 +380,7 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
                                                      c.nmode, c.rmin, c.dr, c.dz);
     k_twiddles<<<(c.fft_m / 2 + 255) / 256, 256, 0, s>>>(c.twiddle, c.fft_m);
     k_sin_table<<<(c.nmode + 255) / 256, 256, 0, s>>>(c.sin_tab, c.nmode);
-    if (!c.lr_direct) {  // needs the edge slabs and the twiddles above
+    {  // needs the edge slabs and the twiddles above (also built in direct mode: the batch uses the FFT chain)
         e = launch_lr_spectra(c, s);
         if (e) return e;
     }
