@@ -149,7 +149,16 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     c.tbb_nchunk = (int)((n + efit::kBatchCh - 1) / efit::kBatchCh);
     c.respb_nchunk = (int)((n + efit::kRespBatchGc - 1) / efit::kRespBatchGc);
     c.respb = false;
-    c.resp_mma = c.nb <= 8 * efit::kRespBatchMaxBlk && getenv("EFIT_RESP_MMA") != nullptr;
+    // single-slice response on the DMMA kernel: for wide bases (nb >= 8: the scalar kernel's nb
+    // accumulators per row limit its loads in flight; measured 117 -> 48 us at C3, nb = 20) and
+    // ~129^2 grids (C2: 18.0 -> 15.5 us); the scalar stream stays at 65^2 (C1: 13.1 vs 14.7 us) and at
+    // 257^2+ with narrow bases (C4: 58 vs 66 us).  EFIT_RESP_MMA=1 / =0 forces either.
+    {
+        const char* ev = getenv("EFIT_RESP_MMA");
+        const long long nn = (long long)c.nw * c.nh;
+        const bool want = ev ? ev[0] != '0' : (c.nb >= 8 || (nn > 96LL * 96LL && nn <= 160LL * 160LL));
+        c.resp_mma = c.nb <= 8 * efit::kRespBatchMaxBlk && want;
+    }
     c.resp_fuse = getenv("EFIT_RESP_NOFUSE") == nullptr;
     t.tb_ch = 2048;
     t.tb_nchunk = (int)((n + t.tb_ch - 1) / t.tb_ch);

@@ -149,7 +149,7 @@ struct Ctx {
     int tbb_nchunk;                // k_bnd_tb_mma chunks (kBatchCh elements)
     int respb_nchunk;              // k_response_mma chunks (kRespBatchGc nodes)
     bool respb;                    // this batch contracts Gd once for all slices (k_response_mma)
-    bool resp_mma;                 // single-slice response on k_response_mma (EFIT_RESP_MMA=1; measured slower)
+    bool resp_mma;                 // single-slice response on k_response_mma (nb >= 8 or ~129^2; EFIT_RESP_MMA=0/1)
     bool resp_fuse;                // k_response evaluates the basis itself (EFIT_RESP_NOFUSE=1: separate k_basis)
     cudaEvent_t bev_fork, bev_tb;  // batch: fork of the slice streams, end of the shared table pass
     cudaEvent_t bev_resp;          // batch: end of the shared Gd pass

@@ -976,11 +976,12 @@ __device__ __forceinline__ bool lsq_chol(double* G, double* R, double* rinv, int
         for (int j = k + lane; j < nb; j += 32) R[k * nb + j] = (j == k) ? r : G[k * nb + j] * ir;
         if (lane == 0) rinv[k] = ir;
         __syncwarp();
-        const int w = nb - k - 1;
-        for (int e = lane; e < w * w; e += 32) {
-            const int i = k + 1 + e / w, j = k + 1 + e % w;
-            if (j >= i) {
-                const double v = G[i * nb + j] - R[k * nb + i] * R[k * nb + j];
+        // trailing update, one lane per row i (its upper entries j >= i are independent updates;
+        // no integer division per entry): same expression per entry as the textbook loop
+        for (int i = k + 1 + lane; i < nb; i += 32) {
+            const double rki = R[k * nb + i];
+            for (int j = i; j < nb; ++j) {
+                const double v = G[i * nb + j] - rki * R[k * nb + j];
                 G[i * nb + j] = v;
                 G[j * nb + i] = v;
             }
@@ -1002,9 +1003,13 @@ __device__ __forceinline__ void lsq_rsolve_rows(double* A, int ld, int nd, int n
     }
 }
 
+// NBT > 0: the basis count as a compile-time constant (loops over it unroll, the final triangular
+// solves keep z in registers); NBT = 0: runtime nb.  Same arithmetic and order either way.
+template <int NBT>
 __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, const double* __restrict__ meas,
-                                             const double* __restrict__ sigma, int nd, int nb,
+                                             const double* __restrict__ sigma, int nd, int nb_arg,
                                              double* __restrict__ coef, double* __restrict__ chi2, int* status) {
+    const int nb = NBT > 0 ? NBT : nb_arg;
     extern __shared__ __align__(16) double sm[];
     const int ld = nb | 1;                         // odd row stride: conflict-free column walks
     double* A = sm;                                // [nd][ld] scaled rows
@@ -1060,7 +1065,42 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
     __syncthreads();
     if (warp == 0 && !s_sing && !lsq_chol(G, R2, r2i, nb) && lane == 0) s_sing = 1;
     __syncthreads();
-    if (tid == 0 && !s_sing) {
+    if (NBT > 0 && tid == 0 && !s_sing) {  // as below, z in registers
+        constexpr int NBC = NBT > 0 ? NBT : 1;
+        double zr[NBC];
+#pragma unroll
+        for (int j = 0; j < NBC; ++j) {
+            double s = z[j];
+#pragma unroll
+            for (int i = 0; i < j; ++i) s = fma(-R2[i * NBC + j], zr[i], s);
+            zr[j] = s * r2i[j];
+        }
+#pragma unroll
+        for (int k = NBC - 1; k >= 0; --k) {
+            double s = zr[k];
+#pragma unroll
+            for (int j = k + 1; j < NBC; ++j) s = fma(-R2[k * NBC + j], zr[j], s);
+            zr[k] = s * r2i[k];
+        }
+#pragma unroll
+        for (int k = NBC - 1; k >= 0; --k) {
+            double s = zr[k];
+#pragma unroll
+            for (int j = k + 1; j < NBC; ++j) s = fma(-R1[k * NBC + j], zr[j], s);
+            zr[k] = s * r1i[k];
+        }
+        double rmax = 0.0, rmin = DBL_MAX;
+#pragma unroll
+        for (int k = 0; k < NBC; ++k) {
+            const double d = fabs(R1[k * NBC + k] * R2[k * NBC + k]);
+            rmax = fmax(rmax, d);
+            rmin = fmin(rmin, d);
+            if (!(sc[k] > 0.0)) s_sing = 1;
+        }
+        if (!(rmin >= 1e-13 * rmax)) s_sing = 1;
+#pragma unroll
+        for (int k = 0; k < NBC; ++k) z[k] = zr[k] / sc[k];
+    } else if (tid == 0 && !s_sing) {
         // z <- R2^-T z (forward), z <- R2^-1 z (back), z <- R1^-1 z (back), c = z / scale
         for (int j = 0; j < nb; ++j) {
             double s = z[j];
@@ -1301,7 +1341,16 @@ cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const dou
         default: break;
     }
     if (done) return cudaGetLastError();
-    launch_pdl(k_lsq, dim3(1), dim3(256), smem, s, resp, meas, sigma, c.ndiag, c.nb, coef, chi2, c.status);
+    switch (c.nb) {
+#define EFIT_LSQ_CASE(V) \
+    case V: launch_pdl(k_lsq<V>, dim3(1), dim3(256), smem, s, resp, meas, sigma, c.ndiag, c.nb, coef, chi2, c.status); break;
+        EFIT_LSQ_CASE(7) EFIT_LSQ_CASE(8) EFIT_LSQ_CASE(9) EFIT_LSQ_CASE(10) EFIT_LSQ_CASE(11) EFIT_LSQ_CASE(12)
+        EFIT_LSQ_CASE(13) EFIT_LSQ_CASE(14) EFIT_LSQ_CASE(15) EFIT_LSQ_CASE(16) EFIT_LSQ_CASE(17) EFIT_LSQ_CASE(18)
+        EFIT_LSQ_CASE(19) EFIT_LSQ_CASE(20) EFIT_LSQ_CASE(21) EFIT_LSQ_CASE(22) EFIT_LSQ_CASE(23) EFIT_LSQ_CASE(24)
+#undef EFIT_LSQ_CASE
+        default:
+            launch_pdl(k_lsq<0>, dim3(1), dim3(256), smem, s, resp, meas, sigma, c.ndiag, c.nb, coef, chi2, c.status);
+    }
     return cudaGetLastError();
 }
 
@@ -2940,7 +2989,12 @@ cudaError_t prepare_kernels(Ctx& c) {
     auto big = [&](const void* f, size_t need) -> cudaError_t {
         return raise_smem_limit(f, need);
     };
-    if ((e = big((const void*)k_lsq, lsq_smem(c)))) return e;
+    if ((e = big((const void*)k_lsq<0>, lsq_smem(c)))) return e;
+#define EFIT_LSQ_BIG(V) if ((e = big((const void*)k_lsq<V>, lsq_smem(c)))) return e;
+    EFIT_LSQ_BIG(7) EFIT_LSQ_BIG(8) EFIT_LSQ_BIG(9) EFIT_LSQ_BIG(10) EFIT_LSQ_BIG(11) EFIT_LSQ_BIG(12)
+    EFIT_LSQ_BIG(13) EFIT_LSQ_BIG(14) EFIT_LSQ_BIG(15) EFIT_LSQ_BIG(16) EFIT_LSQ_BIG(17) EFIT_LSQ_BIG(18)
+    EFIT_LSQ_BIG(19) EFIT_LSQ_BIG(20) EFIT_LSQ_BIG(21) EFIT_LSQ_BIG(22) EFIT_LSQ_BIG(23) EFIT_LSQ_BIG(24)
+#undef EFIT_LSQ_BIG
     if ((e = launch_lr(c, nullptr, true))) return e;
     if ((e = prepare_lr_fft(c))) return e;
     if ((e = big((const void*)k_bnd_tb<kTbGI, kTbUnroll>, 2 * sizeof(double) * c.t.tb_ch))) return e;

@@ -149,6 +149,31 @@ def test_response_spline_mse(torch_mod, efit, orc_mod):
         assert rel(r[:, k], ref[:, k]) < TOL, k
 
 
+@pytest.mark.parametrize("force", ["0", "1"])
+@pytest.mark.parametrize("name,spline", [("65x65", False), ("129x129", True), ("129x129", False)])
+def test_response_kernel_choice(torch_mod, efit, orc_mod, monkeypatch, name, spline, force):
+    """Both single-slice response kernels (scalar stream k_response, EFIT_RESP_MMA=0; DMMA
+    k_response_mma, =1) against the oracle, whatever the automatic choice for the grid/basis."""
+    torch = torch_mod
+    monkeypatch.setenv("EFIT_RESP_MMA", force)
+    nw = int(name.split("x")[0])
+    g = synth.Grid(nw, nw)
+    basis = synth.spline_basis(6) if spline else synth.poly_basis()
+    n_int = 40 if spline else 0
+    cfg = synth.Config(name, g, synth.make_geometry(g, n_int), basis, name)
+    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=0)
+    orc = orc_mod.Oracle.from_config(cfg)
+    psi = synth.perturbed_psi(g, seed=7, rel=1e-3)
+    ref, axbd_ref = orc.response(psi)
+    resp, axbd = ctx.response(T(torch, psi))
+    torch.cuda.synchronize()
+    assert ctx.status() == 0
+    assert np.array_equal(axbd.cpu().numpy(), axbd_ref)
+    r = resp.cpu().numpy()
+    for k in range(ctx.nbasis):
+        assert rel(r[:, k], ref[:, k]) < TOL, (k, rel(r[:, k], ref[:, k]))
+
+
 # ------------------------------------------------------------------ a5: current
 
 @pytest.mark.parametrize("name", SMALL)
@@ -331,6 +356,25 @@ def test_lsq(torch_mod, efit, orc_mod, name):
     sigma = 1e-3 * np.max(np.abs(y)) * np.ones_like(y)
     y = y + sigma * synth.noise(len(y), seed=1)
     st, cref, chi2ref = orc_mod.lsq(resp, y, sigma)
+    coef, chi2 = c.ctx.lsq(T(torch, resp), T(torch, y), T(torch, sigma))
+    assert rel(coef.cpu().numpy(), cref) < TOL_C
+    assert abs(chi2.item() - chi2ref) <= TOL_C * chi2ref
+
+
+@pytest.mark.parametrize("n_int", [1, 6])
+def test_lsq_spline(torch_mod, efit, orc_mod, n_int):
+    """Wide bases (5+5 and 10+10 cubic B-splines, 40 MSE-like rows): the 256-thread CholeskyQR2
+    kernel k_lsq<NB> (nb > 6), C3's solve."""
+    torch = torch_mod
+    c = case("129x129", efit, orc_mod, basis=synth.spline_basis(n_int), n_int=40)
+    assert c.ctx.nbasis == 2 * (n_int + 4)
+    psi = synth.solovev_psi(c.cfg.grid)
+    resp, _ = c.orc.response(psi)
+    y = resp @ synth.c_true(c.cfg.basis)
+    sigma = 1e-3 * np.max(np.abs(y)) * np.ones_like(y)
+    y = y + sigma * synth.noise(len(y), seed=1)
+    st, cref, chi2ref = orc_mod.lsq(resp, y, sigma)
+    assert st == 0
     coef, chi2 = c.ctx.lsq(T(torch, resp), T(torch, y), T(torch, sigma))
     assert rel(coef.cpu().numpy(), cref) < TOL_C
     assert abs(chi2.item() - chi2ref) <= TOL_C * chi2ref
