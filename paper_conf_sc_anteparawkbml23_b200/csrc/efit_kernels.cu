@@ -991,6 +991,39 @@ __device__ __forceinline__ bool lsq_chol(double* G, double* R, double* rinv, int
     return true;
 }
 
+// Same factorisation for a compile-time NB <= 32, held in registers: lane i keeps row i of G
+// (= column i, G stays symmetric), the pivot and the R row are shuffled, so the trailing update is
+// NB independent shuffle + FMA pairs per step instead of shared-memory round trips.  Per entry the
+// same expressions as lsq_chol (G[i][j] - R[k][i] R[k][j]), hence the same bits.
+template <int NB>
+__device__ __forceinline__ bool lsq_chol_warp(const double* G, double* R, double* rinv) {
+    static_assert(NB <= 32, "one lane per row");
+    const int lane = threadIdx.x & 31;
+    double g[NB];
+#pragma unroll
+    for (int j = 0; j < NB; ++j) g[j] = lane < NB ? G[lane * NB + j] : 0.0;
+#pragma unroll
+    for (int k = 0; k < NB; ++k) {
+        const double d = __shfl_sync(0xffffffffu, g[k], k);
+        if (!(d > 0.0)) return false;
+        const double r = sqrt(d), ir = 1.0 / r;
+        const double rki = g[k] * ir;  // R[k][lane] for lane > k
+        if (lane == k) {
+            R[k * NB + k] = r;
+            rinv[k] = ir;
+        } else if (lane > k && lane < NB) {
+            R[k * NB + lane] = rki;
+        }
+#pragma unroll
+        for (int j = k + 1; j < NB; ++j) {
+            const double rkj = __shfl_sync(0xffffffffu, rki, j);
+            g[j] = g[j] - rki * rkj;
+        }
+    }
+    __syncwarp();
+    return true;
+}
+
 // row m of A (in place): a <- a R^-1  (forward substitution with the upper factor)
 __device__ __forceinline__ void lsq_rsolve_rows(double* A, int ld, int nd, int nb, const double* R, const double* rinv) {
     for (int m = threadIdx.x; m < nd; m += blockDim.x) {
@@ -1050,7 +1083,12 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
     // pass 1: G1 = A^T A, R1, Q1 = A R1^-1
     lsq_gram(A, ld, nd, nb, G);
     __syncthreads();
-    if (warp == 0 && !lsq_chol(G, R1, r1i, nb) && lane == 0) s_sing = 1;
+    if (warp == 0) {
+        bool ok;
+        if constexpr (NBT > 0) ok = lsq_chol_warp<NBT>(G, R1, r1i);
+        else ok = lsq_chol(G, R1, r1i, nb);
+        if (!ok && lane == 0) s_sing = 1;
+    }
     __syncthreads();
     if (!s_sing) lsq_rsolve_rows(A, ld, nd, nb, R1, r1i);
     __syncthreads();
@@ -1063,7 +1101,12 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
         if (lane == 0) z[k] = s;
     }
     __syncthreads();
-    if (warp == 0 && !s_sing && !lsq_chol(G, R2, r2i, nb) && lane == 0) s_sing = 1;
+    if (warp == 0 && !s_sing) {
+        bool ok;
+        if constexpr (NBT > 0) ok = lsq_chol_warp<NBT>(G, R2, r2i);
+        else ok = lsq_chol(G, R2, r2i, nb);
+        if (!ok && lane == 0) s_sing = 1;
+    }
     __syncthreads();
     if (NBT > 0 && tid == 0 && !s_sing) {  // as below, z in registers
         constexpr int NBC = NBT > 0 ? NBT : 1;
