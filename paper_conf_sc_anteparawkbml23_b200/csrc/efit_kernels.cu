@@ -1108,41 +1108,44 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
         if (!ok && lane == 0) s_sing = 1;
     }
     __syncthreads();
-    if (NBT > 0 && tid == 0 && !s_sing) {  // as below, z in registers
+    if (NBT > 0 && warp == 0 && !s_sing) {
+        // as below, one lane per unknown: lane j keeps z_j; each step shuffles the finished unknown
+        // and the other lanes apply its term.  The forward solve adds the terms in the serial order;
+        // the back solves add them from the last unknown down (fixed order => deterministic).
         constexpr int NBC = NBT > 0 ? NBT : 1;
-        double zr[NBC];
+        const int j = lane;
+        const bool act = j < NBC;
+        double zj = act ? z[j] : 0.0;
 #pragma unroll
-        for (int j = 0; j < NBC; ++j) {
-            double s = z[j];
-#pragma unroll
-            for (int i = 0; i < j; ++i) s = fma(-R2[i * NBC + j], zr[i], s);
-            zr[j] = s * r2i[j];
+        for (int i = 0; i < NBC; ++i) {  // z <- R2^-T z
+            const double zi = __shfl_sync(0xffffffffu, zj, i) * r2i[i];
+            if (j == i) zj = zi;
+            else if (act && j > i) zj = fma(-R2[i * NBC + j], zi, zj);
         }
 #pragma unroll
-        for (int k = NBC - 1; k >= 0; --k) {
-            double s = zr[k];
-#pragma unroll
-            for (int j = k + 1; j < NBC; ++j) s = fma(-R2[k * NBC + j], zr[j], s);
-            zr[k] = s * r2i[k];
+        for (int k = NBC - 1; k >= 0; --k) {  // z <- R2^-1 z
+            const double zk = __shfl_sync(0xffffffffu, zj, k) * r2i[k];
+            if (j == k) zj = zk;
+            else if (j < k) zj = fma(-R2[j * NBC + k], zk, zj);
         }
 #pragma unroll
-        for (int k = NBC - 1; k >= 0; --k) {
-            double s = zr[k];
-#pragma unroll
-            for (int j = k + 1; j < NBC; ++j) s = fma(-R1[k * NBC + j], zr[j], s);
-            zr[k] = s * r1i[k];
+        for (int k = NBC - 1; k >= 0; --k) {  // z <- R1^-1 z
+            const double zk = __shfl_sync(0xffffffffu, zj, k) * r1i[k];
+            if (j == k) zj = zk;
+            else if (j < k) zj = fma(-R1[j * NBC + k], zk, zj);
         }
-        double rmax = 0.0, rmin = DBL_MAX;
+        if (lane == 0) {
+            double rmax = 0.0, rmin = DBL_MAX;
 #pragma unroll
-        for (int k = 0; k < NBC; ++k) {
-            const double d = fabs(R1[k * NBC + k] * R2[k * NBC + k]);
-            rmax = fmax(rmax, d);
-            rmin = fmin(rmin, d);
-            if (!(sc[k] > 0.0)) s_sing = 1;
+            for (int k = 0; k < NBC; ++k) {
+                const double d = fabs(R1[k * NBC + k] * R2[k * NBC + k]);
+                rmax = fmax(rmax, d);
+                rmin = fmin(rmin, d);
+                if (!(sc[k] > 0.0)) s_sing = 1;
+            }
+            if (!(rmin >= 1e-13 * rmax)) s_sing = 1;
         }
-        if (!(rmin >= 1e-13 * rmax)) s_sing = 1;
-#pragma unroll
-        for (int k = 0; k < NBC; ++k) z[k] = zr[k] / sc[k];
+        if (act) z[j] = zj / sc[j];
     } else if (tid == 0 && !s_sing) {
         // z <- R2^-T z (forward), z <- R2^-1 z (back), z <- R1^-1 z (back), c = z / scale
         for (int j = 0; j < nb; ++j) {
