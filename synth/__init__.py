@@ -178,7 +178,7 @@ def config(name: str) -> Config:
     """The five BASELINE.json configs (C1..C5)."""
     name = name.upper()
     table = {
-        "C1": (65, 0, poly_basis(), "65x65, flux loops + probes, 5+5 polynomial basis, single fit iteration"),
+        "C1": (65, 0, poly_basis(), "65x65, flux loops + probes, 2+3 polynomial basis (5 terms, reading Q8), single fit iteration"),
         "C2": (129, 0, poly_basis(), "129x129, full fit loop on a Solov'ev-derived twin"),
         "C3": (257, 40, spline_basis(6), "257x257, 10+10 cubic-spline basis + 40 MSE-like B_Z points"),
         "C4": (513, 0, poly_basis(), "513x513, response + boundary flux (1/2/4/8 GPUs)"),
@@ -244,12 +244,21 @@ def random_current(grid: Grid, seed: int = 2, signed: bool = False, edge: bool =
     return I.reshape(-1)
 
 
-def c_true(basis: Basis, seed: int = 7) -> np.ndarray:
+def c_true(basis: Basis, seed: int = 7, edge_zero: bool = True) -> np.ndarray:
     """True profile coefficients.  The leading P' and FF' terms are the Solov'ev's
     constant profiles (Delta* psi_S = -scale[(2A+8B)R^2 + 2C] gives
     P'_0 = scale(2A+8B)/mu0 and mu0 FF'_0/(4 pi^2) = 2 C scale/mu0); higher terms are
     seeded at +-10% of the leading one.  For the spline basis every function gets the
-    leading value (partition of unity) times (1 +- 10%)."""
+    leading value (partition of unity) times (1 +- 10%).
+
+    edge_zero (default; reading R2): the profiles vanish at the plasma boundary,
+    P'(1) = FF'(1) = 0 -- the last monomial coefficient is set to minus the sum of the others,
+    the last B-spline coefficient (the only function non-zero at psihat = 1) to 0.  With the
+    Solov'ev's constant profiles the current jumps at the last closed surface, the discrete
+    mask (0 <= psihat < 1) makes the Picard map discontinuous, and a perturbed start converges
+    to a spurious nearby fixed point (2-6 mask nodes off, chi2 ~ 245, c far from c_true;
+    measured with the oracle at 65^2); with an edge-vanishing profile the loop converges to
+    psi_S and c -> c_true (the twin works for any profile: psi_ext absorbs the mismatch)."""
     mu0 = 4e-7 * np.pi
     pp0 = SOL_SCALE * (2 * SOL_A + 8 * SOL_B) / mu0
     ff0 = 2 * SOL_C * SOL_SCALE / mu0 * 4 * np.pi ** 2 / mu0
@@ -257,9 +266,17 @@ def c_true(basis: Basis, seed: int = 7) -> np.ndarray:
     if basis.kind == 0:
         pp = np.concatenate([[pp0], pp0 * 0.1 * rng.uniform(-1, 1, basis.n_pp - 1)])
         ff = np.concatenate([[ff0], ff0 * 0.1 * rng.uniform(-1, 1, basis.n_ff - 1)])
+        if edge_zero:
+            if basis.n_pp > 1:
+                pp[-1] = -np.sum(pp[:-1])
+            if basis.n_ff > 1:
+                ff[-1] = -np.sum(ff[:-1])
     else:
         pp = pp0 * (1 + 0.1 * rng.uniform(-1, 1, basis.n_pp))
         ff = ff0 * (1 + 0.1 * rng.uniform(-1, 1, basis.n_ff))
+        if edge_zero:
+            pp[-1] = 0.0
+            ff[-1] = 0.0
     return np.concatenate([pp, ff]).astype(np.float64)
 
 

@@ -450,17 +450,19 @@ def test_fit_step_graph_replay_matches_eager(torch_mod, efit, orc_mod):
 
 
 def test_fit_loop_c2(torch_mod, efit, orc_mod):
-    """C2: full loop to eps < 1e-5 from a 0.1%-perturbed Solov'ev twin; the GPU
-    loop follows the oracle loop iteration by iteration and stops at the same iteration."""
+    """C2: full loop to eps < 1e-5 from a 1%-perturbed Solov'ev twin (SURVEY 8(d),
+    edge-vanishing profile, reading R2); the GPU loop follows the oracle loop iteration by
+    iteration and stops at the same iteration.  Continued to eps < 1e-10 the GPU iterate is the
+    twin's psi_S with c = c_true (property of the twin construction)."""
     torch = torch_mod
     c = case("C2", efit, orc_mod)
     psi_s, ct, tw = _twin(c, noise_seed=None)
-    psi0 = synth.perturbed_psi(c.cfg.grid, seed=5, rel=1e-3)
+    psi0 = synth.perturbed_psi(c.cfg.grid, seed=5, rel=1e-2)
     ext, y, s = T(torch, tw["psi_ext"]), T(torch, tw["y"]), T(torch, tw["sigma"])
     psi = T(torch, psi0)
     coef, chi2, eps = c.ctx._t(c.ctx.nbasis), c.ctx._t(1), c.ctx._t(1)
     pr = psi0.copy()
-    for it in range(60):
+    for it in range(200):
         st, pr, cr, chr_, er = c.orc.fit_step(pr, tw["psi_ext"], tw["y"], tw["sigma"])
         c.ctx.fit_step(psi, ext, y, s, coef, chi2, eps)
         assert rel(psi.cpu().numpy(), pr) < 1e-10, it
@@ -468,6 +470,13 @@ def test_fit_loop_c2(torch_mod, efit, orc_mod):
         if er < 1e-5:
             break
     assert er < 1e-5
+    for it in range(600):
+        c.ctx.fit_step(psi, ext, y, s, coef, chi2, eps)
+        if eps.item() < 1e-10:
+            break
+    assert eps.item() < 1e-10
+    assert np.max(np.abs(psi.cpu().numpy() - psi_s)) < 1e-8 * np.max(np.abs(psi_s))
+    assert np.max(np.abs(coef.cpu().numpy() - ct)) < 1e-7 * np.max(np.abs(ct))
 
 
 # ------------------------------------------------------------------ multi-rank emulation
@@ -495,49 +504,6 @@ def test_sharded_matches_single_bitwise(torch_mod, efit, orc_mod):
     assert torch.equal(psib, psib1)
 
 
-# ------------------------------------------------------------------ full size (C4 513^2): sampled
-
-@pytest.fixture(scope="module")
-def c4(efit, orc_mod):
-    return case("C4", efit, orc_mod)
-
-
-@pytest.mark.parametrize("mode", [0, 2])
-def test_c4_boundary_sampled(torch_mod, efit, orc_mod, c4, mode):
-    torch = torch_mod
-    c = c4 if mode == 0 else case("C4", efit, orc_mod, mode=mode)
-    I = synth.random_current(c.cfg.grid, seed=2)
-    out = c.ctx.boundary_flux(T(torch, I)).cpu().numpy()
-    rng = np.random.default_rng(0)
-    tg = np.unique(np.concatenate([[0, 512, 513, 1025, 1026, 1536, 2043], rng.integers(0, c.ctx.n_edge, 40)]))
-    ref = c4.orc.boundary_targets(I, tg)
-    assert rel(out[tg], ref) < TOL
-
-
-def test_c4_response_sampled(torch_mod, c4):
-    torch = torch_mod
-    psi = synth.perturbed_psi(c4.cfg.grid, seed=5, rel=1e-3)
-    resp, axbd = c4.ctx.response(T(torch, psi))
-    rows = [0, 7, 43, 44, 80, 119]
-    ref = c4.orc.response_rows(psi, rows)
-    r = resp.cpu().numpy()[rows]
-    for k in range(c4.ctx.nbasis):
-        assert rel(r[:, k], ref[:, k]) < TOL
-
-
-def test_c4_solve_and_current(torch_mod, c4):
-    torch = torch_mod
-    psi = synth.solovev_psi(c4.cfg.grid)
-    coef = synth.c_true(c4.cfg.basis)
-    Iref = c4.orc.current(psi, coef)
-    I = c4.ctx.current(T(torch, psi), T(torch, coef))
-    assert rel(I.cpu().numpy(), Iref) < TOL
-    psib = np.linspace(-0.3, -0.1, c4.ctx.n_edge)
-    ref = c4.orc.interior_solve(Iref, psib)
-    out = c4.ctx.interior_solve(T(torch, Iref), T(torch, psib)).cpu().numpy()
-    assert rel(out, ref) < TOL
-
-
 def test_fit_steps_chained_equals_repeated(torch_mod, efit, orc_mod):
     """efit_fit_steps(n) (axis/boundary of iterations 2..n taken from the previous update kernel)
     is bitwise identical to n separate efit_fit_step calls (each normalising from scratch)."""
@@ -559,37 +525,3 @@ def test_fit_steps_chained_equals_repeated(torch_mod, efit, orc_mod):
         outs.append((psi.clone(), coef.clone(), eps.clone()))
     for a, b in zip(*outs):
         assert torch.equal(a, b)
-
-
-# ------------------------------------------------------------------ stress size (C5 1025^2): sampled
-
-@pytest.mark.parametrize("mode", [0, 2])  # full table (8.6 GB) and half table: the m-chunked SYM path
-def test_c5_boundary_sampled(torch_mod, efit, orc_mod, mode):
-    """configs[4] (1025^2, the largest grid the ABI is quoted on): sampled edge targets, including
-    the corners and both ends of every side, against the oracle's per-target sums."""
-    torch = torch_mod
-    c = case("C5", efit, orc_mod, mode=mode)
-    I = synth.random_current(c.cfg.grid, seed=3, signed=True)
-    out = c.ctx.boundary_flux(T(torch, I)).cpu().numpy()
-    nh, nw = c.cfg.grid.nh, c.cfg.grid.nw
-    fixed = [0, nh - 1, nh, 2 * nh - 1, 2 * nh, 2 * nh + nw - 3, 2 * nh + nw - 2, c.ctx.n_edge - 1]
-    rng = np.random.default_rng(1)
-    tg = np.unique(np.concatenate([fixed, rng.integers(0, c.ctx.n_edge, 24)]))
-    ref = c.orc.boundary_targets(I, tg)
-    assert rel(out[tg], ref) < TOL
-    c.ctx.close()
-    _cases.pop(("C5", mode, None, 0), None)
-
-
-def test_c5_response_sampled(torch_mod, efit, orc_mod):
-    torch = torch_mod
-    c = case("C5", efit, orc_mod, mode=efit.EFIT_GREEN_TABLE_SYM)
-    psi = synth.perturbed_psi(c.cfg.grid, seed=5, rel=1e-3)
-    resp, axbd = c.ctx.response(T(torch, psi))
-    rows = [0, 43, 44, 119]
-    ref = c.orc.response_rows(psi, rows)
-    r = resp.cpu().numpy()[rows]
-    for k in range(c.ctx.nbasis):
-        assert rel(r[:, k], ref[:, k]) < TOL
-    c.ctx.close()
-    _cases.pop(("C5", efit.EFIT_GREEN_TABLE_SYM, None, 0), None)

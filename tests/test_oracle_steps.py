@@ -226,3 +226,29 @@ def test_lsq_exact_recovery_and_singular(oracle_mod):
     A[:, 3] = 2 * A[:, 1]
     st, _, _ = oracle_mod.lsq(A, A @ ct, np.ones(40))
     assert st == -5
+
+
+def test_internal_bz_rows_are_field_of_flux(oracle_mod):
+    """MSE-like internal rows (O5): row m = B_Z at an internal point x from a
+    unit current at every node, B_Z = (1/R) dpsi/dR of the flux Green's function (P:L101;
+    B = grad psi x e_phi / R), by Richardson differences of or_green_psi -- pins the row's
+    kind (B_Z, not B_R or psi) and its offset after the flux-loop and probe rows."""
+    cfg = synth.small_config(65, n_int=10)
+    orc = oracle_mod.Oracle.from_config(cfg)
+    g = cfg.geometry
+    off = len(g.fl_r) + len(g.mp_r)
+    assert orc.ndiag == off + 10
+    Gd = orc.table_Gd()
+    R, Z = cfg.grid.r(), cfg.grid.z()
+    RR, ZZ = np.meshgrid(R, Z, indexing="ij")
+    for k in [0, 3, 9]:
+        x, z = g.int_r[k], g.int_z[k]
+        flux = lambda xr, xz: np.array([oracle_mod.green_psi(xr, xz, r, zz) for r, zz in zip(RR.ravel(), ZZ.ravel())])
+        h = 2e-4
+        d1 = (flux(x + h, z) - flux(x - h, z)) / (2 * h)
+        d2 = (flux(x + h / 2, z) - flux(x - h / 2, z)) / h
+        row = ((4 * d2 - d1) / 3) / x
+        np.testing.assert_allclose(Gd[off + k], row, rtol=0, atol=1e-8 * np.abs(row).max())
+        # and it is not B_R (dpsi/dZ): the two differ at O(1) off the midplane sources
+        dz = (flux(x, z + h) - flux(x, z - h)) / (2 * h)
+        assert np.max(np.abs(Gd[off + k] - (-dz / x))) > 0.1 * np.abs(row).max()
