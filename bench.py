@@ -3,11 +3,13 @@
 
 One "step" = one full Picard fit iteration (normalise, response,
 least squares, current, boundary flux, interior solve, update, eps) over the C4 synthetic
-twin, i.e. one efit_fit_step call (world == 1) or the sharded step (world > 1: targets of the
-response and boundary flux split across ranks, one NCCL all-reduce of each zero-padded slice).
+twin, i.e. one chained efit_fit_steps iteration.  world > 1 (one process per GPU): the same call
+with the in-library NCCL exchange (response rows and the top/bottom boundary stream sharded, two
+all-reduces per iteration; include/efit.h "Multi-GPU"), strong scaling of one reconstruction.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C4] [--impl efit|reference]
 
+--gpus N > 1 outside torchrun re-launches itself under torch.distributed.run (127.0.0.1).
 Prints ONE JSON line on rank 0.  `--impl reference` times the CPU oracle (the reference arm of
 this tier) on the host cores, on the same config/metric/unit.
 """
@@ -39,7 +41,7 @@ UNIT = "fit iterations/s"
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=2000)
+    ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--config", default="C4")
     ap.add_argument("--impl", default="efit", choices=["efit", "reference"])
@@ -52,10 +54,11 @@ def parse():
                     help="time slices per fit step (efit_batch_attach; SURVEY 8(f) f1): S slices share one "
                          "pass over the top/bottom Green's table; value = slice fit iterations/s")
     ap.add_argument("--sharded", action="store_true",
-                    help="run the sharded (world > 1) step even on one rank (NCCL world of 1): exercises the "
-                         "graph-captured exchange path of the scaling run on one GPU")
+                    help="use the in-library NCCL exchange even on one rank (world-1 communicator): exercises "
+                         "the graph-captured exchange path of the scaling run on one GPU")
     ap.add_argument("--no-profile", action="store_true",
                     help="time graph replays without per-kernel events (no roofline breakdown)")
+    ap.add_argument("--reps", type=int, default=5, help="timed repetitions of K steps; value = the median")
     return ap.parse_args()
 
 
@@ -139,9 +142,10 @@ class Clocks:
 
 # ----------------------------------------------------------------------------- GPU arm
 
-def twin_inputs(ctx, cfg, torch, dev, sharded_step=None):
+def twin_inputs(ctx, cfg, torch, dev):
     """Synthetic twin built with the product API: I_S = current(psi_S, c_true),
-    psi_ext = psi_S - solve(boundary(I_S), I_S), y = R(psi_S) c_true + noise."""
+    psi_ext = psi_S - solve(boundary(I_S), I_S), y = R(psi_S) c_true + noise.
+    With the in-library NCCL exchange (world > 1) every call returns replicated outputs."""
     import paper_conf_sc_anteparawkbml23_b200 as efit
     T = lambda a: torch.tensor(np.asarray(a, dtype=np.float64), device=dev)
     psi_s = T(synth.solovev_psi(cfg.grid))
@@ -151,10 +155,6 @@ def twin_inputs(ctx, cfg, torch, dev, sharded_step=None):
     resp = ctx._t(ctx.ndiag * ctx.nbasis)
     efit.efit_boundary_flux(ctx.handle, I_s, psib)
     efit.efit_response(ctx.handle, psi_s, resp)
-    if sharded_step is not None:
-        import torch.distributed as dist
-        dist.all_reduce(psib)
-        dist.all_reduce(resp)
     psi_p = ctx.interior_solve(I_s, psib)
     psi_ext = psi_s - psi_p
     y = resp.view(ctx.ndiag, ctx.nbasis) @ ct
@@ -167,38 +167,6 @@ def twin_inputs(ctx, cfg, torch, dev, sharded_step=None):
     y = y + sigma * T(synth.noise(ctx.ndiag, seed=1))
     psi0 = T(synth.perturbed_psi(cfg.grid, seed=5, rel=1e-3))
     return psi0, psi_ext.contiguous(), y.contiguous(), sigma.contiguous()
-
-
-class ShardedStep:
-    """world > 1: response rows and boundary targets are split across ranks (efit_dist);
-    each rank writes its slice into a zeroed full-size buffer and one NCCL all-reduce per
-    exchange makes it replicated (x + 0 is exact, so results are bitwise those of world = 1).
-    LSQ, current, interior solve and update run replicated."""
-
-    def __init__(self, ctx, torch):
-        self.ctx, self.torch = ctx, torch
-        self.resp = ctx._t(ctx.ndiag * ctx.nbasis)
-        self.psib = ctx._t(ctx.n_edge)
-        self.pcurr = ctx._t(ctx.nw * ctx.nh)
-        self.ev = None
-
-    def __call__(self, psi, psi_ext, meas, sigma, coef, chi2, eps, events=None):
-        import torch.distributed as dist
-        import paper_conf_sc_anteparawkbml23_b200 as efit
-        h = self.ctx.handle
-        self.resp.zero_()
-        efit.efit_response(h, psi, self.resp)
-        dist.all_reduce(self.resp)
-        efit.efit_lsq(h, self.resp, meas, sigma, coef, chi2)
-        efit.efit_current(h, psi, coef, self.pcurr)
-        self.psib.zero_()
-        if events is not None:
-            events[0].record()
-        efit.efit_boundary_flux(h, self.pcurr, self.psib)
-        if events is not None:
-            events[1].record()
-        dist.all_reduce(self.psib)
-        efit.efit_solve_update(h, self.pcurr, self.psib, psi_ext, psi, eps)
 
 
 def batch_inputs(ctx, cfg, torch, dev, S):
@@ -350,124 +318,127 @@ def batch_arm(args, rank, world, local):
     ctx.close()
 
 
+def init_exchange(args, rank, world, dev, torch):
+    """Process group (gloo for host-side broadcasts, NCCL for the max-over-ranks timing) and the
+    library's own NCCL communicator: rank 0 draws the ncclUniqueId (efit_nccl_unique_id), gloo
+    broadcasts it, every rank passes it to efit_green_init (include/efit.h "Multi-GPU")."""
+    import torch.distributed as dist
+    import paper_conf_sc_anteparawkbml23_b200 as efit
+    if world > 1:
+        dist.init_process_group(backend="cpu:gloo,cuda:nccl", device_id=dev)
+    else:  # --sharded on one GPU: a world-1 communicator exercising the same exchange path
+        port = int(os.environ.get("MASTER_PORT", "29533"))
+        dist.init_process_group(backend="cpu:gloo,cuda:nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0,
+                                world_size=1, device_id=dev)
+    buf = torch.zeros(128, dtype=torch.uint8)
+    if rank == 0:
+        buf.copy_(torch.frombuffer(bytearray(efit.efit_nccl_unique_id()), dtype=torch.uint8))
+    dist.broadcast(buf, 0)
+    return bytes(buf.numpy().tobytes())
+
+
+def max_over_ranks(x, torch, dev, use_dist):
+    if not use_dist:
+        return x
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+    return t.item()
+
+
+def barrier(use_dist, torch):
+    if use_dist:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+
+
+def capture_steps(ctx, K, chunk, psi, psi_ext, meas, sigma, coef, chi2, eps, torch):
+    """K chained fit iterations captured into CUDA graphs of <= chunk steps (efit_fit_steps: only
+    the first iteration of a graph normalises psi; the host is out of the timed loop)."""
+    cap = torch.cuda.Stream()
+    graphs, done = [], 0
+    while done < K:
+        n = min(chunk, K - done)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=cap):
+            ctx.fit_steps(n, psi, psi_ext, meas, sigma, coef, chi2, eps)
+        graphs.append(g)
+        done += n
+    torch.cuda.synchronize()
+    return graphs
+
+
 def gpu_arm(args, rank, world, local):
     import torch
     import paper_conf_sc_anteparawkbml23_b200 as efit
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    use_shard = world > 1 or args.sharded
-    if world > 1:
-        import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
-    elif use_shard:
-        import torch.distributed as dist
-        dist.init_process_group("nccl", init_method="tcp://127.0.0.1:29533", rank=0, world_size=1, device_id=dev)
+    use_dist = world > 1 or args.sharded
+    nccl_id = init_exchange(args, rank, world, dev, torch) if use_dist else None
     cfg = synth.config(args.config)
     N, ndiag = cfg.grid.nw, cfg.geometry.ndiag
     mode = MODES[args.mode]
     t0 = time.time()
-    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=mode, rank=rank, world=world, device=dev)
+    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=mode, rank=rank, world=world, device=dev,
+                           nccl_id=nccl_id)
     torch.cuda.synchronize()
     init_s = time.time() - t0
-    sharded = ShardedStep(ctx, torch) if use_shard else None
-    psi0, psi_ext, meas, sigma = twin_inputs(ctx, cfg, torch, dev, sharded)
+    psi0, psi_ext, meas, sigma = twin_inputs(ctx, cfg, torch, dev)
     psi = psi0.clone()
     coef, chi2, eps = ctx._t(ctx.nbasis), ctx._t(1), ctx._t(1)
-
-    def step(events=None):
-        if sharded is None:
-            ctx.fit_step(psi, psi_ext, meas, sigma, coef, chi2, eps)
-        else:
-            sharded(psi, psi_ext, meas, sigma, coef, chi2, eps, events)
-
     for _ in range(args.warmup):
-        step()
+        ctx.fit_step(psi, psi_ext, meas, sigma, coef, chi2, eps)
     torch.cuda.synchronize()
     st = ctx.status()
     if st != 0:
         raise RuntimeError(f"fit step status {st}: {efit.efit_last_error(ctx.handle)}")
 
-    # ---------------- timed region: K steps, per-kernel CUDA events on the launching streams.
-    # world == 1: the K steps are captured ahead of time into CUDA graphs of <= 500 steps and the
-    # timed region replays them back to back (no host in the loop).  Every 10th step carries the
-    # seven event marks (external event-record nodes on the streams the kernels run on); the
-    # per-kernel averages come from those sampled steps of the same timed region.
+    # ---------------- timed region: R repetitions of exactly K steps each (graph replays, no host in
+    # the loop), barrier + synchronize on both sides, CUDA events on the launching stream, max over
+    # ranks; value = the median repetition.  A further repetition of the same K steps carries the
+    # per-kernel event marks (every 10th step) for the breakdown and the roofline.
     K = args.steps
     stream = torch.cuda.current_stream()
-    graphs = []
-    bnd_events = None
-    if sharded is None:
-        if not args.no_profile:
-            # marks on every 10th step: each external event node costs a few us inside a graph
-            efit.efit_profile_begin(ctx.handle, (K + 9) // 10, 10)
-        cap = torch.cuda.Stream()
-        done = 0
-        while done < K:
-            n = min(500, K - done)
-            g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g, stream=cap):
-                # n chained iterations: only the first normalises psi (efit_fit_steps)
-                ctx.fit_steps(n, psi, psi_ext, meas, sigma, coef, chi2, eps)
-            graphs.append(g)
-            done += n
-        torch.cuda.synchronize()
-    else:
-        # sharded: the per-step boundary time comes from an eager event-timed run of the same step
-        # (outside the timed region); the timed region replays captured graphs of <= 100 steps
-        # (kernels + NCCL all-reduces; no host in the loop)
-        nb_ev = min(K, 50)
-        bnd_events = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(nb_ev)]
-        for k in range(nb_ev):
-            step(bnd_events[k])
-        torch.cuda.synchronize()
-        cap = torch.cuda.Stream()
-        done = 0
-        while done < K:
-            n = min(100, K - done)
-            g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g, stream=cap):
-                for _ in range(n):
-                    step()
-            graphs.append(g)
-            done += n
-        torch.cuda.synchronize()
+    graphs = capture_steps(ctx, K, 500, psi, psi_ext, meas, sigma, coef, chi2, eps, torch)
+    if not args.no_profile:
+        efit.efit_profile_begin(ctx.handle, (K + 9) // 10, 10)
+        graphs_prof = capture_steps(ctx, K, 500, psi, psi_ext, meas, sigma, coef, chi2, eps, torch)
     clocks = Clocks(local) if rank == 0 else None
-    if use_shard:
-        torch.distributed.barrier()
-    torch.cuda.synchronize()
     if clocks:
         clocks.start()
         time.sleep(0.3)
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    for g in graphs:
-        g.replay()
-    e1.record(stream)
-    torch.cuda.synchronize()
-    if use_shard:
-        torch.distributed.barrier()
-    clk = clocks.stop() if clocks else None
-    elapsed_ms = e0.elapsed_time(e1)
-    if sharded is None and args.no_profile:
-        prof, nrec = None, 0
-    elif sharded is None:
+    reps = []
+    for _ in range(max(1, args.reps)):
+        barrier(use_dist, torch)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for g in graphs:
+            g.replay()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        reps.append(max_over_ranks(e0.elapsed_time(e1) / K, torch, dev, use_dist))
+    prof, nrec, ms_prof = None, 0, None
+    if not args.no_profile:
+        barrier(use_dist, torch)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for g in graphs_prof:
+            g.replay()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ms_prof = max_over_ranks(e0.elapsed_time(e1) / K, torch, dev, use_dist)
         prof, nrec = efit.efit_profile_end(ctx.handle)
-    else:
-        prof = {"bnd_total": sum(a.elapsed_time(b) for a, b in bnd_events)}
-        nrec = len(bnd_events)
-    ms_step = elapsed_ms / K
-    if use_shard:
-        t = torch.tensor([ms_step], dtype=torch.float64, device=dev)
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        ms_step = t.item()
+    barrier(use_dist, torch)
+    clk = clocks.stop() if clocks else None
+    ms_step = float(np.median(reps))
     st = ctx.status()
     if st != 0:
         raise RuntimeError(f"fit step status {st}")
 
-    # ---------------- roofline of the dominant kernel (k_bnd_tb) and response+boundary GB/s
+    # ---------------- roofline of the dominant kernel and response+boundary GB/s (this rank's bytes)
     peak, peak_kind = measured_peaks()
-    if args.mode in ("sym", "otf-sym"):
+    sym_mode = args.mode in ("sym", "otf-sym")
+    if sym_mode:
         # half table: this rank's 8 x 8 row-pair tiles of 64*nh doubles, streamed once, + (I, I_flipped)
         ntile = ctx.info.sym_tile_hi - ctx.info.sym_tile_lo
         tb_bytes = 8.0 * 64 * N * ntile + 16.0 * N * N
@@ -481,29 +452,28 @@ def gpu_arm(args, rank, world, local):
     gd_bytes = 8.0 * (ctx.info.resp_row_hi - ctx.info.resp_row_lo) * N * N
     if prof is None:
         tb_ms, rb_ms, breakdown = float("nan"), None, {}
-    elif sharded is None:
+    else:
         tb_ms = prof["bnd_tb"] / nrec
         # the left/right chain (bnd_lr) runs concurrently with the top/bottom stream (both from the fork)
         rb_ms = (prof["response"] + max(prof["bnd_tb"], prof["bnd_lr"])) / nrec
         breakdown = {k: round(v / nrec * 1e3, 3) for k, v in prof.items()}  # us per step
-    else:
-        tb_ms = prof["bnd_total"] / nrec  # make_pair + tb + lr + reduce of this rank
-        rb_ms = None
-        breakdown = {"boundary_flux_call": round(tb_ms * 1e3, 3)}
     tb_gbs = tb_bytes / (tb_ms * 1e-3) / 1e9
-    traffic = None
+    traffic, traffic_src = None, None
     ncu_sum = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if os.path.exists(ncu_sum):
         try:
             d = json.load(open(ncu_sum))
             if d.get("config") == args.config and d.get("world", 1) == world:
                 traffic = d.get(tb_kernel, {}).get("dram_bytes_per_launch")
+                traffic_src = d.get(tb_kernel, {}).get("source", "profiles/ncu_summary.json")
         except Exception:
             traffic = None
-    roof = {"kernel": tb_kernel if sharded is None else f"boundary_flux ({tb_kernel}+lr+reduce)",
-            "bound": "hbm", "achieved": round(tb_gbs, 1), "peak": peak, "unit": "GB/s",
-            "frac": round(tb_gbs / peak, 4), "traffic": traffic, "peak_source": peak_kind,
-            "algorithmic_bytes_per_launch": tb_bytes}
+    roof = {"kernel": tb_kernel, "bound": "hbm", "achieved": round(tb_gbs, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(tb_gbs / peak, 4), "traffic": traffic,
+            "traffic_source": (f"ncu --set full capture of this kernel at this config, not measured in this run "
+                               f"({traffic_src})") if traffic is not None else None,
+            "peak_source": peak_kind, "algorithmic_bytes_per_launch": tb_bytes,
+            "timing": "CUDA events on the kernel's stream, every 10th step of a repetition of the K timed steps"}
     if args.mode in ("otf", "otf-sym"):
         # recomputed Green's functions: FP64-ALU bound.  FLOPs per launch = the kernel's executed
         # dadd + dmul + 2 dfma (ncu, profiles/ncu_summary.json) for this config; peak derived from the
@@ -530,24 +500,26 @@ def gpu_arm(args, rank, world, local):
         rb = {"bytes_per_step": tb_bytes + gd_bytes, "us_per_step": round(rb_ms * 1e3, 2),
               "achieved_gbs": round(rb_gbs, 1), "frac": round(rb_gbs / peak, 4)}
 
-    # ---------------- e2e: host buffers through the C ABI, copies inside the timed region
+    # ---------------- e2e: host buffers through the C ABI (efit_fit_host), copies inside the timed region
     e2e = None
     if not args.no_e2e:
-        e2e = e2e_measure(ctx, sharded, psi0, psi_ext, meas, sigma, K_e2e=min(K, 500), torch=torch, dev=dev,
-                          world=world)
+        e2e = e2e_measure(ctx, psi0, psi_ext, meas, sigma, K_e2e=min(K, 400), torch=torch, dev=dev,
+                          use_dist=use_dist)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(args.config)
 
-    # our kernels per step (ncu launch list, profiles/r01_launches_final.csv): response (basis fused),
-    # resp_reduce, lsq, current, lr_fft, lr_mac, lr_ifft, dst_fwd, bnd_tb | (bnd_sym + sym_edge_src),
-    # bnd_reduce, tridiag, dst_inv; + k_normalize at the start of every captured graph.
-    # sharded (step API): + normalize, make_pair (+ sym_pack in the SYM modes) every step
-    sym_mode = args.mode in ("sym", "otf-sym")
+    # our kernels per step (ncu launch list, profiles/): response (basis fused), resp_reduce, lsq,
+    # current, lr_fft, lr_mac, lr_ifft, dst_fwd, bnd_tb | (bnd_sym + sym_edge_src), bnd_reduce,
+    # tridiag, dst_inv; + k_normalize at the start of every captured graph
     per_step = 12 + (1 if sym_mode else 0)
-    launches = per_step * K + len(graphs) if sharded is None else (per_step + 2 + (1 if sym_mode else 0)) * K
+    launches = per_step * K + len(graphs)
     if rank == 0:
+        par = "single GPU"
+        if use_dist:
+            par = (f"sharded x{world}: response rows + top/bottom {'row-pair tiles' if sym_mode else 'rows'}, "
+                   f"in-library NCCL exchange (2 all-reduces per iteration)")
         out = {
             "metric": METRIC, "value": round(1000.0 / ms_step, 2), "unit": UNIT,
             "n_gpus": world, "steps": K, "warmup": args.warmup, "ms_per_step": round(ms_step, 5),
@@ -555,93 +527,53 @@ def gpu_arm(args, rank, world, local):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"{args.config}: {cfg.description}", "grid": f"{N}x{N}",
                        "ndiag": ndiag, "nbasis": cfg.basis.nbasis, "green_mode": args.mode,
-                       "parallelism": f"target-shard x{world}" if use_shard else "single GPU",
+                       "parallelism": par,
                        "l2": f"inputs larger than L2 ({tb_bytes / 1e9:.3f} GB boundary table + {gd_bytes / 1e9:.3f} GB "
-                             f"Gd streamed per step vs 126 MB L2)",
+                             f"Gd streamed per step and rank vs 126 MB L2): no flush",
+                       "reps_ms_per_step": [round(r, 5) for r in reps], "value_from": "median repetition",
+                       "profiled_rep_ms_per_step": round(ms_prof, 5) if ms_prof else None,
                        "init_s": round(init_s, 3), "step_breakdown_us": breakdown},
             "roofline": roof, "response_boundary": rb, "e2e": e2e, "cpu_baseline": cpu,
             "clocks": clk, "gpu_launches": launches,
         }
         print(json.dumps(out), flush=True)
     ctx.close()
-    if use_shard:
+    if use_dist:
         torch.distributed.destroy_process_group()
 
 
-def e2e_measure(ctx, sharded, psi0, psi_ext, meas, sigma, K_e2e, torch, dev, world):
-    """Same metric through the public API with HOST buffers: every step copies its psi, meas and
-    sigma from pinned host memory and reads back its psi, coef, chi2 and eps.  The copies are
-    pipelined across steps (H2D of step k+1 and D2H of step k-1 run on their own streams under the
-    fit step k, double-buffered staging; two 2-MB device copies per step keep the fit step's
-    captured graph on fixed buffers).  Sharded: the same with the step API + NCCL exchange, max over
-    ranks."""
-    n = psi0.numel()
-    nb = ctx.nbasis
-    h_in = [torch.cat([psi0.cpu(), meas.cpu(), sigma.cpu()]).pin_memory() for _ in range(2)]
-    h_out = [torch.empty(n + nb + 2, dtype=torch.float64).pin_memory() for _ in range(2)]
-    psi, m, s = torch.empty_like(psi0), torch.empty_like(meas), torch.empty_like(sigma)
-    coef, chi2, eps = ctx._t(nb), ctx._t(1), ctx._t(1)
-    nin = n + 2 * ctx.ndiag
-    main = torch.cuda.current_stream()
-    cs, hs, ds = torch.cuda.Stream(), torch.cuda.Stream(), torch.cuda.Stream()
-    d_in = [torch.empty(nin, dtype=torch.float64, device=dev) for _ in range(2)]
-    d_out = [torch.empty(n + nb + 2, dtype=torch.float64, device=dev) for _ in range(2)]
-    ev = lambda: torch.cuda.Event()
-    in_ready, in_free = [ev(), ev()], [ev(), ev()]
-    out_ready, out_free = [ev(), ev()], [ev(), ev()]
-    for b in range(2):
-        in_free[b].record(main)
-        out_free[b].record(main)
-
-    def step(k):
-        b = k & 1
-        with torch.cuda.stream(hs):
-            hs.wait_event(in_free[b])
-            d_in[b].copy_(h_in[b], non_blocking=True)
-            in_ready[b].record(hs)
-        with torch.cuda.stream(cs):
-            cs.wait_event(in_ready[b])
-            psi.copy_(d_in[b][:n])
-            m.copy_(d_in[b][n:n + ctx.ndiag])
-            s.copy_(d_in[b][n + ctx.ndiag:])
-            in_free[b].record(cs)
-            if sharded is None:
-                ctx.fit_step(psi, psi_ext, m, s, coef, chi2, eps, stream=cs)
-            else:  # step API + NCCL all-reduces, all on cs
-                sharded(psi, psi_ext, m, s, coef, chi2, eps)
-            cs.wait_event(out_free[b])
-            d_out[b][:n].copy_(psi)
-            d_out[b][n:n + nb].copy_(coef)
-            d_out[b][n + nb:n + nb + 1].copy_(chi2)
-            d_out[b][n + nb + 1:].copy_(eps)
-            out_ready[b].record(cs)
-        with torch.cuda.stream(ds):
-            ds.wait_event(out_ready[b])
-            h_out[b].copy_(d_out[b], non_blocking=True)
-            out_free[b].record(ds)
-
-    for k in range(6):
-        step(k)
+def e2e_measure(ctx, psi0, psi_ext, meas, sigma, K_e2e, torch, dev, use_dist, chunk=50):
+    """The same metric through the public API with HOST buffers: efit_fit_host reconstructs
+    successive time slices, each one fit iteration from its host psi/measurements/sigma (pinned),
+    copying its psi, coefficients, chi2 and eps back to the host; the library double-buffers the
+    copies on its own streams (include/efit.h).  Timed: K_e2e slices in calls of `chunk`."""
+    n, nd, nb = psi0.numel(), ctx.ndiag, ctx.nbasis
+    chunk = min(chunk, K_e2e)
+    h_psi0 = psi0.cpu().repeat(chunk).pin_memory()
+    h_meas = meas.cpu().repeat(chunk).pin_memory()
+    h_sigma = sigma.cpu().repeat(chunk).pin_memory()
+    h_psi = torch.empty(chunk * n, dtype=torch.float64).pin_memory()
+    h_coef = torch.empty(chunk * nb, dtype=torch.float64).pin_memory()
+    h_chi2 = torch.empty(chunk, dtype=torch.float64).pin_memory()
+    h_eps = torch.empty(chunk, dtype=torch.float64).pin_memory()
+    s = torch.cuda.Stream()
+    args = (h_psi0, h_meas, h_sigma, psi_ext, h_psi, h_coef, h_chi2, h_eps)
+    ctx.fit_host(min(chunk, 4), 1, *args, stream=s)   # warm-up: instantiate the slot graphs
     torch.cuda.synchronize()
-    if sharded is not None:
-        torch.distributed.barrier()
+    ncall = max(1, K_e2e // chunk)
+    barrier(use_dist, torch)
     a, z = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    a.record(main)
-    for q in (cs, hs, ds):
-        q.wait_event(a)
-    for k in range(K_e2e):
-        step(k)
-    for q in (cs, hs, ds):
-        main.wait_stream(q)
-    z.record(main)
+    a.record(s)
+    for _ in range(ncall):
+        ctx.fit_host(chunk, 1, *args, stream=s)
+    z.record(s)
     torch.cuda.synchronize()
-    ms = a.elapsed_time(z) / K_e2e
-    if sharded is not None:  # max over ranks
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        ms = t.item()
-    return {"value": round(1000.0 / ms, 2), "unit": UNIT, "h2d_bytes_per_step": 8 * nin,
-            "d2h_bytes_per_step": 8 * (n + nb + 2), "steps": K_e2e, "pipelined": True}
+    ms = max_over_ranks(a.elapsed_time(z) / (ncall * chunk), torch, dev, use_dist)
+    if not np.isfinite(h_eps.numpy()).all():
+        raise RuntimeError("efit_fit_host produced non-finite eps")
+    return {"value": round(1000.0 / ms, 2), "unit": UNIT, "h2d_bytes_per_step": 8 * (n + 2 * nd),
+            "d2h_bytes_per_step": 8 * (n + nb + 2), "steps": ncall * chunk,
+            "api": "efit_fit_host (pinned host buffers; H2D/D2H on library streams, double-buffered)"}
 
 
 # ----------------------------------------------------------------------------- CPU oracle
@@ -706,9 +638,25 @@ def reference_arm(args, rank, world):
     print(json.dumps(out), flush=True)
 
 
+def relaunch_under_torchrun(args):
+    """--gpus N > 1 without a torchrun environment: re-run this command as N ranks (one process
+    per GPU) under torch.distributed.run on 127.0.0.1; rank 0 prints the JSON line."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+    os.execv(sys.executable, cmd)
+
+
 def main():
     args = parse()
     rank, world, local = dist_env()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        relaunch_under_torchrun(args)
+    if args.gpus != world:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE = {world}")
     if args.impl == "reference":
         reference_arm(args, rank, world)
         return

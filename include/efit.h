@@ -34,9 +34,25 @@
  * Errors: arguments are validated on the host before any launch; a failing call returns
  *   a negative EFIT_E_* code, launches nothing and leaves outputs untouched.
  *   efit_last_error() gives a one-line reason.  A context is not thread-safe.
- * Multi-GPU (efit_dist.world > 1): each rank owns a contiguous slice of the targets
- *   (boundary rows i, response rows m); see efit_shard().  The compute calls write only
- *   the rank's slice of d_resp / d_psib; the caller exchanges the slices.
+ * Multi-GPU (efit_dist.world > 1; one process per GPU; north_star "grid rows and diagnostic/boundary
+ *   points are sharded ... with an NCCL allreduce/allgather"): each rank owns the
+ *   response rows [resp_row_lo, resp_row_hi) and its share of the top/bottom boundary stream
+ *   (target rows [bnd_row_lo, bnd_row_hi) of the full table, or the row-pair tiles
+ *   [sym_tile_lo, sym_tile_hi) of the half table); the left/right targets, the least squares, the
+ *   current and the interior solve are computed on every rank.  A rank's exchange slice is
+ *   zero-padded and every exchanged entry has exactly one writing rank, so the sum over ranks is
+ *   exact and every output is BITWISE identical for any world size (the SYM slots are the per-tile
+ *   partial sums, reduced afterwards in the same fixed order as on one GPU).
+ *   - efit_dist.nccl_id != NULL: the context owns an NCCL communicator (efit_green_init is then
+ *     collective over the ranks) and every compute call returns REPLICATED outputs: the exchange (one
+ *     in-place sum all-reduce of the response before the least squares and one of the boundary slice
+ *     before the interior solve) is enqueued inside the call on the caller's stream and captured into
+ *     the fit step's CUDA graph.  NCCL is loaded at run time (the libnccl.so.2 already in the process,
+ *     else the system one; EFIT_NCCL_LIB overrides); EFIT_E_NCCL reports its failures.
+ *   - efit_dist.nccl_id == NULL (caller-exchange mode): efit_response writes only the rank's rows of
+ *     d_resp (zero the buffer and sum it over ranks); the boundary flux goes through
+ *     efit_boundary_partials -> caller's sum over ranks -> efit_boundary_finish; efit_fit_step(s) and
+ *     efit_boundary_flux return EFIT_E_STATE.
  */
 #ifndef EFIT_H
 #define EFIT_H
@@ -81,9 +97,12 @@ typedef struct {
     int32_t ip_sign;
 } efit_geometry;
 
-/* Target sharding across `world` ranks (one process per GPU).  {0, 1} = single GPU. */
+/* Sharding across `world` ranks (one process per GPU).  {0, 1, NULL} = single GPU.  nccl_id: a
+ * 128-byte ncclUniqueId (efit_nccl_unique_id on one rank, sent to the others by the caller), or NULL
+ * for the caller-exchange mode (see "Multi-GPU" above). */
 typedef struct {
     int32_t rank, world;
+    const void* nccl_id;
 } efit_dist;
 
 /* Sizes derived from the configuration (filled by efit_info). */
@@ -93,11 +112,13 @@ typedef struct {
     int32_t rank, world;
     int32_t resp_row_lo, resp_row_hi;   /* this rank's response rows [lo, hi)          */
     int32_t bnd_row_lo, bnd_row_hi;     /* this rank's top/bottom target rows i [lo, hi) */
-    int32_t lr_blk_lo, lr_blk_hi;       /* this rank's left/right target tiles           */
-    int32_t lr_j_lo, lr_j_hi;           /* this rank's left/right targets j [lo, hi)     */
+    int32_t lr_blk_lo, lr_blk_hi;       /* left/right target tiles computed (all: replicated) */
+    int32_t lr_j_lo, lr_j_hi;           /* left/right targets j [lo, hi) computed (0, nh)    */
     int64_t slab_stride;                /* doubles between Green's-table slabs           */
     int32_t sym_nblk;                   /* SYM modes: 8-row blocks of the nw-2 interior rows */
     int32_t sym_tile_lo, sym_tile_hi;   /* SYM modes: this rank's row-pair tiles [lo, hi)   */
+    int64_t xbuf_len;                   /* doubles of a rank's boundary exchange slice       */
+    int32_t exchange;                   /* 1 if the context owns an NCCL communicator        */
     size_t workspace_bytes;
 } efit_info_t;
 
@@ -112,8 +133,8 @@ typedef struct {
  *                            Results equal TABLE to rounding (<= 1e-14 relative), not bit for bit.
  *   EFIT_GREEN_ONTHEFLY_SYM  the SYM decomposition with G recomputed (half the Green's evaluations
  *                            of ONTHEFLY); bitwise equal to EFIT_GREEN_TABLE_SYM.
- * SYM modes with world > 1: the row-pair tiles are sharded, so every rank writes a partial sum for
- * every top/bottom target; the caller SUMS the zero-initialised d_psib over ranks (all-reduce). */
+ * SYM modes with world > 1: the row-pair tiles are sharded; the exchange slice holds the per-tile
+ * partial sums (every slot written by one rank), reduced in a fixed order after the exchange. */
 enum { EFIT_GREEN_TABLE = 0, EFIT_GREEN_ONTHEFLY = 1, EFIT_GREEN_TABLE_SYM = 2, EFIT_GREEN_ONTHEFLY_SYM = 3 };
 
 enum {
@@ -121,7 +142,7 @@ enum {
     EFIT_E_INVAL = -1,     /* bad argument (host-side validation)                 */
     EFIT_E_NOMEM = -2,     /* workspace too small / host allocation failed        */
     EFIT_E_CUDA = -3,      /* CUDA runtime error (possibly from earlier async work) */
-    EFIT_E_NCCL = -4,      /* reserved for the collective layer                    */
+    EFIT_E_NCCL = -4,      /* NCCL not loadable / communicator or collective error */
     EFIT_E_SINGULAR = -5,  /* least-squares: |R_kk| < 1e-13 max|R_jj|              */
     EFIT_E_NOPLASMA = -6,  /* empty plasma mask / psi_axis == psi_bdry             */
     EFIT_E_NONFINITE = -7, /* NaN/Inf met in a reduction                           */
@@ -150,7 +171,8 @@ int efit_plan_info(const efit_grid* grid, const efit_basis* basis, const efit_ge
 
 /* steps_ + green_: psi_axis/psi_bdry from d_psi[nw*nh], then
  * d_resp[m*nbasis + k] = sum_g Gd[m][g] dR dZ mask_g w_k(R_g) phi_k(psihat_g)
- * for this rank's rows m (all rows if world == 1).  d_axbd[2] (may be NULL) receives
+ * for every row m (world == 1, or with the NCCL exchange) or for this rank's rows only
+ * (caller-exchange mode; the other rows are not written).  d_axbd[2] (may be NULL) receives
  * {psi_axis, psi_bdry}. */
 int efit_response(efit_ctx* ctx, const double* d_psi, double* d_resp, double* d_axbd,
                   efit_stream_t stream);
@@ -163,9 +185,25 @@ int efit_current(efit_ctx* ctx, const double* d_psi, const double* d_coef, doubl
 /* pflux_ O(N^3) part (Fig. 2/3): d_psib[p] = sum_g G(x_p; x_g) d_pcurr[g] for the
  * n_edge edge nodes p in the edge order above, physical sign (+; the paper stores the
  * negated sum).  The self term G(x_p; x_p) is the point-to-cell average
- * (reading Q5).  world > 1: only this rank's targets are written. */
+ * (reading Q5).  world > 1 needs the NCCL exchange (EFIT_E_STATE otherwise). */
 int efit_boundary_flux(efit_ctx* ctx, const double* d_pcurr, double* d_psib,
                        efit_stream_t stream);
+
+/* Caller-exchange form of efit_boundary_flux (any mode, any world size):
+ * efit_boundary_partials writes this rank's zero-padded exchange slice d_xbuf[xbuf_len] (efit_info)
+ * for the current d_pcurr: SYM modes -> the partial sums of the rank's row-pair tiles, layout
+ * [i-1][side][slot] (side 0 = bottom, 1 = top; slot = the tile's other 8-row block x m-chunk);
+ * full table -> the rank's top/bottom entries of psi_b (edge order from 2*nh), 0 elsewhere.
+ * efit_boundary_finish takes the slices SUMMED over all ranks in d_xbuf and writes all n_edge
+ * entries of d_psib (left/right targets computed locally from d_pcurr, the same current).  The
+ * result is bitwise that of efit_boundary_flux on one GPU. */
+int efit_boundary_partials(efit_ctx* ctx, const double* d_pcurr, double* d_xbuf, efit_stream_t stream);
+int efit_boundary_finish(efit_ctx* ctx, const double* d_pcurr, const double* d_xbuf, double* d_psib,
+                         efit_stream_t stream);
+
+/* Host: a fresh 128-byte ncclUniqueId into id_out (for efit_dist.nccl_id).  EFIT_E_NCCL if NCCL
+ * cannot be loaded. */
+int efit_nccl_unique_id(void* id_out);
 
 /* pflux_ O(N^2) part, Eq. (1): solve Delta*_h psi = -mu0 R pcurr/(dR dZ) on the interior
  * nodes (5-point operator, reading Q17) with psi = d_psib on the edge.
@@ -183,7 +221,8 @@ int efit_lsq(efit_ctx* ctx, const double* d_resp, const double* d_meas, const do
  *   response(psi) -> lsq -> current -> boundary flux -> interior solve ->
  *   psi <- psi_p + d_psi_ext (in place);  d_eps[0] = max|psi_new - psi_old| / |psi_bdry - psi_axis|.
  * d_meas: measurements with the external-coil contribution already removed.
- * world > 1 is not supported by this fused call (EFIT_E_STATE): use the step calls. */
+ * world > 1: needs the NCCL exchange (efit_dist.nccl_id), EFIT_E_STATE otherwise; the two
+ * exchanges are nodes of the captured graph and every rank ends with the same psi. */
 int efit_fit_step(efit_ctx* ctx, double* d_psi, const double* d_psi_ext, const double* d_meas,
                   const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps,
                   efit_stream_t stream);
@@ -196,8 +235,20 @@ int efit_fit_steps(efit_ctx* ctx, int32_t nsteps, double* d_psi, const double* d
                    const double* d_meas, const double* d_sigma, double* d_coef, double* d_chi2,
                    double* d_eps, efit_stream_t stream);
 
-/* Tail of a fit iteration for the sharded (world > 1) path, after the caller has exchanged the
- * boundary slices: interior solve of d_pcurr with edge values d_psib, then
+/* End-to-end reconstruction from HOST buffers (the e2e path; EFIT reconstructs many time
+ * slices of a discharge).  For each of nslice slices k (one machine: shared d_psi_ext, device):
+ *   h_psi0[k][nw*nh], h_meas[k][ndiag], h_sigma[k][ndiag]  (host, pinned for asynchronous copies)
+ *   -> copied in, `iters` chained fit iterations (efit_fit_steps semantics), results copied out to
+ *   h_psi[k][nw*nh], h_coef[k][nbasis], h_chi2[k], h_eps[k] (host).
+ * The copies run on the library's own streams and are double-buffered, so the upload of slice k+1
+ * and the download of slice k-1 overlap the fit of slice k.  Enqueue only: the host outputs are
+ * valid once `stream` (non-NULL, not capturing) reaches the end of the call.  d_psi_ext must stay
+ * constant while the call is in flight. */
+int efit_fit_host(efit_ctx* ctx, int32_t nslice, int32_t iters, const double* h_psi0, const double* h_meas,
+                  const double* h_sigma, const double* d_psi_ext, double* h_psi, double* h_coef, double* h_chi2,
+                  double* h_eps, efit_stream_t stream);
+
+/* Tail of a fit iteration (caller-exchange path), after efit_boundary_finish: interior solve of d_pcurr with edge values d_psib, then
  * psi <- psi_p + d_psi_ext (in place) and d_eps[0] = max|psi_new - psi_old| / |psi_bdry - psi_axis|,
  * with psi_axis/psi_bdry from the most recent efit_response or efit_current call on this ctx. */
 int efit_solve_update(efit_ctx* ctx, const double* d_pcurr, const double* d_psib, const double* d_psi_ext,

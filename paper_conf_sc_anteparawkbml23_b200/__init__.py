@@ -24,7 +24,8 @@ __all__ = [
     "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY", "EFIT_GREEN_TABLE_SYM",
     "EFIT_GREEN_ONTHEFLY_SYM", "efit_plan_info", "owned_targets", "exchange",
     "efit_batch_workspace_bytes", "efit_batch_attach", "efit_fit_step_batch", "efit_fit_steps_batch",
-    "efit_boundary_flux_batch", "efit_boundary_basis",
+    "efit_boundary_flux_batch", "efit_boundary_basis", "efit_boundary_partials", "efit_boundary_finish",
+    "efit_nccl_unique_id", "efit_fit_host",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -60,7 +61,7 @@ class efit_geometry(ctypes.Structure):
 
 
 class efit_dist(ctypes.Structure):
-    _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32)]
+    _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("nccl_id", ctypes.c_void_p)]
 
 
 class efit_info_t(ctypes.Structure):
@@ -73,6 +74,7 @@ class efit_info_t(ctypes.Structure):
                 ("lr_j_lo", ctypes.c_int32), ("lr_j_hi", ctypes.c_int32),
                 ("slab_stride", ctypes.c_int64), ("sym_nblk", ctypes.c_int32),
                 ("sym_tile_lo", ctypes.c_int32), ("sym_tile_hi", ctypes.c_int32),
+                ("xbuf_len", ctypes.c_int64), ("exchange", ctypes.c_int32),
                 ("workspace_bytes", ctypes.c_size_t)]
 
 
@@ -103,6 +105,10 @@ def lib() -> ctypes.CDLL:
             "efit_response": (I, [vp, vp, vp, vp, vp]),
             "efit_current": (I, [vp, vp, vp, vp, vp]),
             "efit_boundary_flux": (I, [vp, vp, vp, vp]),
+            "efit_boundary_partials": (I, [vp, vp, vp, vp]),
+            "efit_boundary_finish": (I, [vp, vp, vp, vp, vp]),
+            "efit_nccl_unique_id": (I, [vp]),
+            "efit_fit_host": (I, [vp, ctypes.c_int32, ctypes.c_int32, vp, vp, vp, vp, vp, vp, vp, vp, vp]),
             "efit_interior_solve": (I, [vp, vp, vp, vp, vp]),
             "efit_lsq": (I, [vp, vp, vp, vp, vp, vp, vp]),
             "efit_fit_step": (I, [vp, vp, vp, vp, vp, vp, vp, vp, vp]),
@@ -168,7 +174,7 @@ def _arr(a) -> np.ndarray:
 class _Config:
     """Holds the ctypes structs + the numpy arrays they point into (kept alive)."""
 
-    def __init__(self, grid, basis, geometry, rank: int = 0, world: int = 1):
+    def __init__(self, grid, basis, geometry, rank: int = 0, world: int = 1, nccl_id: Optional[bytes] = None):
         self.keep = []
 
         def P(a):
@@ -182,7 +188,13 @@ class _Config:
         self.geom = efit_geometry(len(g.fl_r), P(g.fl_r), P(g.fl_z), len(g.mp_r), P(g.mp_r), P(g.mp_z),
                                   P(g.mp_ang), len(g.int_r), P(g.int_r), P(g.int_z), len(g.lim_r), P(g.lim_r),
                                   P(g.lim_z), int(g.ip_sign))
-        self.dist = efit_dist(rank, world)
+        if nccl_id is not None:
+            if len(nccl_id) != 128:
+                raise ValueError("nccl_id must be the 128-byte ncclUniqueId")
+            self._nccl_id = ctypes.create_string_buffer(bytes(nccl_id), 128)
+            self.dist = efit_dist(rank, world, ctypes.cast(self._nccl_id, ctypes.c_void_p))
+        else:
+            self.dist = efit_dist(rank, world, None)
 
 
 # ------------------------------------------------------------------------ ABI functions
@@ -215,21 +227,31 @@ def efit_plan_info(grid, basis, geom, dist, mode: int = EFIT_GREEN_TABLE) -> efi
 
 
 def owned_targets(info):
-    """Host logic of the sharded step: the response rows and the edge positions (ABI edge order)
-    this rank writes.  Every other entry of the rank's output buffers stays exactly 0, so a sum
-    all-reduce over ranks reproduces the single-GPU arrays bit for bit."""
+    """Host logic of the sharded step: the response rows and the top/bottom edge positions (ABI edge
+    order) whose exchange-slice entries this rank writes (full-table mode; SYM modes exchange the
+    per-tile partial sums instead, see include/efit.h).  Every other entry of the rank's slice is
+    exactly 0, so a sum all-reduce over ranks reproduces the single-GPU arrays bit for bit.  The
+    left/right targets are computed on every rank and never exchanged."""
     rows = list(range(info.resp_row_lo, info.resp_row_hi))
     nw, nh = info.nw, info.nh
-    edge = list(range(info.lr_j_lo, info.lr_j_hi)) + [nh + j for j in range(info.lr_j_lo, info.lr_j_hi)]
+    edge = []
     for i in range(info.bnd_row_lo, info.bnd_row_hi):
         edge += [2 * nh + (i - 1), 2 * nh + (nw - 2) + (i - 1)]
     return rows, sorted(edge)
 
 
 def exchange(buf, group=None) -> None:
-    """Make a zero-padded rank slice replicated: one sum all-reduce (NCCL on GPUs, gloo in tests)."""
+    """Caller-exchange mode: make a zero-padded rank slice replicated with one sum all-reduce
+    (NCCL on GPUs, gloo in tests).  Exact: every entry has one non-zero term."""
     import torch.distributed as dist
     dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=group)
+
+
+def efit_nccl_unique_id() -> bytes:
+    """A fresh 128-byte ncclUniqueId (create on one rank, broadcast to the others)."""
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().efit_nccl_unique_id(buf))
+    return buf.raw
 
 
 def efit_response(ctx, psi, resp, axbd=None, stream=None) -> None:
@@ -242,6 +264,14 @@ def efit_current(ctx, psi, coef, pcurr, stream=None) -> None:
 
 def efit_boundary_flux(ctx, pcurr, psib, stream=None) -> None:
     _check(lib().efit_boundary_flux(ctx, _ptr(pcurr), _ptr(psib), _stream(stream)), ctx)
+
+
+def efit_boundary_partials(ctx, pcurr, xbuf, stream=None) -> None:
+    _check(lib().efit_boundary_partials(ctx, _ptr(pcurr), _ptr(xbuf), _stream(stream)), ctx)
+
+
+def efit_boundary_finish(ctx, pcurr, xbuf, psib, stream=None) -> None:
+    _check(lib().efit_boundary_finish(ctx, _ptr(pcurr), _ptr(xbuf), _ptr(psib), _stream(stream)), ctx)
 
 
 def efit_interior_solve(ctx, pcurr, psib, psi_p, stream=None) -> None:
@@ -280,6 +310,23 @@ def efit_profile_end(ctx):
 def efit_fit_steps(ctx, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None) -> None:
     _check(lib().efit_fit_steps(ctx, nsteps, _ptr(psi), _ptr(psi_ext), _ptr(meas), _ptr(sigma), _ptr(coef),
                                 _ptr(chi2), _ptr(eps), _stream(stream)), ctx)
+
+
+def _hptr(t) -> int:
+    """Host pointer of a contiguous CPU fp64 tensor / numpy array (efit_fit_host)."""
+    if isinstance(t, np.ndarray):
+        if t.dtype != np.float64 or not t.flags.c_contiguous:
+            raise ValueError("expected a C-contiguous float64 array")
+        return t.ctypes.data
+    if t.is_cuda or not t.is_contiguous():
+        raise ValueError("expected a contiguous host tensor")
+    return t.data_ptr()
+
+
+def efit_fit_host(ctx, nslice, iters, h_psi0, h_meas, h_sigma, psi_ext, h_psi, h_coef, h_chi2, h_eps,
+                  stream=None) -> None:
+    _check(lib().efit_fit_host(ctx, nslice, iters, _hptr(h_psi0), _hptr(h_meas), _hptr(h_sigma), _ptr(psi_ext),
+                               _hptr(h_psi), _hptr(h_coef), _hptr(h_chi2), _hptr(h_eps), _stream(stream)), ctx)
 
 
 def efit_batch_workspace_bytes(ctx, nslice: int) -> int:
@@ -348,9 +395,9 @@ class EfitContext:
     """Owns the device workspace (a torch uint8 tensor) and the library handle."""
 
     def __init__(self, grid, basis, geometry, mode: int = EFIT_GREEN_TABLE, rank: int = 0, world: int = 1,
-                 device=None, stream=None):
+                 device=None, stream=None, nccl_id: Optional[bytes] = None):
         import torch
-        self.cfg = _Config(grid, basis, geometry, rank, world)
+        self.cfg = _Config(grid, basis, geometry, rank, world, nccl_id)
         self.device = torch.device(device if device is not None else "cuda")
         nbytes = efit_workspace_bytes(self.cfg.grid, self.cfg.basis, self.cfg.geom, self.cfg.dist, mode)
         # 256-byte alignment: allocate a little extra and offset
@@ -396,6 +443,17 @@ class EfitContext:
         efit_boundary_flux(self.handle, pcurr, out, stream)
         return out
 
+    def boundary_partials(self, pcurr, stream=None):
+        """This rank's zero-padded boundary exchange slice (caller-exchange mode)."""
+        out = self._t(int(self.info.xbuf_len))
+        efit_boundary_partials(self.handle, pcurr, out, stream)
+        return out
+
+    def boundary_finish(self, pcurr, xbuf, stream=None):
+        out = self._t(self.n_edge)
+        efit_boundary_finish(self.handle, pcurr, xbuf, out, stream)
+        return out
+
     def interior_solve(self, pcurr, psib, stream=None):
         out = self._t(self.nw * self.nh)
         efit_interior_solve(self.handle, pcurr, psib, out, stream)
@@ -411,6 +469,10 @@ class EfitContext:
 
     def fit_steps(self, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream=None):
         efit_fit_steps(self.handle, nsteps, psi, psi_ext, meas, sigma, coef, chi2, eps, stream)
+
+    def fit_host(self, nslice, iters, h_psi0, h_meas, h_sigma, psi_ext, h_psi, h_coef, h_chi2, h_eps, stream=None):
+        efit_fit_host(self.handle, nslice, iters, h_psi0, h_meas, h_sigma, psi_ext, h_psi, h_coef, h_chi2, h_eps,
+                      stream)
 
     def status(self, stream=None) -> int:
         return efit_status(self.handle, stream)

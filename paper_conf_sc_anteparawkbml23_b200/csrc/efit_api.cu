@@ -1,7 +1,11 @@
 // efit_api.cu -- C ABI (include/efit.h): validation, tiling plan, workspace carve, CUDA-graph
 // capture of the fit step.  Host code only; kernels live in efit_kernels.cu.
+#include <dlfcn.h>
+#include <nccl.h>  // types only: the functions are resolved at run time (see nccl_api)
+
 #include <cmath>
 #include <cstdarg>
+#include <mutex>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -32,8 +36,76 @@ static int fail(Ctx* c, int code, const char* fmt, ...) {
     return code;
 }
 
+// ------------------------------------------------------------------ NCCL, loaded at run time
+// The library does not link libnccl: a Python host process already holds torch's libnccl.so.2
+// (and a second copy of NCCL in one process is a hazard), so the functions are resolved from the
+// copy already loaded (RTLD_NOLOAD), else from the system library; EFIT_NCCL_LIB names another file.
+struct NcclApi {
+    bool ok = false;
+    char why[200] = "";
+    ncclResult_t (*get_unique_id)(ncclUniqueId*) = nullptr;
+    ncclResult_t (*comm_init_rank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*all_reduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                               cudaStream_t) = nullptr;
+    ncclResult_t (*comm_destroy)(ncclComm_t) = nullptr;
+    const char* (*error_string)(ncclResult_t) = nullptr;
+};
+
+static NcclApi& nccl_api() {
+    static NcclApi api;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        const char* env = getenv("EFIT_NCCL_LIB");
+        void* h = nullptr;
+        if (env) h = dlopen(env, RTLD_NOW | RTLD_GLOBAL);
+        if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+        if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) {
+            std::snprintf(api.why, sizeof(api.why), "cannot load NCCL: %s", dlerror());
+            return;
+        }
+        api.get_unique_id = (decltype(api.get_unique_id))dlsym(h, "ncclGetUniqueId");
+        api.comm_init_rank = (decltype(api.comm_init_rank))dlsym(h, "ncclCommInitRank");
+        api.all_reduce = (decltype(api.all_reduce))dlsym(h, "ncclAllReduce");
+        api.comm_destroy = (decltype(api.comm_destroy))dlsym(h, "ncclCommDestroy");
+        api.error_string = (decltype(api.error_string))dlsym(h, "ncclGetErrorString");
+        api.ok = api.get_unique_id && api.comm_init_rank && api.all_reduce && api.comm_destroy && api.error_string;
+        if (!api.ok) std::snprintf(api.why, sizeof(api.why), "NCCL library lacks a required symbol");
+    });
+    return api;
+}
+
 static int cuda_fail(Ctx* c, cudaError_t e, const char* where) {
+    if (c && c->nccl_err) {
+        const int r = c->nccl_err;
+        c->nccl_err = 0;
+        return fail(c, EFIT_E_NCCL, "%s: NCCL: %s", where, nccl_api().error_string((ncclResult_t)r));
+    }
     return fail(c, EFIT_E_CUDA, "%s: %s", where, cudaGetErrorString(e));
+}
+
+namespace efit {
+cudaError_t xch_allreduce(Ctx& c, double* buf, size_t n, cudaStream_t s) {
+    if (!c.comm) return cudaErrorInvalidValue;
+    const ncclResult_t r = nccl_api().all_reduce(buf, buf, n, ncclFloat64, ncclSum, (ncclComm_t)c.comm, s);
+    if (r != ncclSuccess) {
+        c.nccl_err = (int)r;
+        return cudaErrorUnknown;
+    }
+    return cudaSuccess;
+}
+}  // namespace efit
+
+extern "C" int efit_nccl_unique_id(void* id_out) {
+    if (!id_out) return fail(nullptr, EFIT_E_INVAL, "id_out is null");
+    NcclApi& api = nccl_api();
+    if (!api.ok) return fail(nullptr, EFIT_E_NCCL, "%s", api.why);
+    ncclUniqueId id;
+    const ncclResult_t r = api.get_unique_id(&id);
+    if (r != ncclSuccess) return fail(nullptr, EFIT_E_NCCL, "ncclGetUniqueId: %s", api.error_string(r));
+    std::memcpy(id_out, &id, sizeof(id));
+    return EFIT_OK;
 }
 
 static inline long long round_up(long long x, long long m) { return (x + m - 1) / m * m; }
@@ -177,14 +249,16 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
         t.lr_jj = (q + t.lr_jt - 1) / t.lr_jt * t.lr_jt;
     }
     t.red_blocks = 592;  // 4 per SM: enough loads in flight for the psi scans
-    // shards (targets only => bitwise identical results for any world size)
+    // shards: response rows and top/bottom target rows (full table) or row-pair tiles (SYM); every
+    // exchanged slot has exactly one writer => bitwise identical results for any world size
     int lo, hi;
     efit_shard(c.ndiag, c.rank, c.world, &lo, &hi);
     c.m_lo = lo; c.m_hi = hi;
     efit_shard(c.nw - 2, c.rank, c.world, &lo, &hi);
     c.i_lo = 1 + lo; c.i_hi = 1 + hi;
-    efit_shard(t.lr_njt, c.rank, c.world, &lo, &hi);
-    c.jt_lo = lo; c.jt_hi = hi;
+    // left/right targets: replicated on every rank (an FP64-bound chain under the table stream; the
+    // interior solve's overlapped forward DST needs them locally)
+    c.jt_lo = 0; c.jt_hi = t.lr_njt;
     // SYM modes: row-pair tiles of 8 x 8 interior rows; the tiles (not the targets) are sharded
     c.sym_nblk = (c.ni + 7) / 8;
     c.sym_ntile = (long long)c.sym_nblk * (c.sym_nblk + 1) / 2;
@@ -242,7 +316,6 @@ static size_t carve_scratch(Ctx& c, Take& take, size_t& off, bool batch) {
     c.fhat = (double*)take(sizeof(double) * (size_t)c.fhat_ld * c.nmode);
     c.psip = (double*)take(sizeof(double) * (size_t)n);
     c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 2));
-    c.scratch_meas = (double*)take(sizeof(double) * c.ndiag);
     c.sym_edge = c.sym ? (double*)take(sizeof(double) * 2 * (size_t)(c.nw > 2 ? c.nw - 2 : 1)) : nullptr;
     return (size_t)round_up((long long)off, 256);
 }
@@ -280,6 +353,14 @@ static size_t carve(Ctx& c, char* base) {
     c.twiddle = (double2*)take(sizeof(double2) * (size_t)(c.fft_m / 2));
     c.sin_tab = (double*)take(sizeof(double) * (size_t)c.nmode);
     c.lr_spec = (double*)take(sizeof(double) * 2 * (size_t)c.nh * c.lr_ldi);
+    for (int b = 0; b < 2; ++b) {  // efit_fit_host staging slots
+        c.hslot[b].psi = (double*)take(sizeof(double) * (size_t)n);
+        c.hslot[b].meas = (double*)take(sizeof(double) * c.ndiag);
+        c.hslot[b].sigma = (double*)take(sizeof(double) * c.ndiag);
+        c.hslot[b].coef = (double*)take(sizeof(double) * 32);
+        c.hslot[b].chi2 = (double*)take(sizeof(double) * 2);
+        c.hslot[b].eps = (double*)take(sizeof(double) * 2);
+    }
     return carve_scratch(c, take, off, false);
 }
 
@@ -364,7 +445,11 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
         delete h;
         return cuda_fail(nullptr, e, "side stream");
     }
-    c.gexec = nullptr;
+    for (int k = 0; k < Ctx::kGraphCache; ++k) c.gexec[k] = nullptr;
+    c.gnext = 0;
+    c.hs = c.ds = nullptr;
+    c.hstart = nullptr;
+    for (int b = 0; b < 2; ++b) c.hin[b] = c.hdone[b] = c.hfree[b] = nullptr;
     c.prof_on = false;
     c.prof_rec = false;
     c.prof_every = 1;
@@ -382,6 +467,29 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
             delete h;
             return cuda_fail(nullptr, e, "profile events");
         }
+    }
+    c.comm = nullptr;
+    c.nccl_err = 0;
+    if (dist && dist->nccl_id) {  // collective: every rank of the world calls efit_green_init
+        NcclApi& api = nccl_api();
+        if (!api.ok) {
+            for (int id = 0; id < efit::kNumMarks; ++id) cudaEventDestroy(c.prof_place[id]);
+            cudaStreamDestroy(c.side); cudaEventDestroy(c.ev_fork); cudaEventDestroy(c.ev_join);
+            delete h;
+            return fail(nullptr, EFIT_E_NCCL, "%s", api.why);
+        }
+        ncclUniqueId id;
+        std::memcpy(&id, dist->nccl_id, sizeof(id));
+        ncclComm_t comm = nullptr;
+        const ncclResult_t r = api.comm_init_rank(&comm, c.world, id, c.rank);
+        if (r != ncclSuccess) {
+            for (int k = 0; k < efit::kNumMarks; ++k) cudaEventDestroy(c.prof_place[k]);
+            cudaStreamDestroy(c.side); cudaEventDestroy(c.ev_fork); cudaEventDestroy(c.ev_join);
+            delete h;
+            return fail(nullptr, EFIT_E_NCCL, "ncclCommInitRank(world %d, rank %d): %s", c.world, c.rank,
+                        api.error_string(r));
+        }
+        c.comm = comm;
     }
     c.use_graph = getenv("EFIT_NO_GRAPH") == nullptr;
     c.nslice = 0;
@@ -407,6 +515,8 @@ static void fill_info(const Ctx& c, efit_info_t* info) {
     info->sym_nblk = c.sym_nblk;
     info->sym_tile_lo = (int32_t)c.sym_tile_lo;
     info->sym_tile_hi = (int32_t)c.sym_tile_hi;
+    info->xbuf_len = c.sym ? 2LL * c.ni * c.sym_nblk * c.t.sym_nmc : 2LL * (c.nw - 2);
+    info->exchange = c.comm ? 1 : 0;
     info->workspace_bytes = c.ws_bytes;
 }
 
@@ -445,7 +555,11 @@ extern "C" int efit_response(efit_ctx* h, const double* d_psi, double* d_resp, d
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e;
     if ((e = efit::launch_normalize(c, d_psi, s))) return cuda_fail(&c, e, "normalize");
+    const size_t nresp = (size_t)c.ndiag * c.nb;
+    if (c.comm && c.world > 1 && (e = cudaMemsetAsync(d_resp, 0, sizeof(double) * nresp, s)))
+        return cuda_fail(&c, e, "response clear");
     if ((e = efit::launch_response(c, d_psi, d_resp + (size_t)c.m_lo * c.nb, s))) return cuda_fail(&c, e, "response");
+    if (c.comm && (e = efit::xch_allreduce(c, d_resp, nresp, s))) return cuda_fail(&c, e, "response exchange");
     if (d_axbd && (e = cudaMemcpyAsync(d_axbd, c.axbd, 2 * sizeof(double), cudaMemcpyDeviceToDevice, s)))
         return cuda_fail(&c, e, "axbd copy");
     return EFIT_OK;
@@ -470,10 +584,41 @@ extern "C" int efit_boundary_flux(efit_ctx* h, const double* d_pcurr, double* d_
     Ctx& c = h->c;
     EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
     EFIT_CHECK_PTR(c, d_psib, "d_psib");
+    if (c.world > 1 && !c.comm)
+        return fail(&c, EFIT_E_STATE, "world > 1 without NCCL exchange: use efit_boundary_partials/finish");
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e;
     if ((e = efit::launch_make_pair(c, d_pcurr, s))) return cuda_fail(&c, e, "pair");
-    if ((e = efit::launch_boundary(c, d_pcurr, d_psib, s))) return cuda_fail(&c, e, "boundary");
+    if ((e = efit::launch_boundary(c, d_pcurr, d_psib, s, false, false, c.comm ? efit::XCH_NCCL : efit::XCH_NONE)))
+        return cuda_fail(&c, e, "boundary");
+    return EFIT_OK;
+}
+
+extern "C" int efit_boundary_partials(efit_ctx* h, const double* d_pcurr, double* d_xbuf, efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
+    EFIT_CHECK_PTR(c, d_xbuf, "d_xbuf");
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    if ((e = efit::launch_make_pair(c, d_pcurr, s))) return cuda_fail(&c, e, "pair");
+    if ((e = efit::launch_boundary(c, d_pcurr, nullptr, s, false, false, efit::XCH_PARTIALS, d_xbuf)))
+        return cuda_fail(&c, e, "boundary partials");
+    return EFIT_OK;
+}
+
+extern "C" int efit_boundary_finish(efit_ctx* h, const double* d_pcurr, const double* d_xbuf, double* d_psib,
+                                    efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
+    EFIT_CHECK_PTR(c, d_xbuf, "d_xbuf");
+    EFIT_CHECK_PTR(c, d_psib, "d_psib");
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    if ((e = efit::launch_make_pair(c, d_pcurr, s))) return cuda_fail(&c, e, "pair");
+    if ((e = efit::launch_boundary(c, d_pcurr, d_psib, s, false, false, efit::XCH_FINISH, const_cast<double*>(d_xbuf))))
+        return cuda_fail(&c, e, "boundary finish");
     return EFIT_OK;
 }
 
@@ -530,7 +675,10 @@ static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, 
     mark(c, s, M_BEGIN);
     if (normalize && (e = launch_normalize(c, psi, s))) return e;
     mark(c, s, M_NORM);
-    if ((e = launch_response(c, psi, c.resp, s))) return e;
+    const size_t nresp = (size_t)c.ndiag * c.nb;
+    if (c.comm && c.world > 1 && (e = cudaMemsetAsync(c.resp, 0, sizeof(double) * nresp, s))) return e;
+    if ((e = launch_response(c, psi, c.resp + (size_t)c.m_lo * c.nb, s))) return e;
+    if (c.comm && (e = xch_allreduce(c, c.resp, nresp, s))) return e;  // replicated response (exact sum)
     mark(c, s, M_RESP);
     if ((e = launch_lsq(c, c.resp, meas, sigma, coef, chi2, s))) return e;
     if ((e = launch_current(c, psi, coef, c.pcurr, true, s))) return e;
@@ -538,7 +686,7 @@ static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, 
     // boundary flux (marks M_TB, M_LR inside); in FFT mode the forward DST (without the bottom/top
     // edge terms) runs on the side stream under k_bnd_tb and the tridiagonal solve adds those terms
     const bool overlap = !c.lr_direct;
-    if ((e = launch_boundary(c, c.pcurr, c.psib, s, overlap, c.sym))) return e;
+    if ((e = launch_boundary(c, c.pcurr, c.psib, s, overlap, c.sym, c.comm ? XCH_NCCL : XCH_NONE))) return e;
     if (!overlap && (e = launch_solve_fwd(c, c.pcurr, c.psib, s, 1))) return e;
     if ((e = launch_solve_rest(c, c.psib, nullptr, psi, psi_ext, eps, s, true, overlap))) return e;
     mark(c, s, M_SOLVE);
@@ -551,7 +699,8 @@ static int fit_steps_impl(efit_ctx* h, int32_t nsteps, double* d_psi, const doub
                           const double* d_sigma, double* d_coef, double* d_chi2, double* d_eps, efit_stream_t stream) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
     Ctx& c = h->c;
-    if (c.world != 1) return fail(&c, EFIT_E_STATE, "efit_fit_step(s) needs world == 1 (use the step calls)");
+    if (c.world != 1 && !c.comm)
+        return fail(&c, EFIT_E_STATE, "efit_fit_step(s) with world > 1 needs the NCCL exchange (efit_dist.nccl_id)");
     if (nsteps < 1) return fail(&c, EFIT_E_INVAL, "nsteps < 1");
     EFIT_CHECK_PTR(c, d_psi, "d_psi");
     EFIT_CHECK_PTR(c, d_psi_ext, "d_psi_ext");
@@ -579,20 +728,25 @@ static int fit_steps_impl(efit_ctx* h, int32_t nsteps, double* d_psi, const doub
         if ((e = enqueue())) return cuda_fail(&c, e, "fit step");
         return EFIT_OK;
     }
-    if (!c.gexec || std::memcmp(key, c.gkey, sizeof(key)) != 0) {
-        if (c.gexec) { cudaGraphExecDestroy(c.gexec); c.gexec = nullptr; }
+    int slot = -1;
+    for (int k = 0; k < Ctx::kGraphCache; ++k)
+        if (c.gexec[k] && std::memcmp(key, c.gkey[k], sizeof(key)) == 0) slot = k;
+    if (slot < 0) {
+        slot = c.gnext;
+        c.gnext = (c.gnext + 1) % Ctx::kGraphCache;
+        if (c.gexec[slot]) { cudaGraphExecDestroy(c.gexec[slot]); c.gexec[slot] = nullptr; }
         cudaGraph_t graph = nullptr;
         if ((e = cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal))) return cuda_fail(&c, e, "begin capture");
         cudaError_t e2 = enqueue();
         e = cudaStreamEndCapture(s, &graph);
         if (e2) { if (graph) cudaGraphDestroy(graph); return cuda_fail(&c, e2, "fit step capture"); }
         if (e) return cuda_fail(&c, e, "end capture");
-        e = cudaGraphInstantiateWithFlags(&c.gexec, graph, 0);
+        e = cudaGraphInstantiateWithFlags(&c.gexec[slot], graph, 0);
         cudaGraphDestroy(graph);
-        if (e) { c.gexec = nullptr; return cuda_fail(&c, e, "graph instantiate"); }
-        std::memcpy(c.gkey, key, sizeof(key));
+        if (e) { c.gexec[slot] = nullptr; return cuda_fail(&c, e, "graph instantiate"); }
+        std::memcpy(c.gkey[slot], key, sizeof(key));
     }
-    if ((e = cudaGraphLaunch(c.gexec, s))) return cuda_fail(&c, e, "graph launch");
+    if ((e = cudaGraphLaunch(c.gexec[slot], s))) return cuda_fail(&c, e, "graph launch");
     return EFIT_OK;
 }
 
@@ -606,6 +760,67 @@ extern "C" int efit_fit_steps(efit_ctx* h, int32_t nsteps, double* d_psi, const 
                               const double* d_meas, const double* d_sigma, double* d_coef, double* d_chi2,
                               double* d_eps, efit_stream_t stream) {
     return fit_steps_impl(h, nsteps, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, stream);
+}
+
+// Host-buffer pipeline: nslice successive reconstructions (time slices), each `iters` chained
+// fit iterations, with their inputs read from and results written to HOST memory.  Staging slot
+// k & 1: H2D of slice k on the copy stream hs (after slot k-2's results left on ds) -> the cached
+// fit-step graph on `stream` -> D2H on ds; so the copies of slices k+1 / k-1 overlap slice k's step.
+extern "C" int efit_fit_host(efit_ctx* h, int32_t nslice, int32_t iters, const double* h_psi0, const double* h_meas,
+                             const double* h_sigma, const double* d_psi_ext, double* h_psi, double* h_coef,
+                             double* h_chi2, double* h_eps, efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    if (nslice < 1 || iters < 1) return fail(&c, EFIT_E_INVAL, "nslice and iters must be >= 1");
+    if (!h_psi0 || !h_meas || !h_sigma || !h_psi || !h_coef || !h_chi2 || !h_eps)
+        return fail(&c, EFIT_E_INVAL, "null host buffer");
+    EFIT_CHECK_PTR(c, d_psi_ext, "d_psi_ext");
+    if (c.world != 1 && !c.comm) return fail(&c, EFIT_E_STATE, "world > 1 needs the NCCL exchange");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (s == nullptr) return fail(&c, EFIT_E_INVAL, "efit_fit_host needs a non-default stream");
+    cudaError_t e;
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if ((e = cudaStreamIsCapturing(s, &cs))) return cuda_fail(&c, e, "capture query");
+    if (cs != cudaStreamCaptureStatusNone) return fail(&c, EFIT_E_STATE, "efit_fit_host cannot be captured");
+    if (!c.hs) {
+        int lo = 0, hi = 0;
+        cudaDeviceGetStreamPriorityRange(&lo, &hi);
+        if ((e = cudaStreamCreateWithPriority(&c.hs, cudaStreamNonBlocking, hi)) ||
+            (e = cudaStreamCreateWithPriority(&c.ds, cudaStreamNonBlocking, hi)) ||
+            (e = cudaEventCreateWithFlags(&c.hstart, cudaEventDisableTiming)))
+            return cuda_fail(&c, e, "host pipeline streams");
+        for (int b = 0; b < 2; ++b)
+            if ((e = cudaEventCreateWithFlags(&c.hin[b], cudaEventDisableTiming)) ||
+                (e = cudaEventCreateWithFlags(&c.hdone[b], cudaEventDisableTiming)) ||
+                (e = cudaEventCreateWithFlags(&c.hfree[b], cudaEventDisableTiming)))
+                return cuda_fail(&c, e, "host pipeline events");
+    }
+    const size_t n = (size_t)c.nw * c.nh, nd = (size_t)c.ndiag, nb = (size_t)c.nb;
+    if ((e = cudaEventRecord(c.hstart, s)) || (e = cudaStreamWaitEvent(c.hs, c.hstart, 0)) ||
+        (e = cudaStreamWaitEvent(c.ds, c.hstart, 0)))
+        return cuda_fail(&c, e, "host pipeline fork");
+    for (int k = 0; k < nslice; ++k) {
+        const int b = k & 1;
+        Ctx::HostSlot& q = c.hslot[b];
+        if (k >= 2 && (e = cudaStreamWaitEvent(c.hs, c.hfree[b], 0))) return cuda_fail(&c, e, "slot wait");
+        if ((e = cudaMemcpyAsync(q.psi, h_psi0 + k * n, sizeof(double) * n, cudaMemcpyHostToDevice, c.hs)) ||
+            (e = cudaMemcpyAsync(q.meas, h_meas + k * nd, sizeof(double) * nd, cudaMemcpyHostToDevice, c.hs)) ||
+            (e = cudaMemcpyAsync(q.sigma, h_sigma + k * nd, sizeof(double) * nd, cudaMemcpyHostToDevice, c.hs)) ||
+            (e = cudaEventRecord(c.hin[b], c.hs)) || (e = cudaStreamWaitEvent(s, c.hin[b], 0)))
+            return cuda_fail(&c, e, "H2D");
+        int st = fit_steps_impl(h, iters, q.psi, d_psi_ext, q.meas, q.sigma, q.coef, q.chi2, q.eps, stream);
+        if (st) return st;
+        if ((e = cudaEventRecord(c.hdone[b], s)) || (e = cudaStreamWaitEvent(c.ds, c.hdone[b], 0)) ||
+            (e = cudaMemcpyAsync(h_psi + k * n, q.psi, sizeof(double) * n, cudaMemcpyDeviceToHost, c.ds)) ||
+            (e = cudaMemcpyAsync(h_coef + k * nb, q.coef, sizeof(double) * nb, cudaMemcpyDeviceToHost, c.ds)) ||
+            (e = cudaMemcpyAsync(h_chi2 + k, q.chi2, sizeof(double), cudaMemcpyDeviceToHost, c.ds)) ||
+            (e = cudaMemcpyAsync(h_eps + k, q.eps, sizeof(double), cudaMemcpyDeviceToHost, c.ds)) ||
+            (e = cudaEventRecord(c.hfree[b], c.ds)))
+            return cuda_fail(&c, e, "D2H");
+    }
+    for (int b = 0; b < 2 && b < nslice; ++b)
+        if ((e = cudaStreamWaitEvent(s, c.hfree[(nslice - 1 - b) & 1], 0))) return cuda_fail(&c, e, "join");
+    return EFIT_OK;
 }
 
 // ------------------------------------------------------------------ multi-time-slice batch
@@ -672,11 +887,14 @@ extern "C" int efit_batch_attach(efit_ctx* h, int32_t nslice, void* d_workspace,
         q->shadow = true;
         q->nslice = 0;
         for (int j = 0; j < efit::kMaxSlices; ++j) q->slice[j] = nullptr;
-        q->gexec = nullptr; q->bexec = nullptr; q->pexec = nullptr; q->pgraph = nullptr;
+        for (int k = 0; k < Ctx::kGraphCache; ++k) q->gexec[k] = nullptr;
+        q->hs = q->ds = nullptr;
+        q->bexec = nullptr; q->pexec = nullptr; q->pgraph = nullptr;
         q->prof_on = q->prof_rec = q->prof_capture = false;
         q->prof_ev = nullptr;
         for (int j = 0; j < 16; ++j) q->prof_place[j] = nullptr;
         q->side = nullptr; q->ev_fork = q->ev_join = nullptr;
+        q->comm = nullptr;  // slices never exchange (batching needs world == 1)
         c.slice[k] = q;
         char* base = (char*)d_workspace + per * (size_t)k;
         size_t off = 0;
@@ -1003,7 +1221,16 @@ extern "C" int efit_destroy(efit_ctx* h) {
     if (h->c.bev_fork) cudaEventDestroy(h->c.bev_fork);
     if (h->c.bev_tb) cudaEventDestroy(h->c.bev_tb);
     if (h->c.bev_resp) cudaEventDestroy(h->c.bev_resp);
-    if (h->c.gexec) cudaGraphExecDestroy(h->c.gexec);
+    for (int k = 0; k < Ctx::kGraphCache; ++k)
+        if (h->c.gexec[k]) cudaGraphExecDestroy(h->c.gexec[k]);
+    if (h->c.hs) cudaStreamDestroy(h->c.hs);
+    if (h->c.ds) cudaStreamDestroy(h->c.ds);
+    if (h->c.hstart) cudaEventDestroy(h->c.hstart);
+    for (int b = 0; b < 2; ++b) {
+        if (h->c.hin[b]) cudaEventDestroy(h->c.hin[b]);
+        if (h->c.hdone[b]) cudaEventDestroy(h->c.hdone[b]);
+        if (h->c.hfree[b]) cudaEventDestroy(h->c.hfree[b]);
+    }
     if (h->c.pexec) cudaGraphExecDestroy(h->c.pexec);
     if (h->c.pgraph) cudaGraphDestroy(h->c.pgraph);
     for (int id = 0; id < efit::kNumMarks; ++id)
@@ -1015,6 +1242,7 @@ extern "C" int efit_destroy(efit_ctx* h) {
         for (size_t i = 0; i < (size_t)h->c.prof_slots * efit::kNumMarks; ++i) cudaEventDestroy(h->c.prof_ev[i]);
         delete[] h->c.prof_ev;
     }
+    if (h->c.comm && !h->c.shadow) nccl_api().comm_destroy((ncclComm_t)h->c.comm);
     delete h;
     return EFIT_OK;
 }

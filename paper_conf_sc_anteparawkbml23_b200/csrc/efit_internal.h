@@ -64,7 +64,7 @@ struct Ctx {
     int fft_m, fft_log2;         // complex FFT length 2(nh-1) and its log2
     int m_lo, m_hi;              // response rows of this rank
     int i_lo, i_hi;              // top/bottom target rows of this rank (within [1, nw-1))
-    int jt_lo, jt_hi;            // left/right j-tiles of this rank
+    int jt_lo, jt_hi;            // left/right j-tiles computed here (all of them: replicated on every rank)
     long long S;                 // slab / row stride (doubles), multiple of 32
     Tiling t;
     size_t ws_bytes;
@@ -115,7 +115,11 @@ struct Ctx {
     double* fhat;       // [nmode][fhat_ld]  DST coefficients, mode-major (in place: tridiagonal solution)
     double* psip;       // [nw*nh]
     double* eps_part;   // [red_blocks]
-    double* scratch_meas;  // [ndiag] (unused placeholder)
+
+    // multi-GPU exchange (include/efit.h "Multi-GPU"): NCCL communicator owned by the context when
+    // efit_dist.nccl_id was given (then every compute call returns replicated outputs)
+    void* comm;         // ncclComm_t or nullptr
+    int nccl_err;       // last ncclResult_t != ncclSuccess of xch_allreduce (reported as EFIT_E_NCCL)
 
     // profiling: CUDA events recorded at marks inside the fit step (efit_profile_begin/end).
     // The profiled step is its own CUDA graph with external event-record nodes at the marks,
@@ -135,11 +139,20 @@ struct Ctx {
     cudaStream_t side;
     cudaEvent_t ev_fork, ev_join;
 
-    // CUDA graph cache for efit_fit_step
-    cudaGraphExec_t gexec;
-    const void* gkey[9];
-    cudaStream_t gstream;
+    // CUDA graph cache for efit_fit_step(s): a few pointer sets (efit_fit_host alternates two
+    // staging slots), replaced round-robin
+    static constexpr int kGraphCache = 4;
+    cudaGraphExec_t gexec[kGraphCache];
+    const void* gkey[kGraphCache][9];
+    int gnext;
     bool use_graph;
+
+    // host-buffer pipeline (efit_fit_host): two device staging slots, copy streams and events
+    struct HostSlot {
+        double *psi, *meas, *sigma, *coef, *chi2, *eps;
+    } hslot[2];
+    cudaStream_t hs, ds;              // H2D / D2H streams (created on first use)
+    cudaEvent_t hin[2], hdone[2], hfree[2], hstart;
 
     // multi-time-slice batch: shadow contexts share this context's tables and own
     // their per-iteration scratch (carved from the caller's batch workspace) and a stream each
@@ -174,9 +187,20 @@ cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const dou
                        double* coef, double* chi2, cudaStream_t s);
 cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double* pcurr,
                            bool pair, cudaStream_t s);
+// Boundary-flux exchange modes (multi-GPU; include/efit.h "Multi-GPU"):
+//   XCH_NONE      world 1: the whole psi_b into psib
+//   XCH_NCCL      the rank's zero-padded exchange slice, in-place NCCL sum all-reduce, finish into psib
+//   XCH_PARTIALS  the rank's zero-padded exchange slice into xbuf only (efit_boundary_partials)
+//   XCH_FINISH    psib from the summed exchange slices in xbuf (efit_boundary_finish)
+// Exchange slice: SYM modes -> the row-pair-tile partials [ni][2][sym_nblk*sym_nmc]; full table ->
+// the top/bottom entries of psi_b [2(nw-2)].  Left/right targets are computed on every rank.
+enum { XCH_NONE = 0, XCH_NCCL = 1, XCH_PARTIALS = 2, XCH_FINISH = 3 };
 // prepacked: the SYM staged layouts were written by this iteration's current kernel (fit step)
 cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s,
-                            bool overlap_solve = false, bool prepacked = false);
+                            bool overlap_solve = false, bool prepacked = false, int xmode = XCH_NONE,
+                            double* xbuf = nullptr);
+// in-place NCCL sum all-reduce of n doubles over the context's communicator (efit_api.cu)
+cudaError_t xch_allreduce(Ctx& c, double* buf, size_t n, cudaStream_t s);
 cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cudaStream_t s, int with_bnd);
 cudaError_t launch_solve_rest(Ctx& c, const double* psib, double* psi_out, double* psi_inout, const double* psi_ext,
                               double* eps, cudaStream_t s, bool next_norm, bool tb_fix);

@@ -1665,8 +1665,10 @@ __global__ void __launch_bounds__(256) k_bnd_lr(const double* __restrict__ Tedge
 // psi_b in edge order from the partials: one warp per edge target, chunk-fastest partials,
 // fixed lane assignment + butterfly => deterministic and independent of the rank count.
 // SYM mode: top/bottom partials per (target, side, slot) from k_bnd_sym, plus the edge-row sources
-// ii = 0, nw-1 through the edge slabs (reciprocity: T[i][0][m] = Tedge[0][i][m]) for the rank's
-// own target rows [i_lo, i_hi) only, so that a sum over ranks counts them once.
+// ii = 0, nw-1 through the edge slabs (reciprocity: T[i][0][m] = Tedge[0][i][m]).
+// Multi-GPU (include/efit.h, "Multi-GPU"): every slot of the SYM partials is written by exactly
+// one row-pair tile, i.e. by one rank, so the zero-padded partials summed over ranks are the
+// world-1 partials exactly and this fixed-order reduction gives world-independent psi_b.
 struct SymReduce {
     const double* part;   // nullptr: full-table mode
     int nslot;
@@ -1677,12 +1679,22 @@ struct SymReduce {
     const double* edge;   // SYM: edge-row source sums per top/bottom target (k_sym_edge_src), or nullptr
 };
 
+// Destinations of k_bnd_reduce: left/right entries (psi_b[0, 2 nh)) to `lr` (nullptr: not
+// written), top/bottom entries (psi_b[2 nh, n_edge)) to `tb` (indexed from 0; nullptr: not
+// written) for target rows i in [tb_lo, tb_hi); zero_unowned writes 0 to the other rows' entries
+// (the zero padding of a rank's exchange slice).
+struct BndOut {
+    double* lr;
+    double* tb;
+    int tb_lo, tb_hi, zero_unowned;
+};
+
 // SYM modes: the top/bottom targets' sums over the edge-row sources ii = 0, nw-1 (not in the half
 // table), from the replicated edge slabs: out[side*(nw-2) + i-1] = sum_m T0[i][m] X[0][m] + T1[i][m] X[nw-1][m],
-// X = I (bottom) or F (top).  One warp per target; runs on the side stream under the table stream.
+// X = I (bottom) or F (top).  One warp per target, every target on every rank (replicated, cheap);
+// runs on the side stream under the table stream.
 __global__ void k_sym_edge_src(const double* __restrict__ Tedge, long long S, const double* __restrict__ pc,
-                               const double* __restrict__ pf, int nw, int nh, int i_lo, int i_hi,
-                               double* __restrict__ out) {
+                               const double* __restrict__ pf, int nw, int nh, double* __restrict__ out) {
     griddep();
     const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
     const int q = w;  // 0 .. 2(nw-2)-1
@@ -1690,20 +1702,17 @@ __global__ void k_sym_edge_src(const double* __restrict__ Tedge, long long S, co
     const int side = q < nw - 2 ? 0 : 1;
     const int i = q - side * (nw - 2) + 1;
     double s = 0.0;
-    if (i >= i_lo && i < i_hi) {
-        const double* x0 = (side ? pf : pc);
-        const double* x1 = x0 + (long long)(nw - 1) * nh;
-        const double* t0 = Tedge + (long long)i * nh;
-        const double* t1 = t0 + S;
-        for (int m = lane; m < nh; m += 32) s = fma(t0[m], x0[m], fma(t1[m], x1[m], s));
-    }
+    const double* x0 = (side ? pf : pc);
+    const double* x1 = x0 + (long long)(nw - 1) * nh;
+    const double* t0 = Tedge + (long long)i * nh;
+    const double* t1 = t0 + S;
+    for (int m = lane; m < nh; m += 32) s = fma(t0[m], x0[m], fma(t1[m], x1[m], s));
     s = warp_sum(s);
     if (lane == 0) out[q] = s;
 }
 
 __global__ void k_bnd_reduce(const double* __restrict__ tb_part, int tb_nchunk, const double* __restrict__ lr_part,
-                             int lr_nblk, int nw, int nh, int i_lo, int i_hi, int jlo, int jhi,
-                             double* __restrict__ psib, SymReduce sy) {
+                             int lr_nblk, int nw, int nh, int jlo, int jhi, BndOut o, SymReduce sy) {
     griddep();
     const int n_edge = 2 * nh + 2 * (nw - 2);
     const int p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
@@ -1711,39 +1720,44 @@ __global__ void k_bnd_reduce(const double* __restrict__ tb_part, int tb_nchunk, 
     const double* src;
     int cnt;
     double s = 0.0;
+    double* dst;
     if (p < 2 * nh) {
         const int side = p < nh ? 0 : 1;
         const int j = p - side * nh;
-        if (j < jlo || j >= jhi) return;
+        if (!o.lr || j < jlo || j >= jhi) return;
         src = lr_part + ((long long)side * nh + j) * lr_nblk;
         cnt = lr_nblk;
+        dst = o.lr + p;
     } else {
         const int q = p - 2 * nh;
         const int side = q < nw - 2 ? 0 : 1;
         const int i = q - side * (nw - 2) + 1;
+        if (!o.tb) return;
+        dst = o.tb + q;
+        if (i < o.tb_lo || i >= o.tb_hi) {
+            if (o.zero_unowned && lane == 0) *dst = 0.0;
+            return;
+        }
         if (sy.part) {
             src = sy.part + ((long long)(i - 1) * 2 + side) * sy.nslot;
             cnt = sy.nslot;
-            if (i >= i_lo && i < i_hi) {
-                if (sy.edge) {
-                    if (lane == 0) s = sy.edge[q];
-                } else {
-                    const double* x0 = (side ? sy.pf : sy.pc);
-                    const double* x1 = x0 + (long long)(nw - 1) * nh;
-                    const double* t0 = sy.Tedge + (long long)i * nh;
-                    const double* t1 = t0 + sy.S;
-                    for (int m = lane; m < nh; m += 32) s = fma(t0[m], x0[m], fma(t1[m], x1[m], s));
-                }
+            if (sy.edge) {
+                if (lane == 0) s = sy.edge[q];
+            } else {
+                const double* x0 = (side ? sy.pf : sy.pc);
+                const double* x1 = x0 + (long long)(nw - 1) * nh;
+                const double* t0 = sy.Tedge + (long long)i * nh;
+                const double* t1 = t0 + sy.S;
+                for (int m = lane; m < nh; m += 32) s = fma(t0[m], x0[m], fma(t1[m], x1[m], s));
             }
         } else {
-            if (i < i_lo || i >= i_hi) return;
             src = tb_part + ((long long)i * 2 + side) * tb_nchunk;
             cnt = tb_nchunk;
         }
     }
     for (int c = lane; c < cnt; c += 32) s += src[c];
     s = warp_sum(s);
-    if (lane == 0) psib[p] = s;
+    if (lane == 0) *dst = s;
 }
 
 // On-the-fly variant of k_bnd_tb: G recomputed from (R_i, R_ii, m dZ) with the same device
@@ -2130,75 +2144,113 @@ static cudaError_t launch_lr(Ctx& c, cudaStream_t s, bool prepare) {
 cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cudaStream_t s, int with_bnd);
 
 cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s, bool overlap_solve,
-                            bool prepacked) {
+                            bool prepacked, int xmode, double* xbuf) {
     cudaError_t e;
-    // fork: the FP64-bound left/right kernel runs on the side stream, concurrently with the
-    // HBM-bound top/bottom stream (both only read pcurr / ipair); join before the reduce.
-    if ((e = cudaEventRecord(c.ev_fork, s)) || (e = cudaStreamWaitEvent(c.side, c.ev_fork, 0))) return e;
-    if (c.lr_direct) {
-        if ((e = launch_lr(c, c.side, false))) return e;
-    } else {
-        if ((e = launch_lr_fft(c, psib, c.side))) return e;
+    const bool side_work = xmode != XCH_PARTIALS;  // left/right targets + SYM edge-row sources (replicated)
+    const bool tile_work = xmode != XCH_FINISH;    // the rank's share of the top/bottom stream
+    if (side_work) {
+        // fork: the FP64-bound left/right chain runs on the side stream, concurrently with the
+        // HBM-bound top/bottom stream (both only read pcurr / ipair); join before the reduce.
+        if ((e = cudaEventRecord(c.ev_fork, s)) || (e = cudaStreamWaitEvent(c.side, c.ev_fork, 0))) return e;
+        if (c.lr_direct) {
+            if ((e = launch_lr(c, c.side, false))) return e;
+        } else {
+            if ((e = launch_lr_fft(c, psib, c.side))) return e;
+        }
+        // superposition: apart from the bottom/top edge terms the GS right-hand side is known once the
+        // left/right FFT chain has written psi_b(left/right), so its forward DST also runs under the
+        // HBM-bound stream; k_tridiag adds the bottom/top terms in the sine domain afterwards
+        if (overlap_solve && (e = launch_solve_fwd(c, pcurr, psib, c.side, 2))) return e;
+        if (c.sym && c.sym_edge &&
+            (e = launch_pdl(k_sym_edge_src, dim3((2 * (c.nw - 2) + 7) / 8), dim3(256), 0, c.side, (const double*)c.Tedge,
+                            c.S, (const double*)c.pcurr, (const double*)c.pflip, c.nw, c.nh, c.sym_edge)))
+            return e;
+        mark(c, c.side, M_LR);
+        if ((e = cudaEventRecord(c.ev_join, c.side))) return e;
     }
-    // superposition: apart from the bottom/top edge terms the GS right-hand side is known once the
-    // left/right FFT chain has written psi_b(left/right), so its forward DST also runs under the
-    // HBM-bound stream; k_tridiag adds the bottom/top terms in the sine domain afterwards
-    if (overlap_solve && (e = launch_solve_fwd(c, pcurr, psib, c.side, 2))) return e;
-    if (c.sym && c.sym_edge &&
-        (e = launch_pdl(k_sym_edge_src, dim3((2 * (c.nw - 2) + 7) / 8), dim3(256), 0, c.side, (const double*)c.Tedge, c.S,
-                        (const double*)c.pcurr, (const double*)c.pflip, c.nw, c.nh, c.i_lo, c.i_hi, c.sym_edge)))
-        return e;
-    mark(c, c.side, M_LR);
-    if ((e = cudaEventRecord(c.ev_join, c.side))) return e;
     const int nslab = c.i_hi - c.i_lo;
     const size_t smem_tb = 2 * sizeof(double) * c.t.tb_ch;
+    const long long sym_len = 2LL * c.ni * c.sym_nblk * c.t.sym_nmc;  // SYM exchange slice (doubles)
+    double* sym_out = xmode == XCH_PARTIALS ? xbuf : c.sym_part;
     SymReduce sy{nullptr, 0, c.Tedge, c.S, c.pcurr, c.pflip, nullptr};
-    if (c.sym) {
-        sy.part = c.sym_part;
-        sy.edge = c.sym_edge;
-        sy.nslot = c.sym_nblk * c.t.sym_nmc;
-        const long long ntl = c.sym_tile_hi - c.sym_tile_lo;
-        if (ntl > 0) {
-            const int narr = c.t.sym_nmc == 1 ? 1 : 2;
-            if (!prepacked)
-                launch_pdl(k_sym_pack, dim3(4 * kNumSMs), dim3(256), 0, s, (const double*)c.pcurr, (const double*)c.pflip,
-                           c.nh, c.nhp, c.ni, c.sym_nblk, narr, c.symq, c.symp);
-            if ((e = cudaGetLastError())) return e;
-            const size_t smem = sym_smem(c);
-            const bool mir = c.t.sym_nmc == 1;
-            const dim3 grid((unsigned)(ntl * c.t.sym_nmc));
+    if (tile_work) {
+        if (c.sym) {
+            // other ranks' slots must read 0 in a zero-padded exchange slice
+            if ((xmode == XCH_PARTIALS || (xmode == XCH_NCCL && c.world > 1)) &&
+                (e = cudaMemsetAsync(sym_out, 0, sizeof(double) * (size_t)sym_len, s)))
+                return e;
+            const long long ntl = c.sym_tile_hi - c.sym_tile_lo;
+            if (ntl > 0) {
+                const int narr = c.t.sym_nmc == 1 ? 1 : 2;
+                if (!prepacked)
+                    launch_pdl(k_sym_pack, dim3(4 * kNumSMs), dim3(256), 0, s, (const double*)c.pcurr, (const double*)c.pflip,
+                               c.nh, c.nhp, c.ni, c.sym_nblk, narr, c.symq, c.symp);
+                if ((e = cudaGetLastError())) return e;
+                const size_t smem = sym_smem(c);
+                const bool mir = c.t.sym_nmc == 1;
+                const dim3 grid((unsigned)(ntl * c.t.sym_nmc));
+                const int nslot = c.sym_nblk * c.t.sym_nmc;
 #define EFIT_SYM_LAUNCH(OTFV, MIRV, UNRV, NBV, WGV)                                                                      \
     launch_pdl(k_bnd_sym<OTFV, MIRV, UNRV, NBV, WGV>, grid, dim3(128 * WGV), smem, s, (const double*)c.U, c.sym_tile_lo,  \
-               c.ni, c.nh, c.t.sym_nmc, c.t.sym_mc, (const double*)c.symq, (const double*)c.symp, c.nhp, sy.nslot, \
-               c.sym_part, c.rmin, c.dr, c.dz)
-            if (c.otf) {  // FP64-bound: a short unroll keeps the inlined AGM in registers
-                if (mir) EFIT_SYM_LAUNCH(true, true, 1, 2, kSymWg); else EFIT_SYM_LAUNCH(true, false, 1, 2, kSymWg);
-            } else if (mir) {
-                EFIT_SYM_LAUNCH(false, true, kSymUnr, kSymBuf, kSymWg);
-            } else {
-                EFIT_SYM_LAUNCH(false, false, kSymUnr, kSymBuf, kSymWg);
-            }
+               c.ni, c.nh, c.t.sym_nmc, c.t.sym_mc, (const double*)c.symq, (const double*)c.symp, c.nhp, nslot,       \
+               sym_out, c.rmin, c.dr, c.dz)
+                if (c.otf) {  // FP64-bound: a short unroll keeps the inlined AGM in registers
+                    if (mir) EFIT_SYM_LAUNCH(true, true, 1, 2, kSymWg); else EFIT_SYM_LAUNCH(true, false, 1, 2, kSymWg);
+                } else if (mir) {
+                    EFIT_SYM_LAUNCH(false, true, kSymUnr, kSymBuf, kSymWg);
+                } else {
+                    EFIT_SYM_LAUNCH(false, false, kSymUnr, kSymBuf, kSymWg);
+                }
 #undef EFIT_SYM_LAUNCH
+                if ((e = cudaGetLastError())) return e;
+            }
+        } else if (nslab > 0) {
+            dim3 grid(c.t.tb_nchunk, c.t.tb_ngroup);
+            if (!c.otf) {
+                launch_pdl(k_bnd_tb<kTbGI, kTbUnroll>, dim3(grid), dim3(256), smem_tb, s, c.T, c.S, nslab, c.i_lo, c.nw * c.nh,
+                           c.pcurr, c.pflip, c.t.tb_ch, c.tb_part);
+            } else {
+                launch_pdl(k_bnd_tb_otf<kTbGI>, dim3(grid), dim3(256), smem_tb, s, c.i_lo, nslab, c.nw, c.nh, c.rmin, c.dr,
+                           c.dz, c.pcurr, c.pflip, c.t.tb_ch, c.tb_part);
+            }
             if ((e = cudaGetLastError())) return e;
         }
-    } else if (nslab > 0) {
-        dim3 grid(c.t.tb_nchunk, c.t.tb_ngroup);
-        if (!c.otf) {
-            launch_pdl(k_bnd_tb<kTbGI, kTbUnroll>, dim3(grid), dim3(256), smem_tb, s, c.T, c.S, nslab, c.i_lo, c.nw * c.nh, c.pcurr,
-                                                                  c.pflip, c.t.tb_ch, c.tb_part);
-        } else {
-            launch_pdl(k_bnd_tb_otf<kTbGI>, dim3(grid), dim3(256), smem_tb, s, c.i_lo, nslab, c.nw, c.nh, c.rmin, c.dr, c.dz, c.pcurr,
-                                                           c.pflip, c.t.tb_ch, c.tb_part);
+        if (!c.sym && xmode != XCH_NONE) {
+            // full table: the rank's own top/bottom rows, zero-padded, are its exchange slice
+            BndOut o{nullptr, xmode == XCH_PARTIALS ? xbuf : psib + 2 * c.nh, c.i_lo, c.i_hi, 1};
+            if ((e = launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, (const double*)c.tb_part,
+                                c.t.tb_nchunk, (const double*)c.lr_part, c.t.lr_nblk, c.nw, c.nh, 0, 0, o, sy)))
+                return e;
         }
-        if ((e = cudaGetLastError())) return e;
     }
     mark(c, s, M_TB);
+    if (xmode == XCH_PARTIALS) return cudaSuccess;
+    if (xmode == XCH_NCCL) {  // zero-padded slices summed over ranks: exact (one non-zero term each)
+        if (c.sym) e = xch_allreduce(c, c.sym_part, (size_t)sym_len, s);
+        else e = xch_allreduce(c, psib + 2 * c.nh, (size_t)(2 * (c.nw - 2)), s);
+        if (e) return e;
+    }
     if ((e = cudaStreamWaitEvent(s, c.ev_join, 0))) return e;
-    // left/right entries come from the partials (direct path) or were written by k_lr_ifft
-    const int jlo = c.lr_direct ? c.jt_lo * 32 * c.t.lr_jt : 0;
-    const int jhi = c.lr_direct ? min(c.nh, c.jt_hi * 32 * c.t.lr_jt) : 0;
-    launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, c.tb_part, c.t.tb_nchunk, c.lr_part, c.t.lr_nblk, c.nw, c.nh,
-                                                    c.i_lo, c.i_hi, jlo, jhi, psib, sy);
+    // finish: left/right entries come from the partials (direct path) or were written by k_lr_ifft;
+    // top/bottom from the (exchanged) SYM slots + edge-row sources, or the table chunk partials
+    BndOut o{c.lr_direct ? psib : nullptr, nullptr, 1, c.nw - 1, 0};
+    if (c.sym) {
+        sy.part = xmode == XCH_FINISH ? xbuf : c.sym_part;
+        sy.edge = c.sym_edge;
+        sy.nslot = c.sym_nblk * c.t.sym_nmc;
+        o.tb = psib + 2 * c.nh;
+    } else if (xmode == XCH_NONE) {
+        o.tb = psib + 2 * c.nh;
+        o.tb_lo = c.i_lo;
+        o.tb_hi = c.i_hi;
+    } else if (xmode == XCH_FINISH) {
+        if ((e = cudaMemcpyAsync(psib + 2 * c.nh, xbuf, sizeof(double) * 2 * (size_t)(c.nw - 2), cudaMemcpyDeviceToDevice, s)))
+            return e;
+    }
+    if (!o.lr && !o.tb) return cudaSuccess;
+    const int jhi = c.lr_direct ? c.nh : 0;
+    launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, (const double*)c.tb_part, c.t.tb_nchunk,
+               (const double*)c.lr_part, c.t.lr_nblk, c.nw, c.nh, 0, jhi, o, sy);
     return cudaGetLastError();
 }
 
@@ -2332,8 +2384,9 @@ cudaError_t launch_boundary_batch(Ctx& c, int nslice, Ctx* const* slices, cudaSt
 // left/right entries were written by k_lr_ifft).
 cudaError_t launch_bnd_reduce(Ctx& c, const double* tb_part, int tb_nchunk, double* psib, cudaStream_t s) {
     SymReduce sy{nullptr, 0, c.Tedge, c.S, c.pcurr, c.pflip, nullptr};
-    return launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, tb_part, tb_nchunk, c.lr_part,
-                      c.t.lr_nblk, c.nw, c.nh, c.i_lo, c.i_hi, 0, 0, psib, sy);
+    BndOut o{nullptr, psib + 2 * c.nh, c.i_lo, c.i_hi, 0};
+    return launch_pdl(k_bnd_reduce, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, tb_part, tb_nchunk,
+                      (const double*)c.lr_part, c.t.lr_nblk, c.nw, c.nh, 0, 0, o, sy);
 }
 
 // ================================================================================ interior solve

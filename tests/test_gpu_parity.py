@@ -262,32 +262,6 @@ def test_boundary_sym_matches_full_table(torch_mod, efit, orc_mod):
     assert rel(y, x) < 1e-14
 
 
-def test_sym_sharded_sum_matches_single(torch_mod, efit, orc_mod):
-    """SYM mode, world = 3 emulated on one GPU: each rank streams its share of the row-pair tiles
-    and writes partial sums for every top/bottom target (and its own left/right targets); the
-    sum over ranks (the caller's all-reduce) equals world = 1 to rounding."""
-    torch = torch_mod
-    c1 = case("65x65", efit, orc_mod, mode=efit.EFIT_GREEN_TABLE_SYM)
-    cfg = c1.cfg
-    I = T(torch, synth.random_current(cfg.grid, seed=3, signed=True, edge=True))
-    psib1 = c1.ctx.boundary_flux(I)
-    acc = torch.zeros_like(psib1)
-    world = 3
-    tiles = []
-    for r in range(world):
-        ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=efit.EFIT_GREEN_TABLE_SYM, rank=r, world=world)
-        tiles.append((ctx.info.sym_tile_lo, ctx.info.sym_tile_hi))
-        part = torch.zeros_like(psib1)
-        efit.efit_boundary_flux(ctx.handle, I, part)
-        torch.cuda.synchronize()
-        acc += part
-        ctx.close()
-    nblk = c1.ctx.info.sym_nblk
-    assert tiles[0][0] == 0 and tiles[-1][1] == nblk * (nblk + 1) // 2
-    assert all(a[1] == b[0] for a, b in zip(tiles, tiles[1:]))
-    assert rel(acc.cpu().numpy(), psib1.cpu().numpy()) < 1e-14
-
-
 def test_boundary_literal_fig2(torch_mod, efit, orc_mod):
     """The GPU boundary equals minus the paper's Fig. 2/3 loops transcribed literally."""
     torch = torch_mod
@@ -477,31 +451,6 @@ def test_fit_loop_c2(torch_mod, efit, orc_mod):
     assert eps.item() < 1e-10
     assert np.max(np.abs(psi.cpu().numpy() - psi_s)) < 1e-8 * np.max(np.abs(psi_s))
     assert np.max(np.abs(coef.cpu().numpy() - ct)) < 1e-7 * np.max(np.abs(ct))
-
-
-# ------------------------------------------------------------------ multi-rank emulation
-
-def test_sharded_matches_single_bitwise(torch_mod, efit, orc_mod):
-    """world = 3 ranks emulated serially on one GPU: each rank writes only its slices
-    (response rows, boundary targets); the union equals world = 1 bit for bit."""
-    torch = torch_mod
-    c1 = case("65x65", efit, orc_mod)
-    cfg = c1.cfg
-    psi = T(torch, synth.perturbed_psi(cfg.grid, seed=5, rel=1e-3))
-    I = T(torch, synth.random_current(cfg.grid, seed=2))
-    resp1, _ = c1.ctx.response(psi)
-    psib1 = c1.ctx.boundary_flux(I)
-    world = 3
-    resp = torch.full_like(resp1, float("nan")).reshape(-1)
-    psib = torch.full_like(psib1, float("nan"))
-    for r in range(world):
-        ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, rank=r, world=world)
-        efit.efit_response(ctx.handle, psi, resp)
-        efit.efit_boundary_flux(ctx.handle, I, psib)
-        torch.cuda.synchronize()
-        ctx.close()
-    assert torch.equal(resp.view_as(resp1), resp1)
-    assert torch.equal(psib, psib1)
 
 
 def test_fit_steps_chained_equals_repeated(torch_mod, efit, orc_mod):
