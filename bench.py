@@ -590,22 +590,50 @@ def oracle_setup(config):
     return oracle, orc, tw, psi0
 
 
-def cpu_baseline(config, max_seconds=20.0):
-    """The oracle as it stands (or_fit_step, Green's memo tables prebuilt and untimed, as the
-    paper's pflux_ timing excludes the table precompute) on all host cores; a bounded number
-    of iterations."""
-    oracle, orc, tw, psi = oracle_setup(config)
-    times = []
-    t_all = time.time()
+def _time_iters(fn, psi, tw, max_iters, max_seconds):
+    times, t_all = [], time.time()
     while True:
         t = time.perf_counter()
-        st, psi, coef, chi2, eps = orc.fit_step(psi, tw["psi_ext"], tw["y"], tw["sigma"])
+        st, psi, coef, chi2, eps = fn(psi, tw["psi_ext"], tw["y"], tw["sigma"])
         times.append(time.perf_counter() - t)
-        if time.time() - t_all > max_seconds or len(times) >= 5:
-            break
-    v = len(times) / sum(times)
-    return {"value": round(v, 4), "unit": UNIT, "cores": oracle.get_threads(), "kind": "oracle",
-            "sample": f"{len(times)} oracle fit iteration(s) of {config} (memo tables prebuilt, untimed)"}
+        if st != 0:
+            raise RuntimeError(f"CPU fit step status {st}")
+        if time.time() - t_all > max_seconds or len(times) >= max_iters:
+            return len(times) / sum(times), len(times)
+
+
+def cpu_baseline(config, max_seconds=8.0):
+    """CPU timings beside the GPU number (SURVEY 8(d) "Oracle timing beside it"), same inputs:
+    value = the oracle as it stands (or_fit_step, Green's memo tables prebuilt and untimed, as the
+    paper's pflux_ timing excludes the table precompute) on all host cores; plus the oracle on one
+    core (the paper's one-core baselines) and the paper-literal CPU comparator
+    (baseline/paper_cpu.c: Fig. 2/3 nests + O(N^2) steps, -O3 -march=native -fopenmp) on one
+    core and on all host cores.  Each leg is bounded to a few iterations."""
+    oracle, orc, tw, psi = oracle_setup(config)
+    ncore = host_cores()
+    oracle.set_threads(ncore)
+    v_all, n_all = _time_iters(orc.fit_step, psi, tw, 5, max_seconds)
+    oracle.set_threads(1)
+    v_one, n_one = _time_iters(orc.fit_step, psi, tw, 2, max_seconds)
+    oracle.set_threads(ncore)
+    out = {"value": round(v_all, 4), "unit": UNIT, "cores": ncore, "kind": "oracle",
+           "sample": f"{n_all} oracle fit iteration(s) of {config} on {ncore} cores (memo tables prebuilt, untimed)",
+           "oracle_1core": {"value": round(v_one, 4), "cores": 1, "sample": f"{n_one} iteration(s)"}}
+    try:
+        from baseline import paper_cpu
+        pc = paper_cpu.PaperCPU(synth.config(config), orc)
+        paper_cpu.set_threads(1)
+        p1, n1 = _time_iters(pc.fit_step, psi, tw, 5, max_seconds)
+        paper_cpu.set_threads(ncore)
+        pa, na = _time_iters(pc.fit_step, psi, tw, 20, max_seconds)
+        out["paper_literal_cpu"] = {
+            "what": "baseline/paper_cpu.c: Fig. 2/3 O(N^3) nests + O(N^2) steps, gcc -O3 -march=native -fopenmp",
+            "1core": {"value": round(p1, 4), "cores": 1, "sample": f"{n1} iteration(s)"},
+            "all_cores": {"value": round(pa, 4), "cores": paper_cpu.get_threads(), "sample": f"{na} iteration(s)"},
+            "cpu_model": paper_cpu.cpu_model()}
+    except Exception as ex:  # a missing compiler must not sink the GPU line
+        out["paper_literal_cpu"] = {"unavailable": str(ex)[:200]}
+    return out
 
 
 def reference_arm(args, rank, world):

@@ -261,7 +261,7 @@ int efit_solve_update(efit_ctx* ctx, const double* d_pcurr, const double* d_psib
  * right-hand sides (each slice's current and its mirror), computed on the FP64 tensor cores
  * (mma.sync m8n8k4), while every slice's O(N^2) steps run concurrently on a stream of their own.
  * Each slice's results equal those of efit_fit_step on that slice alone to rounding (the table
- * pass sums in another order; not bit for bit).  Requires mode EFIT_GREEN_TABLE, world == 1.
+ * pass sums in another order; not bit for bit); each slice has its own status word.  Requires mode EFIT_GREEN_TABLE, world == 1.
  *
  * efit_batch_workspace_bytes: device bytes of per-slice scratch for nslice slices.
  * efit_batch_attach: carve that scratch from caller-owned device memory d_workspace (256-byte
@@ -312,9 +312,11 @@ int efit_boundary_basis(efit_ctx* ctx, const double* d_psi, double* d_rb, double
 int efit_profile_begin(efit_ctx* ctx, int32_t nsteps, int32_t every);
 int efit_profile_end(efit_ctx* ctx, double* ms_out, int32_t nout, int32_t* nsteps_out);
 
-/* Synchronise `stream` and return the first data-dependent failure recorded since the last
- * efit_status() call (EFIT_OK, EFIT_E_NOPLASMA, EFIT_E_SINGULAR, EFIT_E_NONFINITE), or
- * EFIT_E_CUDA.  Clears the status word. */
+/* Synchronise `stream` and return the data-dependent failure recorded since the last
+ * efit_status() call (EFIT_OK, EFIT_E_NONFINITE, EFIT_E_NOPLASMA, EFIT_E_SINGULAR -- in that
+ * priority), or EFIT_E_CUDA.  Every batch slice has its own status word (a failing slice sets only
+ * its own outputs to NaN); the words of the context and of all slices are OR-ed, the first failing
+ * slice is named in efit_last_error(), and all words are cleared. */
 int efit_status(efit_ctx* ctx, efit_stream_t stream);
 
 /* Test/inspection access: device pointers into the workspace.  which = 0: top/bottom Green's

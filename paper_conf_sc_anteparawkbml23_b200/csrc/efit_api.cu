@@ -904,8 +904,8 @@ extern "C" int efit_batch_attach(efit_ctx* h, int32_t nslice, void* d_workspace,
             off += bytes;
             return p;
         };
-        carve_scratch(*q, take, off, true);
-        q->status = c.status;  // one sticky status word for the whole batch
+        carve_scratch(*q, take, off, true);  // incl. the slice's own status word (a failing slice, e.g. a
+                                             // pre-plasma time slice, never poisons the others)
         // slice streams at normal priority: the shared table pass (main stream) keeps its SMs while the
         // slices' latency-bound chains fill in (measured +1.7 % at S = 8 over high priority)
         const int prio = getenv("EFIT_BATCH_HIPRIO") ? prio_hi : prio_lo;
@@ -1175,14 +1175,27 @@ extern "C" int efit_status(efit_ctx* h, efit_stream_t stream) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
     Ctx& c = h->c;
     cudaStream_t s = (cudaStream_t)stream;
-    int st = 0;
+    int st[1 + efit::kMaxSlices] = {0};
     cudaError_t e;
-    if ((e = cudaMemcpyAsync(&st, c.status, sizeof(int), cudaMemcpyDeviceToHost, s)) ||
-        (e = cudaMemsetAsync(c.status, 0, sizeof(int), s)) || (e = cudaStreamSynchronize(s)))
-        return cuda_fail(&c, e, "status");
-    if (st & EFIT_ST_NONFINITE) return fail(&c, EFIT_E_NONFINITE, "non-finite psi");
-    if (st & EFIT_ST_NOPLASMA) return fail(&c, EFIT_E_NOPLASMA, "empty plasma mask or psi_axis == psi_bdry");
-    if (st & EFIT_ST_SINGULAR) return fail(&c, EFIT_E_SINGULAR, "singular least-squares matrix");
+    // the context's word and every attached slice's own word (OR-ed; cleared)
+    for (int k = 0; k <= c.nslice; ++k) {
+        int* w = k == 0 ? c.status : c.slice[k - 1]->status;
+        if ((e = cudaMemcpyAsync(&st[k], w, sizeof(int), cudaMemcpyDeviceToHost, s)) ||
+            (e = cudaMemsetAsync(w, 0, sizeof(int), s)))
+            return cuda_fail(&c, e, "status");
+    }
+    if ((e = cudaStreamSynchronize(s))) return cuda_fail(&c, e, "status");
+    int all = 0, first = -1;
+    for (int k = 0; k <= c.nslice; ++k) {
+        all |= st[k];
+        if (st[k] && first < 0) first = k;
+    }
+    const char* where = "";
+    char buf[32] = "";
+    if (first > 0) { std::snprintf(buf, sizeof(buf), " (slice %d)", first - 1); where = buf; }
+    if (all & EFIT_ST_NONFINITE) return fail(&c, EFIT_E_NONFINITE, "non-finite psi%s", where);
+    if (all & EFIT_ST_NOPLASMA) return fail(&c, EFIT_E_NOPLASMA, "empty plasma mask or psi_axis == psi_bdry%s", where);
+    if (all & EFIT_ST_SINGULAR) return fail(&c, EFIT_E_SINGULAR, "singular least-squares matrix%s", where);
     return EFIT_OK;
 }
 

@@ -946,7 +946,12 @@ cudaError_t launch_resp_reduce_batch(Ctx& q, int nchunk, double* resp_rows, cuda
 //   G1 = A^T A = R1^T R1,  Q1 = A R1^-1,  G2 = Q1^T Q1 = R2^T R2  (so A = (Q1 R2^-1)(R2 R1)),
 //   c_hat = R1^-1 R2^-1 R2^-T (Q1^T b),  c = c_hat / column scale,
 // chi2 = sum((meas - resp c)/sigma)^2 from the unscaled system.  Backward stable for
-// cond(A) << eps^-1/2 ~ 1e8 (the synthetic bases: 3.6e3 .. 1.4e7).  Unlike Householder's chain of
+// cond(A) << eps^-1/2 ~ 1e8 (the synthetic bases: 3.6e3 .. 1.4e7).  Beyond that the first Cholesky
+// breaks down; the kernels then fall back to shifted CholeskyQR3 (Fukaya, Kannan, Nakatsukasa,
+// Yamamoto & Yanagisawa, SISC 2020): R0 = chol(A^T A + s I), s = 11 (nd nb + nb(nb+1)) u ||A||^2
+// (||A||_2^2 <= nb for unit columns), A <- A R0^-1 (now cond ~ u^-1/2), then CholeskyQR2 on it and
+// c_hat = R0^-1 (...) -- stable up to cond(A) ~ u^-1, the range of the oracle's Householder QR.
+// Unlike Householder's chain of
 // nb reflections, both Gram matrices are formed with all entries in parallel and the Q1 rows are
 // independent; only the two nb x nb Cholesky factorisations and the triangular solves are serial
 // (one warp).  Fixed summation orders => deterministic.  Singular if a Cholesky pivot is not
@@ -1037,7 +1042,9 @@ __device__ __forceinline__ void lsq_rsolve_rows(double* A, int ld, int nd, int n
 }
 
 // NBT > 0: the basis count as a compile-time constant (loops over it unroll, the final triangular
-// solves keep z in registers); NBT = 0: runtime nb.  Same arithmetic and order either way.
+// solves run one lane per unknown and add the back-substitution terms from the last unknown down);
+// NBT = 0: runtime nb, serial solves adding them in ascending order.  The two paths therefore agree
+// to rounding, not bit for bit (each is deterministic; both are parity-tested against the oracle).
 template <int NBT>
 __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, const double* __restrict__ meas,
                                              const double* __restrict__ sigma, int nd, int nb_arg,
@@ -1056,10 +1063,12 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
     double* sc = r2i + 32;                         // [32] column scales
     double* z = sc + 32;                           // [32]
     double* red = z + 32;                          // [16] chi2 partials
-    __shared__ int s_sing;
+    double* R0 = red + 32;                         // [nb][nb] shifted pass (fallback)
+    double* r0i = R0 + nb * nb;                    // [32]
+    __shared__ int s_sing, s_shift;
     griddep();
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarp = blockDim.x >> 5;
-    if (tid == 0) s_sing = 0;
+    if (tid == 0) { s_sing = 0; s_shift = 0; }
     for (int m = tid; m < nd; m += blockDim.x) {
         const double is = 1.0 / sigma[m];
         isg[m] = is;
@@ -1087,9 +1096,34 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
         bool ok;
         if constexpr (NBT > 0) ok = lsq_chol_warp<NBT>(G, R1, r1i);
         else ok = lsq_chol(G, R1, r1i, nb);
-        if (!ok && lane == 0) s_sing = 1;
+        if (!ok && lane == 0) s_shift = 1;
     }
     __syncthreads();
+    if (s_shift) {  // cond(A) beyond ~1e8: shifted CholeskyQR3 (see above)
+        lsq_gram(A, ld, nd, nb, G);
+        __syncthreads();
+        if (warp == 0) {
+            const double shift = 11.0 * ((double)nd * nb + (double)nb * (nb + 1)) * 0x1p-53 * nb;
+            for (int k = lane; k < nb; k += 32) G[k * nb + k] += shift;
+            __syncwarp();
+            bool ok;
+            if constexpr (NBT > 0) ok = lsq_chol_warp<NBT>(G, R0, r0i);
+            else ok = lsq_chol(G, R0, r0i, nb);
+            if (!ok && lane == 0) s_sing = 1;
+        }
+        __syncthreads();
+        if (!s_sing) lsq_rsolve_rows(A, ld, nd, nb, R0, r0i);
+        __syncthreads();
+        if (!s_sing) lsq_gram(A, ld, nd, nb, G);
+        __syncthreads();
+        if (warp == 0 && !s_sing) {
+            bool ok;
+            if constexpr (NBT > 0) ok = lsq_chol_warp<NBT>(G, R1, r1i);
+            else ok = lsq_chol(G, R1, r1i, nb);
+            if (!ok && lane == 0) s_sing = 1;
+        }
+        __syncthreads();
+    }
     if (!s_sing) lsq_rsolve_rows(A, ld, nd, nb, R1, r1i);
     __syncthreads();
     // pass 2: G2 = Q1^T Q1, R2, z = Q1^T b
@@ -1134,11 +1168,19 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
             if (j == k) zj = zk;
             else if (j < k) zj = fma(-R1[j * NBC + k], zk, zj);
         }
+        if (s_shift) {
+#pragma unroll
+            for (int k = NBC - 1; k >= 0; --k) {  // z <- R0^-1 z
+                const double zk = __shfl_sync(0xffffffffu, zj, k) * r0i[k];
+                if (j == k) zj = zk;
+                else if (j < k) zj = fma(-R0[j * NBC + k], zk, zj);
+            }
+        }
         if (lane == 0) {
             double rmax = 0.0, rmin = DBL_MAX;
 #pragma unroll
             for (int k = 0; k < NBC; ++k) {
-                const double d = fabs(R1[k * NBC + k] * R2[k * NBC + k]);
+                const double d = fabs(R1[k * NBC + k] * R2[k * NBC + k] * (s_shift ? R0[k * NBC + k] : 1.0));
                 rmax = fmax(rmax, d);
                 rmin = fmin(rmin, d);
                 if (!(sc[k] > 0.0)) s_sing = 1;
@@ -1153,9 +1195,9 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
             for (int i = 0; i < j; ++i) s = fma(-R2[i * nb + j], z[i], s);
             z[j] = s * r2i[j];
         }
-        const double* Rs[2] = {R2, R1};
-        const double* Ri[2] = {r2i, r1i};
-        for (int t = 0; t < 2; ++t)
+        const double* Rs[3] = {R2, R1, R0};
+        const double* Ri[3] = {r2i, r1i, r0i};
+        for (int t = 0; t < (s_shift ? 3 : 2); ++t)
             for (int k = nb - 1; k >= 0; --k) {
                 double s = z[k];
                 for (int j = k + 1; j < nb; ++j) s = fma(-Rs[t][k * nb + j], z[j], s);
@@ -1163,7 +1205,7 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
             }
         double rmax = 0.0, rmin = DBL_MAX;
         for (int k = 0; k < nb; ++k) {
-            const double d = fabs(R1[k * nb + k] * R2[k * nb + k]);
+            const double d = fabs(R1[k * nb + k] * R2[k * nb + k] * (s_shift ? R0[k * nb + k] : 1.0));
             rmax = fmax(rmax, d);
             rmin = fmin(rmin, d);
             if (!(sc[k] > 0.0)) s_sing = 1;
@@ -1280,9 +1322,30 @@ __global__ void __launch_bounds__(32) k_lsq_warp(const double* __restrict__ resp
 #pragma unroll
         for (int r = 0; r < RPL; ++r) a[r][k] *= isc;
     }
-    double G[NB][NB], R1[NB][NB], R2[NB][NB], r1i[NB], r2i[NB];
+    double G[NB][NB], R0[NB][NB], R1[NB][NB], R2[NB][NB], r0i[NB], r1i[NB], r2i[NB];
     lsq_gram_reg<NB, RPL>(a, G);
-    lsq_chol_reg<NB>(G, R1, r1i, ok);
+    bool ok1 = true;
+    lsq_chol_reg<NB>(G, R1, r1i, ok1);
+    const bool shifted = !ok1 && ok;  // warp-uniform: cond(A) beyond ~1e8 -> shifted CholeskyQR3
+    if (shifted) {
+        const double shift = 11.0 * ((double)nd * NB + (double)NB * (NB + 1)) * 0x1p-53 * NB;
+#pragma unroll
+        for (int k = 0; k < NB; ++k) G[k][k] += shift;
+        lsq_chol_reg<NB>(G, R0, r0i, ok);
+#pragma unroll
+        for (int r = 0; r < RPL; ++r)  // rows <- rows R0^-1
+#pragma unroll
+            for (int j = 0; j < NB; ++j) {
+                double s = a[r][j];
+#pragma unroll
+                for (int i = 0; i < j; ++i) s = fma(-a[r][i], R0[i][j], s);
+                a[r][j] = s * r0i[j];
+            }
+        lsq_gram_reg<NB, RPL>(a, G);
+        ok1 = true;
+        lsq_chol_reg<NB>(G, R1, r1i, ok1);
+    }
+    ok = ok && ok1;
 #pragma unroll
     for (int r = 0; r < RPL; ++r)  // rows <- rows R1^-1
 #pragma unroll
@@ -1327,10 +1390,19 @@ __global__ void __launch_bounds__(32) k_lsq_warp(const double* __restrict__ resp
         for (int j = k + 1; j < NB; ++j) s = fma(-R1[k][j], z[j], s);
         z[k] = s * r1i[k];
     }
+    if (shifted) {
+#pragma unroll
+        for (int k = NB - 1; k >= 0; --k) {  // R0^-1
+            double s = z[k];
+#pragma unroll
+            for (int j = k + 1; j < NB; ++j) s = fma(-R0[k][j], z[j], s);
+            z[k] = s * r0i[k];
+        }
+    }
     double rmax = 0.0, rmin = DBL_MAX;
 #pragma unroll
     for (int k = 0; k < NB; ++k) {
-        const double d = fabs(R1[k][k] * R2[k][k]);
+        const double d = fabs(R1[k][k] * R2[k][k] * (shifted ? R0[k][k] : 1.0));
         rmax = fmax(rmax, d);
         rmin = fmin(rmin, d);
         z[k] = z[k] / sc[k];
@@ -1370,7 +1442,7 @@ static bool launch_lsq_warp(int nd, const double* resp, const double* meas, cons
 }
 
 static size_t lsq_smem(const Ctx& c) {
-    return sizeof(double) * ((size_t)((c.nb | 1) + 2) * c.ndiag + 3 * (size_t)c.nb * c.nb + 5 * 32);
+    return sizeof(double) * ((size_t)((c.nb | 1) + 2) * c.ndiag + 4 * (size_t)c.nb * c.nb + 7 * 32);
 }
 
 cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const double* sigma, double* coef,

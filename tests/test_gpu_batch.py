@@ -260,3 +260,66 @@ def test_boundary_basis_needs_batch(torch_mod, efit, orc_mod):
     with pytest.raises(efit.EfitError) as ei:
         ctx.boundary_basis(T(torch, synth.perturbed_psi(cfg.grid, seed=5, rel=1e-3)), stream=torch.cuda.Stream())
     assert ei.value.code == efit.EFIT_E_STATE
+
+
+def test_batch_slice_status_isolated(torch_mod, efit, orc_mod):
+    """Every slice has its own status word: a slice without plasma (psi = 0: empty mask, e.g. a
+    pre-plasma time slice) gets NaN results and makes efit_status report EFIT_E_NOPLASMA naming
+    it, while the healthy slices' results are unaffected (equal the oracle's fit step)."""
+    torch = torch_mod
+    cfg, orc, ctx = setup("33x33", efit, orc_mod)
+    S = 3
+    ctx.batch_attach(S)
+    tws, psi0 = _slices(orc, cfg, S)
+    psi0 = [p.copy() for p in psi0]
+    psi0[1][:] = 0.0
+    psi = T(torch, np.stack(psi0))
+    ext = T(torch, np.stack([tw["psi_ext"] for tw in tws]))
+    y = T(torch, np.stack([tw["y"] for tw in tws]))
+    sg = T(torch, np.stack([tw["sigma"] for tw in tws]))
+    coef, chi2, eps = ctx._t(S * ctx.nbasis), ctx._t(S), ctx._t(S)
+    st = torch.cuda.Stream()
+    for _ in range(2):   # twice: the failing slice's sticky bit must not leak into the next call
+        p = psi.clone()
+        with torch.cuda.stream(st):
+            ctx.fit_step_batch(p, ext, y, sg, coef, chi2, eps, stream=st)
+        st.synchronize()
+        cg = coef.cpu().numpy().reshape(S, -1)
+        assert np.all(np.isnan(cg[1]))
+        for k in (0, 2):
+            ok, psi_r, c_r, chi2_r, eps_r = orc.fit_step(psi0[k], tws[k]["psi_ext"], tws[k]["y"], tws[k]["sigma"])
+            assert rel(p.cpu().numpy()[k], psi_r) < TOL
+            assert rel(cg[k], c_r) < TOL_C
+    assert ctx.status() == efit.EFIT_E_NOPLASMA
+    assert "slice 1" in efit.efit_last_error(ctx.handle)
+    assert ctx.status() == 0
+
+
+@pytest.mark.parametrize("nb", [5, 10])
+@pytest.mark.parametrize("cond", [1e6, 1e10, 1e12])
+def test_lsq_ill_conditioned_fallback(torch_mod, efit, orc_mod, nb, cond):
+    """Beyond cond ~ 1e8 CholeskyQR2 breaks down; the kernels fall back to shifted CholeskyQR3
+    (k_lsq_warp for nb <= 6, k_lsq<NB> above).  Against the oracle's Householder QR on a matrix
+    with prescribed singular values: coefficients to 50 cond u (the backward-stable bound), chi2
+    to 1e-10 relative."""
+    torch = torch_mod
+    basis = synth.poly_basis(2, 3) if nb == 5 else synth.poly_basis(5, 5)
+    g = synth.Grid(33, 33)
+    cfg = synth.Config("lsq", g, synth.make_geometry(g, 0), basis, "lsq")
+    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=0)
+    nd = ctx.ndiag
+    rng = np.random.default_rng(int(np.log10(cond)) + nb)
+    U, _ = np.linalg.qr(rng.standard_normal((nd, nb)))
+    V, _ = np.linalg.qr(rng.standard_normal((nb, nb)))
+    A = U @ np.diag(np.logspace(0, -np.log10(cond), nb)) @ V.T
+    A = A * rng.uniform(0.5, 2.0, nb)[None, :]   # unequal column scales
+    x = rng.standard_normal(nb)
+    sigma = rng.uniform(0.5, 1.5, nd)
+    y = A @ x + 1e-3 * sigma * rng.standard_normal(nd)
+    st, cref, chi2ref = orc_mod.lsq(A, y, sigma)
+    assert st == 0
+    coef, chi2 = ctx.lsq(T(torch, A), T(torch, y), T(torch, sigma))
+    assert ctx.status() == 0
+    assert rel(coef.cpu().numpy(), cref) < max(1e-10, 50 * cond * 2.0 ** -53), rel(coef.cpu().numpy(), cref)
+    assert abs(chi2.item() - chi2ref) <= 1e-10 * chi2ref
+    ctx.close()
