@@ -1289,17 +1289,24 @@ template <int NB, int RPL>
 __global__ void __launch_bounds__(32) k_lsq_warp(const double* __restrict__ resp, const double* __restrict__ meas,
                                                  const double* __restrict__ sigma, int nd,
                                                  double* __restrict__ coef, double* __restrict__ chi2, int* status) {
-    griddep();
     const int lane = threadIdx.x;
     double a[RPL][NB], bb[RPL], is[RPL];
+    // sigma and the measurements are inputs of the step (not produced by a predecessor kernel):
+    // their loads and the reciprocal overlap the wait on the response reduction
 #pragma unroll
     for (int r = 0; r < RPL; ++r) {
         const int m = lane + 32 * r;
         const bool ok = m < nd;
         is[r] = ok ? 1.0 / sigma[m] : 0.0;
+        bb[r] = ok ? meas[m] * is[r] : 0.0;
+    }
+    griddep();
+#pragma unroll
+    for (int r = 0; r < RPL; ++r) {
+        const int m = lane + 32 * r;
+        const bool ok = m < nd;
 #pragma unroll
         for (int k = 0; k < NB; ++k) a[r][k] = ok ? resp[(size_t)m * NB + k] * is[r] : 0.0;
-        bb[r] = ok ? meas[m] * is[r] : 0.0;
     }
     double sc[NB];
 #pragma unroll
@@ -1523,30 +1530,32 @@ template <int NB>
 __global__ void k_current_from_basis(const double* __restrict__ Bm, long long ldb, const double* __restrict__ coef,
                                      int nw, int nh, double* __restrict__ pcurr, double* __restrict__ pflip,
                                      SymPackOut sp) {
-    griddep();
     const int n = nw * nh;
-    double cf[NB];
+    const int g = blockIdx.x * blockDim.x + threadIdx.x;  // one node per thread (grid covers n)
+    // the basis values were written by k_response, three kernels back (complete before the
+    // predecessor started), so they are loaded before the wait on the predecessor (the LSQ)
+    double b[NB];
 #pragma unroll
-    for (int k = 0; k < NB; ++k) cf[k] = coef[k];
-    for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += gridDim.x * blockDim.x) {
-        double I = 0.0;
+    for (int k = 0; k < NB; ++k) b[k] = g < n ? Bm[k * ldb + g] : 0.0;
+    griddep();
+    if (g >= n) return;
+    double I = 0.0;
 #pragma unroll
-        for (int k = 0; k < NB; ++k) I = fma(cf[k], Bm[k * ldb + g], I);
-        pcurr[g] = I;
-        const int ii = g / nh, m = g - (g / nh) * nh;
-        pflip[ii * nh + (nh - 1 - m)] = I;
-        const int r = ii - 1;
-        if (sp.q && r >= 0 && r < sp.ni) {  // symq[B][arr][h][m][qh][w], symp[B][arr][p][m] (k_sym_pack)
-            const int B = r >> 3, q = r & 7, qh = q >> 2, h = (q >> 1) & 1, w = q & 1;
-            const long long qb = (long long)B * 16 * nh + (long long)h * 4 * nh + 2 * qh + w;
-            const long long pb = (long long)B * 16 * sp.nhp + (long long)q * sp.nhp;
-            sp.q[qb + 4LL * m] = I;
-            sp.p[pb + m] = I;
-            if (sp.narr == 2) {  // F[ii][nh-1-m] = I
-                const int mf = nh - 1 - m;
-                sp.q[qb + 8LL * nh + 4LL * mf] = I;
-                sp.p[pb + 8LL * sp.nhp + mf] = I;
-            }
+    for (int k = 0; k < NB; ++k) I = fma(coef[k], b[k], I);
+    pcurr[g] = I;
+    const int ii = g / nh, m = g - (g / nh) * nh;
+    pflip[ii * nh + (nh - 1 - m)] = I;
+    const int r = ii - 1;
+    if (sp.q && r >= 0 && r < sp.ni) {  // symq[B][arr][h][m][qh][w], symp[B][arr][p][m] (k_sym_pack)
+        const int B = r >> 3, q = r & 7, qh = q >> 2, h = (q >> 1) & 1, w = q & 1;
+        const long long qb = (long long)B * 16 * nh + (long long)h * 4 * nh + 2 * qh + w;
+        const long long pb = (long long)B * 16 * sp.nhp + (long long)q * sp.nhp;
+        sp.q[qb + 4LL * m] = I;
+        sp.p[pb + m] = I;
+        if (sp.narr == 2) {  // F[ii][nh-1-m] = I
+            const int mf = nh - 1 - m;
+            sp.q[qb + 8LL * nh + 4LL * mf] = I;
+            sp.p[pb + 8LL * sp.nhp + mf] = I;
         }
     }
 }
@@ -2690,20 +2699,25 @@ __global__ void __launch_bounds__(128) k_tridiag_reg(double* __restrict__ fhat, 
                                                      const double* __restrict__ alpha,
                                                      const double* __restrict__ inv, const double* __restrict__ cp,
                                                      int ni, int nmode, TbFix fx) {
-    griddep();
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int mode = blockIdx.x * 4 + warp;
-    if (mode >= nmode) return;
+    const bool act = mode < nmode;
     double* fg = fhat + (long long)mode * ld;
     const long long fo = (long long)mode * 32 * L + lane;
     double f[L], al[L], iv[L], c[L];
+    // the Thomas factors are constant tables: loaded before the wait on the predecessor
+#pragma unroll
+    for (int e = 0; e < L; ++e) {
+        al[e] = act ? alpha[fo + 32 * e] : 0.0;
+        iv[e] = act ? inv[fo + 32 * e] : 0.0;
+        c[e] = act ? cp[fo + 32 * e] : 0.0;
+    }
+    griddep();
+    if (!act) return;
 #pragma unroll
     for (int e = 0; e < L; ++e) {
         const int r = lane * L + e;
         f[e] = r < ni ? (fx.bot ? fg[r] + tb_fix(fx, mode, r) : fg[r]) : 0.0;
-        al[e] = alpha[fo + 32 * e];
-        iv[e] = inv[fo + 32 * e];
-        c[e] = cp[fo + 32 * e];
     }
     double A = 1.0, B = 0.0;
 #pragma unroll
@@ -2774,11 +2788,11 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
     long long bi = LLONG_MAX;
     bool bad = false;
     const double sg = (double)nn.sgn;
-    auto emit = [&](long long g, double pp) {
+    auto emit_v = [&](long long g, double pp, double ext, double old) {
         if (psi_out) psi_out[g] = pp;
         if (psi_inout) {
-            const double nv = pp + psi_ext[g];
-            dmax = fmax(dmax, fabs(nv - psi_inout[g]));
+            const double nv = pp + ext;
+            dmax = fmax(dmax, fabs(nv - old));
             psi_inout[g] = nv;
             if (nn.on) {
                 if (!isfinite(nv)) bad = true;
@@ -2786,6 +2800,30 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
             }
         }
     };
+    auto emit = [&](long long g, double pp) {
+        if (psi_inout) emit_v(g, pp, psi_ext[g], psi_inout[g]);
+        else emit_v(g, pp, 0.0, 0.0);
+    };
+    // one FFT per CTA (FPC = 1): the CTA's two rows of psi_ext (an input) and of the old psi (written
+    // by the previous iteration's update, many kernels back) are loaded before the wait on the
+    // predecessor, into registers, so the update does not start with a memory round trip
+    constexpr int kPre = 8;
+    double pe[2][kPre], po[2][kPre];
+    const bool pre = psi_inout != nullptr && FPC == 1 && (int)blockIdx.x < nrb &&
+                     (nh + (int)blockDim.x - 1) / (int)blockDim.x <= kPre;
+    if (pre) {
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int i = 2 * blockIdx.x + h + 1;
+#pragma unroll
+            for (int q = 0; q < kPre; ++q) {
+                const int j = threadIdx.x + q * blockDim.x;
+                const bool ok = i <= ni && j < nh;
+                pe[h][q] = ok ? psi_ext[(long long)i * nh + j] : 0.0;
+                po[h][q] = ok ? psi_inout[(long long)i * nh + j] : 0.0;
+            }
+        }
+    }
     if ((int)blockIdx.x < nrb) {
         const int rbase = 2 * FPC * blockIdx.x;
         for (int k = threadIdx.x; k < M / 2; k += blockDim.x) Ws[k] = __ldg(W + k);
@@ -2810,12 +2848,16 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
         fft_stockham(a2 + 2 * f * M, a2 + 2 * f * M + M, M, log2m, Ws, lt, TPF);
         const int ro = (fft_stages(log2m) & 1) ? M : 0;
         const double sc = 2.0 / (double)(n + 1);
-        for (int g = 0; g < FPC; ++g) {
-            const double2* res = a2 + 2 * g * M + ro;
+        if (pre) {
+            const double2* res = a2 + ro;
+#pragma unroll
             for (int h = 0; h < 2; ++h) {
-                const int i = rbase + 2 * g + h + 1;
+                const int i = rbase + h + 1;
                 if (i > ni) break;
-                for (int j = threadIdx.x; j < nh; j += blockDim.x) {
+#pragma unroll
+                for (int q = 0; q < kPre; ++q) {
+                    const int j = threadIdx.x + q * blockDim.x;
+                    if (j >= nh) break;
                     double pp;
                     if (j == 0) pp = psib[2 * nh + (i - 1)];
                     else if (j == nh - 1) pp = psib[2 * nh + (nw - 2) + (i - 1)];
@@ -2823,7 +2865,25 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
                         const double2 z = res[j];
                         pp = sc * (h == 0 ? -0.5 * z.y : 0.5 * z.x);
                     }
-                    emit((long long)i * nh + j, pp);
+                    emit_v((long long)i * nh + j, pp, pe[h][q], po[h][q]);
+                }
+            }
+        } else {
+            for (int g = 0; g < FPC; ++g) {
+                const double2* res = a2 + 2 * g * M + ro;
+                for (int h = 0; h < 2; ++h) {
+                    const int i = rbase + 2 * g + h + 1;
+                    if (i > ni) break;
+                    for (int j = threadIdx.x; j < nh; j += blockDim.x) {
+                        double pp;
+                        if (j == 0) pp = psib[2 * nh + (i - 1)];
+                        else if (j == nh - 1) pp = psib[2 * nh + (nw - 2) + (i - 1)];
+                        else {
+                            const double2 z = res[j];
+                            pp = sc * (h == 0 ? -0.5 * z.y : 0.5 * z.x);
+                        }
+                        emit((long long)i * nh + j, pp);
+                    }
                 }
             }
         }
@@ -2882,7 +2942,10 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
 
 static void solve_shape(const Ctx& c, int& fpc, int& threads, size_t& smem) {
     const int M = c.fft_m;
-    fpc = (sizeof(double2) * (size_t)(4 * M + M / 2) <= 160 * 1024) ? 2 : 1;
+    // one FFT (two rows) per CTA: twice the CTAs of the two-FFT shape, so twice the loads in flight
+    // and half the rows per CTA on the latency-bound solve (EFIT_SOLVE_FPC=2 restores it)
+    static const int want = getenv("EFIT_SOLVE_FPC") ? atoi(getenv("EFIT_SOLVE_FPC")) : 1;
+    fpc = (want >= 2 && sizeof(double2) * (size_t)(4 * M + M / 2) <= 160 * 1024) ? 2 : 1;
     int tpf = M / 4;
     if (tpf > 256) tpf = 256;
     if (tpf < 32) tpf = 32;
