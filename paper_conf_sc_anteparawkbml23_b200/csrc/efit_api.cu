@@ -340,7 +340,6 @@ static size_t carve(Ctx& c, char* base) {
     c.symp = c.sym ? (double*)take(sizeof(double) * 16 * (size_t)c.sym_nblk * c.nhp) : nullptr;
     c.sym_part = c.sym ? (double*)take(sizeof(double) * 2 * (size_t)(c.ni > 0 ? c.ni : 1) * c.sym_nblk * c.t.sym_nmc)
                        : nullptr;
-    c.sym_cnt = c.sym ? (unsigned*)take(sizeof(unsigned) * (size_t)c.sym_nblk) : nullptr;
     c.Tedge = (double*)take(sizeof(double) * 2 * (size_t)c.S);
     c.Gd = (double*)take(sizeof(double) * (size_t)(nrows > 0 ? nrows : 1) * c.S);
     c.inlim = (uint8_t*)take((size_t)n);
@@ -431,8 +430,7 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
         delete h;
         return cuda_fail(nullptr, e, "geometry upload");
     }
-    if ((c.sym_cnt && (e = cudaMemsetAsync(c.sym_cnt, 0, sizeof(unsigned) * (size_t)c.sym_nblk, s))) ||
-        (e = efit::prepare_kernels(c)) || (e = efit::launch_init_tables(c, s)) || (e = cudaStreamSynchronize(s))) {
+    if ((e = efit::prepare_kernels(c)) || (e = efit::launch_init_tables(c, s)) || (e = cudaStreamSynchronize(s))) {
         delete h;
         return cuda_fail(nullptr, e, "table build");
     }

@@ -78,7 +78,6 @@ struct Ctx {
     double* symp;       // [sym_nblk][2 (I,F)][8][nhp]             per-iteration block rows, 16-B aligned rows
     int nhp;            // nh rounded up to even (16-byte rows)
     double* sym_edge;   // [2][nw-2] SYM: edge-row source sums of the top/bottom targets (per iteration)
-    unsigned* sym_cnt;  // [sym_nblk] SYM fused finish: CTAs done per 8-row block (zero between launches)
     double* Tedge;      // [2][S]           slabs i = 0 and i = nw-1 (left/right)
     double* Gd;         // [m_hi-m_lo][S]   diagnostic Green's rows
     uint8_t* inlim;     // [nw*nh]

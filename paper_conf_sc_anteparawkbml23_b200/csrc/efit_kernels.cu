@@ -1946,66 +1946,11 @@ __global__ void __launch_bounds__(256) k_bnd_tb_otf(int row_lo, int nslab, int n
 #ifndef EFIT_SYM_MINB
 #define EFIT_SYM_MINB 0
 #endif
-// Fused finish (one GPU, no exchange): a per-block counter counts the CTAs that have written slots
-// of the targets of 8-row block B (nmc x nblk of them: the tiles (B, Q) and (P, B)); the CTA that
-// completes block B reduces its 16 targets exactly as k_bnd_reduce + k_sym_edge_src would (same
-// lane-strided sums and butterflies, so the same bits) and writes them to psi_b -- the separate
-// reduce launch and the edge-source kernel drop out of the iteration.
-struct SymFinish {
-    int on;
-    unsigned* cnt;       // [nblk], zero between launches (reset by the completing CTA)
-    unsigned target;     // nmc * nblk
-    const double* Tedge;
-    long long S;
-    const double* pc;
-    const double* pf;
-    double* tb;          // psi_b + 2 nh: bottom | top entries
-    int nw;
-};
-
-// The completing CTA's reduction (out of line: keeps the streaming loop's register allocation).
-__device__ __noinline__ void sym_finish(const SymFinish& fin, const double* part, int P, int Q, bool diag, int ni,
-                                        int nh, int nslot) {
-    __shared__ int s_last[2];
-    const int t = threadIdx.x, warp = t >> 5, lane = t & 31, nwarp = blockDim.x >> 5;
-    __threadfence();
-    __syncthreads();
-    if (t == 0) {
-        s_last[0] = atomicAdd(fin.cnt + P, 1u) == fin.target - 1u;
-        s_last[1] = !diag && atomicAdd(fin.cnt + Q, 1u) == fin.target - 1u;
-    }
-    __syncthreads();
-    const int nw = fin.nw;
-    for (int e = 0; e < 2; ++e) {
-        if (!s_last[e]) continue;
-        const int B = e == 0 ? P : Q;
-        __threadfence();
-        for (int tg = warp; tg < 16; tg += nwarp) {  // target (row 8B + tg/2, side tg&1)
-            const int r = 8 * B + (tg >> 1), side = tg & 1;
-            if (r >= ni) continue;
-            const int i = r + 1;
-            const double* x0 = side ? fin.pf : fin.pc;
-            const double* x1 = x0 + (long long)(nw - 1) * nh;
-            const double* t0 = fin.Tedge + (long long)i * nh;
-            const double* t1 = t0 + fin.S;
-            double ed = 0.0;
-            for (int m = lane; m < nh; m += 32) ed = fma(t0[m], x0[m], fma(t1[m], x1[m], ed));
-            ed = warp_sum(ed);
-            double sm = lane == 0 ? ed : 0.0;
-            const double* src = part + ((long long)r * 2 + side) * nslot;
-            for (int c = lane; c < nslot; c += 32) sm += __ldcg(src + c);
-            sm = warp_sum(sm);
-            if (lane == 0) fin.tb[side * (nw - 2) + r] = sm;
-        }
-        if (t == 0) fin.cnt[B] = 0u;
-    }
-}
-
 template <bool OTF, bool MIRROR, int UNR, int NBUF, int WG>
 __global__ void __launch_bounds__(128 * WG, EFIT_SYM_MINB ? EFIT_SYM_MINB : (WG == 1 ? 3 : (WG == 2 ? 2 : 1)))
     k_bnd_sym(const double* __restrict__ U, long long tile_lo, int ni, int nh, int nmc, int mc,
               const double* __restrict__ symq, const double* __restrict__ symp, int nhp, int nslot,
-              double* __restrict__ part, double rmin, double dr, double dz, SymFinish fin) {
+              double* __restrict__ part, double rmin, double dr, double dz) {
     extern __shared__ __align__(16) double xs[];
     __shared__ double red[4 * WG][16];
     __shared__ double rrow[4 * WG][4];
@@ -2198,7 +2143,6 @@ __global__ void __launch_bounds__(128 * WG, EFIT_SYM_MINB ? EFIT_SYM_MINB : (WG 
         for (int w = 0; w < 4 * WG; ++w) v += red[w][i];
         if (rq < ni) part[((long long)rq * 2 + side) * nslot + P * nmc + mch] = v;
     }
-    if (fin.on) sym_finish(fin, part, P, Q, diag, ni, nh, nslot);
 }
 
 static size_t sym_smem(const Ctx& c) {
@@ -2282,13 +2226,6 @@ static cudaError_t launch_lr(Ctx& c, cudaStream_t s, bool prepare) {
 
 cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cudaStream_t s, int with_bnd);
 
-// SYM, one GPU without exchange, FFT left/right path: k_bnd_sym finishes psi_b itself (SymFinish)
-static bool sym_fused(const Ctx& c, int xmode) {
-    static const bool off = getenv("EFIT_SYM_NOFUSE") != nullptr;
-    return c.sym && xmode == XCH_NONE && !c.lr_direct && c.sym_cnt && !off && c.sym_tile_lo == 0 &&
-           c.sym_tile_hi == c.sym_ntile;
-}
-
 cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s, bool overlap_solve,
                             bool prepacked, int xmode, double* xbuf) {
     cudaError_t e;
@@ -2307,7 +2244,7 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
         // left/right FFT chain has written psi_b(left/right), so its forward DST also runs under the
         // HBM-bound stream; k_tridiag adds the bottom/top terms in the sine domain afterwards
         if (overlap_solve && (e = launch_solve_fwd(c, pcurr, psib, c.side, 2))) return e;
-        if (c.sym && c.sym_edge && !sym_fused(c, xmode) &&
+        if (c.sym && c.sym_edge &&
             (e = launch_pdl(k_sym_edge_src, dim3((2 * (c.nw - 2) + 7) / 8), dim3(256), 0, c.side, (const double*)c.Tedge,
                             c.S, (const double*)c.pcurr, (const double*)c.pflip, c.nw, c.nh, c.sym_edge)))
             return e;
@@ -2336,13 +2273,10 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
                 const bool mir = c.t.sym_nmc == 1;
                 const dim3 grid((unsigned)(ntl * c.t.sym_nmc));
                 const int nslot = c.sym_nblk * c.t.sym_nmc;
-                SymFinish fin{0, c.sym_cnt, (unsigned)(c.t.sym_nmc * c.sym_nblk), c.Tedge, c.S, c.pcurr, c.pflip,
-                              psib + 2 * c.nh, c.nw};
-                fin.on = sym_fused(c, xmode) ? 1 : 0;
 #define EFIT_SYM_LAUNCH(OTFV, MIRV, UNRV, NBV, WGV)                                                                      \
     launch_pdl(k_bnd_sym<OTFV, MIRV, UNRV, NBV, WGV>, grid, dim3(128 * WGV), smem, s, (const double*)c.U, c.sym_tile_lo,  \
                c.ni, c.nh, c.t.sym_nmc, c.t.sym_mc, (const double*)c.symq, (const double*)c.symp, c.nhp, nslot,       \
-               sym_out, c.rmin, c.dr, c.dz, fin)
+               sym_out, c.rmin, c.dr, c.dz)
                 if (c.otf) {  // FP64-bound: a short unroll keeps the inlined AGM in registers
                     if (mir) EFIT_SYM_LAUNCH(true, true, 1, 2, kSymWg); else EFIT_SYM_LAUNCH(true, false, 1, 2, kSymWg);
                 } else if (mir) {
@@ -2383,9 +2317,7 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
     // finish: left/right entries come from the partials (direct path) or were written by k_lr_ifft;
     // top/bottom from the (exchanged) SYM slots + edge-row sources, or the table chunk partials
     BndOut o{c.lr_direct ? psib : nullptr, nullptr, 1, c.nw - 1, 0};
-    if (sym_fused(c, xmode)) {
-        // top/bottom entries written by k_bnd_sym's completing CTAs; left/right by k_lr_ifft
-    } else if (c.sym) {
+    if (c.sym) {
         sy.part = xmode == XCH_FINISH ? xbuf : c.sym_part;
         sy.edge = c.sym_edge;
         sy.nslot = c.sym_nblk * c.t.sym_nmc;
