@@ -34,7 +34,7 @@ import numpy as np  # noqa: E402
 import synth  # noqa: E402
 
 METRIC = "fit iterations/s and response+boundary GB/s vs B200 HBM peak at 1/2/4/8 GPUs"
-MODES = {"table": 0, "otf": 1, "sym": 2, "otf-sym": 3}  # EFIT_GREEN_* (include/efit.h)
+MODES = {"table": 0, "otf": 1, "sym": 2, "otf-sym": 3, "vh": 4}  # EFIT_GREEN_* (include/efit.h)
 UNIT = "fit iterations/s"
 
 
@@ -49,7 +49,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--mode", default="sym", choices=list(MODES),
                     help="Green's mode of the top/bottom nest (include/efit.h): table = full table "
-                         "(the paper's gridpc), sym = half table by reciprocity, otf / otf-sym = recomputed")
+                         "(the paper's gridpc), sym = half table by reciprocity, otf / otf-sym = recomputed, "
+                         "vh = von Hagenow boundary (no O(N^3) nest; changes the method, SURVEY 8(f) f2)")
     ap.add_argument("--slices", type=int, default=1,
                     help="time slices per fit step (efit_batch_attach; SURVEY 8(f) f1): S slices share one "
                          "pass over the top/bottom Green's table; value = slice fit iterations/s")
@@ -449,6 +450,10 @@ def gpu_arm(args, rank, world, local):
         tb_kernel = "k_bnd_tb"
     if args.mode in ("otf", "otf-sym"):
         tb_bytes = 16.0 * N * N  # no table: only the current pair is read
+    if args.mode == "vh":
+        ne = ctx.n_edge
+        tb_bytes = 8.0 * ne * ne  # the boundary operator, streamed once (+ two O(N^2 log N) solves)
+        tb_kernel = "k_vh_apply (+ zero-Dirichlet solve)"
     gd_bytes = 8.0 * (ctx.info.resp_row_hi - ctx.info.resp_row_lo) * N * N
     if prof is None:
         tb_ms, rb_ms, breakdown = float("nan"), None, {}
@@ -457,6 +462,9 @@ def gpu_arm(args, rank, world, local):
         # the left/right chain (bnd_lr) runs concurrently with the top/bottom stream (both from the fork)
         rb_ms = (prof["response"] + max(prof["bnd_tb"], prof["bnd_lr"])) / nrec
         breakdown = {k: round(v / nrec * 1e3, 3) for k, v in prof.items()}  # us per step
+    if args.mode == "vh" and prof is not None:
+        # no table stream: the roofline kernel is the response (the one HBM stream left)
+        tb_bytes, tb_kernel, tb_ms = gd_bytes, "k_response", prof["response"] / nrec
     tb_gbs = tb_bytes / (tb_ms * 1e-3) / 1e9
     traffic, traffic_src = None, None
     ncu_sum = os.path.join(ROOT, "profiles", "ncu_summary.json")

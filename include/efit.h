@@ -133,9 +133,19 @@ typedef struct {
  *                            Results equal TABLE to rounding (<= 1e-14 relative), not bit for bit.
  *   EFIT_GREEN_ONTHEFLY_SYM  the SYM decomposition with G recomputed (half the Green's evaluations
  *                            of ONTHEFLY); bitwise equal to EFIT_GREEN_TABLE_SYM.
+ *   EFIT_GREEN_VONHAGENOW    no O(N^3) nest at all (the paper's call for "new algorithms that
+ *                            are more suitable for GPUs"): psi0 = the interior solve of the current
+ *                            with ZERO edge values, then by Green's second identity
+ *                            psi_b(p) = -(1/mu0) sum_q G~(x_p; x_q) W_q (1/R_q) dpsi0/dn_q over the edge nodes
+ *                            (second-order one-sided normal derivative, trapezoid weights W = dZ or dR, the
+ *                            log singularity of G integrated exactly on p's own side; reading R3):
+ *                            O(N^2 log N) + an n_edge x n_edge operator table.  Approximates the Green's sum
+ *                            to second order in the grid spacing (~1e-5 relative at 513^2), so results are
+ *                            NOT those of the table modes; world == 1 only.
  * SYM modes with world > 1: the row-pair tiles are sharded; the exchange slice holds the per-tile
  * partial sums (every slot written by one rank), reduced in a fixed order after the exchange. */
-enum { EFIT_GREEN_TABLE = 0, EFIT_GREEN_ONTHEFLY = 1, EFIT_GREEN_TABLE_SYM = 2, EFIT_GREEN_ONTHEFLY_SYM = 3 };
+enum { EFIT_GREEN_TABLE = 0, EFIT_GREEN_ONTHEFLY = 1, EFIT_GREEN_TABLE_SYM = 2, EFIT_GREEN_ONTHEFLY_SYM = 3,
+       EFIT_GREEN_VONHAGENOW = 4 };
 
 enum {
     EFIT_OK = 0,

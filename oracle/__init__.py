@@ -56,6 +56,7 @@ def lib():
                               i, _dp, _dp, i, _dp, _dp, _dp, i, _dp, _dp, i, _dp, _dp, i]),
             "or_destroy": (None, [p]),
             "or_set_self_scale": (None, [p, d]),
+            "or_set_boundary_method": (None, [p, i]),
             "or_set_threads": (None, [i]), "or_get_threads": (i, []),
             "or_get_inlim": (None, [p, _u8p]),
             "or_green_node": (d, [p, i, i, i, i]),
@@ -73,6 +74,7 @@ def lib():
             "or_boundary": (None, [p, _dp, _dp]),
             "or_boundary_targets": (None, [p, _dp, i, _ip, _dp]),
             "or_pflux_literal": (None, [p, _dp, _dp]),
+            "or_boundary_vh": (None, [p, _dp, _dp]),
             "or_apply_gs": (None, [p, _dp, _dp]),
             "or_interior_solve": (None, [p, _dp, _dp, _dp]),
             "or_fit_step": (i, [p, _dp, _dp, _dp, _dp, _dp, _dp, _dp]),
@@ -200,6 +202,10 @@ class Oracle:
         lib().or_get_Gd(self.ptr, _d(out))
         return out
 
+    def set_boundary_method(self, m: int) -> None:
+        """fit_step's boundary flux: 0 = the Green's sum (O12), 1 = von Hagenow (f2)."""
+        lib().or_set_boundary_method(self.ptr, int(m))
+
     def set_self_scale(self, s: float) -> None:
         lib().or_set_self_scale(self.ptr, s)
 
@@ -258,6 +264,13 @@ class Oracle:
         t = np.ascontiguousarray(np.asarray(targets, dtype=np.int32))
         out = np.zeros(len(t))
         lib().or_boundary_targets(self.ptr, _d(I), len(t), t.ctypes.data_as(_ip), _d(out))
+        return out
+
+    def boundary_vh(self, I):
+        """f2: von Hagenow-type boundary flux (zero-Dirichlet solve + boundary Green's operator)."""
+        I = _f64(I)
+        out = np.zeros(self.n_edge)
+        lib().or_boundary_vh(self.ptr, _d(I), _d(out))
         return out
 
     def pflux_literal(self, pcurr):

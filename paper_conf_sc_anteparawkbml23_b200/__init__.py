@@ -22,7 +22,7 @@ __all__ = [
     "efit_solve_update", "efit_profile_begin", "efit_profile_end", "efit_fit_steps",
     "efit_table", "efit_shard", "efit_destroy", "efit_strerror", "efit_last_error", "efit_version",
     "EfitContext", "EFIT_GREEN_TABLE", "EFIT_GREEN_ONTHEFLY", "EFIT_GREEN_TABLE_SYM",
-    "EFIT_GREEN_ONTHEFLY_SYM", "efit_plan_info", "owned_targets", "exchange",
+    "EFIT_GREEN_ONTHEFLY_SYM", "EFIT_GREEN_VONHAGENOW", "efit_plan_info", "owned_targets", "exchange",
     "efit_batch_workspace_bytes", "efit_batch_attach", "efit_fit_step_batch", "efit_fit_steps_batch",
     "efit_boundary_flux_batch", "efit_boundary_basis", "efit_boundary_partials", "efit_boundary_finish",
     "efit_nccl_unique_id", "efit_fit_host",
@@ -36,6 +36,7 @@ EFIT_GREEN_TABLE = 0
 EFIT_GREEN_ONTHEFLY = 1
 EFIT_GREEN_TABLE_SYM = 2       # half table by reciprocity (include/efit.h)
 EFIT_GREEN_ONTHEFLY_SYM = 3
+EFIT_GREEN_VONHAGENOW = 4      # boundary flux by the von Hagenow construction (no O(N^3) nest)
 EFIT_OK, EFIT_E_INVAL, EFIT_E_NOMEM, EFIT_E_CUDA, EFIT_E_NCCL = 0, -1, -2, -3, -4
 EFIT_E_SINGULAR, EFIT_E_NOPLASMA, EFIT_E_NONFINITE, EFIT_E_STATE = -5, -6, -7, -8
 

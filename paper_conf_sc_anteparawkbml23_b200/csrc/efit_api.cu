@@ -168,8 +168,12 @@ static int validate(const efit_grid* g, const efit_basis* b, const efit_geometry
     for (int m = 0; m < geo->n_int; ++m) if (!(geo->int_r[m] > 0)) return fail(nullptr, EFIT_E_INVAL, "internal point R <= 0");
     if (geo->ip_sign != 1 && geo->ip_sign != -1) return fail(nullptr, EFIT_E_INVAL, "ip_sign must be +1 or -1");
     if (mode != EFIT_GREEN_TABLE && mode != EFIT_GREEN_ONTHEFLY && mode != EFIT_GREEN_TABLE_SYM &&
-        mode != EFIT_GREEN_ONTHEFLY_SYM)
+        mode != EFIT_GREEN_ONTHEFLY_SYM && mode != EFIT_GREEN_VONHAGENOW)
         return fail(nullptr, EFIT_E_INVAL, "mode %d", mode);
+    if (mode == EFIT_GREEN_VONHAGENOW && d && d->world > 1)
+        return fail(nullptr, EFIT_E_INVAL, "EFIT_GREEN_VONHAGENOW runs on one GPU (world == 1)");
+    if (mode == EFIT_GREEN_VONHAGENOW && (g->nw < 4 || g->nh < 4))
+        return fail(nullptr, EFIT_E_INVAL, "EFIT_GREEN_VONHAGENOW needs nw, nh >= 4");
     if (d && (d->world < 1 || d->rank < 0 || d->rank >= d->world))
         return fail(nullptr, EFIT_E_INVAL, "rank %d / world %d", d->rank, d->world);
     return EFIT_OK;
@@ -191,6 +195,7 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
     c.mode = mode;
     c.sym = mode == EFIT_GREEN_TABLE_SYM || mode == EFIT_GREEN_ONTHEFLY_SYM;
     c.otf = mode == EFIT_GREEN_ONTHEFLY || mode == EFIT_GREEN_ONTHEFLY_SYM;
+    c.vh = mode == EFIT_GREEN_VONHAGENOW;
     c.rank = d ? d->rank : 0;
     c.world = d ? d->world : 1;
     c.n_edge = 2 * c.nh + 2 * (c.nw - 2);
@@ -317,6 +322,9 @@ static size_t carve_scratch(Ctx& c, Take& take, size_t& off, bool batch) {
     c.psip = (double*)take(sizeof(double) * (size_t)n);
     c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 2));
     c.sym_edge = c.sym ? (double*)take(sizeof(double) * 2 * (size_t)(c.nw > 2 ? c.nw - 2 : 1)) : nullptr;
+    c.vh_psi0 = c.vh ? (double*)take(sizeof(double) * (size_t)n) : nullptr;
+    c.vh_src = c.vh ? (double*)take(sizeof(double) * c.n_edge) : nullptr;
+    c.zero_edge = c.vh ? (double*)take(sizeof(double) * c.n_edge) : nullptr;
     return (size_t)round_up((long long)off, 256);
 }
 
@@ -341,6 +349,7 @@ static size_t carve(Ctx& c, char* base) {
     c.sym_part = c.sym ? (double*)take(sizeof(double) * 2 * (size_t)(c.ni > 0 ? c.ni : 1) * c.sym_nblk * c.t.sym_nmc)
                        : nullptr;
     c.Tedge = (double*)take(sizeof(double) * 2 * (size_t)c.S);
+    c.Kvh = c.vh ? (double*)take(sizeof(double) * (size_t)c.n_edge * c.n_edge) : nullptr;
     c.Gd = (double*)take(sizeof(double) * (size_t)(nrows > 0 ? nrows : 1) * c.S);
     c.inlim = (uint8_t*)take((size_t)n);
     c.dgeo = (double*)take(sizeof(double) * 4 * c.ndiag);
@@ -588,6 +597,12 @@ extern "C" int efit_boundary_flux(efit_ctx* h, const double* d_pcurr, double* d_
         return fail(&c, EFIT_E_STATE, "world > 1 without NCCL exchange: use efit_boundary_partials/finish");
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e;
+    if (c.vh) {  // the caller's current into the internal buffer, then the von Hagenow construction
+        if ((e = cudaMemcpyAsync(c.pcurr, d_pcurr, sizeof(double) * (size_t)c.nw * c.nh, cudaMemcpyDeviceToDevice, s)) ||
+            (e = efit::launch_boundary(c, c.pcurr, d_psib, s)))
+            return cuda_fail(&c, e, "boundary (von Hagenow)");
+        return EFIT_OK;
+    }
     if ((e = efit::launch_make_pair(c, d_pcurr, s))) return cuda_fail(&c, e, "pair");
     if ((e = efit::launch_boundary(c, d_pcurr, d_psib, s, false, false, c.comm ? efit::XCH_NCCL : efit::XCH_NONE)))
         return cuda_fail(&c, e, "boundary");
@@ -597,6 +612,7 @@ extern "C" int efit_boundary_flux(efit_ctx* h, const double* d_pcurr, double* d_
 extern "C" int efit_boundary_partials(efit_ctx* h, const double* d_pcurr, double* d_xbuf, efit_stream_t stream) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
     Ctx& c = h->c;
+    if (c.vh) return fail(&c, EFIT_E_STATE, "no exchange slices in EFIT_GREEN_VONHAGENOW mode");
     EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
     EFIT_CHECK_PTR(c, d_xbuf, "d_xbuf");
     cudaStream_t s = (cudaStream_t)stream;
@@ -611,6 +627,7 @@ extern "C" int efit_boundary_finish(efit_ctx* h, const double* d_pcurr, const do
                                     efit_stream_t stream) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
     Ctx& c = h->c;
+    if (c.vh) return fail(&c, EFIT_E_STATE, "no exchange slices in EFIT_GREEN_VONHAGENOW mode");
     EFIT_CHECK_PTR(c, d_pcurr, "d_pcurr");
     EFIT_CHECK_PTR(c, d_xbuf, "d_xbuf");
     EFIT_CHECK_PTR(c, d_psib, "d_psib");
@@ -681,8 +698,17 @@ static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, 
     if (c.comm && (e = xch_allreduce(c, c.resp, nresp, s))) return e;  // replicated response (exact sum)
     mark(c, s, M_RESP);
     if ((e = launch_lsq(c, c.resp, meas, sigma, coef, chi2, s))) return e;
-    if ((e = launch_current(c, psi, coef, c.pcurr, true, s))) return e;
+    if ((e = launch_current(c, psi, coef, c.pcurr, !c.vh, s))) return e;  // + mirrored pair (table modes)
     mark(c, s, M_CUR);
+    if (c.vh) {  // von Hagenow: zero-Dirichlet solve -> boundary operator -> the Dirichlet solve + update
+        if ((e = launch_boundary(c, c.pcurr, c.psib, s))) return e;
+        mark(c, s, M_LR);
+        if ((e = launch_solve(c, c.pcurr, c.psib, nullptr, psi, psi_ext, eps, s, true))) return e;
+        mark(c, s, M_SOLVE);
+        if (c.prof_on && c.prof_rec && !c.prof_capture && c.prof_next < c.prof_slots) ++c.prof_next;
+        c.prof_rec = false;
+        return cudaSuccess;
+    }
     // boundary flux (marks M_TB, M_LR inside); in FFT mode the forward DST (without the bottom/top
     // edge terms) runs on the side stream under k_bnd_tb and the tridiagonal solve adds those terms
     const bool overlap = !c.lr_direct;

@@ -55,6 +55,7 @@ struct Ctx {
     int n_fl, n_mp, n_int, ndiag, n_lim, ip_sign;
     int mode, rank, world;
     bool sym, otf;               // SYM modes (half table by reciprocity); on-the-fly Green's
+    bool vh;                     // EFIT_GREEN_VONHAGENOW: boundary flux by the von Hagenow construction
     int sym_nblk;                // 8-row blocks of the ni interior rows
     long long sym_ntile;         // sym_nblk (sym_nblk + 1) / 2 row-pair tiles (P <= Q)
     long long sym_tile_lo, sym_tile_hi;  // this rank's tiles
@@ -79,6 +80,7 @@ struct Ctx {
     int nhp;            // nh rounded up to even (16-byte rows)
     double* sym_edge;   // [2][nw-2] SYM: edge-row source sums of the top/bottom targets (per iteration)
     double* Tedge;      // [2][S]           slabs i = 0 and i = nw-1 (left/right)
+    double* Kvh;        // [n_edge][n_edge] von Hagenow boundary operator (VH mode; see k_vh_table)
     double* Gd;         // [m_hi-m_lo][S]   diagnostic Green's rows
     uint8_t* inlim;     // [nw*nh]
     double* dgeo;       // [ndiag][4]       r, z, cos(ang), sin(ang); kind in dkind
@@ -118,6 +120,9 @@ struct Ctx {
 
     // multi-GPU exchange (include/efit.h "Multi-GPU"): NCCL communicator owned by the context when
     // efit_dist.nccl_id was given (then every compute call returns replicated outputs)
+    double* vh_psi0;    // [nw*nh]  VH: zero-Dirichlet solve of the current
+    double* vh_src;     // [n_edge] VH: W_q (1/R_q) dpsi0/dn_q at the edge nodes
+    double* zero_edge;  // [n_edge] zeros (the zero-Dirichlet edge values)
     void* comm;         // ncclComm_t or nullptr
     int nccl_err;       // last ncclResult_t != ncclSuccess of xch_allreduce (reported as EFIT_E_NCCL)
 

@@ -340,6 +340,88 @@ __global__ void k_twiddles(double2* __restrict__ w, int M) {
     w[k] = make_double2(c, -s);
 }
 
+// ------------------------------------------------------------ von Hagenow boundary (VH mode)
+// SURVEY 8(f) f2 / P:L370; include/efit.h EFIT_GREEN_VONHAGENOW.  Green's second identity for
+// Delta* = R div(R^-1 grad) with G(x_p, .) (homogeneous inside the box) and psi0 (the interior solve
+// with zero edge values) gives psi_b(x_p) = -(1/mu0) \oint G(x_p; x') (1/R') dpsi0/dn' dl'.
+// Edge position helpers (edge order of include/efit.h; side 0 left, 1 right, 2 bottom, 3 top).
+__device__ __forceinline__ void vh_edge(int p, int nw, int nh, int& i, int& j, int& side) {
+    if (p < nh) { i = 0; j = p; side = 0; }
+    else if (p < 2 * nh) { i = nw - 1; j = p - nh; side = 1; }
+    else if (p < 2 * nh + nw - 2) { i = p - 2 * nh + 1; j = 0; side = 2; }
+    else { i = p - 2 * nh - (nw - 2) + 1; j = nh - 1; side = 3; }
+}
+
+// K[p][q] = -(1/mu0) G~(x_p; x_q): G itself for q off p's side; on p's side the log singularity's
+// point value -ln(rho) replaced by its exact average over q's segment of length W (dZ or dR),
+// coefficient (mu0/2pi) sqrt(R_p R_q); q = p: the segment average (mu0/2pi) R (ln(16 R/W) - 1).
+// Corner sources are unused (psi0 and its tangential derivatives vanish there): K = 0.
+__global__ void k_vh_table(double* __restrict__ K, int nw, int nh, double rmin, double dr, double zmin, double dz) {
+    const int ne = 2 * nh + 2 * (nw - 2);
+    const long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= (long long)ne * ne) return;
+    const int p = (int)(e / ne), q = (int)(e - (long long)p * ne);
+    int i, j, sp, ii, jj, sq;
+    vh_edge(p, nw, nh, i, j, sp);
+    vh_edge(q, nw, nh, ii, jj, sq);
+    double v = 0.0;
+    if (!((ii == 0 || ii == nw - 1) && (jj == 0 || jj == nh - 1))) {
+        const double Rp = grid_coord(rmin, i, dr), Zp = grid_coord(zmin, j, dz);
+        const double Rq = grid_coord(rmin, ii, dr), Zq = grid_coord(zmin, jj, dz);
+        const double w = sq < 2 ? dz : dr;
+        double G;
+        if (p == q) {
+            G = kMu0Over2Pi * Rp * (log(16.0 * Rp / w) - 1.0);
+        } else {
+            G = green_psi(Rp, Zp, Rq, Zq);
+            if (sp == sq) {
+                const double d = sq < 2 ? fabs(Zq - Zp) : fabs(Rq - Rp);
+                const double a = d - 0.5 * w, b = d + 0.5 * w;
+                const double avg = ((b * log(b) - b) - (a * log(a) - a)) / w;
+                G += kMu0Over2Pi * sqrt(Rp * Rq) * (log(d) - avg);
+            }
+        }
+        v = -G / kMu0;
+    }
+    K[e] = v;
+}
+
+// s_q = W_q (1/R_q) dpsi0/dn_q at every edge node (outward normal, second-order one-sided
+// difference with psi0 = 0 on the edge; 0 at the corners).
+__global__ void k_vh_src(const double* __restrict__ psi0, int nw, int nh, double rmin, double dr, double dz,
+                         double* __restrict__ src) {
+    griddep();
+    const int ne = 2 * nh + 2 * (nw - 2);
+    const int q = blockIdx.x * blockDim.x + threadIdx.x;
+    if (q >= ne) return;
+    int i, j, sd;
+    vh_edge(q, nw, nh, i, j, sd);
+    double v = 0.0;
+    if (!((i == 0 || i == nw - 1) && (j == 0 || j == nh - 1))) {
+        double dn, w;
+        if (sd == 0) { dn = -(4.0 * psi0[(long long)1 * nh + j] - psi0[(long long)2 * nh + j]) / (2.0 * dr); w = dz; }
+        else if (sd == 1) { dn = -(4.0 * psi0[(long long)(nw - 2) * nh + j] - psi0[(long long)(nw - 3) * nh + j]) / (2.0 * dr); w = dz; }
+        else if (sd == 2) { dn = -(4.0 * psi0[(long long)i * nh + 1] - psi0[(long long)i * nh + 2]) / (2.0 * dz); w = dr; }
+        else { dn = -(4.0 * psi0[(long long)i * nh + nh - 2] - psi0[(long long)i * nh + nh - 3]) / (2.0 * dz); w = dr; }
+        v = w * dn / grid_coord(rmin, i, dr);
+    }
+    src[q] = v;
+}
+
+// psi_b[p] = sum_q K[p][q] s_q: one warp per target, lane-strided fixed-order sum + butterfly
+// (deterministic); the operator rows stream once per iteration (n_edge^2 doubles, 33.5 MB at 513^2).
+__global__ void __launch_bounds__(256) k_vh_apply(const double* __restrict__ K, const double* __restrict__ src, int ne,
+                                                  double* __restrict__ psib) {
+    griddep();
+    const int p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+    if (p >= ne) return;
+    const double* kr = K + (long long)p * ne;
+    double s = 0.0;
+    for (int q = lane; q < ne; q += 32) s = fma(__ldcs(kr + q), src[q], s);
+    s = warp_sum(s);
+    if (lane == 0) psib[p] = s;
+}
+
 cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
     const int nw = c.nw, nh = c.nh;
     const long long n = (long long)nw * nh;
@@ -378,6 +460,11 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
         k_green_diag<<<sms * 16, bs, 0, s>>>(c.Gd, c.S, c.m_hi - c.m_lo, c.m_lo, c.dgeo, c.dkind, nw, nh,
                                               c.rmin, c.dr, c.zmin, c.dz);
     k_inlim<<<(int)((n + bs - 1) / bs), bs, 0, s>>>(c.inlim, c.lim, c.n_lim, nw, nh, c.rmin, c.dr, c.zmin, c.dz);
+    if (c.vh) {
+        const long long ne2 = (long long)c.n_edge * c.n_edge;
+        k_vh_table<<<(unsigned)((ne2 + bs - 1) / bs), bs, 0, s>>>(c.Kvh, nw, nh, c.rmin, c.dr, c.zmin, c.dz);
+        if ((e = cudaMemsetAsync(c.zero_edge, 0, sizeof(double) * c.n_edge, s))) return e;
+    }
     k_tri_factors<<<(c.nmode + 63) / 64, 64, 0, s>>>(c.tri_a, c.tri_cp, c.tri_inv, c.tri_alpha, c.ni, c.ni_pad,
                                                      c.nmode, c.rmin, c.dr, c.dz);
     k_twiddles<<<(c.fft_m / 2 + 255) / 256, 256, 0, s>>>(c.twiddle, c.fft_m);
@@ -2229,6 +2316,15 @@ cudaError_t launch_solve_fwd(Ctx& c, const double* pcurr, const double* psib, cu
 cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStream_t s, bool overlap_solve,
                             bool prepacked, int xmode, double* xbuf) {
     cudaError_t e;
+    if (c.vh) {  // von Hagenow: zero-Dirichlet solve, normal derivatives, boundary operator
+        if ((e = launch_solve(c, pcurr, c.zero_edge, c.vh_psi0, nullptr, nullptr, nullptr, s))) return e;
+        if ((e = launch_pdl(k_vh_src, dim3((c.n_edge + 255) / 256), dim3(256), 0, s, (const double*)c.vh_psi0, c.nw,
+                            c.nh, c.rmin, c.dr, c.dz, c.vh_src)))
+            return e;
+        mark(c, s, M_TB);
+        return launch_pdl(k_vh_apply, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, (const double*)c.Kvh,
+                          (const double*)c.vh_src, c.n_edge, psib);
+    }
     const bool side_work = xmode != XCH_PARTIALS;  // left/right targets + SYM edge-row sources (replicated)
     const bool tile_work = xmode != XCH_FINISH;    // the rank's share of the top/bottom stream
     if (side_work) {

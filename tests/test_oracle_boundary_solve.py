@@ -260,3 +260,40 @@ def test_eps_definition(oracle_mod, twin33):
     assert abs(eps - 2e-3) < 1e-9 * 2e-3
     _, pa2, pb2, _, _ = orc.normalize(psi)
     assert abs(np.max(np.abs(v)) / abs(pb2 - pa2) - 2e-3) > 1e-6 * 2e-3  # the new psi's scale differs
+
+
+# ------------------------------------------------------------------ f2: von Hagenow boundary flux
+
+def test_vh_boundary_second_order(oracle_mod):
+    """The von Hagenow construction (or_boundary_vh: zero-Dirichlet solve + boundary Green's
+    operator, P:L370 / SURVEY 8(f) f2) approximates the O12 Green's sum (pinned above) to second
+    order in the grid spacing: the error falls ~4x per halving of h.  A sign error, a missing
+    1/R or 1/mu0, a wrong trapezoid weight or a first-order derivative all break the order."""
+    errs = []
+    for n in [17, 33, 65, 129]:
+        cfg = synth.small_config(n)
+        orc = oracle_mod.Oracle.from_config(cfg)
+        R, Z = cfg.grid.r()[:, None], cfg.grid.z()[None, :]
+        J = np.exp(-((R - 1.7) ** 2 + (Z / 1.5) ** 2) / 0.08)
+        I = (J * cfg.grid.dr * cfg.grid.dz).reshape(-1)
+        exact = orc.boundary_targets(I, list(range(orc.n_edge)))
+        vh = orc.boundary_vh(I)
+        errs.append(np.max(np.abs(vh - exact)) / np.max(np.abs(exact)))
+    assert errs[2] < 1e-3, errs
+    for a, b in zip(errs, errs[1:]):
+        assert a / b > 3.3, errs
+
+
+def test_vh_fit_step_is_oracle_fit_step_with_vh_boundary(oracle_mod):
+    """or_fit_step with the von Hagenow boundary differs from the Green's-sum fit step only
+    through psi_b: at the twin's fixed point both give psi_S up to the boundary approximation."""
+    cfg = synth.small_config(65)
+    orc = oracle_mod.Oracle.from_config(cfg)
+    psi_s = synth.solovev_psi(cfg.grid)
+    tw = orc.twin(psi_s, synth.c_true(cfg.basis))
+    orc.set_boundary_method(1)
+    st, psi, coef, chi2, eps = orc.fit_step(psi_s, tw["psi_ext"], tw["y"], tw["sigma"])
+    orc.set_boundary_method(0)
+    assert st == 0
+    d = np.max(np.abs(psi - psi_s)) / np.max(np.abs(psi_s))
+    assert 1e-9 < d < 1e-3
