@@ -323,8 +323,8 @@ static size_t carve_scratch(Ctx& c, Take& take, size_t& off, bool batch) {
     c.eps_part = (double*)take(sizeof(double) * ((c.ni + 1) / 2 + 2));
     c.sym_edge = c.sym ? (double*)take(sizeof(double) * 2 * (size_t)(c.nw > 2 ? c.nw - 2 : 1)) : nullptr;
     c.vh_psi0 = c.vh ? (double*)take(sizeof(double) * (size_t)n) : nullptr;
-    c.vh_src = c.vh ? (double*)take(sizeof(double) * c.n_edge) : nullptr;
-    c.zero_edge = c.vh ? (double*)take(sizeof(double) * c.n_edge) : nullptr;
+    c.vh_src = c.vh ? (double*)take(sizeof(double) * ((c.n_edge + 3) / 4 * 4)) : nullptr;
+    c.zero_edge = c.vh ? (double*)take(sizeof(double) * ((c.n_edge + 3) / 4 * 4)) : nullptr;
     return (size_t)round_up((long long)off, 256);
 }
 
@@ -349,7 +349,7 @@ static size_t carve(Ctx& c, char* base) {
     c.sym_part = c.sym ? (double*)take(sizeof(double) * 2 * (size_t)(c.ni > 0 ? c.ni : 1) * c.sym_nblk * c.t.sym_nmc)
                        : nullptr;
     c.Tedge = (double*)take(sizeof(double) * 2 * (size_t)c.S);
-    c.Kvh = c.vh ? (double*)take(sizeof(double) * (size_t)c.n_edge * c.n_edge) : nullptr;
+    c.Kvh = c.vh ? (double*)take(sizeof(double) * (size_t)c.n_edge * ((c.n_edge + 3) / 4 * 4)) : nullptr;
     c.Gd = (double*)take(sizeof(double) * (size_t)(nrows > 0 ? nrows : 1) * c.S);
     c.inlim = (uint8_t*)take((size_t)n);
     c.dgeo = (double*)take(sizeof(double) * 4 * c.ndiag);

@@ -356,11 +356,13 @@ __device__ __forceinline__ void vh_edge(int p, int nw, int nh, int& i, int& j, i
 // point value -ln(rho) replaced by its exact average over q's segment of length W (dZ or dR),
 // coefficient (mu0/2pi) sqrt(R_p R_q); q = p: the segment average (mu0/2pi) R (ln(16 R/W) - 1).
 // Corner sources are unused (psi0 and its tangential derivatives vanish there): K = 0.
-__global__ void k_vh_table(double* __restrict__ K, int nw, int nh, double rmin, double dr, double zmin, double dz) {
+__global__ void k_vh_table(double* __restrict__ K, int nw, int nh, int ldk, double rmin, double dr, double zmin,
+                           double dz) {
     const int ne = 2 * nh + 2 * (nw - 2);
     const long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-    if (e >= (long long)ne * ne) return;
-    const int p = (int)(e / ne), q = (int)(e - (long long)p * ne);
+    if (e >= (long long)ne * ldk) return;
+    const int p = (int)(e / ldk), q = (int)(e - (long long)p * ldk);
+    if (q >= ne) { K[e] = 0.0; return; }
     int i, j, sp, ii, jj, sq;
     vh_edge(p, nw, nh, i, j, sp);
     vh_edge(q, nw, nh, ii, jj, sq);
@@ -408,16 +410,36 @@ __global__ void k_vh_src(const double* __restrict__ psi0, int nw, int nh, double
     src[q] = v;
 }
 
-// psi_b[p] = sum_q K[p][q] s_q: one warp per target, lane-strided fixed-order sum + butterfly
-// (deterministic); the operator rows stream once per iteration (n_edge^2 doubles, 33.5 MB at 513^2).
+// psi_b[p] = sum_q K[p][q] s_q: one warp per target, 256-bit streaming loads of the operator row
+// (row stride ldk = n_edge rounded up to 4, zero padded), lane-strided fixed-order partial sums +
+// butterfly (deterministic); the operator streams once per iteration (33.5 MB at 513^2).
 __global__ void __launch_bounds__(256) k_vh_apply(const double* __restrict__ K, const double* __restrict__ src, int ne,
-                                                  double* __restrict__ psib) {
-    griddep();
+                                                  int ldk, double* __restrict__ psib) {
     const int p = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+    const double* kr = K + (long long)(p < ne ? p : 0) * ldk;
+    constexpr int kU = 4;
+    d4 kv[kU];
+    const int nv = ldk >> 2;  // 4-double vectors per row
+#pragma unroll
+    for (int u = 0; u < kU; ++u) {  // the operator is a constant table: first loads before the wait
+        const int v = lane + 32 * u;
+        kv[u] = v < nv ? ld256_stream(kr + 4 * v) : d4{0.0, 0.0, 0.0, 0.0};
+    }
+    griddep();
     if (p >= ne) return;
-    const double* kr = K + (long long)p * ne;
     double s = 0.0;
-    for (int q = lane; q < ne; q += 32) s = fma(__ldcs(kr + q), src[q], s);
+    for (int v0 = 0; v0 < nv; v0 += 32 * kU) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int v = v0 + lane + 32 * u;
+            if (v < nv) {
+                const double4 x = *reinterpret_cast<const double4*>(src + 4 * v);
+                s = dot4(kv[u], d4{x.x, x.y, x.z, x.w}, s);
+            }
+            const int vn = v + 32 * kU;
+            kv[u] = vn < nv ? ld256_stream(kr + 4 * vn) : d4{0.0, 0.0, 0.0, 0.0};
+        }
+    }
     s = warp_sum(s);
     if (lane == 0) psib[p] = s;
 }
@@ -461,9 +483,11 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
                                               c.rmin, c.dr, c.zmin, c.dz);
     k_inlim<<<(int)((n + bs - 1) / bs), bs, 0, s>>>(c.inlim, c.lim, c.n_lim, nw, nh, c.rmin, c.dr, c.zmin, c.dz);
     if (c.vh) {
-        const long long ne2 = (long long)c.n_edge * c.n_edge;
-        k_vh_table<<<(unsigned)((ne2 + bs - 1) / bs), bs, 0, s>>>(c.Kvh, nw, nh, c.rmin, c.dr, c.zmin, c.dz);
-        if ((e = cudaMemsetAsync(c.zero_edge, 0, sizeof(double) * c.n_edge, s))) return e;
+        const int ldk = (c.n_edge + 3) / 4 * 4;
+        const long long ne2 = (long long)c.n_edge * ldk;
+        k_vh_table<<<(unsigned)((ne2 + bs - 1) / bs), bs, 0, s>>>(c.Kvh, nw, nh, ldk, c.rmin, c.dr, c.zmin, c.dz);
+        if ((e = cudaMemsetAsync(c.zero_edge, 0, sizeof(double) * ldk, s))) return e;
+        if ((e = cudaMemsetAsync(c.vh_src, 0, sizeof(double) * ldk, s))) return e;
     }
     k_tri_factors<<<(c.nmode + 63) / 64, 64, 0, s>>>(c.tri_a, c.tri_cp, c.tri_inv, c.tri_alpha, c.ni, c.ni_pad,
                                                      c.nmode, c.rmin, c.dr, c.dz);
@@ -2323,7 +2347,7 @@ cudaError_t launch_boundary(Ctx& c, const double* pcurr, double* psib, cudaStrea
             return e;
         mark(c, s, M_TB);
         return launch_pdl(k_vh_apply, dim3((c.n_edge + 7) / 8), dim3(256), 0, s, (const double*)c.Kvh,
-                          (const double*)c.vh_src, c.n_edge, psib);
+                          (const double*)c.vh_src, c.n_edge, (c.n_edge + 3) / 4 * 4, psib);
     }
     const bool side_work = xmode != XCH_PARTIALS;  // left/right targets + SYM edge-row sources (replicated)
     const bool tile_work = xmode != XCH_FINISH;    // the rank's share of the top/bottom stream
