@@ -489,6 +489,10 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
         if ((e = cudaMemsetAsync(c.zero_edge, 0, sizeof(double) * ldk, s))) return e;
         if ((e = cudaMemsetAsync(c.vh_src, 0, sizeof(double) * ldk, s))) return e;
     }
+    // the factor arrays are padded to 32-row multiples: zero padding makes the padded rows inert in
+    // the warp scans of k_tridiag_reg (compute-sanitizer initcheck, profiles/r02_sanitize_*.txt)
+    for (double* f : {c.tri_cp, c.tri_inv, c.tri_alpha})
+        if ((e = cudaMemsetAsync(f, 0, sizeof(double) * (size_t)c.ni_pad * c.nmode, s))) return e;
     k_tri_factors<<<(c.nmode + 63) / 64, 64, 0, s>>>(c.tri_a, c.tri_cp, c.tri_inv, c.tri_alpha, c.ni, c.ni_pad,
                                                      c.nmode, c.rmin, c.dr, c.dz);
     k_twiddles<<<(c.fft_m / 2 + 255) / 256, 256, 0, s>>>(c.twiddle, c.fft_m);
