@@ -796,13 +796,50 @@ __global__ void __launch_bounds__(256, 2) k_response(const double* __restrict__ 
             }
             if (++pos == npos) {  // row block done: reduce and store its MB x NB partials
                 const int row0 = (warp + j * nwarps) * MB;
+                if constexpr (MB * NB <= 32) {
+                    // transpose reduction: V = MB NB sums over the 32 lanes in log2(32) exchange levels
+                    // that halve the values per lane (2^L/2 + ... + 1 + 1 shuffles instead of 5 V)
+                    constexpr int V = MB * NB;
+                    constexpr int P2 = V <= 1 ? 1 : V <= 2 ? 2 : V <= 4 ? 4 : V <= 8 ? 8 : V <= 16 ? 16 : 32;
+                    double v[P2];
 #pragma unroll
-                for (int r = 0; r < MB; ++r) {
+                    for (int i = 0; i < P2; ++i) v[i] = i < V ? acc[i / NB][i % NB] : 0.0;
 #pragma unroll
-                    for (int k = 0; k < NB; ++k) {
-                        const double v = warp_sum(acc[r][k]);
-                        acc[r][k] = 0.0;
-                        if (lane == 0 && row0 + r < nrows) part[((long long)(row0 + r) * NB + k) * gridDim.x + c] = v;
+                    for (int h = P2 / 2, o = 16; h >= 1; h >>= 1, o >>= 1) {
+                        const bool up = (lane & o) != 0;
+#pragma unroll
+                        for (int i = 0; i < h; ++i) {
+                            const double send = up ? v[i] : v[i + h];
+                            const double keep = up ? v[i + h] : v[i];
+                            v[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+                        }
+                    }
+                    // lane l now holds value index sum_b bit(l, 4 - b) 2^(L-1-b) over the levels done;
+                    // finish the sum over the lanes that still share it
+                    constexpr int L = P2 == 1 ? 0 : P2 == 2 ? 1 : P2 == 4 ? 2 : P2 == 8 ? 3 : P2 == 16 ? 4 : 5;
+#pragma unroll
+                    for (int o = 16 >> L; o >= 1; o >>= 1) v[0] += __shfl_xor_sync(0xffffffffu, v[0], o);
+                    int idx = 0;
+#pragma unroll
+                    for (int b = 0; b < L; ++b) idx |= ((lane >> (4 - b)) & 1) << (L - 1 - b);
+                    const bool writer = (lane & ((32 >> L) - 1)) == 0;
+                    if (writer && idx < V) {
+                        const int r = idx / NB, k = idx % NB;
+                        if (row0 + r < nrows) part[((long long)(row0 + r) * NB + k) * gridDim.x + c] = v[0];
+                    }
+#pragma unroll
+                    for (int r = 0; r < MB; ++r)
+#pragma unroll
+                        for (int k = 0; k < NB; ++k) acc[r][k] = 0.0;
+                } else {
+#pragma unroll
+                    for (int r = 0; r < MB; ++r) {
+#pragma unroll
+                        for (int k = 0; k < NB; ++k) {
+                            const double v = warp_sum(acc[r][k]);
+                            acc[r][k] = 0.0;
+                            if (lane == 0 && row0 + r < nrows) part[((long long)(row0 + r) * NB + k) * gridDim.x + c] = v;
+                        }
                     }
                 }
                 pos = 0;
