@@ -536,6 +536,7 @@ __device__ void normalize_finalize(const double* __restrict__ psi, int nw, int n
     }
     __syncthreads();
     const long long gax = si[0];
+    const double sax = sv[0];  // = s psi[gax] (the partials carry s psi; s = +-1: exact both ways)
     __syncthreads();
     double vb = -DBL_MAX;
     long long vi = LLONG_MAX;
@@ -548,8 +549,9 @@ __device__ void normalize_finalize(const double* __restrict__ psi, int nw, int n
     __syncthreads();
     if (threadIdx.x == 0) {
         for (int q = 1; q < nwarp; ++q) argmax_merge(vb, vi, sv[q], si[q]);
-        const double pa = (gax == LLONG_MAX) ? 0.0 : __ldcg(psi + gax);
-        const double pb = (vi == LLONG_MAX) ? 0.0 : bilinear(psi, nw, nh, rmin, dr, zmin, dz, lim[vi], lim[n_lim + vi]);
+        // the merged values themselves (s times the value): no second round trip to memory
+        const double pa = (gax == LLONG_MAX) ? 0.0 : s * sax;
+        const double pb = (vi == LLONG_MAX) ? 0.0 : s * vb;
         axbd[0] = pa;
         axbd[1] = pb;
         if (gax == LLONG_MAX || !(s * (pa - pb) > 0.0)) atomicOr(status, EFIT_ST_NOPLASMA);
