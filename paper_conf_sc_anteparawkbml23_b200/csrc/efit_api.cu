@@ -693,15 +693,11 @@ static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, 
     if (normalize && (e = launch_normalize(c, psi, s))) return e;
     mark(c, s, M_NORM);
     const size_t nresp = (size_t)c.ndiag * c.nb;
-    if (c.comm) {
-        if (c.world > 1 && (e = cudaMemsetAsync(c.resp, 0, sizeof(double) * nresp, s))) return e;
-        if ((e = launch_response(c, psi, c.resp + (size_t)c.m_lo * c.nb, s))) return e;
-        if ((e = xch_allreduce(c, c.resp, nresp, s))) return e;  // replicated response (exact sum)
-        mark(c, s, M_RESP);
-        if ((e = launch_lsq(c, c.resp, meas, sigma, coef, chi2, s))) return e;
-    } else if ((e = launch_response_lsq(c, psi, c.resp, meas, sigma, coef, chi2, s))) {
-        return e;
-    }
+    if (c.comm && c.world > 1 && (e = cudaMemsetAsync(c.resp, 0, sizeof(double) * nresp, s))) return e;
+    if ((e = launch_response(c, psi, c.resp + (size_t)c.m_lo * c.nb, s))) return e;
+    if (c.comm && (e = xch_allreduce(c, c.resp, nresp, s))) return e;  // replicated response (exact sum)
+    mark(c, s, M_RESP);
+    if ((e = launch_lsq(c, c.resp, meas, sigma, coef, chi2, s))) return e;
     if ((e = launch_current(c, psi, coef, c.pcurr, !c.vh, s))) return e;  // + mirrored pair (table modes)
     mark(c, s, M_CUR);
     if (c.vh) {  // von Hagenow: zero-Dirichlet solve -> boundary operator -> the Dirichlet solve + update

@@ -190,9 +190,6 @@ cudaError_t launch_normalize(Ctx& c, const double* psi, cudaStream_t s);
 cudaError_t launch_response(Ctx& c, const double* psi, double* resp_rows, cudaStream_t s);
 cudaError_t launch_lsq(Ctx& c, const double* resp, const double* meas, const double* sigma,
                        double* coef, double* chi2, cudaStream_t s);
-// response + LSQ of the fit step (fused reduction/LSQ kernel where it applies); marks M_RESP itself
-cudaError_t launch_response_lsq(Ctx& c, const double* psi, double* resp, const double* meas, const double* sigma,
-                                double* coef, double* chi2, cudaStream_t s);
 cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double* pcurr,
                            bool pair, cudaStream_t s);
 // Boundary-flux exchange modes (multi-GPU; include/efit.h "Multi-GPU"):

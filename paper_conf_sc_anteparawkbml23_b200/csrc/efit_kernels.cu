@@ -944,54 +944,6 @@ cudaError_t launch_response(Ctx& c, const double* psi, double* resp_rows, cudaSt
     return response_impl(c, psi, resp_rows, s, false);
 }
 
-template <int NB, int RPL>
-__global__ void __launch_bounds__(256) k_resp_reduce_lsq(const double* __restrict__ part, const double* __restrict__ cnt_part,
-                                                         int nchunk, int ncnt, int total, double* __restrict__ out,
-                                                         int* status, const double* __restrict__ meas,
-                                                         const double* __restrict__ sigma, int nd,
-                                                         double* __restrict__ coef, double* __restrict__ chi2,
-                                                         unsigned* ticket);
-
-// Response + least squares of the fit step: the LSQ fused into the response reduction's last CTA where
-// it applies (one GPU without exchange, scalar response kernel, nb <= 6, nd <= 192), else the two calls.
-cudaError_t launch_response_lsq(Ctx& c, const double* psi, double* resp, const double* meas, const double* sigma,
-                                double* coef, double* chi2, cudaStream_t s) {
-    static const bool off = getenv("EFIT_NO_LSQ_FUSE") != nullptr;
-    const bool fuse = !off && !c.comm && !c.resp_mma && c.nb <= 6 && c.ndiag <= 192 && c.m_lo == 0 &&
-                      c.m_hi == c.ndiag;
-    if (!fuse) {
-        cudaError_t e = launch_response(c, psi, resp, s);
-        if (e) return e;
-        mark(c, s, M_RESP);
-        return launch_lsq(c, resp, meas, sigma, coef, chi2, s);
-    }
-    const int nrows = c.ndiag;
-    switch (c.nb) {
-#define EFIT_NB_CASE(V) case V: launch_resp_nb<V>(c, psi, c.resp_part, s, nrows, false); break;
-        EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
-#undef EFIT_NB_CASE
-        default: return cudaErrorInvalidValue;
-    }
-    cudaError_t e = cudaGetLastError();
-    if (e) return e;
-    mark(c, s, M_RESP);  // (the reduction below now belongs to the lsq interval)
-    const int total = nrows * c.nb;
-    const dim3 g((total + 7) / 8), b(256);
-    const int rpl = c.ndiag <= 64 ? 2 : (c.ndiag <= 128 ? 4 : 6);
-#define EFIT_RL(NBV, RPLV)                                                                                           \
-    launch_pdl(k_resp_reduce_lsq<NBV, RPLV>, g, b, 0, s, (const double*)c.resp_part, (const double*)c.resp_cnt,    \
-               c.t.resp_nchunk, c.t.resp_nchunk, total, resp, c.status, meas, sigma, c.ndiag, coef, chi2, c.tickets + 2)
-#define EFIT_RL_NB(NBV) \
-    case NBV: if (rpl == 2) EFIT_RL(NBV, 2); else if (rpl == 4) EFIT_RL(NBV, 4); else EFIT_RL(NBV, 6); break;
-    switch (c.nb) {
-        EFIT_RL_NB(1) EFIT_RL_NB(2) EFIT_RL_NB(3) EFIT_RL_NB(4) EFIT_RL_NB(5) EFIT_RL_NB(6)
-        default: return cudaErrorInvalidValue;
-    }
-#undef EFIT_RL_NB
-#undef EFIT_RL
-    return cudaGetLastError();
-}
-
 // ------------------------------------------------------------ multi-slice response (tensor cores)
 //
 // S time slices' response matrices in one pass over Gd:
@@ -1489,12 +1441,14 @@ __device__ __forceinline__ void lsq_gram_reg(const double (&a)[RPL][NB], double 
         for (int j = 0; j < i; ++j) G[i][j] = G[j][i];
 }
 
-// Warp LSQ, split so that its input-only part can run before a PDL wait (k_lsq_warp) or in every
-// CTA of the response reduction that may turn out to be the last one (k_resp_reduce_lsq).
 template <int NB, int RPL>
-__device__ __forceinline__ void lsq_warp_prefetch(const double* __restrict__ meas, const double* __restrict__ sigma,
-                                                  int nd, double (&bb)[RPL], double (&is)[RPL]) {
-    const int lane = threadIdx.x & 31;
+__global__ void __launch_bounds__(32) k_lsq_warp(const double* __restrict__ resp, const double* __restrict__ meas,
+                                                 const double* __restrict__ sigma, int nd,
+                                                 double* __restrict__ coef, double* __restrict__ chi2, int* status) {
+    const int lane = threadIdx.x;
+    double a[RPL][NB], bb[RPL], is[RPL];
+    // sigma and the measurements are inputs of the step (not produced by a predecessor kernel):
+    // their loads and the reciprocal overlap the wait on the response reduction
 #pragma unroll
     for (int r = 0; r < RPL; ++r) {
         const int m = lane + 32 * r;
@@ -1502,24 +1456,13 @@ __device__ __forceinline__ void lsq_warp_prefetch(const double* __restrict__ mea
         is[r] = ok ? 1.0 / sigma[m] : 0.0;
         bb[r] = ok ? meas[m] * is[r] : 0.0;
     }
-}
-
-// CG: the response was written by other CTAs of the same kernel (L2 loads; status likewise)
-template <int NB, int RPL, bool CG>
-__device__ __forceinline__ void lsq_warp_solve(const double* __restrict__ resp, const double* __restrict__ meas, int nd,
-                                               double (&bb)[RPL], const double (&is)[RPL], double* __restrict__ coef,
-                                               double* __restrict__ chi2, int* status) {
-    const int lane = threadIdx.x & 31;
-    double a[RPL][NB];
+    griddep();
 #pragma unroll
     for (int r = 0; r < RPL; ++r) {
         const int m = lane + 32 * r;
         const bool ok = m < nd;
 #pragma unroll
-        for (int k = 0; k < NB; ++k) {
-            const double* pr = resp + (size_t)m * NB + k;
-            a[r][k] = ok ? (CG ? __ldcg(pr) : *pr) * is[r] : 0.0;
-        }
+        for (int k = 0; k < NB; ++k) a[r][k] = ok ? resp[(size_t)m * NB + k] * is[r] : 0.0;
     }
     double sc[NB];
 #pragma unroll
@@ -1635,10 +1578,7 @@ __device__ __forceinline__ void lsq_warp_solve(const double* __restrict__ resp, 
         if (m < nd) {
             double res = meas[m];
 #pragma unroll
-            for (int k = 0; k < NB; ++k) {
-                const double* pr = resp + (size_t)m * NB + k;
-                res = fma(-(CG ? __ldcg(pr) : *pr), z[k], res);
-            }
+            for (int k = 0; k < NB; ++k) res = fma(-resp[(size_t)m * NB + k], z[k], res);
             res *= is[r];
             cs = fma(res, res, cs);
         }
@@ -1646,65 +1586,11 @@ __device__ __forceinline__ void lsq_warp_solve(const double* __restrict__ resp, 
     cs = warp_sum(cs);
     if (lane == 0) {
         if (!ok) atomicOr(status, EFIT_ST_SINGULAR);
-        const int stv = CG ? __ldcg(status) : *status;
-        const bool bad = (stv & (EFIT_ST_NOPLASMA | EFIT_ST_NONFINITE)) != 0 || !ok;
+        const bool bad = (*status & (EFIT_ST_NOPLASMA | EFIT_ST_NONFINITE)) != 0 || !ok;
         const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
         *chi2 = bad ? nanv : cs;
 #pragma unroll
         for (int k = 0; k < NB; ++k) coef[k] = bad ? nanv : z[k];
-    }
-}
-
-
-template <int NB, int RPL>
-__global__ void __launch_bounds__(32) k_lsq_warp(const double* __restrict__ resp, const double* __restrict__ meas,
-                                                 const double* __restrict__ sigma, int nd,
-                                                 double* __restrict__ coef, double* __restrict__ chi2, int* status) {
-    // sigma and the measurements are inputs of the step (not produced by a predecessor kernel):
-    // their loads and the reciprocal overlap the wait on the response reduction
-    double bb[RPL], is[RPL];
-    lsq_warp_prefetch<NB, RPL>(meas, sigma, nd, bb, is);
-    griddep();
-    lsq_warp_solve<NB, RPL, false>(resp, meas, nd, bb, is, coef, chi2, status);
-}
-
-// The response reduction with the least squares fused into its last CTA (one GPU, no exchange, nb <=
-// 6): every CTA reduces its (row, k) sums exactly as k_resp_reduce, then the CTA that takes the
-// last ticket runs the warp LSQ on the complete response -- one launch and one PDL boundary fewer.
-template <int NB, int RPL>
-__global__ void __launch_bounds__(256) k_resp_reduce_lsq(const double* __restrict__ part, const double* __restrict__ cnt_part,
-                                                         int nchunk, int ncnt, int total, double* __restrict__ out,
-                                                         int* status, const double* __restrict__ meas,
-                                                         const double* __restrict__ sigma, int nd,
-                                                         double* __restrict__ coef, double* __restrict__ chi2,
-                                                         unsigned* ticket) {
-    double bb[RPL], is[RPL];
-    if (threadIdx.x < 32) lsq_warp_prefetch<NB, RPL>(meas, sigma, nd, bb, is);
-    griddep();
-    const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
-    if (w < total) {
-        const double* p = part + (long long)w * nchunk;
-        double s = 0.0;
-        for (int c = lane; c < nchunk; c += 32) s += p[c];
-        s = warp_sum(s);
-        if (lane == 0) out[w] = s;
-    }
-    if (blockIdx.x == 0 && threadIdx.x < 32) {
-        double cnt = 0.0;
-        for (int c = lane; c < ncnt; c += 32) cnt += cnt_part[c];
-        cnt = warp_sum(cnt);
-        if (lane == 0 && cnt == 0.0) atomicOr(status, EFIT_ST_NOPLASMA);
-    }
-    __shared__ bool last;
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) last = atomicAdd(ticket, 1u) == gridDim.x - 1;
-    __syncthreads();
-    if (!last) return;
-    __threadfence();
-    if (threadIdx.x < 32) {
-        lsq_warp_solve<NB, RPL, true>(out, meas, nd, bb, is, coef, chi2, status);
-        if (lane == 0) *ticket = 0u;
     }
 }
 
