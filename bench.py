@@ -60,6 +60,9 @@ def parse():
     ap.add_argument("--no-profile", action="store_true",
                     help="time graph replays without per-kernel events (no roofline breakdown)")
     ap.add_argument("--reps", type=int, default=5, help="timed repetitions of K steps; value = the median")
+    ap.add_argument("--loop", action="store_true",
+                    help="full fitting loop (P:L103, L287) on the noise-free twin from a 1%% perturbed start: "
+                         "iterations to eps < 1e-5, eps trajectory, time to solution, |c - c_true| (SURVEY 8(d) C2)")
     return ap.parse_args()
 
 
@@ -584,6 +587,76 @@ def e2e_measure(ctx, psi0, psi_ext, meas, sigma, K_e2e, torch, dev, use_dist, ch
             "api": "efit_fit_host (pinned host buffers; H2D/D2H on library streams, double-buffered)"}
 
 
+def loop_arm(args, rank, world, local):
+    """--loop: the full fitting loop (iterate until max|dpsi| / |psi_b - psi_a| < 1e-5)
+    on the noise-free twin (edge-vanishing profile, reading R2) from psi_S + 1% smooth
+    modes (seed 5).  One eps read-back per iteration (as a user polling convergence); time to
+    solution by CUDA events.  Then continued to eps < 1e-10: the iterate must be the twin's psi_S
+    with c = c_true (|c - c_true| and |psi - psi_S| reported at both points)."""
+    import torch
+    import paper_conf_sc_anteparawkbml23_b200 as efit
+    if world > 1:
+        raise SystemExit("--loop runs on one GPU")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    cfg = synth.config(args.config)
+    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=MODES[args.mode], device=dev)
+    T = lambda a: torch.tensor(np.asarray(a, dtype=np.float64), device=dev)
+    psi_s = T(synth.solovev_psi(cfg.grid))
+    ct = T(synth.c_true(cfg.basis))
+    I_s = ctx.current(psi_s, ct)
+    psib = ctx.boundary_flux(I_s)
+    ext = (psi_s - ctx.interior_solve(I_s, psib)).contiguous()
+    resp, _ = ctx.response(psi_s)
+    y = (resp @ ct).contiguous()
+    g = cfg.geometry
+    sigma = torch.zeros_like(y)
+    bounds = np.cumsum([0, len(g.fl_r), len(g.mp_r), len(g.int_r)])
+    for a, b in zip(bounds[:-1], bounds[1:]):
+        if b > a:
+            sigma[a:b] = 1e-3 * y[a:b].abs().max()
+    psi0 = T(synth.perturbed_psi(cfg.grid, seed=5, rel=1e-2))
+    coef, chi2, eps = ctx._t(ctx.nbasis), ctx._t(1), ctx._t(1)
+    st = torch.cuda.Stream()
+    span = psi_s.abs().max().item()
+    cmax = ct.abs().max().item()
+
+    def run(tol, cap):
+        psi = psi0.clone()
+        traj = []
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(st)
+        for it in range(cap):
+            ctx.fit_step(psi, ext, y, sigma, coef, chi2, eps, stream=st)
+            e = eps.item()
+            traj.append(e)
+            if e < tol:
+                break
+        b.record(st)
+        torch.cuda.synchronize()
+        return psi, traj, a.elapsed_time(b)
+
+    run(1e-5, 3)  # warm-up (graph capture)
+    psi, traj, ms = run(1e-5, args.steps)
+    out5 = {"iterations": len(traj), "eps": traj[-1], "time_to_solution_ms": round(ms, 3),
+            "ms_per_iteration": round(ms / len(traj), 4),
+            "psi_rel_err_vs_psi_S": (psi - psi_s).abs().max().item() / span,
+            "coef_rel_err_vs_c_true": (coef - ct).abs().max().item() / cmax}
+    psi, traj2, ms2 = run(1e-10, 20 * args.steps)
+    out10 = {"iterations": len(traj2), "eps": traj2[-1],
+             "psi_rel_err_vs_psi_S": (psi - psi_s).abs().max().item() / span,
+             "coef_rel_err_vs_c_true": (coef - ct).abs().max().item() / cmax}
+    st_code = ctx.status()
+    rate = float(np.exp(np.mean(np.log(np.array(traj2[-20:])[1:] / np.array(traj2[-20:])[:-1])))) if len(traj2) > 21 else None
+    print(json.dumps({"metric": "full fitting loop to eps < 1e-5 (P:L103, L287)", "config": {
+        "workload": f"{args.config}: {cfg.description}", "grid": f"{cfg.grid.nw}x{cfg.grid.nh}",
+        "green_mode": args.mode, "start": "psi_S + 1% smooth modes (seed 5)", "twin": "noise-free, edge-vanishing profile"},
+        "status": st_code, "to_1e-5": out5, "to_1e-10": out10, "contraction_rate": rate,
+        "eps_trajectory": [float(f"{e:.3e}") for e in traj]}), flush=True)
+    ctx.close()
+
+
 # ----------------------------------------------------------------------------- CPU oracle
 
 def oracle_setup(config):
@@ -695,6 +768,9 @@ def main():
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE = {world}")
     if args.impl == "reference":
         reference_arm(args, rank, world)
+        return
+    if args.loop:
+        loop_arm(args, rank, world, local)
         return
     if args.slices > 1:
         batch_arm(args, rank, world, local)
