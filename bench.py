@@ -617,7 +617,7 @@ def loop_arm(args, rank, world, local):
             sigma[a:b] = 1e-3 * y[a:b].abs().max()
     psi0 = T(synth.perturbed_psi(cfg.grid, seed=5, rel=1e-2))
     coef, chi2, eps = ctx._t(ctx.nbasis), ctx._t(1), ctx._t(1)
-    st = torch.cuda.Stream()
+    st = torch.cuda.current_stream()  # eps.item() reads on this stream: each read sees its iteration
     span = psi_s.abs().max().item()
     cmax = ct.abs().max().item()
 
