@@ -1594,179 +1594,9 @@ __global__ void __launch_bounds__(32) k_lsq_warp(const double* __restrict__ resp
     }
 }
 
-// Sum of V <= 32 per-thread values over the CTA, result in every thread (fixed order: transpose
-// reduction inside each warp -- log2 levels that halve the values per lane -- then the per-warp
-// totals summed in warp order from shared memory).  `red` holds [nwarps][32] doubles.
-template <int V>
-__device__ __forceinline__ void cta_sum_vec(double (&v)[V], double* red) {
-    static_assert(V >= 1 && V <= 32, "1..32 values");
-    constexpr int P2 = V <= 1 ? 1 : V <= 2 ? 2 : V <= 4 ? 4 : V <= 8 ? 8 : V <= 16 ? 16 : 32;
-    constexpr int L = P2 == 1 ? 0 : P2 == 2 ? 1 : P2 == 4 ? 2 : P2 == 8 ? 3 : P2 == 16 ? 4 : 5;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
-    double w[P2];
-#pragma unroll
-    for (int i = 0; i < P2; ++i) w[i] = i < V ? v[i] : 0.0;
-#pragma unroll
-    for (int h = P2 / 2, o = 16; h >= 1; h >>= 1, o >>= 1) {
-        const bool up = (lane & o) != 0;
-#pragma unroll
-        for (int i = 0; i < h; ++i) {
-            const double send = up ? w[i] : w[i + h];
-            const double keep = up ? w[i + h] : w[i];
-            w[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
-        }
-    }
-#pragma unroll
-    for (int o = 16 >> L; o >= 1; o >>= 1) w[0] += __shfl_xor_sync(0xffffffffu, w[0], o);
-    int idx = 0;
-#pragma unroll
-    for (int b = 0; b < L; ++b) idx |= ((lane >> (4 - b)) & 1) << (L - 1 - b);
-    __syncthreads();  // red may still be read by a previous call
-    if ((lane & ((32 >> L) - 1)) == 0 && idx < V) red[warp * 32 + idx] = w[0];
-    __syncthreads();
-#pragma unroll
-    for (int i = 0; i < V; ++i) {
-        double t = 0.0;
-        for (int q = 0; q < nwarp; ++q) t += red[q * 32 + i];
-        v[i] = t;
-    }
-}
-
-// CholeskyQR2 (+ shifted CholeskyQR3 fallback) with one diagnostic row per thread (nd <= 256): the
-// Gram matrices and Q^T b are CTA transpose reductions, the nb x nb factorisations and triangular
-// solves run redundantly in every thread's registers (no serial single-warp sections).  Same
-// arithmetic definition as k_lsq / k_lsq_warp, another summation order.
-template <int NB>
-__global__ void __launch_bounds__(256) k_lsq_cta(const double* __restrict__ resp, const double* __restrict__ meas,
-                                                 const double* __restrict__ sigma, int nd, double* __restrict__ coef,
-                                                 double* __restrict__ chi2, int* status) {
-    constexpr int NG = NB * (NB + 1) / 2;
-    static_assert(NG + NB <= 32, "Gram + right-hand side in one reduction");
-    __shared__ double red[8 * 32];
-    const int m = threadIdx.x;
-    const bool act = m < nd;
-    // sigma and the measurements are inputs of the step: before the wait on the response
-    const double is = act ? 1.0 / sigma[m] : 0.0;
-    const double ym = act ? meas[m] : 0.0;
-    const double bm = ym * is;
-    griddep();
-    double rr[NB], a[NB];
-#pragma unroll
-    for (int k = 0; k < NB; ++k) {
-        rr[k] = act ? resp[(size_t)m * NB + k] : 0.0;
-        a[k] = rr[k] * is;
-    }
-    double sc[NB];
-#pragma unroll
-    for (int k = 0; k < NB; ++k) sc[k] = a[k] * a[k];
-    cta_sum_vec<NB>(sc, red);
-    bool ok = true;
-#pragma unroll
-    for (int k = 0; k < NB; ++k) {
-        sc[k] = sqrt(sc[k]);
-        ok = ok && (sc[k] > 0.0);
-        a[k] *= sc[k] > 0.0 ? 1.0 / sc[k] : 0.0;
-    }
-    double G[NB][NB], R0[NB][NB], R1[NB][NB], R2[NB][NB], r0i[NB], r1i[NB], r2i[NB];
-    auto gram = [&](double (&g)[NB][NB], double (&z)[NB], bool with_b) {
-        double v[NG + NB];
-        int e = 0;
-#pragma unroll
-        for (int i = 0; i < NB; ++i)
-#pragma unroll
-            for (int j = i; j < NB; ++j) v[e++] = a[i] * a[j];
-#pragma unroll
-        for (int k = 0; k < NB; ++k) v[NG + k] = with_b ? a[k] * bm : 0.0;
-        cta_sum_vec<NG + NB>(v, red);
-        e = 0;
-#pragma unroll
-        for (int i = 0; i < NB; ++i)
-#pragma unroll
-            for (int j = i; j < NB; ++j) { g[i][j] = v[e]; g[j][i] = v[e]; ++e; }
-#pragma unroll
-        for (int k = 0; k < NB; ++k) z[k] = v[NG + k];
-    };
-    auto apply_rinv = [&](const double (&R)[NB][NB], const double (&ri)[NB]) {  // a <- a R^-1
-#pragma unroll
-        for (int j = 0; j < NB; ++j) {
-            double t = a[j];
-#pragma unroll
-            for (int i = 0; i < j; ++i) t = fma(-a[i], R[i][j], t);
-            a[j] = t * ri[j];
-        }
-    };
-    double z[NB];
-    gram(G, z, false);
-    bool ok1 = true;
-    lsq_chol_reg<NB>(G, R1, r1i, ok1);
-    const bool shifted = !ok1 && ok;  // CTA-uniform: cond(A) beyond ~1e8 -> shifted CholeskyQR3
-    if (shifted) {
-        const double shift = 11.0 * ((double)nd * NB + (double)NB * (NB + 1)) * 0x1p-53 * NB;
-#pragma unroll
-        for (int k = 0; k < NB; ++k) G[k][k] += shift;
-        lsq_chol_reg<NB>(G, R0, r0i, ok);
-        apply_rinv(R0, r0i);
-        gram(G, z, false);
-        ok1 = true;
-        lsq_chol_reg<NB>(G, R1, r1i, ok1);
-    }
-    ok = ok && ok1;
-    apply_rinv(R1, r1i);
-    gram(G, z, true);
-    lsq_chol_reg<NB>(G, R2, r2i, ok);
-#pragma unroll
-    for (int j = 0; j < NB; ++j) {  // R2^-T
-        double t = z[j];
-#pragma unroll
-        for (int i = 0; i < j; ++i) t = fma(-R2[i][j], z[i], t);
-        z[j] = t * r2i[j];
-    }
-    auto back = [&](const double (&R)[NB][NB], const double (&ri)[NB]) {
-#pragma unroll
-        for (int k = NB - 1; k >= 0; --k) {
-            double t = z[k];
-#pragma unroll
-            for (int j = k + 1; j < NB; ++j) t = fma(-R[k][j], z[j], t);
-            z[k] = t * ri[k];
-        }
-    };
-    back(R2, r2i);
-    back(R1, r1i);
-    if (shifted) back(R0, r0i);
-    double rmax = 0.0, rmin = DBL_MAX;
-#pragma unroll
-    for (int k = 0; k < NB; ++k) {
-        const double d = fabs(R1[k][k] * R2[k][k] * (shifted ? R0[k][k] : 1.0));
-        rmax = fmax(rmax, d);
-        rmin = fmin(rmin, d);
-        z[k] = z[k] / sc[k];
-    }
-    ok = ok && (rmin >= 1e-13 * rmax);
-    double res = ym;
-#pragma unroll
-    for (int k = 0; k < NB; ++k) res = fma(-rr[k], z[k], res);
-    res *= is;
-    double cs[1] = {res * res};
-    cta_sum_vec<1>(cs, red);
-    if (threadIdx.x == 0) {
-        if (!ok) atomicOr(status, EFIT_ST_SINGULAR);
-        const bool bad = (*status & (EFIT_ST_NOPLASMA | EFIT_ST_NONFINITE)) != 0 || !ok;
-        const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
-        *chi2 = bad ? nanv : cs[0];
-#pragma unroll
-        for (int k = 0; k < NB; ++k) coef[k] = bad ? nanv : z[k];
-    }
-}
-
 template <int NB>
 static bool launch_lsq_warp(int nd, const double* resp, const double* meas, const double* sigma, double* coef,
                             double* chi2, int* status, cudaStream_t s) {
-    static const bool warp_only = getenv("EFIT_LSQ_WARP") != nullptr;  // A/B: the single-warp kernel
-    if (!warp_only && nd <= 256) {
-        const int threads = (nd + 31) / 32 * 32;
-        launch_pdl(k_lsq_cta<NB>, dim3(1), dim3(threads), 0, s, resp, meas, sigma, nd, coef, chi2, status);
-        return true;
-    }
     if (nd <= 64) launch_pdl(k_lsq_warp<NB, 2>, dim3(1), dim3(32), 0, s, resp, meas, sigma, nd, coef, chi2, status);
     else if (nd <= 128) launch_pdl(k_lsq_warp<NB, 4>, dim3(1), dim3(32), 0, s, resp, meas, sigma, nd, coef, chi2, status);
     else if (nd <= 192) launch_pdl(k_lsq_warp<NB, 6>, dim3(1), dim3(32), 0, s, resp, meas, sigma, nd, coef, chi2, status);
