@@ -459,6 +459,8 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
     c.hs = c.ds = nullptr;
     c.hstart = nullptr;
     for (int b = 0; b < 2; ++b) c.hin[b] = c.hdone[b] = c.hfree[b] = nullptr;
+    c.hgexec[0] = c.hgexec[1] = nullptr;
+    c.hkey[0] = c.hkey[1] = nullptr;
     c.prof_on = false;
     c.prof_rec = false;
     c.prof_every = 1;
@@ -788,6 +790,90 @@ extern "C" int efit_fit_steps(efit_ctx* h, int32_t nsteps, double* d_psi, const 
     return fit_steps_impl(h, nsteps, d_psi, d_psi_ext, d_meas, d_sigma, d_coef, d_chi2, d_eps, stream);
 }
 
+// Pipelined host path (efit_fit_host): one graph launch per slice.  Graph b (slot b) = the chained
+// fit of slot b's staging buffers, plus a parallel branch that downloads the previous slice's results
+// from slot b^1 and then uploads the next slice's inputs into it; the branch's 7 copy nodes are
+// re-pointed at the neighbouring slices' host arrays before every launch (and disabled at the ends).
+// Returns EFIT_OK, 1 if the graphs cannot be built for these buffers (caller falls back to the stream
+// pipeline), or an error code.
+static int fit_host_graphs(efit_ctx* h, int32_t nslice, int32_t iters, const double* h_psi0, const double* h_meas,
+                           const double* h_sigma, const double* d_psi_ext, double* h_psi, double* h_coef,
+                           double* h_chi2, double* h_eps, cudaStream_t s) {
+    Ctx& c = h->c;
+    const size_t n = (size_t)c.nw * c.nh, nd = (size_t)c.ndiag, nb = (size_t)c.nb;
+    cudaError_t e;
+    const void* key0 = (const void*)(intptr_t)iters;
+    if (!c.hgexec[0] || c.hkey[0] != key0 || c.hkey[1] != (const void*)d_psi_ext) {
+        for (int b = 0; b < 2; ++b)
+            if (c.hgexec[b]) { cudaGraphExecDestroy(c.hgexec[b]); c.hgexec[b] = nullptr; }
+        for (int b = 0; b < 2; ++b) {
+            Ctx::HostSlot& q = c.hslot[b];
+            Ctx::HostSlot& o = c.hslot[b ^ 1];
+            cudaGraph_t g = nullptr;
+            if ((e = cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal))) return cuda_fail(&c, e, "begin capture");
+            cudaError_t e2 = cudaSuccess;
+            for (int k = 0; k < iters && !e2; ++k)
+                e2 = enqueue_fit_step(c, q.psi, d_psi_ext, q.meas, q.sigma, q.coef, q.chi2, q.eps, s, k == 0);
+            e = cudaStreamEndCapture(s, &g);
+            if (e2 || e) { if (g) cudaGraphDestroy(g); return cuda_fail(&c, e2 ? e2 : e, "host graph capture"); }
+            // the copy branch: D2H of slot b^1 (roots), then H2D into it
+            cudaGraphNode_t* nd7 = c.hnode[b];
+            const bool ok =
+                cudaGraphAddMemcpyNode1D(&nd7[0], g, nullptr, 0, h_psi, o.psi, sizeof(double) * n, cudaMemcpyDeviceToHost) == cudaSuccess &&
+                cudaGraphAddMemcpyNode1D(&nd7[1], g, nullptr, 0, h_coef, o.coef, sizeof(double) * nb, cudaMemcpyDeviceToHost) == cudaSuccess &&
+                cudaGraphAddMemcpyNode1D(&nd7[2], g, nullptr, 0, h_chi2, o.chi2, sizeof(double), cudaMemcpyDeviceToHost) == cudaSuccess &&
+                cudaGraphAddMemcpyNode1D(&nd7[3], g, nullptr, 0, h_eps, o.eps, sizeof(double), cudaMemcpyDeviceToHost) == cudaSuccess &&
+                cudaGraphAddMemcpyNode1D(&nd7[4], g, nd7, 4, o.psi, h_psi0, sizeof(double) * n, cudaMemcpyHostToDevice) == cudaSuccess &&
+                cudaGraphAddMemcpyNode1D(&nd7[5], g, nd7, 4, o.meas, h_meas, sizeof(double) * nd, cudaMemcpyHostToDevice) == cudaSuccess &&
+                cudaGraphAddMemcpyNode1D(&nd7[6], g, nd7, 4, o.sigma, h_sigma, sizeof(double) * nd, cudaMemcpyHostToDevice) == cudaSuccess &&
+                cudaGraphInstantiateWithFlags(&c.hgexec[b], g, 0) == cudaSuccess;
+            cudaGraphDestroy(g);
+            if (!ok) {
+                cudaGetLastError();
+                for (int q2 = 0; q2 < 2; ++q2)
+                    if (c.hgexec[q2]) { cudaGraphExecDestroy(c.hgexec[q2]); c.hgexec[q2] = nullptr; }
+                return 1;
+            }
+        }
+        c.hkey[0] = key0;
+        c.hkey[1] = (const void*)d_psi_ext;
+    }
+    // slice 0's inputs into slot 0
+    Ctx::HostSlot& q0 = c.hslot[0];
+    if ((e = cudaMemcpyAsync(q0.psi, h_psi0, sizeof(double) * n, cudaMemcpyHostToDevice, s)) ||
+        (e = cudaMemcpyAsync(q0.meas, h_meas, sizeof(double) * nd, cudaMemcpyHostToDevice, s)) ||
+        (e = cudaMemcpyAsync(q0.sigma, h_sigma, sizeof(double) * nd, cudaMemcpyHostToDevice, s)))
+        return cuda_fail(&c, e, "H2D");
+    for (int k = 0; k < nslice; ++k) {
+        const int b = k & 1;
+        Ctx::HostSlot& o = c.hslot[b ^ 1];
+        cudaGraphExec_t x = c.hgexec[b];
+        cudaGraphNode_t* nd7 = c.hnode[b];
+        const bool dn = k >= 1, up = k + 1 < nslice;
+        const size_t kp = dn ? (size_t)(k - 1) : 0, kn = up ? (size_t)(k + 1) : 0;
+        if ((e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[0], h_psi + kp * n, o.psi, sizeof(double) * n, cudaMemcpyDeviceToHost)) ||
+            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[1], h_coef + kp * nb, o.coef, sizeof(double) * nb, cudaMemcpyDeviceToHost)) ||
+            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[2], h_chi2 + kp, o.chi2, sizeof(double), cudaMemcpyDeviceToHost)) ||
+            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[3], h_eps + kp, o.eps, sizeof(double), cudaMemcpyDeviceToHost)) ||
+            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[4], o.psi, h_psi0 + kn * n, sizeof(double) * n, cudaMemcpyHostToDevice)) ||
+            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[5], o.meas, h_meas + kn * nd, sizeof(double) * nd, cudaMemcpyHostToDevice)) ||
+            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[6], o.sigma, h_sigma + kn * nd, sizeof(double) * nd, cudaMemcpyHostToDevice)))
+            return cuda_fail(&c, e, "host graph update");
+        for (int q = 0; q < 7; ++q)
+            if ((e = cudaGraphNodeSetEnabled(x, nd7[q], q < 4 ? dn : up))) return cuda_fail(&c, e, "host graph update");
+        if ((e = cudaGraphLaunch(x, s))) return cuda_fail(&c, e, "host graph launch");
+    }
+    // the last slice's results
+    const size_t kl = (size_t)(nslice - 1);
+    Ctx::HostSlot& ql = c.hslot[(nslice - 1) & 1];
+    if ((e = cudaMemcpyAsync(h_psi + kl * n, ql.psi, sizeof(double) * n, cudaMemcpyDeviceToHost, s)) ||
+        (e = cudaMemcpyAsync(h_coef + kl * nb, ql.coef, sizeof(double) * nb, cudaMemcpyDeviceToHost, s)) ||
+        (e = cudaMemcpyAsync(h_chi2 + kl, ql.chi2, sizeof(double), cudaMemcpyDeviceToHost, s)) ||
+        (e = cudaMemcpyAsync(h_eps + kl, ql.eps, sizeof(double), cudaMemcpyDeviceToHost, s)))
+        return cuda_fail(&c, e, "D2H");
+    return EFIT_OK;
+}
+
 // Host-buffer pipeline: nslice successive reconstructions (time slices), each `iters` chained
 // fit iterations, with their inputs read from and results written to HOST memory.  Staging slot
 // k & 1: H2D of slice k on the copy stream hs (after slot k-2's results left on ds) -> the cached
@@ -822,6 +908,11 @@ extern "C" int efit_fit_host(efit_ctx* h, int32_t nslice, int32_t iters, const d
                 return cuda_fail(&c, e, "host pipeline events");
     }
     const size_t n = (size_t)c.nw * c.nh, nd = (size_t)c.ndiag, nb = (size_t)c.nb;
+    if (c.use_graph && !c.prof_on && getenv("EFIT_HOST_STREAMS") == nullptr) {
+        const int st = fit_host_graphs(h, nslice, iters, h_psi0, h_meas, h_sigma, d_psi_ext, h_psi, h_coef, h_chi2,
+                                       h_eps, s);
+        if (st != 1) return st;  // 1: graphs not available for these buffers -> stream pipeline below
+    }
     if ((e = cudaEventRecord(c.hstart, s)) || (e = cudaStreamWaitEvent(c.hs, c.hstart, 0)) ||
         (e = cudaStreamWaitEvent(c.ds, c.hstart, 0)))
         return cuda_fail(&c, e, "host pipeline fork");
@@ -915,6 +1006,7 @@ extern "C" int efit_batch_attach(efit_ctx* h, int32_t nslice, void* d_workspace,
         for (int j = 0; j < efit::kMaxSlices; ++j) q->slice[j] = nullptr;
         for (int k = 0; k < Ctx::kGraphCache; ++k) q->gexec[k] = nullptr;
         q->hs = q->ds = nullptr;
+        q->hgexec[0] = q->hgexec[1] = nullptr;
         q->bexec = nullptr; q->pexec = nullptr; q->pgraph = nullptr;
         q->prof_on = q->prof_rec = q->prof_capture = false;
         q->prof_ev = nullptr;
@@ -1262,6 +1354,8 @@ extern "C" int efit_destroy(efit_ctx* h) {
     if (h->c.bev_resp) cudaEventDestroy(h->c.bev_resp);
     for (int k = 0; k < Ctx::kGraphCache; ++k)
         if (h->c.gexec[k]) cudaGraphExecDestroy(h->c.gexec[k]);
+    for (int b = 0; b < 2; ++b)
+        if (h->c.hgexec[b]) cudaGraphExecDestroy(h->c.hgexec[b]);
     if (h->c.hs) cudaStreamDestroy(h->c.hs);
     if (h->c.ds) cudaStreamDestroy(h->c.ds);
     if (h->c.hstart) cudaEventDestroy(h->c.hstart);

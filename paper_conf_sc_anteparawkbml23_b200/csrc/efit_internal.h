@@ -156,8 +156,13 @@ struct Ctx {
     struct HostSlot {
         double *psi, *meas, *sigma, *coef, *chi2, *eps;
     } hslot[2];
-    cudaStream_t hs, ds;              // H2D / D2H streams (created on first use)
+    cudaStream_t hs, ds;              // H2D / D2H streams (created on first use; fallback pipeline)
     cudaEvent_t hin[2], hdone[2], hfree[2], hstart;
+    // pipelined per-slice graphs: graph b = the fit of slot b + (D2H of slot b^1 -> H2D into slot b^1)
+    // as a parallel branch; its 7 copy nodes are re-pointed at the neighbouring slices per launch
+    cudaGraphExec_t hgexec[2];
+    cudaGraphNode_t hnode[2][7];      // D2H psi, coef, chi2, eps | H2D psi, meas, sigma
+    const void* hkey[2];              // (iters, d_psi_ext) the graphs were built for
 
     // multi-time-slice batch: shadow contexts share this context's tables and own
     // their per-iteration scratch (carved from the caller's batch workspace) and a stream each

@@ -179,3 +179,43 @@ def test_nccl_world1_exchange_bitwise(torch_mod, efit, mode, name):
         assert torch.equal(a, b)
     xch.close()
     plain.close()
+
+
+@pytest.mark.parametrize("path", ["graphs", "streams"])
+@pytest.mark.parametrize("pinned", [True, False])
+def test_fit_host_matches_device_steps(torch_mod, efit, monkeypatch, path, pinned):
+    """efit_fit_host (the e2e path: host buffers in and out, copies overlapped with the fits of the
+    neighbouring slices) equals efit_fit_steps on device buffers slice by slice, bit for bit, in both
+    pipelines (per-slice graphs with re-pointed copy nodes; the stream fallback) and for pinned and
+    pageable host memory."""
+    torch = torch_mod
+    if path == "streams":
+        monkeypatch.setenv("EFIT_HOST_STREAMS", "1")
+    cfg = synth.config("C2")
+    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=2)
+    psi0, ext, y, s = _twin_inputs(torch, cfg, ctx)
+    S, iters = 5, 2
+    n, nd, nb = psi0.numel(), ctx.ndiag, ctx.nbasis
+    P = torch.stack([psi0 * (1.0 + 1e-4 * k) for k in range(S)]).cpu()
+    Y = torch.stack([y * (1.0 + 1e-3 * k) for k in range(S)]).cpu()
+    G = torch.stack([s for _ in range(S)]).cpu()
+    outs = [torch.empty(S * n, dtype=torch.float64), torch.empty(S * nb, dtype=torch.float64),
+            torch.empty(S, dtype=torch.float64), torch.empty(S, dtype=torch.float64)]
+    ins = [P.reshape(-1).contiguous(), Y.reshape(-1).contiguous(), G.reshape(-1).contiguous()]
+    if pinned:
+        ins = [t.pin_memory() for t in ins]
+        outs = [t.pin_memory() for t in outs]
+    st = torch.cuda.Stream()
+    for _ in range(2):   # twice: the second call reuses the cached graphs
+        ctx.fit_host(S, iters, *ins, ext, *outs, stream=st)
+        st.synchronize()
+    assert ctx.status() == 0
+    for k in range(S):
+        psi = P[k].cuda().contiguous()
+        coef, chi2, eps = ctx._t(nb), ctx._t(1), ctx._t(1)
+        ctx.fit_steps(iters, psi, ext, Y[k].cuda().contiguous(), G[k].cuda().contiguous(), coef, chi2, eps)
+        torch.cuda.synchronize()
+        assert torch.equal(outs[0][k * n:(k + 1) * n], psi.cpu()), k
+        assert torch.equal(outs[1][k * nb:(k + 1) * nb], coef.cpu()), k
+        assert outs[2][k].item() == chi2.item() and outs[3][k].item() == eps.item(), k
+    ctx.close()
