@@ -584,7 +584,7 @@ def e2e_measure(ctx, psi0, psi_ext, meas, sigma, K_e2e, torch, dev, use_dist, ch
         raise RuntimeError("efit_fit_host produced non-finite eps")
     return {"value": round(1000.0 / ms, 2), "unit": UNIT, "h2d_bytes_per_step": 8 * (n + 2 * nd),
             "d2h_bytes_per_step": 8 * (n + nb + 2), "steps": ncall * chunk,
-            "api": "efit_fit_host (pinned host buffers; H2D/D2H on library streams, double-buffered)"}
+            "api": "efit_fit_host (pinned host buffers; one graph launch per slice, the neighbouring slices' H2D/D2H as parallel graph branches)"}
 
 
 def loop_arm(args, rank, world, local):

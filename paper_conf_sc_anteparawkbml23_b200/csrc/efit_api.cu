@@ -460,6 +460,7 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
     c.hstart = nullptr;
     for (int b = 0; b < 2; ++b) c.hin[b] = c.hdone[b] = c.hfree[b] = nullptr;
     c.hgexec[0] = c.hgexec[1] = nullptr;
+    c.hgraph[0] = c.hgraph[1] = nullptr;
     c.hkey[0] = c.hkey[1] = nullptr;
     c.prof_on = false;
     c.prof_rec = false;
@@ -804,8 +805,13 @@ static int fit_host_graphs(efit_ctx* h, int32_t nslice, int32_t iters, const dou
     cudaError_t e;
     const void* key0 = (const void*)(intptr_t)iters;
     if (!c.hgexec[0] || c.hkey[0] != key0 || c.hkey[1] != (const void*)d_psi_ext) {
-        for (int b = 0; b < 2; ++b)
-            if (c.hgexec[b]) { cudaGraphExecDestroy(c.hgexec[b]); c.hgexec[b] = nullptr; }
+        auto drop = [&c]() {
+            for (int b = 0; b < 2; ++b) {
+                if (c.hgexec[b]) { cudaGraphExecDestroy(c.hgexec[b]); c.hgexec[b] = nullptr; }
+                if (c.hgraph[b]) { cudaGraphDestroy(c.hgraph[b]); c.hgraph[b] = nullptr; }
+            }
+        };
+        drop();
         for (int b = 0; b < 2; ++b) {
             Ctx::HostSlot& q = c.hslot[b];
             Ctx::HostSlot& o = c.hslot[b ^ 1];
@@ -827,11 +833,10 @@ static int fit_host_graphs(efit_ctx* h, int32_t nslice, int32_t iters, const dou
                 cudaGraphAddMemcpyNode1D(&nd7[5], g, nd7, 4, o.meas, h_meas, sizeof(double) * nd, cudaMemcpyHostToDevice) == cudaSuccess &&
                 cudaGraphAddMemcpyNode1D(&nd7[6], g, nd7, 4, o.sigma, h_sigma, sizeof(double) * nd, cudaMemcpyHostToDevice) == cudaSuccess &&
                 cudaGraphInstantiateWithFlags(&c.hgexec[b], g, 0) == cudaSuccess;
-            cudaGraphDestroy(g);
+            c.hgraph[b] = g;
             if (!ok) {
                 cudaGetLastError();
-                for (int q2 = 0; q2 < 2; ++q2)
-                    if (c.hgexec[q2]) { cudaGraphExecDestroy(c.hgexec[q2]); c.hgexec[q2] = nullptr; }
+                drop();
                 return 1;
             }
         }
@@ -851,16 +856,20 @@ static int fit_host_graphs(efit_ctx* h, int32_t nslice, int32_t iters, const dou
         cudaGraphNode_t* nd7 = c.hnode[b];
         const bool dn = k >= 1, up = k + 1 < nslice;
         const size_t kp = dn ? (size_t)(k - 1) : 0, kn = up ? (size_t)(k + 1) : 0;
-        if ((e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[0], h_psi + kp * n, o.psi, sizeof(double) * n, cudaMemcpyDeviceToHost)) ||
-            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[1], h_coef + kp * nb, o.coef, sizeof(double) * nb, cudaMemcpyDeviceToHost)) ||
-            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[2], h_chi2 + kp, o.chi2, sizeof(double), cudaMemcpyDeviceToHost)) ||
-            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[3], h_eps + kp, o.eps, sizeof(double), cudaMemcpyDeviceToHost)) ||
-            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[4], o.psi, h_psi0 + kn * n, sizeof(double) * n, cudaMemcpyHostToDevice)) ||
-            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[5], o.meas, h_meas + kn * nd, sizeof(double) * nd, cudaMemcpyHostToDevice)) ||
-            (e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[6], o.sigma, h_sigma + kn * nd, sizeof(double) * nd, cudaMemcpyHostToDevice)))
-            return cuda_fail(&c, e, "host graph update");
+        struct { void* dst; const void* src; size_t bytes; cudaMemcpyKind kind; } cp[7] = {
+            {h_psi + kp * n, o.psi, sizeof(double) * n, cudaMemcpyDeviceToHost},
+            {h_coef + kp * nb, o.coef, sizeof(double) * nb, cudaMemcpyDeviceToHost},
+            {h_chi2 + kp, o.chi2, sizeof(double), cudaMemcpyDeviceToHost},
+            {h_eps + kp, o.eps, sizeof(double), cudaMemcpyDeviceToHost},
+            {o.psi, h_psi0 + kn * n, sizeof(double) * n, cudaMemcpyHostToDevice},
+            {o.meas, h_meas + kn * nd, sizeof(double) * nd, cudaMemcpyHostToDevice},
+            {o.sigma, h_sigma + kn * nd, sizeof(double) * nd, cudaMemcpyHostToDevice}};
         for (int q = 0; q < 7; ++q)
-            if ((e = cudaGraphNodeSetEnabled(x, nd7[q], q < 4 ? dn : up))) return cuda_fail(&c, e, "host graph update");
+            if ((e = cudaGraphExecMemcpyNodeSetParams1D(x, nd7[q], cp[q].dst, cp[q].src, cp[q].bytes, cp[q].kind)))
+                return fail(&c, EFIT_E_CUDA, "host graph update: copy node %d of slice %d: %s", q, k, cudaGetErrorString(e));
+        for (int q = 0; q < 7; ++q)
+            if ((e = cudaGraphNodeSetEnabled(x, nd7[q], q < 4 ? dn : up)))
+                return fail(&c, EFIT_E_CUDA, "host graph enable: node %d of slice %d: %s", q, k, cudaGetErrorString(e));
         if ((e = cudaGraphLaunch(x, s))) return cuda_fail(&c, e, "host graph launch");
     }
     // the last slice's results
@@ -1007,6 +1016,7 @@ extern "C" int efit_batch_attach(efit_ctx* h, int32_t nslice, void* d_workspace,
         for (int k = 0; k < Ctx::kGraphCache; ++k) q->gexec[k] = nullptr;
         q->hs = q->ds = nullptr;
         q->hgexec[0] = q->hgexec[1] = nullptr;
+        q->hgraph[0] = q->hgraph[1] = nullptr;
         q->bexec = nullptr; q->pexec = nullptr; q->pgraph = nullptr;
         q->prof_on = q->prof_rec = q->prof_capture = false;
         q->prof_ev = nullptr;
@@ -1354,8 +1364,10 @@ extern "C" int efit_destroy(efit_ctx* h) {
     if (h->c.bev_resp) cudaEventDestroy(h->c.bev_resp);
     for (int k = 0; k < Ctx::kGraphCache; ++k)
         if (h->c.gexec[k]) cudaGraphExecDestroy(h->c.gexec[k]);
-    for (int b = 0; b < 2; ++b)
+    for (int b = 0; b < 2; ++b) {
         if (h->c.hgexec[b]) cudaGraphExecDestroy(h->c.hgexec[b]);
+        if (h->c.hgraph[b]) cudaGraphDestroy(h->c.hgraph[b]);
+    }
     if (h->c.hs) cudaStreamDestroy(h->c.hs);
     if (h->c.ds) cudaStreamDestroy(h->c.ds);
     if (h->c.hstart) cudaEventDestroy(h->c.hstart);

@@ -161,6 +161,7 @@ struct Ctx {
     // pipelined per-slice graphs: graph b = the fit of slot b + (D2H of slot b^1 -> H2D into slot b^1)
     // as a parallel branch; its 7 copy nodes are re-pointed at the neighbouring slices per launch
     cudaGraphExec_t hgexec[2];
+    cudaGraph_t hgraph[2];            // kept alive: the copy-node handles below belong to it
     cudaGraphNode_t hnode[2][7];      // D2H psi, coef, chi2, eps | H2D psi, meas, sigma
     const void* hkey[2];              // (iters, d_psi_ext) the graphs were built for
 
