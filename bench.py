@@ -357,13 +357,14 @@ def barrier(use_dist, torch):
 
 def capture_steps(ctx, K, chunk, psi, psi_ext, meas, sigma, coef, chi2, eps, torch):
     """K chained fit iterations captured into CUDA graphs of <= chunk steps (efit_fit_steps: only
-    the first iteration of a graph normalises psi; the host is out of the timed loop)."""
+    the first iteration of a graph normalises psi; the host is out of the timed loop).  Thread-local
+    capture: with the in-library NCCL exchange, NCCL's proxy thread may call CUDA concurrently."""
     cap = torch.cuda.Stream()
     graphs, done = [], 0
     while done < K:
         n = min(chunk, K - done)
         g = torch.cuda.CUDAGraph()
-        with torch.cuda.graph(g, stream=cap):
+        with torch.cuda.graph(g, stream=cap, capture_error_mode="thread_local"):
             ctx.fit_steps(n, psi, psi_ext, meas, sigma, coef, chi2, eps)
         graphs.append(g)
         done += n
