@@ -2336,11 +2336,14 @@ __global__ void k_sym_pack(const double* __restrict__ I, const double* __restric
 
 // table vectors per row and lane per round, rounds in the register ring (EFIT_SYM_UNR/BUF
 // override at build time for tuning)
+// u1b4 (one 32-byte vector per row and ring round, four rounds: three in flight while one is
+// consumed) -- measured 100.8 vs 109.8 us per boundary call at 513^2 against u2b2 (same 64 ring
+// registers, finer rounds: the next loads issue after a quarter of the compute); u1b5 / u2b3 spill
 #ifndef EFIT_SYM_UNR
-#define EFIT_SYM_UNR 2
+#define EFIT_SYM_UNR 1
 #endif
 #ifndef EFIT_SYM_BUF
-#define EFIT_SYM_BUF 2
+#define EFIT_SYM_BUF 4
 #endif
 #ifndef EFIT_SYM_WG
 #define EFIT_SYM_WG 2
