@@ -57,6 +57,10 @@ def lib():
             "or_destroy": (None, [p]),
             "or_set_self_scale": (None, [p, d]),
             "or_set_boundary_method": (None, [p, i]),
+            "or_set_steps_mode": (None, [p, i]),
+            "or_get_steps_info": (None, [p, _dp]),
+            "or_hermite_eval": (None, [p, _dp, d, d, _dp]),
+            "or_newton_stationary": (i, [p, _dp, d, d, _dp]),
             "or_set_threads": (None, [i]), "or_get_threads": (i, []),
             "or_get_inlim": (None, [p, _u8p]),
             "or_green_node": (d, [p, i, i, i, i]),
@@ -205,6 +209,30 @@ class Oracle:
     def set_boundary_method(self, m: int) -> None:
         """fit_step's boundary flux: 0 = the Green's sum (O12), 1 = von Hagenow (f2)."""
         lib().or_set_boundary_method(self.ptr, int(m))
+
+    def set_steps_mode(self, m: int) -> None:
+        """Normalisation (steps_): 0 = O8 limited rule (Q9), 1 = full steps_ (f3, reading R4)."""
+        lib().or_set_steps_mode(self.ptr, int(m))
+
+    def steps_info(self) -> np.ndarray:
+        """f3 record of the last normalisation (layout in efit_oracle.c, f3 section)."""
+        out = np.zeros(16)
+        lib().or_get_steps_info(self.ptr, _d(out))
+        return out
+
+    def hermite_eval(self, psi, xt: float, xu: float) -> np.ndarray:
+        """p, pt, pu, ptt, puu, ptu of the f3 bicubic Hermite interpolant (index coordinates)."""
+        psi = _f64(psi)
+        out = np.zeros(6)
+        lib().or_hermite_eval(self.ptr, _d(psi), xt, xu, _d(out))
+        return out
+
+    def newton_stationary(self, psi, xt: float, xu: float):
+        """f3 Newton search: (converged, [xt, xu, p, det, ptt])."""
+        psi = _f64(psi)
+        out = np.zeros(5)
+        conv = lib().or_newton_stationary(self.ptr, _d(psi), xt, xu, _d(out))
+        return bool(conv), out
 
     def set_self_scale(self, s: float) -> None:
         lib().or_set_self_scale(self.ptr, s)

@@ -205,6 +205,31 @@ def solovev_psi(grid: Grid) -> np.ndarray:
     return (-SOL_SCALE * p).reshape(-1).astype(np.float64)
 
 
+# Diverted (X-point) Solov'ev for the f3 steps_ row (reading R4): with C < 0 the
+# polynomial Solov'ev has saddle points at R_x^2 = -C/A, Z_x^2 = 2B(R0^2 - R_x^2)/A (both inside
+# the limiter for R_x = 1.45 m); the homogeneous term D*Z (Delta* Z = 0, same current profile)
+# raises the lower one, which becomes the primary X-point (lower single null, DIII-D's usual shape).
+DIV_RX = 1.45
+DIV_C = -SOL_A * DIV_RX ** 2
+DIV_D = 0.045
+
+
+def solovev_diverted_psi(grid: Grid, d: float = DIV_D) -> np.ndarray:
+    """psi = -scale*(A R^2 Z^2 + B (R^2-R0^2)^2 + C_div Z^2 + d Z) on the nodes (g = i*nh + j)."""
+    R = grid.r()[:, None]
+    Z = grid.z()[None, :]
+    p = SOL_A * R ** 2 * Z ** 2 + SOL_B * (R ** 2 - SOL_R0 ** 2) ** 2 + DIV_C * Z ** 2 + d * Z
+    return (-SOL_SCALE * p).reshape(-1).astype(np.float64)
+
+
+def diverted_xpoints(d: float = 0.0):
+    """Analytic X-points (R, +-Z, psi) of the d = 0 double null."""
+    rx = math.sqrt(-DIV_C / SOL_A)
+    zx = math.sqrt(2 * SOL_B * (SOL_R0 ** 2 - rx ** 2) / SOL_A)
+    psi_x = -SOL_SCALE * SOL_B * (SOL_R0 ** 2 - rx ** 2) ** 2
+    return rx, zx, psi_x
+
+
 def solovev_poly(grid: Grid, A: float, B: float, C: float, R0: float) -> np.ndarray:
     """Un-negated polynomial Solov'ev A R^2 Z^2 + B (R^2-R0^2)^2 + C Z^2 (interior-solve pin)."""
     R = grid.r()[:, None]
@@ -244,7 +269,7 @@ def random_current(grid: Grid, seed: int = 2, signed: bool = False, edge: bool =
     return I.reshape(-1)
 
 
-def c_true(basis: Basis, seed: int = 7, edge_zero: bool = True) -> np.ndarray:
+def c_true(basis: Basis, seed: int = 7, edge_zero: bool = True, sol_c: float = SOL_C) -> np.ndarray:
     """True profile coefficients.  The leading P' and FF' terms are the Solov'ev's
     constant profiles (Delta* psi_S = -scale[(2A+8B)R^2 + 2C] gives
     P'_0 = scale(2A+8B)/mu0 and mu0 FF'_0/(4 pi^2) = 2 C scale/mu0); higher terms are
@@ -261,7 +286,7 @@ def c_true(basis: Basis, seed: int = 7, edge_zero: bool = True) -> np.ndarray:
     psi_S and c -> c_true (the twin works for any profile: psi_ext absorbs the mismatch)."""
     mu0 = 4e-7 * np.pi
     pp0 = SOL_SCALE * (2 * SOL_A + 8 * SOL_B) / mu0
-    ff0 = 2 * SOL_C * SOL_SCALE / mu0 * 4 * np.pi ** 2 / mu0
+    ff0 = 2 * sol_c * SOL_SCALE / mu0 * 4 * np.pi ** 2 / mu0
     rng = np.random.default_rng(seed)
     if basis.kind == 0:
         pp = np.concatenate([[pp0], pp0 * 0.1 * rng.uniform(-1, 1, basis.n_pp - 1)])
