@@ -221,6 +221,38 @@ int efit_nccl_unique_id(void* id_out);
 int efit_interior_solve(efit_ctx* ctx, const double* d_pcurr, const double* d_psib,
                         double* d_psi_p, efit_stream_t stream);
 
+/* ---- steps_ rule -----------------------------------------------------------------
+ * steps_ computes "the dimensionless poloidal fluxes and the location of the plasma boundary";
+ * the paper gives no algorithm.  Two rules (readings Q9 and R4):
+ *   EFIT_STEPS_LIMITER (default)  axis = in-limiter grid argmax of s psi; boundary = max of s psi
+ *                                 (bilinear) over the limiter vertices; mask = in-limiter and
+ *                                 0 <= psihat < 1 (a limited plasma).
+ *   EFIT_STEPS_FULL               axis refined by Newton's method on the bicubic Hermite interpolant of
+ *                                 psi (central-difference nodal derivatives); X-points = Newton-refined
+ *                                 saddles from the 8 best discrete candidates (indefinite discrete
+ *                                 Hessian, local minimum of |grad psi|^2) inside the limiter; boundary =
+ *                                 the largest in s of {limiter value over the vertices between the lower and
+ *                                 upper X-point heights, lower X-point, upper X-point}; mask = the
+ *                                 4-connected component of the axis node in {in-limiter, 0 <= psihat < 1}
+ *                                 (private-flux regions excluded).  Every decision is plain IEEE fp64 in
+ *                                 the reading's order (bit-reproducible).  Adds three launches per
+ *                                 iteration (the chained fit steps then normalise before every iteration).
+ *                                 Needs 6 <= nw, nh and nw * ceil(nh/32) * 4 bytes of bitmap in shared
+ *                                 memory (up to ~1025^2); not with a batch attached (EFIT_E_STATE).
+ * efit_set_steps: host-only switch (drops the cached fit-step graphs); EFIT_E_INVAL for a bad mode or
+ *   a grid outside the limits above. */
+enum { EFIT_STEPS_LIMITER = 0, EFIT_STEPS_FULL = 1 };
+int efit_set_steps(efit_ctx* ctx, int32_t steps_mode);
+
+/* The context's steps_ of d_psi[nw*nh] alone.  d_info[16] (device):
+ *   [0] psi_axis [1] psi_bdry [2] R_axis [3] Z_axis [4] 1 if the axis was refined off the node
+ *   [5] limiter value [6..8] lower X-point (R, Z, psi) [9..11] upper X-point [12] boundary kind
+ *   (0 limiter, 1 lower X, 2 upper X) [13] masked nodes [14] X candidates examined [15] axis node g;
+ *   NaN where absent (EFIT_STEPS_LIMITER fills [0], [1] and [12] only).
+ * d_mask (device uint8[nw*nh], may be NULL) receives the plasma mask.  Not capturable (LIMITER mode
+ * uploads a small host record). */
+int efit_normalize(efit_ctx* ctx, const double* d_psi, double* d_info, uint8_t* d_mask, efit_stream_t stream);
+
 /* Weighted least squares: minimise sum_m ((meas_m - sum_k resp_mk c_k)/sigma_m)^2
  * over all ndiag rows.  d_coef[nbasis], d_chi2[1]. */
 int efit_lsq(efit_ctx* ctx, const double* d_resp, const double* d_meas, const double* d_sigma,

@@ -25,7 +25,8 @@ __all__ = [
     "EFIT_GREEN_ONTHEFLY_SYM", "EFIT_GREEN_VONHAGENOW", "efit_plan_info", "owned_targets", "exchange",
     "efit_batch_workspace_bytes", "efit_batch_attach", "efit_fit_step_batch", "efit_fit_steps_batch",
     "efit_boundary_flux_batch", "efit_boundary_basis", "efit_boundary_partials", "efit_boundary_finish",
-    "efit_nccl_unique_id", "efit_fit_host",
+    "efit_nccl_unique_id", "efit_fit_host", "efit_set_steps", "efit_normalize", "EFIT_STEPS_LIMITER",
+    "EFIT_STEPS_FULL",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -37,6 +38,8 @@ EFIT_GREEN_ONTHEFLY = 1
 EFIT_GREEN_TABLE_SYM = 2       # half table by reciprocity (include/efit.h)
 EFIT_GREEN_ONTHEFLY_SYM = 3
 EFIT_GREEN_VONHAGENOW = 4      # boundary flux by the von Hagenow construction (no O(N^3) nest)
+EFIT_STEPS_LIMITER = 0         # steps_ rule (include/efit.h): limited plasma, O8 / reading Q9
+EFIT_STEPS_FULL = 1            # full steps_ (f3): bicubic axis, X-points, connectivity-filtered mask
 EFIT_OK, EFIT_E_INVAL, EFIT_E_NOMEM, EFIT_E_CUDA, EFIT_E_NCCL = 0, -1, -2, -3, -4
 EFIT_E_SINGULAR, EFIT_E_NOPLASMA, EFIT_E_NONFINITE, EFIT_E_STATE = -5, -6, -7, -8
 
@@ -105,6 +108,8 @@ def lib() -> ctypes.CDLL:
             "efit_plan_info": (I, [P(efit_grid), P(efit_basis), P(efit_geometry), P(efit_dist), I, P(efit_info_t)]),
             "efit_response": (I, [vp, vp, vp, vp, vp]),
             "efit_current": (I, [vp, vp, vp, vp, vp]),
+            "efit_set_steps": (I, [vp, ctypes.c_int32]),
+            "efit_normalize": (I, [vp, vp, vp, vp, vp]),
             "efit_boundary_flux": (I, [vp, vp, vp, vp]),
             "efit_boundary_partials": (I, [vp, vp, vp, vp]),
             "efit_boundary_finish": (I, [vp, vp, vp, vp, vp]),
@@ -257,6 +262,14 @@ def efit_nccl_unique_id() -> bytes:
 
 def efit_response(ctx, psi, resp, axbd=None, stream=None) -> None:
     _check(lib().efit_response(ctx, _ptr(psi), _ptr(resp), _ptr(axbd), _stream(stream)), ctx)
+
+
+def efit_set_steps(ctx, steps_mode: int) -> None:
+    _check(lib().efit_set_steps(ctx, int(steps_mode)), ctx)
+
+
+def efit_normalize(ctx, psi, info, mask=None, stream=None) -> None:
+    _check(lib().efit_normalize(ctx, _ptr(psi), _ptr(info), _ptr(mask), _stream(stream)), ctx)
 
 
 def efit_current(ctx, psi, coef, pcurr, stream=None) -> None:
@@ -433,6 +446,17 @@ class EfitContext:
         axbd = self._t(2)
         efit_response(self.handle, psi, resp, axbd, stream)
         return resp.view(self.ndiag, self.nbasis), axbd
+
+    def set_steps(self, steps_mode: int) -> None:
+        efit_set_steps(self.handle, steps_mode)
+
+    def normalize(self, psi, stream=None):
+        """(info[16], uint8 mask[nw*nh]) of the context's steps_ rule (include/efit.h efit_normalize)."""
+        import torch
+        info = self._t(16)
+        mask = torch.zeros(self.nw * self.nh, dtype=torch.uint8, device=self.device)
+        efit_normalize(self.handle, psi, info, mask, stream)
+        return info, mask
 
     def current(self, psi, coef, stream=None):
         out = self._t(self.nw * self.nh)

@@ -7,7 +7,10 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libefit_b200.so")
-SOURCES = ["efit_api.cu", "efit_kernels.cu"]
+SOURCES = ["efit_api.cu", "efit_kernels.cu", "efit_steps.cu"]
+# per-source flags: the steps_ kernels take discrete decisions from fp64 expressions that must round
+# exactly as written (no FMA contraction anywhere in that translation unit)
+SOURCE_FLAGS = {"efit_steps.cu": ["-fmad=false"]}
 HEADERS = ["efit_internal.h", "efit_device.cuh"]
 
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
@@ -33,7 +36,8 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str = LIB
     for src in SOURCES:
         tag = "" if out == LIB else "." + os.path.basename(out).replace(".so", "")
         obj = os.path.join(CSRC, src.replace(".cu", tag + ".o"))
-        cmd = ["nvcc", *NVCC_FLAGS, *["-D" + d for d in defines], "-c", os.path.join(CSRC, src), "-o", obj]
+        cmd = ["nvcc", *NVCC_FLAGS, *SOURCE_FLAGS.get(src, []), *["-D" + d for d in defines], "-c",
+               os.path.join(CSRC, src), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         log.append(r.stdout + r.stderr)
         if r.returncode != 0:

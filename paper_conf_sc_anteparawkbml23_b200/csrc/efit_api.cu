@@ -325,6 +325,12 @@ static size_t carve_scratch(Ctx& c, Take& take, size_t& off, bool batch) {
     c.vh_psi0 = c.vh ? (double*)take(sizeof(double) * (size_t)n) : nullptr;
     c.vh_src = c.vh ? (double*)take(sizeof(double) * ((c.n_edge + 3) / 4 * 4)) : nullptr;
     c.zero_edge = c.vh ? (double*)take(sizeof(double) * ((c.n_edge + 3) / 4 * 4)) : nullptr;
+    // full steps_ (f3): always carved (efit_set_steps switches without a new workspace)
+    c.pmask = (uint8_t*)take((size_t)n);
+    c.st_info = (double*)take(sizeof(double) * 16);
+    c.st_cnt = (unsigned*)take(sizeof(unsigned) * 4);
+    c.st_cand = (double2*)take(sizeof(double2) * (size_t)efit::steps_cand_cap(c.nw, c.nh));
+    c.st_bits = (uint32_t*)take(sizeof(uint32_t) * (size_t)c.nw * efit::steps_words(c.nh));
     return (size_t)round_up((long long)off, 256);
 }
 
@@ -577,6 +583,62 @@ extern "C" int efit_response(efit_ctx* h, const double* d_psi, double* d_resp, d
     return EFIT_OK;
 }
 
+// cached fit-step graphs were captured for one normalisation rule: drop them when it changes
+static void drop_fit_graphs(Ctx& c) {
+    for (int k = 0; k < Ctx::kGraphCache; ++k)
+        if (c.gexec[k]) { cudaGraphExecDestroy(c.gexec[k]); c.gexec[k] = nullptr; }
+    for (int b = 0; b < 2; ++b) {
+        if (c.hgexec[b]) { cudaGraphExecDestroy(c.hgexec[b]); c.hgexec[b] = nullptr; }
+        if (c.hgraph[b]) { cudaGraphDestroy(c.hgraph[b]); c.hgraph[b] = nullptr; }
+    }
+    c.hkey[0] = c.hkey[1] = nullptr;
+}
+
+extern "C" int efit_set_steps(efit_ctx* h, int32_t steps_mode) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    if (steps_mode != EFIT_STEPS_LIMITER && steps_mode != EFIT_STEPS_FULL)
+        return fail(&c, EFIT_E_INVAL, "steps_mode must be EFIT_STEPS_LIMITER or EFIT_STEPS_FULL");
+    if (steps_mode == EFIT_STEPS_FULL) {
+        if (c.nslice > 0) return fail(&c, EFIT_E_STATE, "EFIT_STEPS_FULL with a batch attached");
+        int optin = 0;
+        cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, c.device);
+        if (c.nw < 6 || c.nh < 6 || efit::steps_fill_smem(c.nw, c.nh, nullptr) > (size_t)optin)
+            return fail(&c, EFIT_E_INVAL, "EFIT_STEPS_FULL needs 6 <= nw, nh and a plasma bitmap in shared memory (nw*nh <= ~1025^2)");
+    }
+    if (c.steps != steps_mode) drop_fit_graphs(c);
+    c.steps = steps_mode;
+    return EFIT_OK;
+}
+
+extern "C" int efit_normalize(efit_ctx* h, const double* d_psi, double* d_info, uint8_t* d_mask, efit_stream_t stream) {
+    if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
+    Ctx& c = h->c;
+    EFIT_CHECK_PTR(c, d_psi, "d_psi");
+    EFIT_CHECK_PTR(c, d_info, "d_info");
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    if ((e = efit::launch_normalize(c, d_psi, s))) return cuda_fail(&c, e, "normalize");
+    if (c.steps) {
+        if ((e = cudaMemcpyAsync(d_info, c.st_info, 16 * sizeof(double), cudaMemcpyDeviceToDevice, s)))
+            return cuda_fail(&c, e, "info copy");
+        if (d_mask && (e = cudaMemcpyAsync(d_mask, c.pmask, (size_t)c.nw * c.nh, cudaMemcpyDeviceToDevice, s)))
+            return cuda_fail(&c, e, "mask copy");
+        return EFIT_OK;
+    }
+    // limiter rule: {psi_axis, psi_bdry}, kind 0, the rest NaN
+    const double nan = __builtin_nan("");
+    double hinfo[16];
+    for (int k = 0; k < 16; ++k) hinfo[k] = nan;
+    hinfo[12] = 0.0;
+    if ((e = cudaMemcpyAsync(c.st_info, hinfo, sizeof(hinfo), cudaMemcpyHostToDevice, s)) ||
+        (e = cudaMemcpyAsync(c.st_info, c.axbd, 2 * sizeof(double), cudaMemcpyDeviceToDevice, s)) ||
+        (e = cudaMemcpyAsync(d_info, c.st_info, 16 * sizeof(double), cudaMemcpyDeviceToDevice, s)))
+        return cuda_fail(&c, e, "info copy");
+    if (d_mask && (e = efit::launch_mask_o8(c, d_psi, d_mask, s))) return cuda_fail(&c, e, "mask");
+    return EFIT_OK;
+}
+
 extern "C" int efit_current(efit_ctx* h, const double* d_psi, const double* d_coef, double* d_pcurr,
                             efit_stream_t stream) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
@@ -693,7 +755,7 @@ static cudaError_t enqueue_fit_step(Ctx& c, double* psi, const double* psi_ext, 
     cudaError_t e;
     c.prof_rec = c.prof_on && (c.prof_calls++ % c.prof_every == 0);
     mark(c, s, M_BEGIN);
-    if (normalize && (e = launch_normalize(c, psi, s))) return e;
+    if ((normalize || c.steps) && (e = launch_normalize(c, psi, s))) return e;  // f3: steps_ every iteration
     mark(c, s, M_NORM);
     const size_t nresp = (size_t)c.ndiag * c.nb;
     if (c.comm && c.world > 1 && (e = cudaMemsetAsync(c.resp, 0, sizeof(double) * nresp, s))) return e;
@@ -991,6 +1053,7 @@ extern "C" int efit_batch_workspace_bytes(const efit_ctx* h, int32_t nslice, siz
 extern "C" int efit_batch_attach(efit_ctx* h, int32_t nslice, void* d_workspace, size_t ws_bytes) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
     Ctx& c = h->c;
+    if (c.steps) return fail(&c, EFIT_E_STATE, "batch with EFIT_STEPS_FULL is not supported");
     int st = batch_check(c, nslice);
     if (st) return st;
     const size_t per = slice_bytes(c);

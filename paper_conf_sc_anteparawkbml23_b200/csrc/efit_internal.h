@@ -123,6 +123,13 @@ struct Ctx {
     double* vh_psi0;    // [nw*nh]  VH: zero-Dirichlet solve of the current
     double* vh_src;     // [n_edge] VH: W_q (1/R_q) dpsi0/dn_q at the edge nodes
     double* zero_edge;  // [n_edge] zeros (the zero-Dirichlet edge values)
+    // full steps_ (efit_set_steps): per-iteration plasma mask replacing the limiter flags
+    int steps;          // EFIT_STEPS_LIMITER (0) or EFIT_STEPS_FULL (1)
+    uint8_t* pmask;     // [nw*nh]  connectivity-filtered plasma mask (steps == 1)
+    double* st_info;    // [16]     axis / X-point / boundary record (efit_normalize layout)
+    unsigned* st_cnt;   // [4]      candidate count, axis node, non-finite flag
+    double2* st_cand;   // [steps_cand_cap] X-point candidates (|grad|^2, g)
+    uint32_t* st_bits;  // [nw][steps_words] candidate bitmap
     void* comm;         // ncclComm_t or nullptr
     int nccl_err;       // last ncclResult_t != ncclSuccess of xch_allreduce (reported as EFIT_E_NCCL)
 
@@ -189,6 +196,18 @@ struct Ctx {
 enum Mark { M_BEGIN = 0, M_NORM, M_RESP, M_CUR, M_TB, M_LR, M_SOLVE, kNumMarks };
 constexpr int kNumProfileFields = 7;  // step, normalize, response, lsq+current, bnd_tb, bnd_lr, tail
 void mark(Ctx& c, cudaStream_t s, int id);  // efit_api.cu; no-op unless profiling
+
+// plasma-region flags read by the basis / response / current kernels: the limiter flags (O8 rule,
+// psihat tested per node) or the connectivity-filtered mask of the full steps_ (f3)
+inline const uint8_t* mask_of(const Ctx& c) { return c.steps ? c.pmask : c.inlim; }
+
+// ---- full steps_ (efit_steps.cu) -------------------------------------------------
+int steps_words(int nh);
+int steps_cand_cap(int nw, int nh);
+size_t steps_fill_smem(int nw, int nh, bool* cand_smem);
+cudaError_t prepare_steps(Ctx& c, int smem_optin);
+cudaError_t launch_steps(Ctx& c, const double* psi, cudaStream_t s);
+cudaError_t launch_mask_o8(Ctx& c, const double* psi, uint8_t* mask, cudaStream_t s);
 
 // ---- launchers (efit_kernels.cu) -------------------------------------------------
 cudaError_t launch_init_tables(Ctx& c, cudaStream_t s);

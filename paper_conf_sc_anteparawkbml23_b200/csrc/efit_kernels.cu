@@ -505,6 +505,7 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
     if (e) return e;
     e = cudaMemsetAsync(c.tickets, 0, sizeof(unsigned) * 8, s);
     if (e) return e;
+    if (c.st_cnt && (e = cudaMemsetAsync(c.st_cnt, 0, sizeof(unsigned) * 4, s))) return e;
     return cudaGetLastError();
 }
 
@@ -605,6 +606,7 @@ __global__ void __launch_bounds__(256) k_normalize(const double* __restrict__ ps
 }
 
 cudaError_t launch_normalize(Ctx& c, const double* psi, cudaStream_t s) {
+    if (c.steps) return launch_steps(c, psi, s);
     launch_pdl(k_normalize, dim3(c.t.red_blocks), dim3(256), 0, s, psi, c.inlim, c.nw, c.nh, c.rmin, c.dr, c.zmin, c.dz,
                                                c.ip_sign, c.lim, c.n_lim, c.norm_part, c.tickets + 0,
                                                c.axbd, c.status);
@@ -890,11 +892,11 @@ static void launch_resp_nb(Ctx& c, const double* psi, double* part, cudaStream_t
     const int gc = c.t.resp_gc;
     const size_t smem = sizeof(double) * NB * gc;
     const long long ldb = (long long)c.t.resp_nchunk * gc;
-    FusedBasis fb{c.resp_fuse ? 1 : 0, psi, c.inlim, c.axbd, c.nh, c.rmin, c.dr, c.dr * c.dz, basis_params(c),
+    FusedBasis fb{c.resp_fuse ? 1 : 0, psi, mask_of(c), c.axbd, c.nh, c.rmin, c.dr, c.dr * c.dz, basis_params(c),
                   c.bmat, c.resp_cnt};
     if (!prepare && !c.resp_fuse) {
         BasisParams bp = basis_params(c);
-        launch_pdl(k_basis<NB>, dim3(c.t.resp_nchunk), dim3(gc <= 1024 ? gc : 1024), 0, s, psi, c.inlim, c.axbd, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp,
+        launch_pdl(k_basis<NB>, dim3(c.t.resp_nchunk), dim3(gc <= 1024 ? gc : 1024), 0, s, psi, mask_of(c), c.axbd, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp,
                                                     gc, ldb, c.bmat, c.resp_cnt);
     }
     int mb = c.t.resp_mb;
@@ -1044,7 +1046,7 @@ cudaError_t launch_basis(Ctx& c, const double* psi, cudaStream_t s) {
     switch (c.nb) {
 #define EFIT_NB_CASE(V)                                                                                              \
     case V:                                                                                                          \
-        return launch_pdl(k_basis<V>, dim3(c.t.resp_nchunk), dim3(gc <= 1024 ? gc : 1024), 0, s, psi, c.inlim, c.axbd, \
+        return launch_pdl(k_basis<V>, dim3(c.t.resp_nchunk), dim3(gc <= 1024 ? gc : 1024), 0, s, psi, mask_of(c), c.axbd, \
                           c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp, gc, ldb, c.bmat, c.resp_cnt);
         EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
         EFIT_NB_CASE(7) EFIT_NB_CASE(8) EFIT_NB_CASE(9) EFIT_NB_CASE(10) EFIT_NB_CASE(11) EFIT_NB_CASE(12)
@@ -1745,7 +1747,7 @@ cudaError_t launch_current(Ctx& c, const double* psi, const double* coef, double
     double* fl = pair ? c.pflip : nullptr;
     switch (c.nb) {
 #define EFIT_NB_CASE(V) \
-    case V: launch_pdl(k_current<V>, dim3(blocks), dim3(256), 0, s, psi, c.inlim, c.axbd, coef, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp, pcurr, fl); break;
+    case V: launch_pdl(k_current<V>, dim3(blocks), dim3(256), 0, s, psi, mask_of(c), c.axbd, coef, c.nw, c.nh, c.rmin, c.dr, c.dr * c.dz, bp, pcurr, fl); break;
         EFIT_NB_CASE(1) EFIT_NB_CASE(2) EFIT_NB_CASE(3) EFIT_NB_CASE(4) EFIT_NB_CASE(5) EFIT_NB_CASE(6)
         EFIT_NB_CASE(7) EFIT_NB_CASE(8) EFIT_NB_CASE(9) EFIT_NB_CASE(10) EFIT_NB_CASE(11) EFIT_NB_CASE(12)
         EFIT_NB_CASE(13) EFIT_NB_CASE(14) EFIT_NB_CASE(15) EFIT_NB_CASE(16) EFIT_NB_CASE(17) EFIT_NB_CASE(18)
@@ -3160,7 +3162,7 @@ cudaError_t launch_solve_rest(Ctx& c, const double* psib, double* psi_out, doubl
     }
     if (e) return e;
     NextNorm nn;
-    nn.on = (next_norm && psi_inout) ? 1 : 0;
+    nn.on = (next_norm && psi_inout && !c.steps) ? 1 : 0;  // f3: steps_ runs before every iteration
     nn.sgn = c.ip_sign;
     nn.n_lim = c.n_lim;
     nn.inlim = c.inlim;
@@ -3423,7 +3425,7 @@ cudaError_t prepare_kernels(Ctx& c) {
         if ((e = big((const void*)k_dst_inv, smem))) return e;
         if ((e = big((const void*)k_tridiag, sizeof(double) * 4 * ((size_t)c.ni_pad + 32)))) return e;
     }
-    return cudaSuccess;
+    return prepare_steps(c, g_smem_optin);
 }
 
 }  // namespace efit

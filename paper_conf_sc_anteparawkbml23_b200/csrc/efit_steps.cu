@@ -1,0 +1,618 @@
+// efit_steps.cu -- the full steps_ normalisation on sm_100a.
+//
+// steps_ computes "the dimensionless poloidal fluxes and the location of the plasma boundary"
+// (P:L107); the algorithm is DESIGN.md reading R4: magnetic axis refined on the bicubic Hermite
+// interpolant of psi (central-difference nodal derivatives, index units) by Newton's method,
+// X-points found the same way from saddle candidates, the boundary = the first of {limiter contact
+// between the X-point heights, lower X-point, upper X-point} met going out from the axis, and the
+// plasma mask = the 4-connected component of the axis node in {in-limiter, 0 <= psihat < 1}.
+//
+// This translation unit is compiled with -fmad=false: every floating-point expression below is a
+// sequence of plain IEEE fp64 operations in the written order (that of the reading), so every
+// discrete decision (candidate test, Newton acceptance, boundary choice, mask bit) is reproducible
+// bit for bit.  Three launches per normalisation:
+//   k_steps_scan   all CTAs: in-limiter argmax partials of s psi + X-point candidate list;
+//                  the last CTA: axis / X-point Newton searches, limiter value, boundary
+//   k_steps_bits   candidate bitmap {inlim, 0 <= psihat < 1}, one 32-bit word per warp (ballot)
+//   k_steps_fill   one CTA: bit-parallel flood fill from the axis node in shared memory (row runs by
+//                  carry propagation, column runs by a segmented scan), then the byte mask
+#include <cuda_runtime.h>
+#include <float.h>
+#include <limits.h>
+#include <stdint.h>
+
+#include <utility>
+
+#include "efit_internal.h"
+
+namespace efit {
+
+namespace {
+
+constexpr int kNewtonIters = 20;
+constexpr int kMaxXCand = 8;
+constexpr int kFillThreads = 1024;
+constexpr int kSegRows = 16;  // rows per segment of the column scans
+
+__device__ __forceinline__ void am_merge(double& v, long long& i, double v2, long long i2) {
+    if (v2 > v || (v2 == v && i2 < i)) { v = v2; i = i2; }
+}
+
+__device__ __forceinline__ void am_warp(double& v, long long& i) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const double v2 = __shfl_xor_sync(0xffffffffu, v, o);
+        const long long i2 = __shfl_xor_sync(0xffffffffu, i, o);
+        am_merge(v, i, v2, i2);
+    }
+}
+
+struct Field {
+    const double* psi;
+    int nw, nh;
+    __device__ __forceinline__ double at(int i, int j) const { return __ldg(psi + (long long)i * nh + j); }
+};
+
+// Hermite basis on [0, 1]: values at 0 / 1, slopes at 0 / 1, and their first and second derivatives
+__device__ __forceinline__ void herm_basis(double t, double h[4], double d[4], double e[4]) {
+    const double t2 = t * t;
+    h[0] = (2.0 * t - 3.0) * t2 + 1.0;
+    h[1] = (3.0 - 2.0 * t) * t2;
+    h[2] = ((t - 2.0) * t + 1.0) * t;
+    h[3] = (t - 1.0) * t2;
+    d[0] = (6.0 * t) * (t - 1.0);
+    d[1] = -d[0];
+    d[2] = (3.0 * t - 4.0) * t + 1.0;
+    d[3] = (3.0 * t - 2.0) * t;
+    e[0] = 12.0 * t - 6.0;
+    e[1] = -e[0];
+    e[2] = 6.0 * t - 4.0;
+    e[3] = 6.0 * t - 2.0;
+}
+
+// sum_a A[a] (sum_b Q[a][b] B[b]), both sums left to right
+__device__ __forceinline__ double herm_form(const double Q[4][4], const double* A, const double* B) {
+    double v[4];
+#pragma unroll
+    for (int a = 0; a < 4; ++a) v[a] = ((Q[a][0] * B[0] + Q[a][1] * B[1]) + Q[a][2] * B[2]) + Q[a][3] * B[3];
+    return ((A[0] * v[0] + A[1] * v[1]) + A[2] * v[2]) + A[3] * v[3];
+}
+
+// p, pt, pu, ptt, puu, ptu of the interpolant at index coordinates (xt, xu); cell clamped to
+// 1 <= ci <= nw-3, 1 <= cj <= nh-3 (both corners interior: central differences defined)
+__device__ void herm_eval(const Field& F, double xt, double xu, double out[6]) {
+    int ci = (int)floor(xt), cj = (int)floor(xu);
+    ci = ci < 1 ? 1 : (ci > F.nw - 3 ? F.nw - 3 : ci);
+    cj = cj < 1 ? 1 : (cj > F.nh - 3 ? F.nh - 3 : cj);
+    const double t = xt - (double)ci, u = xu - (double)cj;
+    double Q[4][4];
+#pragma unroll
+    for (int a = 0; a < 2; ++a) {
+        const int i = ci + a;
+#pragma unroll
+        for (int b = 0; b < 2; ++b) {
+            const int j = cj + b;
+            Q[a][b] = F.at(i, j);
+            Q[a][2 + b] = 0.5 * (F.at(i, j + 1) - F.at(i, j - 1));
+            Q[2 + a][b] = 0.5 * (F.at(i + 1, j) - F.at(i - 1, j));
+            Q[2 + a][2 + b] = 0.25 * (((F.at(i + 1, j + 1) - F.at(i + 1, j - 1)) - F.at(i - 1, j + 1)) + F.at(i - 1, j - 1));
+        }
+    }
+    double ht[4], dt[4], et[4], hu[4], du[4], eu[4];
+    herm_basis(t, ht, dt, et);
+    herm_basis(u, hu, du, eu);
+    out[0] = herm_form(Q, ht, hu);
+    out[1] = herm_form(Q, dt, hu);
+    out[2] = herm_form(Q, ht, du);
+    out[3] = herm_form(Q, et, hu);
+    out[4] = herm_form(Q, ht, eu);
+    out[5] = herm_form(Q, dt, du);
+}
+
+// Newton's method for grad p = 0 from (xt, xu): <= 20 steps, step components clamped to [-1/2, 1/2],
+// converged when both are below 1e-10.  out = xt, xu, p, det, ptt at the final point.
+__device__ bool newton_stationary(const Field& F, double xt, double xu, double out[5]) {
+    double d[6];
+    bool conv = false;
+    for (int it = 0; it < kNewtonIters; ++it) {
+        herm_eval(F, xt, xu, d);
+        const double det = d[3] * d[4] - d[5] * d[5];
+        if (!(det != 0.0)) break;
+        double st = (d[4] * d[1] - d[5] * d[2]) / det;
+        double su = (d[3] * d[2] - d[5] * d[1]) / det;
+        if (!(fabs(st) < 1e300) || !(fabs(su) < 1e300)) break;
+        st = st > 0.5 ? 0.5 : st;
+        st = st < -0.5 ? -0.5 : st;
+        su = su > 0.5 ? 0.5 : su;
+        su = su < -0.5 ? -0.5 : su;
+        xt = xt - st;
+        xu = xu - su;
+        if (fabs(st) < 1e-10 && fabs(su) < 1e-10) { conv = true; break; }
+    }
+    herm_eval(F, xt, xu, d);
+    out[0] = xt; out[1] = xu; out[2] = d[0]; out[3] = d[3] * d[4] - d[5] * d[5]; out[4] = d[3];
+    return conv;
+}
+
+__device__ __forceinline__ double grad2(const Field& F, int i, int j) {
+    const double gt = 0.5 * (F.at(i + 1, j) - F.at(i - 1, j));
+    const double gu = 0.5 * (F.at(i, j + 1) - F.at(i, j - 1));
+    return gt * gt + gu * gu;
+}
+
+// X-point candidate test of node (i, j), 2 <= i <= nw-3, 2 <= j <= nh-3, in the limiter: indefinite
+// discrete Hessian and |grad|^2 a local minimum over the 8 neighbours (strict against lower node
+// indices, <= against higher ones)
+__device__ bool xcand(const Field& F, int i, int j, double& key) {
+    const double p0 = F.at(i, j);
+    const double dtt = (F.at(i + 1, j) - 2.0 * p0) + F.at(i - 1, j);
+    const double duu = (F.at(i, j + 1) - 2.0 * p0) + F.at(i, j - 1);
+    const double dtu = 0.25 * (((F.at(i + 1, j + 1) - F.at(i + 1, j - 1)) - F.at(i - 1, j + 1)) + F.at(i - 1, j - 1));
+    if (!(dtt * duu - dtu * dtu < 0.0)) return false;
+    const double g2 = grad2(F, i, j);
+    for (int di = -1; di <= 1; ++di)
+        for (int dj = -1; dj <= 1; ++dj) {
+            if (!di && !dj) continue;
+            const double v = grad2(F, i + di, j + dj);
+            const bool lower = (di < 0) || (di == 0 && dj < 0);  // neighbour has the lower node index
+            if (lower ? !(g2 < v) : !(g2 <= v)) return false;
+        }
+    key = g2;
+    return true;
+}
+
+// even-odd rule of O7 (same expression as the limiter table)
+__device__ bool in_polygon(double R, double Z, const double* lim, int n_lim) {
+    bool inside = false;
+    for (int k = 0; k < n_lim; ++k) {
+        const int k1 = (k + 1 == n_lim) ? 0 : k + 1;
+        const double r0 = lim[k], z0 = lim[n_lim + k], r1 = lim[k1], z1 = lim[n_lim + k1];
+        if ((z0 > Z) != (z1 > Z)) {
+            const double x = ((r1 - r0) * (Z - z0)) / (z1 - z0) + r0;
+            if (R < x) inside = !inside;
+        }
+    }
+    return inside;
+}
+
+// O8's bilinear value at (R, Z)
+__device__ double bilin(const Field& F, double rmin, double dr, double zmin, double dz, double R, double Z) {
+    const double x = (R - rmin) / dr, y = (Z - zmin) / dz;
+    int i = (int)floor(x), j = (int)floor(y);
+    i = i < 0 ? 0 : (i > F.nw - 2 ? F.nw - 2 : i);
+    j = j < 0 ? 0 : (j > F.nh - 2 ? F.nh - 2 : j);
+    const double t = x - (double)i, u = y - (double)j;
+    const double w00 = (1.0 - t) * (1.0 - u), w10 = t * (1.0 - u), w01 = (1.0 - t) * u, w11 = t * u;
+    return ((w00 * F.at(i, j) + w10 * F.at(i + 1, j)) + w01 * F.at(i, j + 1)) + w11 * F.at(i + 1, j + 1);
+}
+
+struct ScanArgs {
+    const double* psi;
+    const uint8_t* inlim;
+    int nw, nh, sgn;
+    double rmin, dr, zmin, dz;
+    const double* lim;
+    int n_lim;
+    double* part;        // [gridDim.x][2] (s psi, g) argmax partials
+    unsigned* ticket;
+    double2* cand;       // [cap] (|grad|^2, g)
+    unsigned* cnt;       // [0] candidates found, [1] axis node g0 (or UINT_MAX), [2] non-finite psi seen
+    int cap;
+    double* info;        // [16] (efit.h efit_normalize layout)
+    double* axbd;        // [2]
+    int* status;
+};
+
+__global__ void __launch_bounds__(256) k_steps_scan(ScanArgs a) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    __shared__ double sv[8];
+    __shared__ long long si[8];
+    __shared__ bool last;
+    __shared__ double selk[kMaxXCand];
+    __shared__ long long selg[kMaxXCand];
+    __shared__ double res[kMaxXCand + 1][5];
+    __shared__ int rconv[kMaxXCand + 1];
+    __shared__ double lv[8];
+    __shared__ long long li[8];
+    __shared__ double zlim[2];
+    __shared__ int nsel_s, bad_s;
+    const Field F{a.psi, a.nw, a.nh};
+    const int n = a.nw * a.nh, nh = a.nh;
+    const double s = (double)a.sgn;
+    double best = -DBL_MAX;
+    long long bi = LLONG_MAX;
+    bool bad = false;
+    for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += gridDim.x * blockDim.x) {
+        const double p = __ldcg(a.psi + g);
+        const uint8_t in = __ldg(a.inlim + g);
+        if (!isfinite(p)) bad = true;
+        if (in) {
+            am_merge(best, bi, s * p, (long long)g);
+            const int i = g / nh, j = g - (g / nh) * nh;
+            double key;
+            if (i >= 2 && i <= a.nw - 3 && j >= 2 && j <= nh - 3 && xcand(F, i, j, key)) {
+                const unsigned k = atomicAdd(a.cnt, 1u);
+                if (k < (unsigned)a.cap) a.cand[k] = make_double2(key, (double)g);
+            }
+        }
+    }
+    __threadfence();  // this thread's candidate entries before the block's ticket
+    if (__syncthreads_or(bad) && threadIdx.x == 0) {
+        atomicOr(a.status, EFIT_ST_NONFINITE);
+        atomicOr(a.cnt + 2, 1u);
+    }
+    am_warp(best, bi);
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+    if (l == 0) { sv[w] = best; si[w] = bi; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int q = 1; q < 8; ++q) am_merge(best, bi, sv[q], si[q]);
+        a.part[2 * blockIdx.x] = best;
+        a.part[2 * blockIdx.x + 1] = (double)bi;
+        __threadfence();
+        last = (atomicAdd(a.ticket, 1u) == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    // ---- last CTA: (3) axis node, (4) X-point candidates, Newton searches
+    best = -DBL_MAX; bi = LLONG_MAX;
+    for (int b = threadIdx.x; b < (int)gridDim.x; b += blockDim.x)
+        am_merge(best, bi, __ldcg(a.part + 2 * b), (long long)__ldcg(a.part + 2 * b + 1));
+    am_warp(best, bi);
+    if (l == 0) { sv[w] = best; si[w] = bi; }
+    if (threadIdx.x == 0) { nsel_s = 0; bad_s = *((volatile unsigned*)(a.cnt + 2)) ? 1 : 0; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int q = 1; q < 8; ++q) am_merge(best, bi, sv[q], si[q]);
+        si[0] = bi;
+    }
+    const unsigned ncand_all = *((volatile unsigned*)a.cnt);
+    const int ncand = (int)(ncand_all < (unsigned)a.cap ? ncand_all : (unsigned)a.cap);
+    // the 8 smallest (|grad|^2, g): rank of each candidate in that total order
+    for (int q = threadIdx.x; q < ncand; q += blockDim.x) {
+        const double2 cq = __ldcg(a.cand + q);
+        int rank = 0;
+        for (int r = 0; r < ncand && rank < kMaxXCand; ++r) {
+            const double2 cr = __ldcg(a.cand + r);
+            if (cr.x < cq.x || (cr.x == cq.x && cr.y < cq.y)) ++rank;
+        }
+        if (rank < kMaxXCand) { selk[rank] = cq.x; selg[rank] = (long long)cq.y; atomicMax(&nsel_s, rank + 1); }
+    }
+    __syncthreads();
+    const long long g0 = si[0];
+    const int nsel = nsel_s;
+    const bool ok0 = (g0 != LLONG_MAX) && !bad_s;
+    // thread 0: the axis; threads 1..nsel: the X-point candidates (concurrently)
+    if (ok0 && threadIdx.x <= nsel) {
+        const long long gs = threadIdx.x == 0 ? g0 : selg[threadIdx.x - 1];
+        const int i = (int)(gs / nh), j = (int)(gs - (gs / nh) * nh);
+        double o[5];
+        bool conv = false;
+        if (threadIdx.x > 0 || (a.nw >= 4 && nh >= 4 && i >= 1 && i <= a.nw - 2 && j >= 1 && j <= nh - 2))
+            conv = newton_stationary(F, (double)i, (double)j, o);
+        rconv[threadIdx.x] = conv ? 1 : 0;
+        for (int k = 0; k < 5; ++k) res[threadIdx.x][k] = o[k];
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double* info = a.info;
+        for (int k = 0; k < 16; ++k) info[k] = __longlong_as_double(0x7ff8000000000000LL);  // NaN
+        double pa = 0.0, Za = 0.0;
+        bool lo = false, hi = false;
+        double xlo[3], xhi[3];
+        if (ok0) {
+            const int i0 = (int)(g0 / nh), j0 = (int)(g0 - (g0 / nh) * nh);
+            const double p0 = F.at(i0, j0);
+            pa = p0;
+            double xa = (double)i0, ya = (double)j0;
+            int ref = 0;
+            const double* o = res[0];
+            if (rconv[0] && o[3] > 0.0 && s * o[4] < 0.0 && fabs(o[0] - (double)i0) <= 1.0 &&
+                fabs(o[1] - (double)j0) <= 1.0 && s * o[2] >= s * p0) {
+                pa = o[2]; xa = o[0]; ya = o[1]; ref = 1;
+            }
+            Za = a.zmin + ya * a.dz;
+            info[0] = pa; info[2] = a.rmin + xa * a.dr; info[3] = Za; info[4] = (double)ref; info[15] = (double)g0;
+            info[14] = (double)nsel;
+            for (int q = 0; q < nsel; ++q) {
+                const long long gq = selg[q];
+                const int i = (int)(gq / nh), j = (int)(gq - (gq / nh) * nh);
+                const double* x = res[q + 1];
+                if (!(rconv[q + 1] && x[3] < 0.0 && fabs(x[0] - (double)i) <= 1.5 && fabs(x[1] - (double)j) <= 1.5))
+                    continue;
+                const double Rx = a.rmin + x[0] * a.dr, Zx = a.zmin + x[1] * a.dz;
+                if (!in_polygon(Rx, Zx, a.lim, a.n_lim)) continue;
+                if (!(s * (pa - x[2]) > 0.0)) continue;
+                if (Zx < Za) {
+                    if (!lo || s * x[2] > s * xlo[2]) { lo = true; xlo[0] = Rx; xlo[1] = Zx; xlo[2] = x[2]; }
+                } else if (Zx > Za) {
+                    if (!hi || s * x[2] > s * xhi[2]) { hi = true; xhi[0] = Rx; xhi[1] = Zx; xhi[2] = x[2]; }
+                }
+            }
+            if (lo) { info[6] = xlo[0]; info[7] = xlo[1]; info[8] = xlo[2]; }
+            if (hi) { info[9] = xhi[0]; info[10] = xhi[1]; info[11] = xhi[2]; }
+        }
+        zlim[0] = lo ? xlo[1] : -DBL_MAX;
+        zlim[1] = hi ? xhi[1] : DBL_MAX;
+        res[0][0] = pa;
+        rconv[0] = ok0 ? 1 : 0;
+    }
+    __syncthreads();
+    // ---- (5) limiter value between the X-point heights (ties: lowest vertex)
+    double vb = -DBL_MAX;
+    long long vi = LLONG_MAX;
+    if (rconv[0]) {
+        const bool lo = zlim[0] != -DBL_MAX, hi = zlim[1] != DBL_MAX;
+        for (int v = threadIdx.x; v < a.n_lim; v += blockDim.x) {
+            const double z = a.lim[a.n_lim + v];
+            if (lo && !(z > zlim[0])) continue;
+            if (hi && !(z < zlim[1])) continue;
+            am_merge(vb, vi, s * bilin(F, a.rmin, a.dr, a.zmin, a.dz, a.lim[v], z), (long long)v);
+        }
+    }
+    am_warp(vb, vi);
+    if (l == 0) { lv[w] = vb; li[w] = vi; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int q = 1; q < 8; ++q) am_merge(vb, vi, lv[q], li[q]);
+        double* info = a.info;
+        const double pa = res[0][0];
+        // (6) boundary: the largest in s of {limiter, lower X, upper X}, ties in that order
+        int kind = -1;
+        double pb = 0.0;
+        if (rconv[0]) {
+            if (vi != LLONG_MAX) { kind = 0; pb = s * vb; info[5] = pb; }
+            const double plo = info[8], phi = info[11];
+            if (plo == plo && (kind < 0 || s * plo > s * pb)) { kind = 1; pb = plo; }
+            if (phi == phi && (kind < 0 || s * phi > s * pb)) { kind = 2; pb = phi; }
+        }
+        info[1] = pb;
+        info[12] = (double)kind;
+        a.axbd[0] = pa;
+        a.axbd[1] = pb;
+        const bool plasma = kind >= 0 && s * (pa - pb) > 0.0;
+        if (!plasma) atomicOr(a.status, EFIT_ST_NOPLASMA);
+        a.cnt[1] = plasma ? (unsigned)g0 : UINT_MAX;
+        a.cnt[0] = 0u;    // candidate counter and non-finite flag ready for the next launch
+        a.cnt[2] = 0u;
+        *a.ticket = 0u;
+    }
+}
+
+// bits[i][k] bit b = node (i, 32k + b) is in the limiter with 0 <= psihat < 1 (one warp per word)
+__global__ void __launch_bounds__(256) k_steps_bits(const double* __restrict__ psi, const uint8_t* __restrict__ inlim,
+                                                   int nw, int nh, int W, const double* __restrict__ axbd,
+                                                   uint32_t* __restrict__ bits) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    const long long word = (long long)blockIdx.x * 8 + (threadIdx.x >> 5);
+    if (word >= (long long)nw * W) return;
+    const int i = (int)(word / W), k = (int)(word - (word / W) * W);
+    const int j = 32 * k + (threadIdx.x & 31);
+    const double pa = __ldcg(axbd), pb = __ldcg(axbd + 1);
+    bool in = false;
+    if (j < nh) {
+        const long long g = (long long)i * nh + j;
+        if (__ldg(inlim + g)) {
+            const double h = (__ldcg(psi + g) - pa) / (pb - pa);
+            in = h >= 0.0 && h < 1.0;
+        }
+    }
+    const uint32_t b = __ballot_sync(0xffffffffu, in);
+    if ((threadIdx.x & 31) == 0) bits[word] = b;
+}
+
+// run fill within one 32-bit word, upwards in bit index: every bit of c connected through a run
+// of c's bits to a seed bit of x (x subset of c); the carry out says the fill reached bit 31
+__device__ __forceinline__ uint32_t fill_up(uint32_t c, uint32_t x, uint32_t& carry) {
+    const unsigned long long sum = (unsigned long long)c + x;
+    carry = (uint32_t)(sum >> 32);
+    return ((((uint32_t)sum) ^ c) & c) | x;
+}
+
+template <bool CSMEM>
+__global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(const uint32_t* __restrict__ bits_g, int nw, int nh,
+                                                               int W, const unsigned* __restrict__ cnt,
+                                                               uint8_t* __restrict__ mask, double* __restrict__ info,
+                                                               int* status) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    extern __shared__ uint32_t sm[];
+    const int nseg = (nw + kSegRows - 1) / kSegRows;
+    uint32_t* R = sm;                                  // [nw][W] reached
+    uint32_t* Cs = sm + (size_t)nw * W;                // [nw][W] candidates (CSMEM)
+    uint32_t* G = Cs + (CSMEM ? (size_t)nw * W : 0);   // [nseg][W] segment results
+    uint32_t* P = G + (size_t)nseg * W;                // [nseg][W] segment pass-through
+    uint32_t* I = P + (size_t)nseg * W;                // [nseg][W] segment carry-in
+    __shared__ int cnt_s[32];
+    const uint32_t* C = CSMEM ? Cs : bits_g;
+    const int tid = threadIdx.x;
+    const long long nwords = (long long)nw * W;
+    const unsigned g0 = __ldcg(cnt + 1);
+    for (long long q = tid; q < nwords; q += kFillThreads) {
+        R[q] = 0u;
+        if (CSMEM) Cs[q] = __ldcg(bits_g + q);
+    }
+    __syncthreads();
+    if (tid == 0 && g0 != UINT_MAX) {
+        const int i0 = (int)(g0 / (unsigned)nh), j0 = (int)(g0 - (g0 / (unsigned)nh) * (unsigned)nh);
+        const uint32_t bit = 1u << (j0 & 31);
+        const long long q = (long long)i0 * W + (j0 >> 5);
+        const uint32_t cw = CSMEM ? C[q] : __ldcg(C + q);
+        R[q] = cw & bit;
+    }
+    __syncthreads();
+    auto ldc = [&](long long q) -> uint32_t { return CSMEM ? C[q] : __ldcg(C + q); };
+    const int nitem = nseg * W;
+    for (;;) {
+        bool changed = false;
+        // rows: runs along Z (bits), right then left, carries across words
+        for (int i = tid; i < nw; i += kFillThreads) {
+            uint32_t* r = R + (long long)i * W;
+            const long long cb = (long long)i * W;
+            uint32_t carry = 0u;
+            for (int k = 0; k < W; ++k) {
+                const uint32_t c = ldc(cb + k), old = r[k];
+                const uint32_t x = old | (carry & c & 1u);
+                const uint32_t f = fill_up(c, x, carry);
+                if (f != old) { r[k] = f; changed = true; }
+            }
+            carry = 0u;
+            for (int k = W - 1; k >= 0; --k) {
+                const uint32_t c = __brev(ldc(cb + k)), old = r[k];
+                const uint32_t x = __brev(old) | (carry & c & 1u);
+                const uint32_t f = __brev(fill_up(c, x, carry));
+                if (f != old) { r[k] = f; changed = true; }
+            }
+        }
+        __syncthreads();
+        // columns: runs along R (rows), down then up, by segments of kSegRows rows
+        for (int dir = 0; dir < 2; ++dir) {
+            for (int it = tid; it < nitem; it += kFillThreads) {  // segment transfer (G, P) without input
+                const int sg = it / W, k = it - (it / W) * W;
+                const int i0 = sg * kSegRows, i1 = min(nw, i0 + kSegRows);
+                uint32_t prev = 0u, pass = 0xffffffffu;
+                for (int q = 0; q < i1 - i0; ++q) {
+                    const int i = dir == 0 ? i0 + q : i1 - 1 - q;
+                    const uint32_t c = ldc((long long)i * W + k);
+                    prev = R[(long long)i * W + k] | (c & prev);
+                    pass &= c;
+                }
+                G[it] = prev;
+                P[it] = pass;
+            }
+            __syncthreads();
+            for (int k = tid; k < W; k += kFillThreads) {  // carries across segments
+                uint32_t in = 0u;
+                for (int q = 0; q < nseg; ++q) {
+                    const int sg = dir == 0 ? q : nseg - 1 - q;
+                    I[sg * W + k] = in;
+                    in = G[sg * W + k] | (P[sg * W + k] & in);
+                }
+            }
+            __syncthreads();
+            for (int it = tid; it < nitem; it += kFillThreads) {
+                const int sg = it / W, k = it - (it / W) * W;
+                const int i0 = sg * kSegRows, i1 = min(nw, i0 + kSegRows);
+                uint32_t prev = I[it];
+                for (int q = 0; q < i1 - i0; ++q) {
+                    const int i = dir == 0 ? i0 + q : i1 - 1 - q;
+                    const long long p = (long long)i * W + k;
+                    const uint32_t old = R[p];
+                    const uint32_t v = old | (ldc(p) & prev);
+                    if (v != old) { R[p] = v; changed = true; }
+                    prev = v;
+                }
+            }
+            __syncthreads();
+        }
+        if (!__syncthreads_or(changed)) break;
+    }
+    // byte mask and its count
+    int c = 0;
+    const long long n = (long long)nw * nh;
+    for (long long g = tid; g < n; g += kFillThreads) {
+        const int i = (int)(g / nh), j = (int)(g - (g / nh) * nh);
+        const uint8_t m = (uint8_t)((R[(long long)i * W + (j >> 5)] >> (j & 31)) & 1u);
+        mask[g] = m;
+        c += m;
+    }
+    c = __reduce_add_sync(0xffffffffu, c);
+    if ((tid & 31) == 0) cnt_s[tid >> 5] = c;
+    __syncthreads();
+    if (tid == 0) {
+        int t = 0;
+        for (int q = 0; q < kFillThreads / 32; ++q) t += cnt_s[q];
+        info[13] = (double)t;
+        if (t == 0) atomicOr(status, EFIT_ST_NOPLASMA);
+    }
+}
+
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl_s(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args&&... args) {
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+
+}  // namespace
+
+int steps_words(int nh) { return (nh + 31) / 32; }
+int steps_cand_cap(int nw, int nh) { return ((nw + 1) / 2) * ((nh + 1) / 2); }
+
+// dynamic shared memory of k_steps_fill; the candidate bitmap is staged when both maps fit
+size_t steps_fill_smem(int nw, int nh, bool* cand_smem) {
+    const size_t W = (size_t)steps_words(nh), nseg = (size_t)(nw + kSegRows - 1) / kSegRows;
+    const size_t base = 4 * (W * nw + 3 * nseg * W);
+    const bool both = base + 4 * W * nw <= 200 * 1024;
+    if (cand_smem) *cand_smem = both;
+    return both ? base + 4 * W * nw : base;
+}
+
+cudaError_t prepare_steps(Ctx& c, int smem_optin) {
+    bool cs;
+    const size_t sm = steps_fill_smem(c.nw, c.nh, &cs);
+    if ((long long)sm > smem_optin) return cudaSuccess;  // reported by efit_set_steps
+    cudaError_t e = cudaFuncSetAttribute((const void*)k_steps_fill<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e) return e;
+    return cudaFuncSetAttribute((const void*)k_steps_fill<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+}
+
+// full steps_ of psi: c.axbd, c.st_info, c.pmask (the plasma mask used downstream in place of the
+// limiter flags)
+cudaError_t launch_steps(Ctx& c, const double* psi, cudaStream_t s) {
+    ScanArgs a;
+    a.psi = psi; a.inlim = c.inlim; a.nw = c.nw; a.nh = c.nh; a.sgn = c.ip_sign;
+    a.rmin = c.rmin; a.dr = c.dr; a.zmin = c.zmin; a.dz = c.dz; a.lim = c.lim; a.n_lim = c.n_lim;
+    a.part = c.norm_part; a.ticket = c.tickets + 2; a.cand = c.st_cand; a.cnt = c.st_cnt;
+    a.cap = steps_cand_cap(c.nw, c.nh); a.info = c.st_info; a.axbd = c.axbd; a.status = c.status;
+    cudaError_t e = launch_pdl_s(k_steps_scan, dim3(c.t.red_blocks), dim3(256), 0, s, a);
+    if (e) return e;
+    const int W = steps_words(c.nh);
+    const long long nwords = (long long)c.nw * W;
+    e = launch_pdl_s(k_steps_bits, dim3((unsigned)((nwords + 7) / 8)), dim3(256), 0, s, psi, c.inlim, c.nw, c.nh, W,
+                     (const double*)c.axbd, c.st_bits);
+    if (e) return e;
+    bool cs;
+    const size_t sm = steps_fill_smem(c.nw, c.nh, &cs);
+    if (cs)
+        e = launch_pdl_s(k_steps_fill<true>, dim3(1), dim3(kFillThreads), sm, s, (const uint32_t*)c.st_bits, c.nw, c.nh,
+                         W, (const unsigned*)c.st_cnt, c.pmask, c.st_info, c.status);
+    else
+        e = launch_pdl_s(k_steps_fill<false>, dim3(1), dim3(kFillThreads), sm, s, (const uint32_t*)c.st_bits, c.nw,
+                         c.nh, W, (const unsigned*)c.st_cnt, c.pmask, c.st_info, c.status);
+    if (e) return e;
+    return cudaGetLastError();
+}
+
+// O8 byte mask (limiter rule) for efit_normalize in EFIT_STEPS_LIMITER mode
+__global__ void k_mask_o8(const double* __restrict__ psi, const uint8_t* __restrict__ inlim, int n,
+                          const double* __restrict__ axbd, uint8_t* __restrict__ mask) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    const double pa = __ldcg(axbd), pb = __ldcg(axbd + 1);
+    for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += gridDim.x * blockDim.x) {
+        bool m = false;
+        if (inlim[g]) {
+            const double h = (__ldcg(psi + g) - pa) / (pb - pa);
+            m = h >= 0.0 && h < 1.0;
+        }
+        mask[g] = (uint8_t)m;
+    }
+}
+
+cudaError_t launch_mask_o8(Ctx& c, const double* psi, uint8_t* mask, cudaStream_t s) {
+    const int n = c.nw * c.nh;
+    cudaError_t e = launch_pdl_s(k_mask_o8, dim3((n + 255) / 256 < 1184 ? (n + 255) / 256 : 1184), dim3(256), 0, s, psi,
+                                 (const uint8_t*)c.inlim, n, (const double*)c.axbd, mask);
+    if (e) return e;
+    return cudaGetLastError();
+}
+
+}  // namespace efit

@@ -62,7 +62,7 @@ def test_workspace_bytes_scales(efit):
     assert 8.6e9 < sizes["C5"] < 9.9e9
     c = _cfg(synth.config("C4"))
     otf = efit.efit_workspace_bytes(c.grid, c.basis, c.geom, c.dist, efit.EFIT_GREEN_ONTHEFLY)
-    assert otf < 0.3e9
+    assert otf < 0.32e9  # Gd (253 MB) + per-iteration scratch, no boundary table
 
 
 @pytest.mark.parametrize("mutate,expect", [
