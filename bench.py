@@ -60,6 +60,13 @@ def parse():
     ap.add_argument("--no-profile", action="store_true",
                     help="time graph replays without per-kernel events (no roofline breakdown)")
     ap.add_argument("--reps", type=int, default=5, help="timed repetitions of K steps; value = the median")
+    ap.add_argument("--rule", default="limiter", choices=["limiter", "full"],
+                    help="steps_ rule (include/efit.h efit_set_steps): limiter = O8 limited-plasma rule, "
+                         "full = bicubic axis, X-point boundary, connectivity-filtered mask (SURVEY 8(f) f3)")
+    ap.add_argument("--shape", default=None, choices=["limited", "diverted"],
+                    help="twin equilibrium: the limited Solov'ev (default for --rule limiter) or the lower-single-"
+                         "null Solov'ev (default for --rule full; its Picard loop is vertically unstable, so psi is "
+                         "restored to the start before every timed iteration, DESIGN.md R4)")
     ap.add_argument("--loop", action="store_true",
                     help="full fitting loop (P:L103, L287) on the noise-free twin from a 1%% perturbed start: "
                          "iterations to eps < 1e-5, eps trajectory, time to solution, |c - c_true| (SURVEY 8(d) C2)")
@@ -146,14 +153,18 @@ class Clocks:
 
 # ----------------------------------------------------------------------------- GPU arm
 
-def twin_inputs(ctx, cfg, torch, dev):
+def twin_inputs(ctx, cfg, torch, dev, shape="limited"):
     """Synthetic twin built with the product API: I_S = current(psi_S, c_true),
     psi_ext = psi_S - solve(boundary(I_S), I_S), y = R(psi_S) c_true + noise.
     With the in-library NCCL exchange (world > 1) every call returns replicated outputs."""
     import paper_conf_sc_anteparawkbml23_b200 as efit
     T = lambda a: torch.tensor(np.asarray(a, dtype=np.float64), device=dev)
-    psi_s = T(synth.solovev_psi(cfg.grid))
-    ct = T(synth.c_true(cfg.basis))
+    if shape == "diverted":
+        psi_s = T(synth.solovev_diverted_psi(cfg.grid))
+        ct = T(synth.c_true(cfg.basis, sol_c=synth.DIV_C))
+    else:
+        psi_s = T(synth.solovev_psi(cfg.grid))
+        ct = T(synth.c_true(cfg.basis))
     I_s = ctx.current(psi_s, ct)
     psib = ctx._t(ctx.n_edge)
     resp = ctx._t(ctx.ndiag * ctx.nbasis)
@@ -169,7 +180,11 @@ def twin_inputs(ctx, cfg, torch, dev):
         if b > a:
             sigma[a:b] = 1e-3 * y[a:b].abs().max()
     y = y + sigma * T(synth.noise(ctx.ndiag, seed=1))
-    psi0 = T(synth.perturbed_psi(cfg.grid, seed=5, rel=1e-3))
+    if shape == "diverted":
+        ps = synth.solovev_diverted_psi(cfg.grid)
+        psi0 = T(ps + 1e-4 * (ps.max() - ps.min()) * synth.smooth_modes(cfg.grid, 5) / 3.0)
+    else:
+        psi0 = T(synth.perturbed_psi(cfg.grid, seed=5, rel=1e-3))
     return psi0, psi_ext.contiguous(), y.contiguous(), sigma.contiguous()
 
 
@@ -355,7 +370,7 @@ def barrier(use_dist, torch):
     torch.cuda.synchronize()
 
 
-def capture_steps(ctx, K, chunk, psi, psi_ext, meas, sigma, coef, chi2, eps, torch):
+def capture_steps(ctx, K, chunk, psi, psi_ext, meas, sigma, coef, chi2, eps, torch, restore=None):
     """K chained fit iterations captured into CUDA graphs of <= chunk steps (efit_fit_steps: only
     the first iteration of a graph normalises psi; the host is out of the timed loop).  Thread-local
     capture: with the in-library NCCL exchange, NCCL's proxy thread may call CUDA concurrently."""
@@ -365,7 +380,12 @@ def capture_steps(ctx, K, chunk, psi, psi_ext, meas, sigma, coef, chi2, eps, tor
         n = min(chunk, K - done)
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=cap, capture_error_mode="thread_local"):
-            ctx.fit_steps(n, psi, psi_ext, meas, sigma, coef, chi2, eps)
+            if restore is None:
+                ctx.fit_steps(n, psi, psi_ext, meas, sigma, coef, chi2, eps)
+            else:  # every iteration from the same start (a 2.1 MB device copy before each)
+                for _ in range(n):
+                    psi.copy_(restore)
+                    ctx.fit_steps(1, psi, psi_ext, meas, sigma, coef, chi2, eps)
         graphs.append(g)
         done += n
     torch.cuda.synchronize()
@@ -388,10 +408,17 @@ def gpu_arm(args, rank, world, local):
                            nccl_id=nccl_id)
     torch.cuda.synchronize()
     init_s = time.time() - t0
-    psi0, psi_ext, meas, sigma = twin_inputs(ctx, cfg, torch, dev)
+    full = args.rule == "full"
+    shape = args.shape or ("diverted" if full else "limited")
+    if full:
+        ctx.set_steps(efit.EFIT_STEPS_FULL)
+    psi0, psi_ext, meas, sigma = twin_inputs(ctx, cfg, torch, dev, shape)
+    restore = psi0 if shape == "diverted" else None
     psi = psi0.clone()
     coef, chi2, eps = ctx._t(ctx.nbasis), ctx._t(1), ctx._t(1)
     for _ in range(args.warmup):
+        if restore is not None:
+            psi.copy_(restore)
         ctx.fit_step(psi, psi_ext, meas, sigma, coef, chi2, eps)
     torch.cuda.synchronize()
     st = ctx.status()
@@ -404,10 +431,10 @@ def gpu_arm(args, rank, world, local):
     # per-kernel event marks (every 10th step) for the breakdown and the roofline.
     K = args.steps
     stream = torch.cuda.current_stream()
-    graphs = capture_steps(ctx, K, 500, psi, psi_ext, meas, sigma, coef, chi2, eps, torch)
+    graphs = capture_steps(ctx, K, 500, psi, psi_ext, meas, sigma, coef, chi2, eps, torch, restore)
     if not args.no_profile:
         efit.efit_profile_begin(ctx.handle, (K + 9) // 10, 10)
-        graphs_prof = capture_steps(ctx, K, 500, psi, psi_ext, meas, sigma, coef, chi2, eps, torch)
+        graphs_prof = capture_steps(ctx, K, 500, psi, psi_ext, meas, sigma, coef, chi2, eps, torch, restore)
     clocks = Clocks(local) if rank == 0 else None
     if clocks:
         clocks.start()
@@ -514,12 +541,12 @@ def gpu_arm(args, rank, world, local):
 
     # ---------------- e2e: host buffers through the C ABI (efit_fit_host), copies inside the timed region
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and restore is None:
         e2e = e2e_measure(ctx, psi0, psi_ext, meas, sigma, K_e2e=min(K, 400), torch=torch, dev=dev,
                           use_dist=use_dist)
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not full:
         cpu = cpu_baseline(args.config)
 
     # our kernels per step (ncu launch list, profiles/): response (basis fused), resp_reduce, lsq,
@@ -527,6 +554,8 @@ def gpu_arm(args, rank, world, local):
     # tridiag, dst_inv; + k_normalize at the start of every captured graph
     per_step = 12 + (1 if sym_mode else 0)
     launches = per_step * K + len(graphs)
+    if full:  # steps_ (3 kernels) before every iteration instead of once per graph
+        launches = (per_step + 3) * K
     if rank == 0:
         par = "single GPU"
         if use_dist:
@@ -539,6 +568,10 @@ def gpu_arm(args, rank, world, local):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"{args.config}: {cfg.description}", "grid": f"{N}x{N}",
                        "ndiag": ndiag, "nbasis": cfg.basis.nbasis, "green_mode": args.mode,
+                       "steps_rule": args.rule, "equilibrium": shape,
+                       **({"psi_restored_each_step": "psi <- psi_start (device copy) before every timed "
+                           "iteration: the diverted Picard loop is vertically unstable (DESIGN.md R4)"}
+                          if restore is not None else {}),
                        "parallelism": par,
                        "l2": f"inputs larger than L2 ({tb_bytes / 1e9:.3f} GB boundary table + {gd_bytes / 1e9:.3f} GB "
                              f"Gd streamed per step and rank vs 126 MB L2): no flush",
@@ -602,6 +635,8 @@ def loop_arm(args, rank, world, local):
     dev = torch.device("cuda", local)
     cfg = synth.config(args.config)
     ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=MODES[args.mode], device=dev)
+    if args.rule == "full":  # the limited twin under the full steps_ rule (the diverted loop is unstable)
+        ctx.set_steps(efit.EFIT_STEPS_FULL)
     T = lambda a: torch.tensor(np.asarray(a, dtype=np.float64), device=dev)
     psi_s = T(synth.solovev_psi(cfg.grid))
     ct = T(synth.c_true(cfg.basis))
@@ -652,7 +687,7 @@ def loop_arm(args, rank, world, local):
     rate = float(np.exp(np.mean(np.log(np.array(traj2[-20:])[1:] / np.array(traj2[-20:])[:-1])))) if len(traj2) > 21 else None
     print(json.dumps({"metric": "full fitting loop to eps < 1e-5 (P:L103, L287)", "config": {
         "workload": f"{args.config}: {cfg.description}", "grid": f"{cfg.grid.nw}x{cfg.grid.nh}",
-        "green_mode": args.mode, "start": "psi_S + 1% smooth modes (seed 5)", "twin": "noise-free, edge-vanishing profile"},
+        "green_mode": args.mode, "steps_rule": args.rule, "start": "psi_S + 1% smooth modes (seed 5)", "twin": "noise-free, edge-vanishing profile"},
         "status": st_code, "to_1e-5": out5, "to_1e-10": out10, "contraction_rate": rate,
         "eps_trajectory": [float(f"{e:.3e}") for e in traj]}), flush=True)
     ctx.close()

@@ -36,6 +36,11 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str = LIB
     for src in SOURCES:
         tag = "" if out == LIB else "." + os.path.basename(out).replace(".so", "")
         obj = os.path.join(CSRC, src.replace(".cu", tag + ".o"))
+        hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", "efit.h"), __file__]
+        if (not force and not defines and os.path.exists(obj) and
+                all(os.path.getmtime(obj) > os.path.getmtime(d) for d in hdrs + [os.path.join(CSRC, src)])):
+            objs.append(obj)  # object up to date (incremental build)
+            continue
         cmd = ["nvcc", *NVCC_FLAGS, *SOURCE_FLAGS.get(src, []), *["-D" + d for d in defines], "-c",
                os.path.join(CSRC, src), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)

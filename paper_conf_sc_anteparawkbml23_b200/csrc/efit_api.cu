@@ -330,7 +330,7 @@ static size_t carve_scratch(Ctx& c, Take& take, size_t& off, bool batch) {
     c.st_info = (double*)take(sizeof(double) * 16);
     c.st_cnt = (unsigned*)take(sizeof(unsigned) * 4);
     c.st_cand = (double2*)take(sizeof(double2) * (size_t)efit::steps_cand_cap(c.nw, c.nh));
-    c.st_bits = (uint32_t*)take(sizeof(uint32_t) * (size_t)c.nw * efit::steps_words(c.nh));
+    c.st_bits = (uint64_t*)take(sizeof(uint64_t) * (size_t)c.nw * efit::steps_words(c.nh));
     return (size_t)round_up((long long)off, 256);
 }
 
@@ -603,7 +603,7 @@ extern "C" int efit_set_steps(efit_ctx* h, int32_t steps_mode) {
         if (c.nslice > 0) return fail(&c, EFIT_E_STATE, "EFIT_STEPS_FULL with a batch attached");
         int optin = 0;
         cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, c.device);
-        if (c.nw < 6 || c.nh < 6 || efit::steps_fill_smem(c.nw, c.nh, nullptr) > (size_t)optin)
+        if (c.nw < 6 || c.nh < 6 || efit::steps_words(c.nh) > 32 || efit::steps_fill_smem(c.nw, c.nh, nullptr) > (size_t)optin)
             return fail(&c, EFIT_E_INVAL, "EFIT_STEPS_FULL needs 6 <= nw, nh and a plasma bitmap in shared memory (nw*nh <= ~1025^2)");
     }
     if (c.steps != steps_mode) drop_fit_graphs(c);

@@ -129,7 +129,7 @@ struct Ctx {
     double* st_info;    // [16]     axis / X-point / boundary record (efit_normalize layout)
     unsigned* st_cnt;   // [4]      candidate count, axis node, non-finite flag
     double2* st_cand;   // [steps_cand_cap] X-point candidates (|grad|^2, g)
-    uint32_t* st_bits;  // [nw][steps_words] candidate bitmap
+    uint64_t* st_bits;  // [nw][steps_words] candidate bitmap, then the plasma component (64-bit words)
     void* comm;         // ncclComm_t or nullptr
     int nccl_err;       // last ncclResult_t != ncclSuccess of xch_allreduce (reported as EFIT_E_NCCL)
 

@@ -186,36 +186,30 @@ __device__ double bilin(const Field& F, double rmin, double dr, double zmin, dou
     return ((w00 * F.at(i, j) + w10 * F.at(i + 1, j)) + w01 * F.at(i, j + 1)) + w11 * F.at(i + 1, j + 1);
 }
 
-struct ScanArgs {
+struct StepsArgs {
     const double* psi;
     const uint8_t* inlim;
     int nw, nh, sgn;
     double rmin, dr, zmin, dz;
     const double* lim;
     int n_lim;
-    double* part;        // [gridDim.x][2] (s psi, g) argmax partials
-    unsigned* ticket;
-    double2* cand;       // [cap] (|grad|^2, g)
-    unsigned* cnt;       // [0] candidates found, [1] axis node g0 (or UINT_MAX), [2] non-finite psi seen
+    double* part;        // [red_blocks][2] (s psi, g) argmax partials of k_steps_scan
+    int nparts;
+    double2* cand;       // [cap] X-point candidates (|grad|^2, g)
+    unsigned* cnt;       // [0] candidates found, [1] axis node g0 (UINT_MAX: no plasma), [2] non-finite psi seen
     int cap;
     double* info;        // [16] (efit.h efit_normalize layout)
     double* axbd;        // [2]
     int* status;
 };
 
-__global__ void __launch_bounds__(256) k_steps_scan(ScanArgs a) {
+// All CTAs: per-block in-limiter argmax of s psi (ties: lowest g), X-point candidates appended to a
+// list (at most one per 2 x 2 node block: two 8-neighbours cannot both be local minima under the
+// strict/non-strict tie rule, so the list never overflows its ceil(nw/2) ceil(nh/2) slots).
+__global__ void __launch_bounds__(256) k_steps_scan(StepsArgs a) {
     asm volatile("griddepcontrol.wait;" ::: "memory");
     __shared__ double sv[8];
     __shared__ long long si[8];
-    __shared__ bool last;
-    __shared__ double selk[kMaxXCand];
-    __shared__ long long selg[kMaxXCand];
-    __shared__ double res[kMaxXCand + 1][5];
-    __shared__ int rconv[kMaxXCand + 1];
-    __shared__ double lv[8];
-    __shared__ long long li[8];
-    __shared__ double zlim[2];
-    __shared__ int nsel_s, bad_s;
     const Field F{a.psi, a.nw, a.nh};
     const int n = a.nw * a.nh, nh = a.nh;
     const double s = (double)a.sgn;
@@ -223,10 +217,9 @@ __global__ void __launch_bounds__(256) k_steps_scan(ScanArgs a) {
     long long bi = LLONG_MAX;
     bool bad = false;
     for (int g = blockIdx.x * blockDim.x + threadIdx.x; g < n; g += gridDim.x * blockDim.x) {
-        const double p = __ldcg(a.psi + g);
-        const uint8_t in = __ldg(a.inlim + g);
+        const double p = __ldg(a.psi + g);
         if (!isfinite(p)) bad = true;
-        if (in) {
+        if (__ldg(a.inlim + g)) {
             am_merge(best, bi, s * p, (long long)g);
             const int i = g / nh, j = g - (g / nh) * nh;
             double key;
@@ -236,7 +229,6 @@ __global__ void __launch_bounds__(256) k_steps_scan(ScanArgs a) {
             }
         }
     }
-    __threadfence();  // this thread's candidate entries before the block's ticket
     if (__syncthreads_or(bad) && threadIdx.x == 0) {
         atomicOr(a.status, EFIT_ST_NONFINITE);
         atomicOr(a.cnt + 2, 1u);
@@ -249,56 +241,92 @@ __global__ void __launch_bounds__(256) k_steps_scan(ScanArgs a) {
         for (int q = 1; q < 8; ++q) am_merge(best, bi, sv[q], si[q]);
         a.part[2 * blockIdx.x] = best;
         a.part[2 * blockIdx.x + 1] = (double)bi;
-        __threadfence();
-        last = (atomicAdd(a.ticket, 1u) == gridDim.x - 1);
     }
-    __syncthreads();
-    if (!last) return;
-    __threadfence();
-    // ---- last CTA: (3) axis node, (4) X-point candidates, Newton searches
-    best = -DBL_MAX; bi = LLONG_MAX;
-    for (int b = threadIdx.x; b < (int)gridDim.x; b += blockDim.x)
-        am_merge(best, bi, __ldcg(a.part + 2 * b), (long long)__ldcg(a.part + 2 * b + 1));
+}
+
+constexpr int kFinalWarps = kMaxXCand + 1;  // warp 0: the axis, warps 1..8: X-point candidates
+
+// One CTA: (3) axis, (4) X-points, (5) limiter value, (6) boundary.  Newton searches run one per
+// warp (lane 0) concurrently; the in-limiter test of an X-point is the parity of the crossings over
+// the limiter edges (an order-independent count: the same decision as the sequential even-odd rule).
+__global__ void __launch_bounds__(32 * kFinalWarps) k_steps_final(StepsArgs a) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    __shared__ double sv[kFinalWarps];
+    __shared__ long long si[kFinalWarps];
+    __shared__ long long selg[kMaxXCand];
+    __shared__ double res[kFinalWarps][4];  // xt, xu, p, det (after Newton)
+    __shared__ int racc[kFinalWarps];        // converged (+ saddle, near, inside for candidates)
+    __shared__ double zlim[2];
+    __shared__ int nsel_s;
+    const Field F{a.psi, a.nw, a.nh};
+    const int nh = a.nh, tid = threadIdx.x, w = tid >> 5, l = tid & 31;
+    const double s = (double)a.sgn;
+    double best = -DBL_MAX;
+    long long bi = LLONG_MAX;
+    for (int b = tid; b < a.nparts; b += blockDim.x) am_merge(best, bi, a.part[2 * b], (long long)a.part[2 * b + 1]);
     am_warp(best, bi);
     if (l == 0) { sv[w] = best; si[w] = bi; }
-    if (threadIdx.x == 0) { nsel_s = 0; bad_s = *((volatile unsigned*)(a.cnt + 2)) ? 1 : 0; }
+    if (tid == 0) nsel_s = 0;
     __syncthreads();
-    if (threadIdx.x == 0) {
-        for (int q = 1; q < 8; ++q) am_merge(best, bi, sv[q], si[q]);
+    if (tid == 0) {
+        for (int q = 1; q < kFinalWarps; ++q) am_merge(best, bi, sv[q], si[q]);
         si[0] = bi;
     }
-    const unsigned ncand_all = *((volatile unsigned*)a.cnt);
+    const unsigned ncand_all = a.cnt[0];
     const int ncand = (int)(ncand_all < (unsigned)a.cap ? ncand_all : (unsigned)a.cap);
-    // the 8 smallest (|grad|^2, g): rank of each candidate in that total order
-    for (int q = threadIdx.x; q < ncand; q += blockDim.x) {
-        const double2 cq = __ldcg(a.cand + q);
+    for (int q = tid; q < ncand; q += blockDim.x) {  // the 8 smallest (|grad|^2, g): ranks in that order
+        const double2 cq = a.cand[q];
         int rank = 0;
         for (int r = 0; r < ncand && rank < kMaxXCand; ++r) {
-            const double2 cr = __ldcg(a.cand + r);
+            const double2 cr = a.cand[r];
             if (cr.x < cq.x || (cr.x == cq.x && cr.y < cq.y)) ++rank;
         }
-        if (rank < kMaxXCand) { selk[rank] = cq.x; selg[rank] = (long long)cq.y; atomicMax(&nsel_s, rank + 1); }
+        if (rank < kMaxXCand) { selg[rank] = (long long)cq.y; atomicMax(&nsel_s, rank + 1); }
     }
     __syncthreads();
     const long long g0 = si[0];
     const int nsel = nsel_s;
-    const bool ok0 = (g0 != LLONG_MAX) && !bad_s;
-    // thread 0: the axis; threads 1..nsel: the X-point candidates (concurrently)
-    if (ok0 && threadIdx.x <= nsel) {
-        const long long gs = threadIdx.x == 0 ? g0 : selg[threadIdx.x - 1];
+    const bool ok0 = (g0 != LLONG_MAX) && a.cnt[2] == 0u;
+    if (ok0 && w <= nsel) {
+        const long long gs = w == 0 ? g0 : selg[w - 1];
         const int i = (int)(gs / nh), j = (int)(gs - (gs / nh) * nh);
-        double o[5];
-        bool conv = false;
-        if (threadIdx.x > 0 || (a.nw >= 4 && nh >= 4 && i >= 1 && i <= a.nw - 2 && j >= 1 && j <= nh - 2))
-            conv = newton_stationary(F, (double)i, (double)j, o);
-        rconv[threadIdx.x] = conv ? 1 : 0;
-        for (int k = 0; k < 5; ++k) res[threadIdx.x][k] = o[k];
+        int acc = 0;
+        double o[5] = {0.0, 0.0, 0.0, 0.0, 0.0};
+        if (l == 0) {
+            if (w > 0 || (a.nw >= 4 && nh >= 4 && i >= 1 && i <= a.nw - 2 && j >= 1 && j <= nh - 2)) {
+                const bool conv = newton_stationary(F, (double)i, (double)j, o);
+                if (w == 0)
+                    acc = conv ? 1 : 0;
+                else
+                    acc = (conv && o[3] < 0.0 && fabs(o[0] - (double)i) <= 1.5 && fabs(o[1] - (double)j) <= 1.5) ? 1 : 0;
+            }
+        }
+        acc = __shfl_sync(0xffffffffu, acc, 0);
+        if (w > 0 && acc) {  // inside the limiter: parity of the edge crossings (O7 rule), lanes over edges
+            const double Rx = __shfl_sync(0xffffffffu, a.rmin + o[0] * a.dr, 0);
+            const double Zx = __shfl_sync(0xffffffffu, a.zmin + o[1] * a.dz, 0);
+            unsigned par = 0u;
+            for (int k = l; k < a.n_lim; k += 32) {
+                const int k1 = (k + 1 == a.n_lim) ? 0 : k + 1;
+                const double r0 = a.lim[k], z0 = a.lim[a.n_lim + k], r1 = a.lim[k1], z1 = a.lim[a.n_lim + k1];
+                if ((z0 > Zx) != (z1 > Zx)) {
+                    const double x = ((r1 - r0) * (Zx - z0)) / (z1 - z0) + r0;
+                    if (Rx < x) par ^= 1u;
+                }
+            }
+            acc = (__popc(__ballot_sync(0xffffffffu, par != 0u)) & 1) ? 1 : 0;
+        }
+        if (l == 0) {
+            racc[w] = acc;
+            res[w][0] = o[0]; res[w][1] = o[1]; res[w][2] = o[2]; res[w][3] = o[3];
+            if (w == 0) res[0][3] = o[3] > 0.0 && a.sgn * o[4] < 0.0 ? 1.0 : 0.0;  // maximum of s psi
+        }
     }
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (tid == 0) {
         double* info = a.info;
         for (int k = 0; k < 16; ++k) info[k] = __longlong_as_double(0x7ff8000000000000LL);  // NaN
-        double pa = 0.0, Za = 0.0;
+        double pa = 0.0;
         bool lo = false, hi = false;
         double xlo[3], xhi[3];
         if (ok0) {
@@ -307,27 +335,22 @@ __global__ void __launch_bounds__(256) k_steps_scan(ScanArgs a) {
             pa = p0;
             double xa = (double)i0, ya = (double)j0;
             int ref = 0;
-            const double* o = res[0];
-            if (rconv[0] && o[3] > 0.0 && s * o[4] < 0.0 && fabs(o[0] - (double)i0) <= 1.0 &&
-                fabs(o[1] - (double)j0) <= 1.0 && s * o[2] >= s * p0) {
-                pa = o[2]; xa = o[0]; ya = o[1]; ref = 1;
+            if (racc[0] && res[0][3] == 1.0 && fabs(res[0][0] - (double)i0) <= 1.0 &&
+                fabs(res[0][1] - (double)j0) <= 1.0 && s * res[0][2] >= s * p0) {
+                pa = res[0][2]; xa = res[0][0]; ya = res[0][1]; ref = 1;
             }
-            Za = a.zmin + ya * a.dz;
+            const double Za = a.zmin + ya * a.dz;
             info[0] = pa; info[2] = a.rmin + xa * a.dr; info[3] = Za; info[4] = (double)ref; info[15] = (double)g0;
             info[14] = (double)nsel;
-            for (int q = 0; q < nsel; ++q) {
-                const long long gq = selg[q];
-                const int i = (int)(gq / nh), j = (int)(gq - (gq / nh) * nh);
-                const double* x = res[q + 1];
-                if (!(rconv[q + 1] && x[3] < 0.0 && fabs(x[0] - (double)i) <= 1.5 && fabs(x[1] - (double)j) <= 1.5))
-                    continue;
-                const double Rx = a.rmin + x[0] * a.dr, Zx = a.zmin + x[1] * a.dz;
-                if (!in_polygon(Rx, Zx, a.lim, a.n_lim)) continue;
-                if (!(s * (pa - x[2]) > 0.0)) continue;
+            for (int q = 0; q < nsel; ++q) {  // candidate order (ties: the earlier one)
+                if (!racc[q + 1]) continue;
+                const double px = res[q + 1][2];
+                if (!(s * (pa - px) > 0.0)) continue;
+                const double Rx = a.rmin + res[q + 1][0] * a.dr, Zx = a.zmin + res[q + 1][1] * a.dz;
                 if (Zx < Za) {
-                    if (!lo || s * x[2] > s * xlo[2]) { lo = true; xlo[0] = Rx; xlo[1] = Zx; xlo[2] = x[2]; }
+                    if (!lo || s * px > s * xlo[2]) { lo = true; xlo[0] = Rx; xlo[1] = Zx; xlo[2] = px; }
                 } else if (Zx > Za) {
-                    if (!hi || s * x[2] > s * xhi[2]) { hi = true; xhi[0] = Rx; xhi[1] = Zx; xhi[2] = x[2]; }
+                    if (!hi || s * px > s * xhi[2]) { hi = true; xhi[0] = Rx; xhi[1] = Zx; xhi[2] = px; }
                 }
             }
             if (lo) { info[6] = xlo[0]; info[7] = xlo[1]; info[8] = xlo[2]; }
@@ -335,16 +358,16 @@ __global__ void __launch_bounds__(256) k_steps_scan(ScanArgs a) {
         }
         zlim[0] = lo ? xlo[1] : -DBL_MAX;
         zlim[1] = hi ? xhi[1] : DBL_MAX;
-        res[0][0] = pa;
-        rconv[0] = ok0 ? 1 : 0;
+        res[0][2] = pa;
+        racc[0] = ok0 ? 1 : 0;
     }
     __syncthreads();
-    // ---- (5) limiter value between the X-point heights (ties: lowest vertex)
+    // (5) limiter value between the X-point heights (ties: lowest vertex)
     double vb = -DBL_MAX;
     long long vi = LLONG_MAX;
-    if (rconv[0]) {
+    if (racc[0]) {
         const bool lo = zlim[0] != -DBL_MAX, hi = zlim[1] != DBL_MAX;
-        for (int v = threadIdx.x; v < a.n_lim; v += blockDim.x) {
+        for (int v = tid; v < a.n_lim; v += blockDim.x) {
             const double z = a.lim[a.n_lim + v];
             if (lo && !(z > zlim[0])) continue;
             if (hi && !(z < zlim[1])) continue;
@@ -352,16 +375,17 @@ __global__ void __launch_bounds__(256) k_steps_scan(ScanArgs a) {
         }
     }
     am_warp(vb, vi);
-    if (l == 0) { lv[w] = vb; li[w] = vi; }
     __syncthreads();
-    if (threadIdx.x == 0) {
-        for (int q = 1; q < 8; ++q) am_merge(vb, vi, lv[q], li[q]);
+    if (l == 0) { sv[w] = vb; si[w] = vi; }
+    __syncthreads();
+    if (tid == 0) {
+        for (int q = 1; q < kFinalWarps; ++q) am_merge(vb, vi, sv[q], si[q]);
         double* info = a.info;
-        const double pa = res[0][0];
+        const double pa = res[0][2];
         // (6) boundary: the largest in s of {limiter, lower X, upper X}, ties in that order
         int kind = -1;
         double pb = 0.0;
-        if (rconv[0]) {
+        if (racc[0]) {
             if (vi != LLONG_MAX) { kind = 0; pb = s * vb; info[5] = pb; }
             const double plo = info[8], phi = info[11];
             if (plo == plo && (kind < 0 || s * plo > s * pb)) { kind = 1; pb = plo; }
@@ -374,156 +398,180 @@ __global__ void __launch_bounds__(256) k_steps_scan(ScanArgs a) {
         const bool plasma = kind >= 0 && s * (pa - pb) > 0.0;
         if (!plasma) atomicOr(a.status, EFIT_ST_NOPLASMA);
         a.cnt[1] = plasma ? (unsigned)g0 : UINT_MAX;
-        a.cnt[0] = 0u;    // candidate counter and non-finite flag ready for the next launch
+        a.cnt[0] = 0u;  // candidate counter and non-finite flag ready for the next scan
         a.cnt[2] = 0u;
-        *a.ticket = 0u;
     }
 }
 
-// bits[i][k] bit b = node (i, 32k + b) is in the limiter with 0 <= psihat < 1 (one warp per word)
+// bits[i][k] bit b = node (i, 64k + b) is in the limiter with 0 <= psihat < 1 (one warp per word)
 __global__ void __launch_bounds__(256) k_steps_bits(const double* __restrict__ psi, const uint8_t* __restrict__ inlim,
                                                    int nw, int nh, int W, const double* __restrict__ axbd,
-                                                   uint32_t* __restrict__ bits) {
+                                                   unsigned long long* __restrict__ bits) {
     asm volatile("griddepcontrol.wait;" ::: "memory");
     const long long word = (long long)blockIdx.x * 8 + (threadIdx.x >> 5);
     if (word >= (long long)nw * W) return;
     const int i = (int)(word / W), k = (int)(word - (word / W) * W);
-    const int j = 32 * k + (threadIdx.x & 31);
-    const double pa = __ldcg(axbd), pb = __ldcg(axbd + 1);
-    bool in = false;
-    if (j < nh) {
-        const long long g = (long long)i * nh + j;
-        if (__ldg(inlim + g)) {
-            const double h = (__ldcg(psi + g) - pa) / (pb - pa);
-            in = h >= 0.0 && h < 1.0;
+    const double pa = axbd[0], pb = axbd[1];
+    uint32_t half[2];
+#pragma unroll
+    for (int hh = 0; hh < 2; ++hh) {
+        const int j = 64 * k + 32 * hh + (threadIdx.x & 31);
+        bool in = false;
+        if (j < nh) {
+            const long long g = (long long)i * nh + j;
+            if (__ldg(inlim + g)) {
+                const double h = (__ldg(psi + g) - pa) / (pb - pa);
+                in = h >= 0.0 && h < 1.0;
+            }
         }
+        half[hh] = __ballot_sync(0xffffffffu, in);
     }
-    const uint32_t b = __ballot_sync(0xffffffffu, in);
-    if ((threadIdx.x & 31) == 0) bits[word] = b;
+    if ((threadIdx.x & 31) == 0) bits[word] = (unsigned long long)half[0] | ((unsigned long long)half[1] << 32);
 }
 
-// run fill within one 32-bit word, upwards in bit index: every bit of c connected through a run
-// of c's bits to a seed bit of x (x subset of c); the carry out says the fill reached bit 31
-__device__ __forceinline__ uint32_t fill_up(uint32_t c, uint32_t x, uint32_t& carry) {
-    const unsigned long long sum = (unsigned long long)c + x;
-    carry = (uint32_t)(sum >> 32);
-    return ((((uint32_t)sum) ^ c) & c) | x;
+// run fill upwards in bit index within a 64-bit word: every bit of c connected through a run of c's
+// bits to a seed bit of x (x subset of c); carry = the fill ran out through bit 63
+__device__ __forceinline__ unsigned long long fill_up64(unsigned long long c, unsigned long long x, bool& carry) {
+    const unsigned long long sum = c + x;
+    carry = sum < c;
+    return ((sum ^ c) & c) | x;
 }
 
+// One CTA: bit-parallel flood fill from the axis node in shared memory.  Rounds of (a) runs along Z
+// within each row (one thread per row, carries from word to word) and (b) runs along R within each
+// bit column, down then up (one warp per 64-bit column word; 32 row segments: a sequential pass
+// inside each segment, the segment transfers (G, P) composed by a warp scan, a second pass with the
+// carry-in).  Only rows changed since their last (a) and word columns changed since their last (b)
+// are processed (both passes are idempotent on unchanged data); the fill ends when nothing is dirty.
+// The component is written back over the candidate bitmap (bits_g) with its size.
 template <bool CSMEM>
-__global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(const uint32_t* __restrict__ bits_g, int nw, int nh,
-                                                               int W, const unsigned* __restrict__ cnt,
-                                                               uint8_t* __restrict__ mask, double* __restrict__ info,
-                                                               int* status) {
+__global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long long* __restrict__ bits_g, int nw,
+                                                               int nh, int W, const unsigned* __restrict__ cnt,
+                                                               double* __restrict__ info, int* status) {
     asm volatile("griddepcontrol.wait;" ::: "memory");
-    extern __shared__ uint32_t sm[];
-    const int nseg = (nw + kSegRows - 1) / kSegRows;
-    uint32_t* R = sm;                                  // [nw][W] reached
-    uint32_t* Cs = sm + (size_t)nw * W;                // [nw][W] candidates (CSMEM)
-    uint32_t* G = Cs + (CSMEM ? (size_t)nw * W : 0);   // [nseg][W] segment results
-    uint32_t* P = G + (size_t)nseg * W;                // [nseg][W] segment pass-through
-    uint32_t* I = P + (size_t)nseg * W;                // [nseg][W] segment carry-in
+    extern __shared__ unsigned long long sm[];
+    unsigned long long* R = sm;                                  // [nw][W] reached
+    unsigned long long* Cs = sm + (size_t)nw * W;                // [nw][W] candidates (CSMEM)
+    uint8_t* rdirty = reinterpret_cast<uint8_t*>(sm + (CSMEM ? 2 : 1) * (size_t)nw * W);  // [nw]
+    __shared__ uint8_t cdirty[32];
     __shared__ int cnt_s[32];
-    const uint32_t* C = CSMEM ? Cs : bits_g;
-    const int tid = threadIdx.x;
-    const long long nwords = (long long)nw * W;
-    const unsigned g0 = __ldcg(cnt + 1);
-    for (long long q = tid; q < nwords; q += kFillThreads) {
-        R[q] = 0u;
-        if (CSMEM) Cs[q] = __ldcg(bits_g + q);
+    const unsigned long long* C = CSMEM ? Cs : bits_g;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    constexpr int nwarp = kFillThreads / 32;
+    const int nwords = nw * W;
+    const unsigned g0 = cnt[1];
+    for (int q = tid; q < nwords; q += kFillThreads) {
+        R[q] = 0ull;
+        if (CSMEM) Cs[q] = bits_g[q];
     }
+    for (int i = tid; i < nw; i += kFillThreads) rdirty[i] = 0;
+    if (tid < 32) cdirty[tid] = 0;
     __syncthreads();
     if (tid == 0 && g0 != UINT_MAX) {
         const int i0 = (int)(g0 / (unsigned)nh), j0 = (int)(g0 - (g0 / (unsigned)nh) * (unsigned)nh);
-        const uint32_t bit = 1u << (j0 & 31);
-        const long long q = (long long)i0 * W + (j0 >> 5);
-        const uint32_t cw = CSMEM ? C[q] : __ldcg(C + q);
-        R[q] = cw & bit;
+        const int q = i0 * W + (j0 >> 6);
+        R[q] = C[q] & (1ull << (j0 & 63));
+        rdirty[i0] = 1;
+        cdirty[j0 >> 6] = 1;
     }
     __syncthreads();
-    auto ldc = [&](long long q) -> uint32_t { return CSMEM ? C[q] : __ldcg(C + q); };
-    const int nitem = nseg * W;
+    const int L = (nw + 31) / 32;  // rows per segment
     for (;;) {
-        bool changed = false;
-        // rows: runs along Z (bits), right then left, carries across words
-        for (int i = tid; i < nw; i += kFillThreads) {
-            uint32_t* r = R + (long long)i * W;
-            const long long cb = (long long)i * W;
-            uint32_t carry = 0u;
+        bool work = false;
+        for (int i = tid; i < nw; i += kFillThreads) {  // (a) rows along Z
+            if (!rdirty[i]) continue;
+            rdirty[i] = 0;
+            work = true;
+            unsigned long long* r = R + (size_t)i * W;
+            const unsigned long long* cr = C + (size_t)i * W;
+            bool carry = false;
             for (int k = 0; k < W; ++k) {
-                const uint32_t c = ldc(cb + k), old = r[k];
-                const uint32_t x = old | (carry & c & 1u);
-                const uint32_t f = fill_up(c, x, carry);
-                if (f != old) { r[k] = f; changed = true; }
+                const unsigned long long c = cr[k], old = r[k];
+                const unsigned long long x = old | (carry ? (c & 1ull) : 0ull);
+                const unsigned long long f = fill_up64(c, x, carry);
+                if (f != old) { r[k] = f; cdirty[k] = 1; }
             }
-            carry = 0u;
+            carry = false;
             for (int k = W - 1; k >= 0; --k) {
-                const uint32_t c = __brev(ldc(cb + k)), old = r[k];
-                const uint32_t x = __brev(old) | (carry & c & 1u);
-                const uint32_t f = __brev(fill_up(c, x, carry));
-                if (f != old) { r[k] = f; changed = true; }
+                const unsigned long long c = __brevll(cr[k]), old = r[k];
+                const unsigned long long x = __brevll(old) | (carry ? (c & 1ull) : 0ull);
+                const unsigned long long f = __brevll(fill_up64(c, x, carry));
+                if (f != old) { r[k] = f; cdirty[k] = 1; }
             }
         }
         __syncthreads();
-        // columns: runs along R (rows), down then up, by segments of kSegRows rows
-        for (int dir = 0; dir < 2; ++dir) {
-            for (int it = tid; it < nitem; it += kFillThreads) {  // segment transfer (G, P) without input
-                const int sg = it / W, k = it - (it / W) * W;
-                const int i0 = sg * kSegRows, i1 = min(nw, i0 + kSegRows);
-                uint32_t prev = 0u, pass = 0xffffffffu;
+        for (int k = warp; k < W; k += nwarp) {  // (b) word columns along R; lane = row segment
+            if (!cdirty[k]) continue;
+            work = true;
+            const int i0 = lane * L, i1 = min(nw, i0 + L);
+#pragma unroll 1
+            for (int dir = 0; dir < 2; ++dir) {
+                unsigned long long gv = 0ull, pv = ~0ull;
                 for (int q = 0; q < i1 - i0; ++q) {
                     const int i = dir == 0 ? i0 + q : i1 - 1 - q;
-                    const uint32_t c = ldc((long long)i * W + k);
-                    prev = R[(long long)i * W + k] | (c & prev);
-                    pass &= c;
+                    const unsigned long long c = C[(size_t)i * W + k];
+                    gv = R[(size_t)i * W + k] | (c & gv);
+                    pv &= c;
                 }
-                G[it] = prev;
-                P[it] = pass;
-            }
-            __syncthreads();
-            for (int k = tid; k < W; k += kFillThreads) {  // carries across segments
-                uint32_t in = 0u;
-                for (int q = 0; q < nseg; ++q) {
-                    const int sg = dir == 0 ? q : nseg - 1 - q;
-                    I[sg * W + k] = in;
-                    in = G[sg * W + k] | (P[sg * W + k] & in);
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {  // inclusive composition of the segment transfers
+                    const unsigned long long go = dir == 0 ? __shfl_up_sync(0xffffffffu, gv, d) : __shfl_down_sync(0xffffffffu, gv, d);
+                    const unsigned long long po = dir == 0 ? __shfl_up_sync(0xffffffffu, pv, d) : __shfl_down_sync(0xffffffffu, pv, d);
+                    if (dir == 0 ? lane >= d : lane + d < 32) { gv |= pv & go; pv &= po; }
                 }
-            }
-            __syncthreads();
-            for (int it = tid; it < nitem; it += kFillThreads) {
-                const int sg = it / W, k = it - (it / W) * W;
-                const int i0 = sg * kSegRows, i1 = min(nw, i0 + kSegRows);
-                uint32_t prev = I[it];
+                unsigned long long prev = dir == 0 ? __shfl_up_sync(0xffffffffu, gv, 1) : __shfl_down_sync(0xffffffffu, gv, 1);
+                if (dir == 0 ? lane == 0 : lane == 31) prev = 0ull;
                 for (int q = 0; q < i1 - i0; ++q) {
                     const int i = dir == 0 ? i0 + q : i1 - 1 - q;
-                    const long long p = (long long)i * W + k;
-                    const uint32_t old = R[p];
-                    const uint32_t v = old | (ldc(p) & prev);
-                    if (v != old) { R[p] = v; changed = true; }
+                    const size_t p = (size_t)i * W + k;
+                    const unsigned long long old = R[p];
+                    const unsigned long long v = old | (C[p] & prev);
+                    if (v != old) { R[p] = v; rdirty[i] = 1; }
                     prev = v;
                 }
             }
-            __syncthreads();
+            __syncwarp();
+            if (lane == 0) cdirty[k] = 0;
         }
-        if (!__syncthreads_or(changed)) break;
+        if (!__syncthreads_or(work)) break;
     }
-    // byte mask and its count
     int c = 0;
-    const long long n = (long long)nw * nh;
-    for (long long g = tid; g < n; g += kFillThreads) {
-        const int i = (int)(g / nh), j = (int)(g - (g / nh) * nh);
-        const uint8_t m = (uint8_t)((R[(long long)i * W + (j >> 5)] >> (j & 31)) & 1u);
-        mask[g] = m;
-        c += m;
+    for (int q = tid; q < nwords; q += kFillThreads) {
+        bits_g[q] = R[q];
+        c += __popcll(R[q]);
     }
     c = __reduce_add_sync(0xffffffffu, c);
-    if ((tid & 31) == 0) cnt_s[tid >> 5] = c;
+    if (lane == 0) cnt_s[warp] = c;
     __syncthreads();
     if (tid == 0) {
         int t = 0;
-        for (int q = 0; q < kFillThreads / 32; ++q) t += cnt_s[q];
+        for (int q = 0; q < nwarp; ++q) t += cnt_s[q];
         info[13] = (double)t;
         if (t == 0) atomicOr(status, EFIT_ST_NOPLASMA);
+    }
+}
+
+// byte mask from the component bitmap, 16 nodes per thread (one 16-byte store; pmask 256-B aligned)
+__global__ void __launch_bounds__(256) k_steps_mask(const unsigned long long* __restrict__ bits, int nw, int nh, int W,
+                                                   uint8_t* __restrict__ mask) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    const unsigned n = (unsigned)nw * (unsigned)nh;
+    const unsigned t = blockIdx.x * blockDim.x + threadIdx.x;
+    const unsigned g0 = 16u * t;
+    if (g0 >= n) return;
+    int i = (int)(g0 / (unsigned)nh), j = (int)(g0 - (unsigned)i * (unsigned)nh);
+    uint32_t v[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+    for (int b = 0; b < 16; ++b) {
+        if (g0 + b < n) v[b >> 2] |= (uint32_t)((bits[i * W + (j >> 6)] >> (j & 63)) & 1ull) << (8 * (b & 3));
+        if (++j == nh) { j = 0; ++i; }
+    }
+    if (g0 + 16u <= n) {
+        *reinterpret_cast<uint4*>(mask + g0) = make_uint4(v[0], v[1], v[2], v[3]);
+    } else {
+#pragma unroll
+        for (int b = 0; b < 16; ++b)
+            if (g0 + b < n) mask[g0 + b] = (uint8_t)(v[b >> 2] >> (8 * (b & 3)));
     }
 }
 
@@ -544,16 +592,15 @@ cudaError_t launch_pdl_s(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t s
 
 }  // namespace
 
-int steps_words(int nh) { return (nh + 31) / 32; }
+int steps_words(int nh) { return (nh + 63) / 64; }  // 64-bit words per bitmap row
 int steps_cand_cap(int nw, int nh) { return ((nw + 1) / 2) * ((nh + 1) / 2); }
 
-// dynamic shared memory of k_steps_fill; the candidate bitmap is staged when both maps fit
+// dynamic shared memory of k_steps_fill; the candidate bitmap is staged too when both maps fit
 size_t steps_fill_smem(int nw, int nh, bool* cand_smem) {
-    const size_t W = (size_t)steps_words(nh), nseg = (size_t)(nw + kSegRows - 1) / kSegRows;
-    const size_t base = 4 * (W * nw + 3 * nseg * W);
-    const bool both = base + 4 * W * nw <= 200 * 1024;
+    const size_t one = 8 * (size_t)steps_words(nh) * nw;
+    const bool both = 2 * one + nw <= 200 * 1024;
     if (cand_smem) *cand_smem = both;
-    return both ? base + 4 * W * nw : base;
+    return (both ? 2 * one : one) + (size_t)nw;  // + the row dirty flags
 }
 
 cudaError_t prepare_steps(Ctx& c, int smem_optin) {
@@ -566,28 +613,35 @@ cudaError_t prepare_steps(Ctx& c, int smem_optin) {
 }
 
 // full steps_ of psi: c.axbd, c.st_info, c.pmask (the plasma mask used downstream in place of the
-// limiter flags)
+// limiter flags).  Five launches: scan (all CTAs) -> final (1 CTA) -> bits -> fill (1 CTA) -> mask.
 cudaError_t launch_steps(Ctx& c, const double* psi, cudaStream_t s) {
-    ScanArgs a;
+    StepsArgs a;
     a.psi = psi; a.inlim = c.inlim; a.nw = c.nw; a.nh = c.nh; a.sgn = c.ip_sign;
     a.rmin = c.rmin; a.dr = c.dr; a.zmin = c.zmin; a.dz = c.dz; a.lim = c.lim; a.n_lim = c.n_lim;
-    a.part = c.norm_part; a.ticket = c.tickets + 2; a.cand = c.st_cand; a.cnt = c.st_cnt;
+    a.part = c.norm_part; a.nparts = c.t.red_blocks; a.cand = c.st_cand; a.cnt = c.st_cnt;
     a.cap = steps_cand_cap(c.nw, c.nh); a.info = c.st_info; a.axbd = c.axbd; a.status = c.status;
+    unsigned long long* bits = reinterpret_cast<unsigned long long*>(c.st_bits);
     cudaError_t e = launch_pdl_s(k_steps_scan, dim3(c.t.red_blocks), dim3(256), 0, s, a);
-    if (e) return e;
+    if (!e) e = launch_pdl_s(k_steps_final, dim3(1), dim3(32 * kFinalWarps), 0, s, a);
     const int W = steps_words(c.nh);
     const long long nwords = (long long)c.nw * W;
-    e = launch_pdl_s(k_steps_bits, dim3((unsigned)((nwords + 7) / 8)), dim3(256), 0, s, psi, c.inlim, c.nw, c.nh, W,
-                     (const double*)c.axbd, c.st_bits);
-    if (e) return e;
+    if (!e)
+        e = launch_pdl_s(k_steps_bits, dim3((unsigned)((nwords + 7) / 8)), dim3(256), 0, s, psi, (const uint8_t*)c.inlim,
+                         c.nw, c.nh, W, (const double*)c.axbd, bits);
     bool cs;
     const size_t sm = steps_fill_smem(c.nw, c.nh, &cs);
-    if (cs)
-        e = launch_pdl_s(k_steps_fill<true>, dim3(1), dim3(kFillThreads), sm, s, (const uint32_t*)c.st_bits, c.nw, c.nh,
-                         W, (const unsigned*)c.st_cnt, c.pmask, c.st_info, c.status);
-    else
-        e = launch_pdl_s(k_steps_fill<false>, dim3(1), dim3(kFillThreads), sm, s, (const uint32_t*)c.st_bits, c.nw,
-                         c.nh, W, (const unsigned*)c.st_cnt, c.pmask, c.st_info, c.status);
+    if (!e) {
+        if (cs)
+            e = launch_pdl_s(k_steps_fill<true>, dim3(1), dim3(kFillThreads), sm, s, bits, c.nw, c.nh, W,
+                             (const unsigned*)c.st_cnt, c.st_info, c.status);
+        else
+            e = launch_pdl_s(k_steps_fill<false>, dim3(1), dim3(kFillThreads), sm, s, bits, c.nw, c.nh, W,
+                             (const unsigned*)c.st_cnt, c.st_info, c.status);
+    }
+    const unsigned n16 = (unsigned)(((long long)c.nw * c.nh + 15) / 16);
+    if (!e)
+        e = launch_pdl_s(k_steps_mask, dim3((n16 + 255) / 256), dim3(256), 0, s, (const unsigned long long*)bits, c.nw,
+                         c.nh, W, c.pmask);
     if (e) return e;
     return cudaGetLastError();
 }
