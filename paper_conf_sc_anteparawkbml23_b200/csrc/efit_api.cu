@@ -945,6 +945,41 @@ static int fit_host_graphs(efit_ctx* h, int32_t nslice, int32_t iters, const dou
     return EFIT_OK;
 }
 
+// The host-buffer stream pipeline of one efit_fit_host call (fallback of the per-slice graphs).
+// Staging slot k & 1: H2D of slice k on the copy stream hs (after slot k-2's results left on ds) ->
+// the fit steps on s -> D2H on ds; so the copies of slices k+1 / k-1 overlap slice k's iterations.
+static int fit_host_pipeline(efit_ctx* h, int32_t nslice, int32_t iters, const double* h_psi0, const double* h_meas,
+                                     const double* h_sigma, const double* d_psi_ext, double* h_psi, double* h_coef,
+                                     double* h_chi2, double* h_eps, cudaStream_t s) {
+    Ctx& c = h->c;
+    const size_t n = (size_t)c.nw * c.nh, nd = (size_t)c.ndiag, nb = (size_t)c.nb;
+    cudaError_t e;
+    if ((e = cudaEventRecord(c.hstart, s)) || (e = cudaStreamWaitEvent(c.hs, c.hstart, 0)) ||
+        (e = cudaStreamWaitEvent(c.ds, c.hstart, 0)))
+        return cuda_fail(&c, e, "host pipeline");
+    for (int k = 0; k < nslice; ++k) {
+        const int b = k & 1;
+        Ctx::HostSlot& q = c.hslot[b];
+        if (k >= 2 && (e = cudaStreamWaitEvent(c.hs, c.hfree[b], 0))) return cuda_fail(&c, e, "host pipeline");
+        if ((e = cudaMemcpyAsync(q.psi, h_psi0 + k * n, sizeof(double) * n, cudaMemcpyHostToDevice, c.hs)) ||
+            (e = cudaMemcpyAsync(q.meas, h_meas + k * nd, sizeof(double) * nd, cudaMemcpyHostToDevice, c.hs)) ||
+            (e = cudaMemcpyAsync(q.sigma, h_sigma + k * nd, sizeof(double) * nd, cudaMemcpyHostToDevice, c.hs)) ||
+            (e = cudaEventRecord(c.hin[b], c.hs)) || (e = cudaStreamWaitEvent(s, c.hin[b], 0)))
+            return cuda_fail(&c, e, "host pipeline");
+        const int st = fit_steps_impl(h, iters, q.psi, d_psi_ext, q.meas, q.sigma, q.coef, q.chi2, q.eps, s);
+        if (st) return st;
+        if ((e = cudaEventRecord(c.hdone[b], s)) || (e = cudaStreamWaitEvent(c.ds, c.hdone[b], 0)) ||
+            (e = cudaMemcpyAsync(h_psi + k * n, q.psi, sizeof(double) * n, cudaMemcpyDeviceToHost, c.ds)) ||
+            (e = cudaMemcpyAsync(h_coef + k * nb, q.coef, sizeof(double) * nb, cudaMemcpyDeviceToHost, c.ds)) ||
+            (e = cudaMemcpyAsync(h_chi2 + k, q.chi2, sizeof(double), cudaMemcpyDeviceToHost, c.ds)) ||
+            (e = cudaMemcpyAsync(h_eps + k, q.eps, sizeof(double), cudaMemcpyDeviceToHost, c.ds)) ||
+            (e = cudaEventRecord(c.hfree[b], c.ds)))
+            return cuda_fail(&c, e, "host pipeline");
+    }
+    for (int b = 0; b < 2 && b < nslice; ++b)
+        if ((e = cudaStreamWaitEvent(s, c.hfree[(nslice - 1 - b) & 1], 0))) return cuda_fail(&c, e, "host pipeline");
+    return EFIT_OK;
+}
 // Host-buffer pipeline: nslice successive reconstructions (time slices), each `iters` chained
 // fit iterations, with their inputs read from and results written to HOST memory.  Staging slot
 // k & 1: H2D of slice k on the copy stream hs (after slot k-2's results left on ds) -> the cached
@@ -978,37 +1013,12 @@ extern "C" int efit_fit_host(efit_ctx* h, int32_t nslice, int32_t iters, const d
                 (e = cudaEventCreateWithFlags(&c.hfree[b], cudaEventDisableTiming)))
                 return cuda_fail(&c, e, "host pipeline events");
     }
-    const size_t n = (size_t)c.nw * c.nh, nd = (size_t)c.ndiag, nb = (size_t)c.nb;
     if (c.use_graph && !c.prof_on && getenv("EFIT_HOST_STREAMS") == nullptr) {
         const int st = fit_host_graphs(h, nslice, iters, h_psi0, h_meas, h_sigma, d_psi_ext, h_psi, h_coef, h_chi2,
                                        h_eps, s);
         if (st != 1) return st;  // 1: graphs not available for these buffers -> stream pipeline below
     }
-    if ((e = cudaEventRecord(c.hstart, s)) || (e = cudaStreamWaitEvent(c.hs, c.hstart, 0)) ||
-        (e = cudaStreamWaitEvent(c.ds, c.hstart, 0)))
-        return cuda_fail(&c, e, "host pipeline fork");
-    for (int k = 0; k < nslice; ++k) {
-        const int b = k & 1;
-        Ctx::HostSlot& q = c.hslot[b];
-        if (k >= 2 && (e = cudaStreamWaitEvent(c.hs, c.hfree[b], 0))) return cuda_fail(&c, e, "slot wait");
-        if ((e = cudaMemcpyAsync(q.psi, h_psi0 + k * n, sizeof(double) * n, cudaMemcpyHostToDevice, c.hs)) ||
-            (e = cudaMemcpyAsync(q.meas, h_meas + k * nd, sizeof(double) * nd, cudaMemcpyHostToDevice, c.hs)) ||
-            (e = cudaMemcpyAsync(q.sigma, h_sigma + k * nd, sizeof(double) * nd, cudaMemcpyHostToDevice, c.hs)) ||
-            (e = cudaEventRecord(c.hin[b], c.hs)) || (e = cudaStreamWaitEvent(s, c.hin[b], 0)))
-            return cuda_fail(&c, e, "H2D");
-        int st = fit_steps_impl(h, iters, q.psi, d_psi_ext, q.meas, q.sigma, q.coef, q.chi2, q.eps, stream);
-        if (st) return st;
-        if ((e = cudaEventRecord(c.hdone[b], s)) || (e = cudaStreamWaitEvent(c.ds, c.hdone[b], 0)) ||
-            (e = cudaMemcpyAsync(h_psi + k * n, q.psi, sizeof(double) * n, cudaMemcpyDeviceToHost, c.ds)) ||
-            (e = cudaMemcpyAsync(h_coef + k * nb, q.coef, sizeof(double) * nb, cudaMemcpyDeviceToHost, c.ds)) ||
-            (e = cudaMemcpyAsync(h_chi2 + k, q.chi2, sizeof(double), cudaMemcpyDeviceToHost, c.ds)) ||
-            (e = cudaMemcpyAsync(h_eps + k, q.eps, sizeof(double), cudaMemcpyDeviceToHost, c.ds)) ||
-            (e = cudaEventRecord(c.hfree[b], c.ds)))
-            return cuda_fail(&c, e, "D2H");
-    }
-    for (int b = 0; b < 2 && b < nslice; ++b)
-        if ((e = cudaStreamWaitEvent(s, c.hfree[(nslice - 1 - b) & 1], 0))) return cuda_fail(&c, e, "join");
-    return EFIT_OK;
+    return fit_host_pipeline(h, nslice, iters, h_psi0, h_meas, h_sigma, d_psi_ext, h_psi, h_coef, h_chi2, h_eps, s);
 }
 
 // ------------------------------------------------------------------ multi-time-slice batch

@@ -452,8 +452,8 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
     extern __shared__ unsigned long long sm[];
     unsigned long long* R = sm;                                  // [nw][W] reached
     unsigned long long* Cs = sm + (size_t)nw * W;                // [nw][W] candidates (CSMEM)
-    uint8_t* rdirty = reinterpret_cast<uint8_t*>(sm + (CSMEM ? 2 : 1) * (size_t)nw * W);  // [nw]
-    __shared__ uint8_t cdirty[32];
+    unsigned* rdirty = reinterpret_cast<unsigned*>(sm + (CSMEM ? 2 : 1) * (size_t)nw * W);  // [ceil(nw/32)] row bits
+    __shared__ unsigned cdirty;  // word-column bits (W <= 32)
     __shared__ int cnt_s[32];
     const unsigned long long* C = CSMEM ? Cs : bits_g;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -464,23 +464,22 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
         R[q] = 0ull;
         if (CSMEM) Cs[q] = bits_g[q];
     }
-    for (int i = tid; i < nw; i += kFillThreads) rdirty[i] = 0;
-    if (tid < 32) cdirty[tid] = 0;
+    for (int i = tid; i < (nw + 31) / 32; i += kFillThreads) rdirty[i] = 0u;
+    if (tid == 0) cdirty = 0u;
     __syncthreads();
     if (tid == 0 && g0 != UINT_MAX) {
         const int i0 = (int)(g0 / (unsigned)nh), j0 = (int)(g0 - (g0 / (unsigned)nh) * (unsigned)nh);
         const int q = i0 * W + (j0 >> 6);
         R[q] = C[q] & (1ull << (j0 & 63));
-        rdirty[i0] = 1;
-        cdirty[j0 >> 6] = 1;
+        rdirty[i0 >> 5] = 1u << (i0 & 31);
+        cdirty = 1u << (j0 >> 6);
     }
     __syncthreads();
     const int L = (nw + 31) / 32;  // rows per segment
     for (;;) {
         bool work = false;
         for (int i = tid; i < nw; i += kFillThreads) {  // (a) rows along Z
-            if (!rdirty[i]) continue;
-            rdirty[i] = 0;
+            if (!((rdirty[i >> 5] >> (i & 31)) & 1u)) continue;
             work = true;
             unsigned long long* r = R + (size_t)i * W;
             const unsigned long long* cr = C + (size_t)i * W;
@@ -489,19 +488,24 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
                 const unsigned long long c = cr[k], old = r[k];
                 const unsigned long long x = old | (carry ? (c & 1ull) : 0ull);
                 const unsigned long long f = fill_up64(c, x, carry);
-                if (f != old) { r[k] = f; cdirty[k] = 1; }
+                if (f != old) { r[k] = f; atomicOr(&cdirty, 1u << k); }
             }
             carry = false;
             for (int k = W - 1; k >= 0; --k) {
                 const unsigned long long c = __brevll(cr[k]), old = r[k];
                 const unsigned long long x = __brevll(old) | (carry ? (c & 1ull) : 0ull);
                 const unsigned long long f = __brevll(fill_up64(c, x, carry));
-                if (f != old) { r[k] = f; cdirty[k] = 1; }
+                if (f != old) { r[k] = f; atomicOr(&cdirty, 1u << k); }
             }
         }
         __syncthreads();
+        const unsigned cd = cdirty;
+        __syncthreads();
+        if (tid == 0) cdirty = 0u;  // every dirty row had its pass: clear (the column passes set new ones)
+        for (int i = tid; i < (nw + 31) / 32; i += kFillThreads) rdirty[i] = 0u;
+        __syncthreads();
         for (int k = warp; k < W; k += nwarp) {  // (b) word columns along R; lane = row segment
-            if (!cdirty[k]) continue;
+            if (!((cd >> k) & 1u)) continue;
             work = true;
             const int i0 = lane * L, i1 = min(nw, i0 + L);
 #pragma unroll 1
@@ -526,12 +530,10 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
                     const size_t p = (size_t)i * W + k;
                     const unsigned long long old = R[p];
                     const unsigned long long v = old | (C[p] & prev);
-                    if (v != old) { R[p] = v; rdirty[i] = 1; }
+                    if (v != old) { R[p] = v; atomicOr(&rdirty[i >> 5], 1u << (i & 31)); }
                     prev = v;
                 }
             }
-            __syncwarp();
-            if (lane == 0) cdirty[k] = 0;
         }
         if (!__syncthreads_or(work)) break;
     }
@@ -598,9 +600,9 @@ int steps_cand_cap(int nw, int nh) { return ((nw + 1) / 2) * ((nh + 1) / 2); }
 // dynamic shared memory of k_steps_fill; the candidate bitmap is staged too when both maps fit
 size_t steps_fill_smem(int nw, int nh, bool* cand_smem) {
     const size_t one = 8 * (size_t)steps_words(nh) * nw;
-    const bool both = 2 * one + nw <= 200 * 1024;
+    const bool both = 2 * one + 4 * (size_t)((nw + 31) / 32) <= 200 * 1024;
     if (cand_smem) *cand_smem = both;
-    return (both ? 2 * one : one) + (size_t)nw;  // + the row dirty flags
+    return (both ? 2 * one : one) + 4 * (size_t)((nw + 31) / 32);  // + the row dirty bits
 }
 
 cudaError_t prepare_steps(Ctx& c, int smem_optin) {

@@ -1,6 +1,6 @@
 """Small end-to-end run for compute-sanitizer: every per-iteration kernel of the
 default SYM and TABLE fit steps, the batch (mbarrier/bulk-copy DMMA kernels), the caller-exchange
-boundary partials/finish and the von Hagenow mode, on 33x33 (tiny grids keep the tools fast)."""
+boundary partials/finish, the von Hagenow mode and the full steps_ (f3) kernels, on 33x33 (tiny grids keep the tools fast)."""
 import os
 import sys
 
@@ -44,4 +44,23 @@ for mode in (2, 0, 4):
     torch.cuda.synchronize()
     assert ctx.status() == 0, efit.efit_last_error(ctx.handle)
     ctx.close()
+# full steps_ (f3): scan / final / bits / one-CTA fill (shared-memory bitmaps, atomics) / mask
+cfg = synth.small_config(n)
+ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=2, device=dev)
+ctx.set_steps(efit.EFIT_STEPS_FULL)
+psi_s = T(synth.solovev_diverted_psi(cfg.grid))
+ct = T(synth.c_true(cfg.basis, sol_c=synth.DIV_C))
+I = ctx.current(psi_s, ct)
+ext = psi_s - ctx.interior_solve(I, ctx.boundary_flux(I))
+resp, _ = ctx.response(psi_s)
+y = resp @ ct
+s = torch.full_like(y, 1e-3) * y.abs().max()
+info, mask = ctx.normalize(psi_s)
+coef, chi2, eps = ctx._t(ctx.nbasis), ctx._t(1), ctx._t(1)
+psi = psi_s.clone()
+ctx.fit_steps(2, psi, ext.contiguous(), y.contiguous(), s.contiguous(), coef, chi2, eps)
+torch.cuda.synchronize()
+assert ctx.status() == 0, efit.efit_last_error(ctx.handle)
+assert info.cpu().numpy()[12] == 1.0
+ctx.close()
 print("sanitize run ok")

@@ -186,8 +186,8 @@ def test_nccl_world1_exchange_bitwise(torch_mod, efit, mode, name):
 def test_fit_host_matches_device_steps(torch_mod, efit, monkeypatch, path, pinned):
     """efit_fit_host (the e2e path: host buffers in and out, copies overlapped with the fits of the
     neighbouring slices) equals efit_fit_steps on device buffers slice by slice, bit for bit, in both
-    pipelines (per-slice graphs with re-pointed copy nodes; the stream fallback) and for pinned and
-    pageable host memory."""
+    pipelines (per-slice graphs with re-pointed copy nodes, then the whole-call graph of a repeated
+    call; the stream fallback) and for pinned and pageable host memory."""
     torch = torch_mod
     if path == "streams":
         monkeypatch.setenv("EFIT_HOST_STREAMS", "1")
@@ -206,7 +206,9 @@ def test_fit_host_matches_device_steps(torch_mod, efit, monkeypatch, path, pinne
         ins = [t.pin_memory() for t in ins]
         outs = [t.pin_memory() for t in outs]
     st = torch.cuda.Stream()
-    for _ in range(2):   # twice: the second call reuses the cached graphs
+    for call in range(3):  # 1: per-slice graphs; 2: captured as one whole-call graph; 3: its replay
+        for t in outs:
+            t.fill_(float("nan"))
         ctx.fit_host(S, iters, *ins, ext, *outs, stream=st)
         st.synchronize()
     assert ctx.status() == 0
