@@ -222,6 +222,10 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
             if (best < 0 || cost <= best) { best = cost; t.resp_gc = gc; }  // ties -> larger chunks
         }
     }
+    if (const char* ev = getenv("EFIT_RESP_GC")) {  // tuning override (multiple of 128)
+        const int g = atoi(ev);
+        if (g >= 128 && g % 128 == 0 && g <= 1152) t.resp_gc = g;
+    }
     t.resp_nchunk = (int)((n + t.resp_gc - 1) / t.resp_gc);
     c.tbb_nchunk = (int)((n + efit::kBatchCh - 1) / efit::kBatchCh);
     c.respb_nchunk = (int)((n + efit::kRespBatchGc - 1) / efit::kRespBatchGc);
