@@ -245,11 +245,21 @@ __global__ void __launch_bounds__(256) k_steps_scan(StepsArgs a) {
 }
 
 constexpr int kFinalWarps = kMaxXCand + 1;  // warp 0: the axis, warps 1..8: X-point candidates
+constexpr int kFinalLimStage = 1024;         // limiter vertices staged in shared memory (24 KB)
 
 // One CTA: (3) axis, (4) X-points, (5) limiter value, (6) boundary.  Newton searches run one per
 // warp (lane 0) concurrently; the in-limiter test of an X-point is the parity of the crossings over
 // the limiter edges (an order-independent count: the same decision as the sequential even-odd rule).
 __global__ void __launch_bounds__(32 * kFinalWarps) k_steps_final(StepsArgs a) {
+    // limiter vertices (constant: staged before the wait on the predecessor) and, right after it,
+    // s psi_bilin at every vertex, so that the X-point in-limiter tests and the limiter value after
+    // the Newton searches read shared memory only
+    extern __shared__ double lsm[];  // [2 n_lim] vertices (r then z), [n_lim] s psi_bilin
+    const bool lstage = a.n_lim <= kFinalLimStage;
+    double* vval = lsm + 2 * kFinalLimStage;
+    if (lstage)
+        for (int k = threadIdx.x; k < 2 * a.n_lim; k += blockDim.x) lsm[k] = __ldg(a.lim + k);
+    const double* lim = lstage ? lsm : a.lim;
     asm volatile("griddepcontrol.wait;" ::: "memory");
     __shared__ double sv[kFinalWarps];
     __shared__ long long si[kFinalWarps];
@@ -261,6 +271,10 @@ __global__ void __launch_bounds__(32 * kFinalWarps) k_steps_final(StepsArgs a) {
     const Field F{a.psi, a.nw, a.nh};
     const int nh = a.nh, tid = threadIdx.x, w = tid >> 5, l = tid & 31;
     const double s = (double)a.sgn;
+    __syncthreads();  // staged vertices visible
+    if (lstage)
+        for (int v = tid; v < a.n_lim; v += blockDim.x)
+            vval[v] = s * bilin(F, a.rmin, a.dr, a.zmin, a.dz, lim[v], lim[a.n_lim + v]);
     double best = -DBL_MAX;
     long long bi = LLONG_MAX;
     for (int b = tid; b < a.nparts; b += blockDim.x) am_merge(best, bi, a.part[2 * b], (long long)a.part[2 * b + 1]);
@@ -308,7 +322,7 @@ __global__ void __launch_bounds__(32 * kFinalWarps) k_steps_final(StepsArgs a) {
             unsigned par = 0u;
             for (int k = l; k < a.n_lim; k += 32) {
                 const int k1 = (k + 1 == a.n_lim) ? 0 : k + 1;
-                const double r0 = a.lim[k], z0 = a.lim[a.n_lim + k], r1 = a.lim[k1], z1 = a.lim[a.n_lim + k1];
+                const double r0 = lim[k], z0 = lim[a.n_lim + k], r1 = lim[k1], z1 = lim[a.n_lim + k1];
                 if ((z0 > Zx) != (z1 > Zx)) {
                     const double x = ((r1 - r0) * (Zx - z0)) / (z1 - z0) + r0;
                     if (Rx < x) par ^= 1u;
@@ -368,10 +382,10 @@ __global__ void __launch_bounds__(32 * kFinalWarps) k_steps_final(StepsArgs a) {
     if (racc[0]) {
         const bool lo = zlim[0] != -DBL_MAX, hi = zlim[1] != DBL_MAX;
         for (int v = tid; v < a.n_lim; v += blockDim.x) {
-            const double z = a.lim[a.n_lim + v];
+            const double z = lim[a.n_lim + v];
             if (lo && !(z > zlim[0])) continue;
             if (hi && !(z < zlim[1])) continue;
-            am_merge(vb, vi, s * bilin(F, a.rmin, a.dr, a.zmin, a.dz, a.lim[v], z), (long long)v);
+            am_merge(vb, vi, lstage ? vval[v] : s * bilin(F, a.rmin, a.dr, a.zmin, a.dz, lim[v], z), (long long)v);
         }
     }
     am_warp(vb, vi);
@@ -548,7 +562,7 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
     if (tid == 0) {
         int t = 0;
         for (int q = 0; q < nwarp; ++q) t += cnt_s[q];
-        info[13] = (double)t;
+        if (g0 != UINT_MAX) info[13] = (double)t;  // no boundary / no plasma: left NaN (as the oracle)
         if (t == 0) atomicOr(status, EFIT_ST_NOPLASMA);
     }
 }
@@ -624,7 +638,7 @@ cudaError_t launch_steps(Ctx& c, const double* psi, cudaStream_t s) {
     a.cap = steps_cand_cap(c.nw, c.nh); a.info = c.st_info; a.axbd = c.axbd; a.status = c.status;
     unsigned long long* bits = reinterpret_cast<unsigned long long*>(c.st_bits);
     cudaError_t e = launch_pdl_s(k_steps_scan, dim3(c.t.red_blocks), dim3(256), 0, s, a);
-    if (!e) e = launch_pdl_s(k_steps_final, dim3(1), dim3(32 * kFinalWarps), 0, s, a);
+    if (!e) e = launch_pdl_s(k_steps_final, dim3(1), dim3(32 * kFinalWarps), sizeof(double) * 3 * kFinalLimStage, s, a);
     const int W = steps_words(c.nh);
     const long long nwords = (long long)c.nw * W;
     if (!e)

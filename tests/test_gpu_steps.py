@@ -101,6 +101,66 @@ def test_normalize_bitwise(torch_mod, efit, orc_mod, n, kind):
     ctx.close()
 
 
+@pytest.mark.parametrize("shape", [(65, 129), (129, 65), (97, 65)], ids=["65x129", "129x65", "97x65"])
+@pytest.mark.parametrize("sign", [1, -1], ids=["ip+", "ip-"])
+def test_normalize_bitwise_nonsquare_and_sign(torch_mod, efit, orc_mod, shape, sign):
+    """Ragged (non-square) grids and a negative plasma current (ip_sign = -1, psi minimal on the
+    axis): the same bit-for-bit agreement (nh - 1 need not be a power of two for steps_ itself, but
+    the context requires it, so nh is 65 or 129)."""
+    import dataclasses
+    torch = torch_mod
+    g = synth.Grid(*shape)
+    geo = dataclasses.replace(synth.make_geometry(g), ip_sign=sign)
+    cfg = synth.Config("ns", g, geo, synth.poly_basis(), "non-square")
+    orc = orc_mod.Oracle.from_config(cfg)
+    orc.set_steps_mode(1)
+    psi = sign * synth.solovev_diverted_psi(g)
+    cnt, pa, pb, mask, _ = orc.normalize(psi)
+    oinfo = orc.steps_info()
+    ctx = efit.EfitContext(g, cfg.basis, geo, mode=efit.EFIT_GREEN_TABLE_SYM)
+    ctx.set_steps(efit.EFIT_STEPS_FULL)
+    info, gmask = ctx.normalize(T(torch, psi))
+    torch.cuda.synchronize()
+    assert ctx.status() == 0 and cnt > 0
+    assert np.array_equal(gmask.cpu().numpy(), mask)
+    _same_info(info.cpu().numpy(), oinfo)
+    assert oinfo[12] == 1.0  # the lower X-point bounds the plasma for either sign
+    ctx.close()
+
+
+def test_minimum_grid_and_no_plasma(torch_mod, efit, orc_mod):
+    """The smallest grid the full rule accepts (9 x 9, nh - 1 a power of two; rejected below 6) and a
+    psi with no plasma (a plane: no interior maximum, no X-point): both sides report no plasma."""
+    torch = torch_mod
+    cfg = synth.small_config(9)
+    orc = orc_mod.Oracle.from_config(cfg)
+    orc.set_steps_mode(1)
+    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=efit.EFIT_GREEN_TABLE_SYM)
+    ctx.set_steps(efit.EFIT_STEPS_FULL)
+    psi = synth.solovev_diverted_psi(cfg.grid)
+    cnt, pa, pb, mask, _ = orc.normalize(psi)
+    info, gmask = ctx.normalize(T(torch, psi))
+    torch.cuda.synchronize()
+    st = ctx.status()
+    assert (st == 0) == (cnt > 0)
+    _same_info(info.cpu().numpy(), orc.steps_info())
+    if cnt > 0:
+        assert np.array_equal(gmask.cpu().numpy(), mask)
+    R = np.repeat(cfg.grid.r(), cfg.grid.nh)
+    plane = 0.01 * (R - R.mean())
+    cnt, *_ = orc.normalize(plane)
+    info, gmask = ctx.normalize(T(torch, plane))
+    torch.cuda.synchronize()
+    assert cnt < 0 and ctx.status() == efit.EFIT_E_NOPLASMA and int(gmask.sum().item()) == 0
+    _same_info(info.cpu().numpy(), orc.steps_info())
+    ctx.close()
+    small = synth.small_config(5)
+    ctx5 = efit.EfitContext(small.grid, small.basis, small.geometry, mode=efit.EFIT_GREEN_TABLE)
+    with pytest.raises(efit.EfitError):
+        ctx5.set_steps(efit.EFIT_STEPS_FULL)
+    ctx5.close()
+
+
 def test_limiter_mode_normalize_matches_o8(torch_mod, efit, orc_mod):
     torch = torch_mod
     cfg = synth.small_config(65)
