@@ -21,6 +21,7 @@
 #include <limits.h>
 #include <stdint.h>
 
+#include <cstdio>
 #include <utility>
 
 #include "efit_internal.h"
@@ -32,7 +33,6 @@ namespace {
 constexpr int kNewtonIters = 20;
 constexpr int kMaxXCand = 8;
 constexpr int kFillThreads = 1024;
-constexpr int kSegRows = 16;  // rows per segment of the column scans
 
 __device__ __forceinline__ void am_merge(double& v, long long& i, double v2, long long i2) {
     if (v2 > v || (v2 == v && i2 < i)) { v = v2; i = i2; }
@@ -159,20 +159,6 @@ __device__ bool xcand(const Field& F, int i, int j, double& key) {
         }
     key = g2;
     return true;
-}
-
-// even-odd rule of O7 (same expression as the limiter table)
-__device__ bool in_polygon(double R, double Z, const double* lim, int n_lim) {
-    bool inside = false;
-    for (int k = 0; k < n_lim; ++k) {
-        const int k1 = (k + 1 == n_lim) ? 0 : k + 1;
-        const double r0 = lim[k], z0 = lim[n_lim + k], r1 = lim[k1], z1 = lim[n_lim + k1];
-        if ((z0 > Z) != (z1 > Z)) {
-            const double x = ((r1 - r0) * (Z - z0)) / (z1 - z0) + r0;
-            if (R < x) inside = !inside;
-        }
-    }
-    return inside;
 }
 
 // O8's bilinear value at (R, Z)
@@ -468,6 +454,7 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
     unsigned long long* Cs = sm + (size_t)nw * W;                // [nw][W] candidates (CSMEM)
     unsigned* rdirty = reinterpret_cast<unsigned*>(sm + (CSMEM ? 2 : 1) * (size_t)nw * W);  // [ceil(nw/32)] row bits
     __shared__ unsigned cdirty;  // word-column bits (W <= 32)
+    __shared__ unsigned long long wtot[kFillThreads / 32][2];  // per-warp segment-scan totals (G, P)
     __shared__ int cnt_s[32];
     const unsigned long long* C = CSMEM ? Cs : bits_g;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -489,7 +476,15 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
         cdirty = 1u << (j0 >> 6);
     }
     __syncthreads();
-    const int L = (nw + 31) / 32;  // rows per segment
+#ifdef EFIT_STEPS_DEBUG
+    long long t_dbg0 = clock64(), t_dbg[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    int rounds_dbg = 0;
+#endif
+#ifdef EFIT_STEPS_DEBUG
+    long long t_init = clock64() - t_dbg0, t_h[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#endif
+    const int WPC = min(4, max(1, nwarp / W));  // warps per column word
+    const int L = (nw + 32 * WPC - 1) / (32 * WPC);  // rows per segment
     for (;;) {
         bool work = false;
         for (int i = tid; i < nw; i += kFillThreads) {  // (a) rows along Z
@@ -514,17 +509,23 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
         }
         __syncthreads();
         const unsigned cd = cdirty;
+#ifdef EFIT_STEPS_DEBUG
+        if (rounds_dbg < 8) t_h[rounds_dbg] = clock64() - t_dbg0;
+#endif
         __syncthreads();
         if (tid == 0) cdirty = 0u;  // every dirty row had its pass: clear (the column passes set new ones)
         for (int i = tid; i < (nw + 31) / 32; i += kFillThreads) rdirty[i] = 0u;
         __syncthreads();
-        for (int k = warp; k < W; k += nwarp) {  // (b) word columns along R; lane = row segment
-            if (!((cd >> k) & 1u)) continue;
-            work = true;
-            const int i0 = lane * L, i1 = min(nw, i0 + L);
-#pragma unroll 1
-            for (int dir = 0; dir < 2; ++dir) {
-                unsigned long long gv = 0ull, pv = ~0ull;
+        // (b) word columns along R: WPC warps per column word, lane = one of 32 WPC row segments; the
+        // segment transfers are composed by a warp scan, the warps' totals through shared memory
+        for (int dir = 0; dir < 2; ++dir) {
+            const bool act = warp < W * WPC && ((cd >> (warp / WPC)) & 1u);
+            const int k = warp / WPC, part = warp - (warp / WPC) * WPC;
+            const int seg = part * 32 + lane;
+            const int i0 = min(nw, seg * L), i1 = min(nw, i0 + L);
+            unsigned long long gv = 0ull, pv = ~0ull;
+            if (act) {
+                work = true;
                 for (int q = 0; q < i1 - i0; ++q) {
                     const int i = dir == 0 ? i0 + q : i1 - 1 - q;
                     const unsigned long long c = C[(size_t)i * W + k];
@@ -532,13 +533,26 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
                     pv &= c;
                 }
 #pragma unroll
-                for (int d = 1; d < 32; d <<= 1) {  // inclusive composition of the segment transfers
+                for (int d = 1; d < 32; d <<= 1) {  // inclusive composition in scan order
                     const unsigned long long go = dir == 0 ? __shfl_up_sync(0xffffffffu, gv, d) : __shfl_down_sync(0xffffffffu, gv, d);
                     const unsigned long long po = dir == 0 ? __shfl_up_sync(0xffffffffu, pv, d) : __shfl_down_sync(0xffffffffu, pv, d);
                     if (dir == 0 ? lane >= d : lane + d < 32) { gv |= pv & go; pv &= po; }
                 }
-                unsigned long long prev = dir == 0 ? __shfl_up_sync(0xffffffffu, gv, 1) : __shfl_down_sync(0xffffffffu, gv, 1);
-                if (dir == 0 ? lane == 0 : lane == 31) prev = 0ull;
+                if (lane == (dir == 0 ? 31 : 0)) { wtot[warp][0] = gv; wtot[warp][1] = pv; }
+            }
+            __syncthreads();
+            if (act) {
+                unsigned long long cin = 0ull;  // carry into this warp: the totals of the warps before it
+                if (dir == 0) {
+                    for (int p2 = 0; p2 < part; ++p2) cin = wtot[k * WPC + p2][0] | (wtot[k * WPC + p2][1] & cin);
+                } else {
+                    for (int p2 = WPC - 1; p2 > part; --p2) cin = wtot[k * WPC + p2][0] | (wtot[k * WPC + p2][1] & cin);
+                }
+                // exclusive prefix of this lane = the previous lane's inclusive value applied to cin
+                unsigned long long ge = dir == 0 ? __shfl_up_sync(0xffffffffu, gv, 1) : __shfl_down_sync(0xffffffffu, gv, 1);
+                unsigned long long pe = dir == 0 ? __shfl_up_sync(0xffffffffu, pv, 1) : __shfl_down_sync(0xffffffffu, pv, 1);
+                if (lane == (dir == 0 ? 0 : 31)) { ge = 0ull; pe = ~0ull; }
+                unsigned long long prev = ge | (pe & cin);
                 for (int q = 0; q < i1 - i0; ++q) {
                     const int i = dir == 0 ? i0 + q : i1 - 1 - q;
                     const size_t p = (size_t)i * W + k;
@@ -548,7 +562,12 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
                     prev = v;
                 }
             }
+            __syncthreads();
         }
+#ifdef EFIT_STEPS_DEBUG
+        if (rounds_dbg < 8) t_dbg[rounds_dbg] = clock64() - t_dbg0;
+        ++rounds_dbg;
+#endif
         if (!__syncthreads_or(work)) break;
     }
     int c = 0;
@@ -563,6 +582,11 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
         int t = 0;
         for (int q = 0; q < nwarp; ++q) t += cnt_s[q];
         if (g0 != UINT_MAX) info[13] = (double)t;  // no boundary / no plasma: left NaN (as the oracle)
+#ifdef EFIT_STEPS_DEBUG
+        printf("fill rounds=%d end t=%lld count=%d rounds at %lld %lld %lld %lld %lld\n", rounds_dbg, clock64() - t_dbg0, t,
+               t_dbg[0], t_dbg[1], t_dbg[2], t_dbg[3], t_dbg[4]);
+        printf("  init %lld, after H: %lld %lld %lld %lld\n", t_init, t_h[0], t_h[1], t_h[2], t_h[3]);
+#endif
         if (t == 0) atomicOr(status, EFIT_ST_NOPLASMA);
     }
 }
