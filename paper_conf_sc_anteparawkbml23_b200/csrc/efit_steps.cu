@@ -487,6 +487,7 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
     const int L = (nw + 32 * WPC - 1) / (32 * WPC);  // rows per segment
     for (;;) {
         bool work = false;
+        unsigned cmask = 0u;  // word columns this thread changed (one warp-aggregated atomic per pass)
         for (int i = tid; i < nw; i += kFillThreads) {  // (a) rows along Z
             if (!((rdirty[i >> 5] >> (i & 31)) & 1u)) continue;
             work = true;
@@ -497,16 +498,18 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
                 const unsigned long long c = cr[k], old = r[k];
                 const unsigned long long x = old | (carry ? (c & 1ull) : 0ull);
                 const unsigned long long f = fill_up64(c, x, carry);
-                if (f != old) { r[k] = f; atomicOr(&cdirty, 1u << k); }
+                if (f != old) { r[k] = f; cmask |= 1u << k; }
             }
             carry = false;
             for (int k = W - 1; k >= 0; --k) {
                 const unsigned long long c = __brevll(cr[k]), old = r[k];
                 const unsigned long long x = __brevll(old) | (carry ? (c & 1ull) : 0ull);
                 const unsigned long long f = __brevll(fill_up64(c, x, carry));
-                if (f != old) { r[k] = f; atomicOr(&cdirty, 1u << k); }
+                if (f != old) { r[k] = f; cmask |= 1u << k; }
             }
         }
+        cmask = __reduce_or_sync(0xffffffffu, cmask);
+        if (lane == 0 && cmask) atomicOr(&cdirty, cmask);
         __syncthreads();
         const unsigned cd = cdirty;
 #ifdef EFIT_STEPS_DEBUG
@@ -553,13 +556,21 @@ __global__ void __launch_bounds__(kFillThreads, 1) k_steps_fill(unsigned long lo
                 unsigned long long pe = dir == 0 ? __shfl_up_sync(0xffffffffu, pv, 1) : __shfl_down_sync(0xffffffffu, pv, 1);
                 if (lane == (dir == 0 ? 0 : 31)) { ge = 0ull; pe = ~0ull; }
                 unsigned long long prev = ge | (pe & cin);
+                unsigned long long rmask = 0ull;  // rows i0 + q changed (L <= 64), set with <= 3 atomics
                 for (int q = 0; q < i1 - i0; ++q) {
                     const int i = dir == 0 ? i0 + q : i1 - 1 - q;
                     const size_t p = (size_t)i * W + k;
                     const unsigned long long old = R[p];
                     const unsigned long long v = old | (C[p] & prev);
-                    if (v != old) { R[p] = v; atomicOr(&rdirty[i >> 5], 1u << (i & 31)); }
+                    if (v != old) { R[p] = v; rmask |= 1ull << (i - i0); }
                     prev = v;
+                }
+                while (rmask) {  // the changed rows' dirty bits, one atomic per 32-row word touched
+                    const int b = __ffsll((long long)rmask) - 1, i = i0 + b, w0 = i >> 5;
+                    const int nb = min(32 - (i & 31), 64 - b);
+                    const unsigned long long chunk = (nb == 64 ? ~0ull : ((1ull << nb) - 1ull)) & (rmask >> b);
+                    atomicOr(&rdirty[w0], (unsigned)(chunk << (i & 31)));
+                    rmask &= ~(nb == 64 ? ~0ull : (((1ull << nb) - 1ull) << b));
                 }
             }
             __syncthreads();
