@@ -238,7 +238,8 @@ int efit_interior_solve(efit_ctx* ctx, const double* d_pcurr, const double* d_ps
  *                                 the reading's order (bit-reproducible).  Adds three launches per
  *                                 iteration (the chained fit steps then normalise before every iteration).
  *                                 Needs 6 <= nw, nh and nw * ceil(nh/32) * 4 bytes of bitmap in shared
- *                                 memory (up to ~1025^2); not with a batch attached (EFIT_E_STATE).
+ *                                 memory (up to ~1025^2).  Applies to the attached batch slices too
+ *                                 (each slice normalises its own psi).
  * efit_set_steps: host-only switch (drops the cached fit-step graphs); EFIT_E_INVAL for a bad mode or
  *   a grid outside the limits above. */
 enum { EFIT_STEPS_LIMITER = 0, EFIT_STEPS_FULL = 1 };

@@ -604,14 +604,17 @@ extern "C" int efit_set_steps(efit_ctx* h, int32_t steps_mode) {
     if (steps_mode != EFIT_STEPS_LIMITER && steps_mode != EFIT_STEPS_FULL)
         return fail(&c, EFIT_E_INVAL, "steps_mode must be EFIT_STEPS_LIMITER or EFIT_STEPS_FULL");
     if (steps_mode == EFIT_STEPS_FULL) {
-        if (c.nslice > 0) return fail(&c, EFIT_E_STATE, "EFIT_STEPS_FULL with a batch attached");
         int optin = 0;
         cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, c.device);
         if (c.nw < 6 || c.nh < 6 || efit::steps_words(c.nh) > 32 || efit::steps_fill_smem(c.nw, c.nh, nullptr) > (size_t)optin)
             return fail(&c, EFIT_E_INVAL, "EFIT_STEPS_FULL needs 6 <= nw, nh and a plasma bitmap in shared memory (nw*nh <= ~1025^2)");
     }
-    if (c.steps != steps_mode) drop_fit_graphs(c);
+    if (c.steps != steps_mode) {
+        drop_fit_graphs(c);
+        if (c.bexec) { cudaGraphExecDestroy(c.bexec); c.bexec = nullptr; }
+    }
     c.steps = steps_mode;
+    for (int k = 0; k < c.nslice; ++k) c.slice[k]->steps = steps_mode;  // batch slices normalise alike
     return EFIT_OK;
 }
 
@@ -1067,7 +1070,6 @@ extern "C" int efit_batch_workspace_bytes(const efit_ctx* h, int32_t nslice, siz
 extern "C" int efit_batch_attach(efit_ctx* h, int32_t nslice, void* d_workspace, size_t ws_bytes) {
     if (!h) return fail(nullptr, EFIT_E_INVAL, "ctx is null");
     Ctx& c = h->c;
-    if (c.steps) return fail(&c, EFIT_E_STATE, "batch with EFIT_STEPS_FULL is not supported");
     int st = batch_check(c, nslice);
     if (st) return st;
     const size_t per = slice_bytes(c);
@@ -1142,7 +1144,7 @@ static cudaError_t enqueue_fit_step_batch(Ctx& c, double* psi, const double* psi
             cudaStream_t sk = q.side;
             double* pk = psi + k * n;
             if ((e = cudaStreamWaitEvent(sk, c.bev_fork, 0))) return e;
-            if (normalize && (e = launch_normalize(q, pk, sk))) return e;
+            if ((normalize || q.steps) && (e = launch_normalize(q, pk, sk))) return e;  // f3: every iteration
             if ((e = launch_basis(q, pk, sk))) return e;
             if ((e = cudaEventRecord(q.ev_join, sk))) return e;
         }
@@ -1160,7 +1162,7 @@ static cudaError_t enqueue_fit_step_batch(Ctx& c, double* psi, const double* psi
             if ((e = launch_resp_reduce_batch(q, c.respb_nchunk, q.resp, sk))) return e;
         } else {
             if ((e = cudaStreamWaitEvent(sk, c.bev_fork, 0))) return e;
-            if (normalize && (e = launch_normalize(q, pk, sk))) return e;
+            if ((normalize || q.steps) && (e = launch_normalize(q, pk, sk))) return e;
             if ((e = launch_response(q, pk, q.resp, sk))) return e;
         }
         if ((e = launch_lsq(q, q.resp, meas + (size_t)k * c.ndiag, sigma + (size_t)k * c.ndiag, coef + (size_t)k * c.nb,

@@ -268,7 +268,7 @@ def test_c4_full_steps_fit_step(torch_mod, efit, orc_mod):
 
 def test_steps_mode_switch_and_errors(torch_mod, efit, orc_mod):
     """Switching the rule drops the cached graphs (the same pointers give the other rule's result);
-    bad modes are rejected on the host; a batch cannot be attached in EFIT_STEPS_FULL."""
+    bad modes are rejected on the host."""
     torch = torch_mod
     cfg = synth.small_config(65)
     orc = orc_mod.Oracle.from_config(cfg)
@@ -295,9 +295,41 @@ def test_steps_mode_switch_and_errors(torch_mod, efit, orc_mod):
     assert rel(results[0], results[1]) > 1e-6  # the two rules differ on a diverted psi
     with pytest.raises(efit.EfitError):
         ctx.set_steps(7)
-    ctx.set_steps(efit.EFIT_STEPS_FULL)
-    with pytest.raises(efit.EfitError):
-        ctx.batch_attach(2)
+    ctx.close()
+
+
+def test_batch_full_steps_per_slice(torch_mod, efit, orc_mod):
+    """A batch of 3 time slices (shared table pass on the tensor cores) under the full steps_ rule:
+    every slice normalises its own psi (axis, X-point, connected mask) and equals the oracle's f3
+    fit step on that slice (the table pass sums in another order: rounding-level agreement)."""
+    torch = torch_mod
+    cfg = synth.small_config(65)
+    orc = orc_mod.Oracle.from_config(cfg)
+    orc.set_steps_mode(1)
+    psi_s = synth.solovev_diverted_psi(cfg.grid)
+    ct = synth.c_true(cfg.basis, sol_c=synth.DIV_C)
+    tw = orc.twin(psi_s, ct, noise_seed=1)
+    S, n = 3, cfg.grid.n
+    starts = [psi_s + 1e-4 * (k + 1) * (psi_s.max() - psi_s.min()) * synth.smooth_modes(cfg.grid, 5 + k) / 3.0
+              for k in range(S)]
+    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=efit.EFIT_GREEN_TABLE)
+    ctx.batch_attach(S)
+    ctx.set_steps(efit.EFIT_STEPS_FULL)  # after attaching: propagated to the slices
+    P = T(torch, np.concatenate(starts))
+    E = T(torch, np.tile(tw["psi_ext"], S))
+    Y = T(torch, np.tile(tw["y"], S))
+    G = T(torch, np.tile(tw["sigma"], S))
+    coef, chi2, eps = ctx._t(S * ctx.nbasis), ctx._t(S), ctx._t(S)
+    st = torch.cuda.Stream()
+    ctx.fit_step_batch(P, E, Y, G, coef, chi2, eps, stream=st)
+    st.synchronize()
+    assert ctx.status() == 0
+    Pg, Cg = P.cpu().numpy(), coef.cpu().numpy()
+    for k in range(S):
+        s0, pr, cr, chr_, er = orc.fit_step(starts[k], tw["psi_ext"], tw["y"], tw["sigma"])
+        assert s0 == 0
+        assert rel(Pg[k * n:(k + 1) * n], pr) < TOL, k
+        assert rel(Cg[k * ctx.nbasis:(k + 1) * ctx.nbasis], cr) < TOL_C, k
     ctx.close()
 
 
