@@ -2884,12 +2884,34 @@ __global__ void __launch_bounds__(128) k_tridiag_reg(double* __restrict__ fhat, 
         iv[e] = act ? inv[fo + 32 * e] : 0.0;
         c[e] = act ? cp[fo + 32 * e] : 0.0;
     }
+    // staging through shared memory: coalesced loads of the mode column (row r at r + r/L: the lane
+    // segments r = lane L + e are then conflict-free) and of the bottom/top edge rows (the same for
+    // every mode of the CTA), instead of 32-way scattered per-lane segment loads
+    __shared__ double sf[4][32 * (L + 1)];
+    __shared__ double sbt[2][32 * L];
     griddep();
+    if (fx.bot)
+        for (int r = threadIdx.x; r < ni; r += blockDim.x) {
+            sbt[0][r] = fx.bot[r];
+            sbt[1][r] = fx.top[r];
+        }
+    double* sw = sf[warp];
+    if (act) {
+#pragma unroll
+        for (int e = 0; e < L; ++e) {
+            const int r = 32 * e + lane;
+            sw[r + r / L] = r < ni ? fg[r] : 0.0;
+        }
+    }
+    __syncthreads();
     if (!act) return;
+    const double sgn_fx = (mode & 1) ? -1.0 : 1.0;  // tb_fix's expression, edge rows from shared memory
+    const double sk_fx = fx.bot ? fx.sink[mode] * fx.idz2 : 0.0;
 #pragma unroll
     for (int e = 0; e < L; ++e) {
         const int r = lane * L + e;
-        f[e] = r < ni ? (fx.bot ? fg[r] + tb_fix(fx, mode, r) : fg[r]) : 0.0;
+        const double v = sw[r + lane];
+        f[e] = r < ni ? (fx.bot ? v + -(sbt[0][r] + sgn_fx * sbt[1][r]) * sk_fx : v) : 0.0;
     }
     double A = 1.0, B = 0.0;
 #pragma unroll
@@ -2929,10 +2951,14 @@ __global__ void __launch_bounds__(128) k_tridiag_reg(double* __restrict__ fhat, 
         x = fma(-c[e], x, f[e]);
         f[e] = x;
     }
+    // back through the skewed shared column: coalesced stores
+#pragma unroll
+    for (int e = 0; e < L; ++e) sw[lane * (L + 1) + e] = f[e];
+    __syncwarp();
 #pragma unroll
     for (int e = 0; e < L; ++e) {
-        const int r = lane * L + e;
-        if (r < ni) fg[r] = f[e];
+        const int r = 32 * e + lane;
+        if (r < ni) fg[r] = sw[r + r / L];
     }
 }
 
