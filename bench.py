@@ -602,11 +602,11 @@ def gpu_arm(args, rank, world, local):
 
     # our kernels per step (ncu launch list, profiles/): response (basis fused), resp_reduce, lsq,
     # current, lr_fft, lr_mac, lr_ifft, dst_fwd, bnd_tb | (bnd_sym + sym_edge_src), bnd_reduce,
-    # tridiag, dst_inv; + k_normalize at the start of every captured graph
-    per_step = 12 + (1 if sym_mode else 0)
+    # tridiag, dst_inv, dst_fin; + k_normalize at the start of every captured graph
+    per_step = 13 + (1 if sym_mode else 0)
     launches = per_step * K + len(graphs)
-    if full:  # steps_ (3 kernels) before every iteration instead of once per graph
-        launches = (per_step + 3) * K
+    if full:  # steps_ (5 kernels) before every iteration instead of once per graph
+        launches = (per_step + 5) * K
     if rank == 0:
         par = "single GPU"
         if use_dist:

@@ -9,7 +9,7 @@
 //   k_bnd_tb      top/bottom targets, T slabs streamed once     (pflux_ 2nd O(N^3) nest) HBM-bound
 //   k_bnd_lr      left/right targets, Toeplitz in registers     (pflux_ Fig. 2 nest)  FP64-bound
 //   k_bnd_reduce  fixed-order partial sums -> psi_b (edge order)
-//   k_dst_fwd / k_tridiag / k_dst_inv   interior GS solve + update + eps (pflux_ O(N^2), Eq. (1))
+//   k_dst_fwd / k_tridiag / k_dst_inv / k_dst_fin   interior GS solve + update + eps (pflux_ O(N^2), Eq. (1))
 // Every reduction has a fixed order, so results are bitwise reproducible run to run and
 // independent of the number of ranks.
 #include <cfloat>
@@ -3114,14 +3114,21 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
             nn.part[2 * blockIdx.x] = best;
             nn.part[2 * blockIdx.x + 1] = (double)bi;
         }
-        __threadfence();
-        last = (atomicAdd(ticket, 1u) == gridDim.x - 1);
     }
-    __syncthreads();
-    if (!last) return;
-    __threadfence();
+}
+
+// eps = max over the k_dst_inv blocks' partials / |psi_bdry - psi_axis| (the old psi's values), then
+// the new psi's axis / boundary for the next chained iteration (replaces its k_normalize).  A kernel
+// of its own (one CTA, launched programmatically behind k_dst_inv): the kernel boundary orders the
+// partials, so the update blocks need no fence and no completion ticket.
+__global__ void __launch_bounds__(256) k_dst_fin(const double* __restrict__ eps_part, int nparts,
+                                                 const double* __restrict__ psi_inout, int nw, int nh,
+                                                 double* __restrict__ axbd, double* __restrict__ eps, NextNorm nn) {
+    griddep();
+    __shared__ double wmax[8];
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
     double m = 0.0;
-    for (int b = threadIdx.x; b < (int)gridDim.x; b += blockDim.x) m = fmax(m, __ldcg(eps_part + b));
+    for (int b = threadIdx.x; b < nparts; b += blockDim.x) m = fmax(m, eps_part[b]);
     m = warp_max(m);
     if (l == 0) wmax[w] = m;
     __syncthreads();
@@ -3129,13 +3136,11 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
         double mm = 0.0;
         for (int q = 0; q < (int)(blockDim.x >> 5); ++q) mm = fmax(mm, wmax[q]);
         *eps = mm / fabs(axbd[1] - axbd[0]);
-        *ticket = 0u;
     }
     __syncthreads();
-    // the new psi's axis/boundary for the next chained iteration (replaces its k_normalize)
     if (nn.on)
         normalize_finalize(psi_inout, nw, nh, nn.rmin, nn.dr, nn.zmin, nn.dz, nn.sgn, nn.lim, nn.n_lim, nn.part,
-                           gridDim.x, axbd, nn.status);
+                           nparts, axbd, nn.status);
 }
 
 static void solve_shape(const Ctx& c, int& fpc, int& threads, size_t& smem) {
@@ -3196,9 +3201,12 @@ cudaError_t launch_solve_rest(Ctx& c, const double* psib, double* psi_out, doubl
     nn.rmin = c.rmin; nn.dr = c.dr; nn.zmin = c.zmin; nn.dz = c.dz;
     nn.part = c.norm_part;
     nn.status = c.status;
-    return launch_pdl(k_dst_inv, dim3(nrb + 1), dim3(threads), smem, s, c.fhat, c.fhat_ld, psib, c.nw, c.nh,
-                      c.twiddle, c.fft_m, c.fft_log2, fpc, psi_out, psi_inout, psi_ext, c.eps_part, c.tickets + 1,
-                      c.axbd, eps, nn);
+    e = launch_pdl(k_dst_inv, dim3(nrb + 1), dim3(threads), smem, s, c.fhat, c.fhat_ld, psib, c.nw, c.nh,
+                   c.twiddle, c.fft_m, c.fft_log2, fpc, psi_out, psi_inout, psi_ext, c.eps_part, c.tickets + 1,
+                   c.axbd, eps, nn);
+    if (e || !psi_inout) return e;
+    return launch_pdl(k_dst_fin, dim3(1), dim3(256), 0, s, (const double*)c.eps_part, nrb + 1, (const double*)psi_inout,
+                      c.nw, c.nh, c.axbd, eps, nn);
 }
 
 cudaError_t launch_solve(Ctx& c, const double* pcurr, const double* psib, double* psi_out, double* psi_inout,
