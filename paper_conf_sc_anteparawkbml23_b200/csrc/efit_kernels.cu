@@ -3124,23 +3124,54 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
 __global__ void __launch_bounds__(256) k_dst_fin(const double* __restrict__ eps_part, int nparts,
                                                  const double* __restrict__ psi_inout, int nw, int nh,
                                                  double* __restrict__ axbd, double* __restrict__ eps, NextNorm nn) {
+    // latency-shaped: the limiter vertices (constant) are read before the wait on k_dst_inv; after it,
+    // the eps and argmax partials come in one round trip, the vertex values in a second one
+    __shared__ double wv[8], av[8], bv[8];
+    __shared__ long long ai[8], bi_s[8];
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31, nwarp = blockDim.x >> 5;
+    double lr = 0.0, lz = 0.0;
+    const bool hasv = nn.on && (int)threadIdx.x < nn.n_lim;
+    if (hasv) { lr = nn.lim[threadIdx.x]; lz = nn.lim[nn.n_lim + threadIdx.x]; }
     griddep();
-    __shared__ double wmax[8];
-    const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
-    double m = 0.0;
-    for (int b = threadIdx.x; b < nparts; b += blockDim.x) m = fmax(m, eps_part[b]);
+    const double sg = (double)nn.sgn;
+    double m = 0.0, best = -DBL_MAX;
+    long long bi = LLONG_MAX;
+    for (int b = threadIdx.x; b < nparts; b += blockDim.x) {
+        m = fmax(m, eps_part[b]);
+        if (nn.on) argmax_merge(best, bi, nn.part[2 * b], (long long)nn.part[2 * b + 1]);
+    }
+    // the old axis / boundary (this iteration's eps) before they are replaced below
+    const double pa_old = axbd[0], pb_old = axbd[1];
+    // limiter-vertex values of the new psi (thread v; n_lim <= blockDim handled by the loop below)
+    double vb = -DBL_MAX;
+    long long vi = LLONG_MAX;
+    if (nn.on) {
+        if (hasv) argmax_merge(vb, vi, sg * bilinear(psi_inout, nw, nh, nn.rmin, nn.dr, nn.zmin, nn.dz, lr, lz),
+                               (long long)threadIdx.x);
+        for (int v = threadIdx.x + blockDim.x; v < nn.n_lim; v += blockDim.x)
+            argmax_merge(vb, vi, sg * bilinear(psi_inout, nw, nh, nn.rmin, nn.dr, nn.zmin, nn.dz, nn.lim[v],
+                                               nn.lim[nn.n_lim + v]), (long long)v);
+    }
     m = warp_max(m);
-    if (l == 0) wmax[w] = m;
+    warp_argmax(best, bi);
+    warp_argmax(vb, vi);
+    if (l == 0) { wv[w] = m; av[w] = best; ai[w] = bi; bv[w] = vb; bi_s[w] = vi; }
     __syncthreads();
     if (threadIdx.x == 0) {
-        double mm = 0.0;
-        for (int q = 0; q < (int)(blockDim.x >> 5); ++q) mm = fmax(mm, wmax[q]);
-        *eps = mm / fabs(axbd[1] - axbd[0]);
+        for (int q = 1; q < nwarp; ++q) {
+            m = fmax(m, wv[q]);
+            argmax_merge(best, bi, av[q], ai[q]);
+            argmax_merge(vb, vi, bv[q], bi_s[q]);
+        }
+        *eps = m / fabs(pb_old - pa_old);
+        if (nn.on) {  // as normalize_finalize: the merged values themselves (s times the value)
+            const double pa = (bi == LLONG_MAX) ? 0.0 : sg * best;
+            const double pb = (vi == LLONG_MAX) ? 0.0 : sg * vb;
+            axbd[0] = pa;
+            axbd[1] = pb;
+            if (bi == LLONG_MAX || !(sg * (pa - pb) > 0.0)) atomicOr(nn.status, EFIT_ST_NOPLASMA);
+        }
     }
-    __syncthreads();
-    if (nn.on)
-        normalize_finalize(psi_inout, nw, nh, nn.rmin, nn.dr, nn.zmin, nn.dz, nn.sgn, nn.lim, nn.n_lim, nn.part,
-                           nparts, axbd, nn.status);
 }
 
 static void solve_shape(const Ctx& c, int& fpc, int& threads, size_t& smem) {
