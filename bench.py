@@ -624,7 +624,7 @@ def gpu_arm(args, rank, world, local):
                            "iteration: the diverted Picard loop is vertically unstable (DESIGN.md R4)"}
                           if restore is not None else {}),
                        "parallelism": par,
-                       "l2": (f"tables fit in L2 ({table_bytes / 1e9:.3f} GB boundary + {gd_bytes / 1e9:.3f} GB Gd): value = "
+                       "l2": (f"tables within 2 x L2 ({table_bytes / 1e9:.3f} GB boundary + {gd_bytes / 1e9:.3f} GB Gd): value = "
                               f"cold L2, a 256 MB write before every timed iteration ({flush_ms * 1e3:.1f} us, timed "
                               f"alone and subtracted; each iteration normalises psi first); L2-warm chained "
                               f"iterations: {1000.0 / warm_ms:.1f} it/s" if warm_ms is not None else
