@@ -602,9 +602,9 @@ def gpu_arm(args, rank, world, local):
 
     # our kernels per step (ncu launch list, profiles/): response (basis fused), resp_reduce, lsq,
     # current, lr_fft, lr_mac, lr_ifft, dst_fwd, bnd_tb | (bnd_sym + sym_edge_src), bnd_reduce,
-    # tridiag, dst_inv, dst_fin; + k_normalize at the start of every captured graph
+    # tridiag, dst_inv, norm_fin; + k_normalize and its k_norm_fin at the start of every captured graph
     per_step = 13 + (1 if sym_mode else 0)
-    launches = per_step * K + len(graphs)
+    launches = per_step * K + 2 * len(graphs)
     if full:  # steps_ (5 kernels) before every iteration instead of once per graph
         launches = (per_step + 5) * K
     if rank == 0:

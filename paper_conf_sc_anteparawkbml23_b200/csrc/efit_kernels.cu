@@ -9,7 +9,7 @@
 //   k_bnd_tb      top/bottom targets, T slabs streamed once     (pflux_ 2nd O(N^3) nest) HBM-bound
 //   k_bnd_lr      left/right targets, Toeplitz in registers     (pflux_ Fig. 2 nest)  FP64-bound
 //   k_bnd_reduce  fixed-order partial sums -> psi_b (edge order)
-//   k_dst_fwd / k_tridiag / k_dst_inv / k_dst_fin   interior GS solve + update + eps (pflux_ O(N^2), Eq. (1))
+//   k_dst_fwd / k_tridiag / k_dst_inv / k_norm_fin   interior GS solve + update + eps (pflux_ O(N^2), Eq. (1))
 // Every reduction has a fixed order, so results are bitwise reproducible run to run and
 // independent of the number of ranks.
 #include <cfloat>
@@ -511,58 +511,10 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
 
 // ================================================================================ normalize
 
-// Last-block part of the normalisation (called by exactly one block after all `nparts` block
-// partials (value, index) are visible): psi_axis from the partials, psi_bdry from the limiter
-// vertices, status if there is no plasma.  Uses 256 threads.
-__device__ void normalize_finalize(const double* __restrict__ psi, int nw, int nh, double rmin, double dr,
-                                   double zmin, double dz, int sgn, const double* __restrict__ lim, int n_lim,
-                                   const double* part, int nparts, double* __restrict__ axbd, int* status) {
-    __shared__ double sv[32];
-    __shared__ long long si[32];
-    const double s = (double)sgn;
-    const int w = threadIdx.x >> 5, l = threadIdx.x & 31, nwarp = blockDim.x >> 5;
-    double best = -DBL_MAX;
-    long long bi = LLONG_MAX;
-    for (int b = threadIdx.x; b < nparts; b += blockDim.x) {
-        double v = __ldcg(part + 2 * b);
-        double ix = __ldcg(part + 2 * b + 1);
-        argmax_merge(best, bi, v, (long long)ix);
-    }
-    warp_argmax(best, bi);
-    if (l == 0) { sv[w] = best; si[w] = bi; }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        for (int q = 1; q < nwarp; ++q) argmax_merge(best, bi, sv[q], si[q]);
-        sv[0] = best; si[0] = bi;
-    }
-    __syncthreads();
-    const long long gax = si[0];
-    const double sax = sv[0];  // = s psi[gax] (the partials carry s psi; s = +-1: exact both ways)
-    __syncthreads();
-    double vb = -DBL_MAX;
-    long long vi = LLONG_MAX;
-    for (int v = threadIdx.x; v < n_lim; v += blockDim.x) {
-        double pv = bilinear(psi, nw, nh, rmin, dr, zmin, dz, lim[v], lim[n_lim + v]);
-        argmax_merge(vb, vi, s * pv, (long long)v);
-    }
-    warp_argmax(vb, vi);
-    if (l == 0) { sv[w] = vb; si[w] = vi; }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        for (int q = 1; q < nwarp; ++q) argmax_merge(vb, vi, sv[q], si[q]);
-        // the merged values themselves (s times the value): no second round trip to memory
-        const double pa = (gax == LLONG_MAX) ? 0.0 : s * sax;
-        const double pb = (vi == LLONG_MAX) ? 0.0 : s * vb;
-        axbd[0] = pa;
-        axbd[1] = pb;
-        if (gax == LLONG_MAX || !(s * (pa - pb) > 0.0)) atomicOr(status, EFIT_ST_NOPLASMA);
-    }
-    __syncthreads();
-}
 
 // psi_axis = s * max_{g in limiter} s psi_g (ties: lowest g);  psi_bdry = s * max over limiter
-// vertices of s * bilinear(psi) (ties: lowest vertex).  Last-block pattern: the final block
-// combines the per-block partials; `ticket` returns to 0 for the next launch.
+// vertices of s * bilinear(psi) (ties: lowest vertex).  Per-block (value, index) partials here; the
+// one-CTA k_norm_fin behind it merges them and evaluates the limiter vertices.
 __global__ void __launch_bounds__(256) k_normalize(const double* __restrict__ psi, const uint8_t* __restrict__ inlim,
                                                    int nw, int nh, double rmin, double dr, double zmin, double dz,
                                                    int sgn, const double* __restrict__ lim, int n_lim,
@@ -571,7 +523,6 @@ __global__ void __launch_bounds__(256) k_normalize(const double* __restrict__ ps
     griddep();
     __shared__ double sv[8];
     __shared__ long long si[8];
-    __shared__ bool last;
     const int n = nw * nh;
     const double s = (double)sgn;
     double best = -DBL_MAX;
@@ -594,23 +545,19 @@ __global__ void __launch_bounds__(256) k_normalize(const double* __restrict__ ps
         for (int q = 1; q < (int)(blockDim.x >> 5); ++q) argmax_merge(best, bi, sv[q], si[q]);
         part[2 * blockIdx.x] = best;
         part[2 * blockIdx.x + 1] = (double)bi;
-        __threadfence();
-        unsigned t = atomicAdd(ticket, 1u);
-        last = (t == gridDim.x - 1);
     }
-    __syncthreads();
-    if (!last) return;
-    __threadfence();
-    normalize_finalize(psi, nw, nh, rmin, dr, zmin, dz, sgn, lim, n_lim, part, gridDim.x, axbd, status);
-    if (threadIdx.x == 0) *ticket = 0u;
 }
+
+static cudaError_t launch_norm_fin(Ctx& c, const double* psi, int nparts, const double* eps_part, double* eps,
+                                   cudaStream_t s);  // after k_norm_fin below
 
 cudaError_t launch_normalize(Ctx& c, const double* psi, cudaStream_t s) {
     if (c.steps) return launch_steps(c, psi, s);
-    launch_pdl(k_normalize, dim3(c.t.red_blocks), dim3(256), 0, s, psi, c.inlim, c.nw, c.nh, c.rmin, c.dr, c.zmin, c.dz,
-                                               c.ip_sign, c.lim, c.n_lim, c.norm_part, c.tickets + 0,
-                                               c.axbd, c.status);
-    return cudaGetLastError();
+    cudaError_t e = launch_pdl(k_normalize, dim3(c.t.red_blocks), dim3(256), 0, s, psi, c.inlim, c.nw, c.nh, c.rmin,
+                               c.dr, c.zmin, c.dz, c.ip_sign, c.lim, c.n_lim, c.norm_part, c.tickets + 0, c.axbd,
+                               c.status);
+    if (e) return e;
+    return launch_norm_fin(c, psi, c.t.red_blocks, nullptr, nullptr, s);
 }
 
 static BasisParams basis_params(const Ctx& c) {
@@ -3117,11 +3064,12 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
     }
 }
 
-// eps = max over the k_dst_inv blocks' partials / |psi_bdry - psi_axis| (the old psi's values), then
-// the new psi's axis / boundary for the next chained iteration (replaces its k_normalize).  A kernel
-// of its own (one CTA, launched programmatically behind k_dst_inv): the kernel boundary orders the
-// partials, so the update blocks need no fence and no completion ticket.
-__global__ void __launch_bounds__(256) k_dst_fin(const double* __restrict__ eps_part, int nparts,
+// Finish of an axis / boundary search (one CTA, launched programmatically behind the partials'
+// producer, so the producer's blocks need no fence and no completion ticket):
+//   behind k_dst_inv: eps = max over its blocks' partials / |psi_bdry - psi_axis| (the old values),
+//     then the new psi's axis / boundary for the next chained iteration;
+//   behind k_normalize (eps_part = eps = nullptr): psi_axis / psi_bdry of the given psi.
+__global__ void __launch_bounds__(256) k_norm_fin(const double* __restrict__ eps_part, int nparts,
                                                  const double* __restrict__ psi_inout, int nw, int nh,
                                                  double* __restrict__ axbd, double* __restrict__ eps, NextNorm nn) {
     // latency-shaped: the limiter vertices (constant) are read before the wait on k_dst_inv; after it,
@@ -3137,11 +3085,11 @@ __global__ void __launch_bounds__(256) k_dst_fin(const double* __restrict__ eps_
     double m = 0.0, best = -DBL_MAX;
     long long bi = LLONG_MAX;
     for (int b = threadIdx.x; b < nparts; b += blockDim.x) {
-        m = fmax(m, eps_part[b]);
+        if (eps_part) m = fmax(m, eps_part[b]);
         if (nn.on) argmax_merge(best, bi, nn.part[2 * b], (long long)nn.part[2 * b + 1]);
     }
     // the old axis / boundary (this iteration's eps) before they are replaced below
-    const double pa_old = axbd[0], pb_old = axbd[1];
+    const double pa_old = eps ? axbd[0] : 0.0, pb_old = eps ? axbd[1] : 0.0;
     // limiter-vertex values of the new psi (thread v; n_lim <= blockDim handled by the loop below)
     double vb = -DBL_MAX;
     long long vi = LLONG_MAX;
@@ -3163,8 +3111,8 @@ __global__ void __launch_bounds__(256) k_dst_fin(const double* __restrict__ eps_
             argmax_merge(best, bi, av[q], ai[q]);
             argmax_merge(vb, vi, bv[q], bi_s[q]);
         }
-        *eps = m / fabs(pb_old - pa_old);
-        if (nn.on) {  // as normalize_finalize: the merged values themselves (s times the value)
+        if (eps) *eps = m / fabs(pb_old - pa_old);
+        if (nn.on) {  // psi_axis / psi_bdry: the merged values themselves (s times the value), rule Q9
             const double pa = (bi == LLONG_MAX) ? 0.0 : sg * best;
             const double pb = (vi == LLONG_MAX) ? 0.0 : sg * vb;
             axbd[0] = pa;
@@ -3172,6 +3120,25 @@ __global__ void __launch_bounds__(256) k_dst_fin(const double* __restrict__ eps_
             if (bi == LLONG_MAX || !(sg * (pa - pb) > 0.0)) atomicOr(nn.status, EFIT_ST_NOPLASMA);
         }
     }
+}
+
+static NextNorm next_norm_args(const Ctx& c, bool on) {
+    NextNorm nn;
+    nn.on = on ? 1 : 0;
+    nn.sgn = c.ip_sign;
+    nn.n_lim = c.n_lim;
+    nn.inlim = c.inlim;
+    nn.lim = c.lim;
+    nn.rmin = c.rmin; nn.dr = c.dr; nn.zmin = c.zmin; nn.dz = c.dz;
+    nn.part = c.norm_part;
+    nn.status = c.status;
+    return nn;
+}
+
+static cudaError_t launch_norm_fin(Ctx& c, const double* psi, int nparts, const double* eps_part, double* eps,
+                                   cudaStream_t s) {
+    return launch_pdl(k_norm_fin, dim3(1), dim3(256), 0, s, eps_part, nparts, psi, c.nw, c.nh, c.axbd, eps,
+                      next_norm_args(c, true));
 }
 
 static void solve_shape(const Ctx& c, int& fpc, int& threads, size_t& smem) {
@@ -3223,20 +3190,12 @@ cudaError_t launch_solve_rest(Ctx& c, const double* psib, double* psi_out, doubl
                            c.tri_alpha, c.tri_inv, c.tri_cp, c.ni, L, c.nmode, fx);
     }
     if (e) return e;
-    NextNorm nn;
-    nn.on = (next_norm && psi_inout && !c.steps) ? 1 : 0;  // f3: steps_ runs before every iteration
-    nn.sgn = c.ip_sign;
-    nn.n_lim = c.n_lim;
-    nn.inlim = c.inlim;
-    nn.lim = c.lim;
-    nn.rmin = c.rmin; nn.dr = c.dr; nn.zmin = c.zmin; nn.dz = c.dz;
-    nn.part = c.norm_part;
-    nn.status = c.status;
+    const NextNorm nn = next_norm_args(c, next_norm && psi_inout && !c.steps);  // f3: steps_ before every iteration
     e = launch_pdl(k_dst_inv, dim3(nrb + 1), dim3(threads), smem, s, c.fhat, c.fhat_ld, psib, c.nw, c.nh,
                    c.twiddle, c.fft_m, c.fft_log2, fpc, psi_out, psi_inout, psi_ext, c.eps_part, c.tickets + 1,
                    c.axbd, eps, nn);
     if (e || !psi_inout) return e;
-    return launch_pdl(k_dst_fin, dim3(1), dim3(256), 0, s, (const double*)c.eps_part, nrb + 1, (const double*)psi_inout,
+    return launch_pdl(k_norm_fin, dim3(1), dim3(256), 0, s, (const double*)c.eps_part, nrb + 1, (const double*)psi_inout,
                       c.nw, c.nh, c.axbd, eps, nn);
 }
 
