@@ -456,7 +456,7 @@ extern "C" int efit_green_init(efit_ctx** out, const efit_grid* grid, const efit
     c.side = nullptr; c.ev_fork = nullptr; c.ev_join = nullptr;
     int prio_lo = 0, prio_hi = 0;
     cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
-    if ((e = cudaStreamCreateWithPriority(&c.side, cudaStreamNonBlocking, prio_hi)) ||
+    if ((e = cudaStreamCreateWithPriority(&c.side, cudaStreamNonBlocking, getenv("EFIT_SIDE_LOPRIO") ? prio_lo : prio_hi)) ||
         (e = cudaEventCreateWithFlags(&c.ev_fork, cudaEventDisableTiming)) ||
         (e = cudaEventCreateWithFlags(&c.ev_join, cudaEventDisableTiming))) {
         if (c.side) cudaStreamDestroy(c.side);
