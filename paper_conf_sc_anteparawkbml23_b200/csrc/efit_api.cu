@@ -383,6 +383,12 @@ static size_t carve(Ctx& c, char* base) {
     return carve_scratch(c, take, off, false);
 }
 
+// Captured graphs keep the priorities of the streams their kernels were enqueued on: the left/right
+// chain and the forward DST run on the high-priority side stream so that their CTAs are placed
+// between the waves of the table stream (without this flag every node takes the launch stream's
+// priority and the side chain is starved: 196 instead of 179 us per C4 iteration).
+static constexpr unsigned long long kGraphFlags = cudaGraphInstantiateFlagUseNodePriority;
+
 static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 
 extern "C" int efit_workspace_bytes(const efit_grid* grid, const efit_basis* basis, const efit_geometry* geom,
@@ -839,7 +845,7 @@ static int fit_steps_impl(efit_ctx* h, int32_t nsteps, double* d_psi, const doub
         e = cudaStreamEndCapture(s, &graph);
         if (e2) { if (graph) cudaGraphDestroy(graph); return cuda_fail(&c, e2, "fit step capture"); }
         if (e) return cuda_fail(&c, e, "end capture");
-        e = cudaGraphInstantiateWithFlags(&c.gexec[slot], graph, 0);
+        e = cudaGraphInstantiateWithFlags(&c.gexec[slot], graph, kGraphFlags);
         cudaGraphDestroy(graph);
         if (e) { c.gexec[slot] = nullptr; return cuda_fail(&c, e, "graph instantiate"); }
         std::memcpy(c.gkey[slot], key, sizeof(key));
@@ -901,7 +907,7 @@ static int fit_host_graphs(efit_ctx* h, int32_t nslice, int32_t iters, const dou
                 cudaGraphAddMemcpyNode1D(&nd7[4], g, nd7, 4, o.psi, h_psi0, sizeof(double) * n, cudaMemcpyHostToDevice) == cudaSuccess &&
                 cudaGraphAddMemcpyNode1D(&nd7[5], g, nd7, 4, o.meas, h_meas, sizeof(double) * nd, cudaMemcpyHostToDevice) == cudaSuccess &&
                 cudaGraphAddMemcpyNode1D(&nd7[6], g, nd7, 4, o.sigma, h_sigma, sizeof(double) * nd, cudaMemcpyHostToDevice) == cudaSuccess &&
-                cudaGraphInstantiateWithFlags(&c.hgexec[b], g, 0) == cudaSuccess;
+                cudaGraphInstantiateWithFlags(&c.hgexec[b], g, kGraphFlags) == cudaSuccess;
             c.hgraph[b] = g;
             if (!ok) {
                 cudaGetLastError();
@@ -1230,7 +1236,7 @@ static int fit_steps_batch_impl(efit_ctx* h, int32_t nsteps, double* d_psi, cons
         e = cudaStreamEndCapture(s, &graph);
         if (e2) { if (graph) cudaGraphDestroy(graph); return cuda_fail(&c, e2, "batched fit step capture"); }
         if (e) return cuda_fail(&c, e, "end capture");
-        e = cudaGraphInstantiateWithFlags(&c.bexec, graph, 0);
+        e = cudaGraphInstantiateWithFlags(&c.bexec, graph, kGraphFlags);
         cudaGraphDestroy(graph);
         if (e) { c.bexec = nullptr; return cuda_fail(&c, e, "graph instantiate"); }
         std::memcpy(c.bkey, key, sizeof(key));
