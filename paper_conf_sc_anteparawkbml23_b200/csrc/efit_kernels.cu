@@ -518,8 +518,7 @@ cudaError_t launch_init_tables(Ctx& c, cudaStream_t s) {
 __global__ void __launch_bounds__(256) k_normalize(const double* __restrict__ psi, const uint8_t* __restrict__ inlim,
                                                    int nw, int nh, double rmin, double dr, double zmin, double dz,
                                                    int sgn, const double* __restrict__ lim, int n_lim,
-                                                   double* __restrict__ part, unsigned* ticket,
-                                                   double* __restrict__ axbd, int* status) {
+                                                   double* __restrict__ part, int* status) {
     griddep();
     __shared__ double sv[8];
     __shared__ long long si[8];
@@ -554,8 +553,7 @@ static cudaError_t launch_norm_fin(Ctx& c, const double* psi, int nparts, const 
 cudaError_t launch_normalize(Ctx& c, const double* psi, cudaStream_t s) {
     if (c.steps) return launch_steps(c, psi, s);
     cudaError_t e = launch_pdl(k_normalize, dim3(c.t.red_blocks), dim3(256), 0, s, psi, c.inlim, c.nw, c.nh, c.rmin,
-                               c.dr, c.zmin, c.dz, c.ip_sign, c.lim, c.n_lim, c.norm_part, c.tickets + 0, c.axbd,
-                               c.status);
+                               c.dr, c.zmin, c.dz, c.ip_sign, c.lim, c.n_lim, c.norm_part, c.status);
     if (e) return e;
     return launch_norm_fin(c, psi, c.t.red_blocks, nullptr, nullptr, s);
 }
@@ -2918,12 +2916,10 @@ __global__ void __launch_bounds__(512) k_dst_inv(const double* __restrict__ fhat
                                                  int nw, int nh, const double2* __restrict__ W, int M, int log2m,
                                                  int FPC, double* __restrict__ psi_out, double* __restrict__ psi_inout,
                                                  const double* __restrict__ psi_ext, double* __restrict__ eps_part,
-                                                 unsigned* ticket, double* __restrict__ axbd,
-                                                 double* __restrict__ eps, NextNorm nn) {
+                                                 NextNorm nn) {
     extern __shared__ __align__(16) double2 a2[];  // FPC x ([M] data, [M] scratch), then [M/2] twiddles
     double2* Ws = a2 + 2 * FPC * M;
     __shared__ double wmax[16];
-    __shared__ bool last;
     const int n = nh - 2, ni = nw - 2;
     const int nrb = (ni + 2 * FPC - 1) / (2 * FPC);  // row blocks; block nrb does the edge rows
     const int TPF = blockDim.x / FPC;
@@ -3192,8 +3188,7 @@ cudaError_t launch_solve_rest(Ctx& c, const double* psib, double* psi_out, doubl
     if (e) return e;
     const NextNorm nn = next_norm_args(c, next_norm && psi_inout && !c.steps);  // f3: steps_ before every iteration
     e = launch_pdl(k_dst_inv, dim3(nrb + 1), dim3(threads), smem, s, c.fhat, c.fhat_ld, psib, c.nw, c.nh,
-                   c.twiddle, c.fft_m, c.fft_log2, fpc, psi_out, psi_inout, psi_ext, c.eps_part, c.tickets + 1,
-                   c.axbd, eps, nn);
+                   c.twiddle, c.fft_m, c.fft_log2, fpc, psi_out, psi_inout, psi_ext, c.eps_part, nn);
     if (e || !psi_inout) return e;
     return launch_pdl(k_norm_fin, dim3(1), dim3(256), 0, s, (const double*)c.eps_part, nrb + 1, (const double*)psi_inout,
                       c.nw, c.nh, c.axbd, eps, nn);
