@@ -1203,8 +1203,10 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
     }
     __syncthreads();
     if (s_shift) {  // cond(A) beyond ~1e8: shifted CholeskyQR3 (see above)
-        lsq_gram(A, ld, nd, nb, G);
-        __syncthreads();
+        if (NBT == 0) {  // lsq_chol factorised G in place: form it again (lsq_chol_warp only read it)
+            lsq_gram(A, ld, nd, nb, G);
+            __syncthreads();
+        }
         if (warp == 0) {
             const double shift = 11.0 * ((double)nd * nb + (double)nb * (nb + 1)) * 0x1p-53 * nb;
             for (int k = lane; k < nb; k += 32) G[k * nb + k] += shift;
