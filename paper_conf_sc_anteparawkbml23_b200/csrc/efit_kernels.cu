@@ -1110,12 +1110,18 @@ __device__ __forceinline__ bool lsq_chol_warp(const double* G, double* R, double
     double g[NB];
 #pragma unroll
     for (int j = 0; j < NB; ++j) g[j] = lane < NB ? G[lane * NB + j] : 0.0;
-#pragma unroll
+    // the pivot loop is not unrolled: one copy of the step's code, reused NB times (an unrolled NB = 20
+    // factorisation is ~2.5k instructions executed once per iteration, fetched cold: ~100k cycles);
+    // g[k] (runtime k) is selected from the register array, the update predicated on j > k
+#pragma unroll 1
     for (int k = 0; k < NB; ++k) {
-        const double d = __shfl_sync(0xffffffffu, g[k], k);
+        double gk = 0.0;
+#pragma unroll
+        for (int j = 0; j < NB; ++j) gk = (j == k) ? g[j] : gk;
+        const double d = __shfl_sync(0xffffffffu, gk, k);
         if (!(d > 0.0)) return false;
         const double r = sqrt(d), ir = 1.0 / r;
-        const double rki = g[k] * ir;  // R[k][lane] for lane > k
+        const double rki = gk * ir;  // R[k][lane] for lane > k
         if (lane == k) {
             R[k * NB + k] = r;
             rinv[k] = ir;
@@ -1123,9 +1129,9 @@ __device__ __forceinline__ bool lsq_chol_warp(const double* G, double* R, double
             R[k * NB + lane] = rki;
         }
 #pragma unroll
-        for (int j = k + 1; j < NB; ++j) {
+        for (int j = 0; j < NB; ++j) {
             const double rkj = __shfl_sync(0xffffffffu, rki, j);
-            g[j] = g[j] - rki * rkj;
+            if (j > k) g[j] = g[j] - rki * rkj;
         }
     }
     __syncwarp();
@@ -1255,26 +1261,27 @@ __global__ void __launch_bounds__(256) k_lsq(const double* __restrict__ resp, co
         const int j = lane;
         const bool act = j < NBC;
         double zj = act ? z[j] : 0.0;
-#pragma unroll
+        // step loops not unrolled (code reuse; see lsq_chol_warp)
+#pragma unroll 1
         for (int i = 0; i < NBC; ++i) {  // z <- R2^-T z
             const double zi = __shfl_sync(0xffffffffu, zj, i) * r2i[i];
             if (j == i) zj = zi;
             else if (act && j > i) zj = fma(-R2[i * NBC + j], zi, zj);
         }
-#pragma unroll
+#pragma unroll 1
         for (int k = NBC - 1; k >= 0; --k) {  // z <- R2^-1 z
             const double zk = __shfl_sync(0xffffffffu, zj, k) * r2i[k];
             if (j == k) zj = zk;
             else if (j < k) zj = fma(-R2[j * NBC + k], zk, zj);
         }
-#pragma unroll
+#pragma unroll 1
         for (int k = NBC - 1; k >= 0; --k) {  // z <- R1^-1 z
             const double zk = __shfl_sync(0xffffffffu, zj, k) * r1i[k];
             if (j == k) zj = zk;
             else if (j < k) zj = fma(-R1[j * NBC + k], zk, zj);
         }
         if (s_shift) {
-#pragma unroll
+#pragma unroll 1
             for (int k = NBC - 1; k >= 0; --k) {  // z <- R0^-1 z
                 const double zk = __shfl_sync(0xffffffffu, zj, k) * r0i[k];
                 if (j == k) zj = zk;
