@@ -161,6 +161,29 @@ def test_minimum_grid_and_no_plasma(torch_mod, efit, orc_mod):
     ctx5.close()
 
 
+@pytest.mark.parametrize("kind", ["diverted", "diverted_perturbed"])
+def test_c5_normalize_bitwise_global_bitmap(torch_mod, efit, orc_mod, kind):
+    """1025^2 (C5): the candidate bitmap no longer fits in shared memory next to the component, so the
+    flood fill reads it from global memory (k_steps_fill<false>); same bit-for-bit agreement.  An
+    on-the-fly Green's context (no table to build): steps_ does not depend on the Green's mode."""
+    torch = torch_mod
+    cfg = synth.config("C5")
+    orc = orc_mod.Oracle.from_config(cfg)
+    orc.set_steps_mode(1)
+    psi = _psi(kind, cfg.grid)
+    cnt, pa, pb, mask, _ = orc.normalize(psi)
+    oinfo = orc.steps_info()
+    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=efit.EFIT_GREEN_ONTHEFLY_SYM)
+    ctx.set_steps(efit.EFIT_STEPS_FULL)
+    info, gmask = ctx.normalize(T(torch, psi))
+    torch.cuda.synchronize()
+    assert ctx.status() == 0 and cnt > 0
+    assert np.array_equal(gmask.cpu().numpy(), mask)
+    _same_info(info.cpu().numpy(), oinfo)
+    assert oinfo[12] == 1.0
+    ctx.close()
+
+
 def test_limiter_mode_normalize_matches_o8(torch_mod, efit, orc_mod):
     torch = torch_mod
     cfg = synth.small_config(65)
