@@ -184,6 +184,42 @@ def test_c5_normalize_bitwise_global_bitmap(torch_mod, efit, orc_mod, kind):
     ctx.close()
 
 
+def test_fit_host_full_steps_matches_device(torch_mod, efit, orc_mod):
+    """The host-buffer pipeline (efit_fit_host) under the full steps_ rule equals efit_fit_steps on
+    device buffers slice by slice, bit for bit (every iteration normalises under the rule)."""
+    torch = torch_mod
+    cfg = synth.small_config(129)
+    orc = orc_mod.Oracle.from_config(cfg)
+    orc.set_steps_mode(1)
+    psi_s = synth.solovev_diverted_psi(cfg.grid)
+    ct = synth.c_true(cfg.basis, sol_c=synth.DIV_C)
+    tw = orc.twin(psi_s, ct, noise_seed=1)
+    ctx = efit.EfitContext(cfg.grid, cfg.basis, cfg.geometry, mode=efit.EFIT_GREEN_TABLE_SYM)
+    ctx.set_steps(efit.EFIT_STEPS_FULL)
+    S, iters, n, nb = 3, 2, cfg.grid.n, ctx.nbasis
+    starts = [psi_s + 1e-4 * (k + 1) * (psi_s.max() - psi_s.min()) * synth.smooth_modes(cfg.grid, 5 + k) / 3.0
+              for k in range(S)]
+    ext = T(torch, tw["psi_ext"])
+    h_psi0 = torch.tensor(np.concatenate(starts)).pin_memory()
+    h_meas = torch.tensor(np.tile(tw["y"], S)).pin_memory()
+    h_sig = torch.tensor(np.tile(tw["sigma"], S)).pin_memory()
+    outs = [torch.empty(S * n, dtype=torch.float64).pin_memory(), torch.empty(S * nb, dtype=torch.float64).pin_memory(),
+            torch.empty(S, dtype=torch.float64).pin_memory(), torch.empty(S, dtype=torch.float64).pin_memory()]
+    st = torch.cuda.Stream()
+    for _ in range(2):
+        ctx.fit_host(S, iters, h_psi0, h_meas, h_sig, ext, *outs, stream=st)
+        st.synchronize()
+    assert ctx.status() == 0
+    for k in range(S):
+        psi = T(torch, starts[k])
+        coef, chi2, eps = ctx._t(nb), ctx._t(1), ctx._t(1)
+        ctx.fit_steps(iters, psi, ext, T(torch, tw["y"]), T(torch, tw["sigma"]), coef, chi2, eps)
+        torch.cuda.synchronize()
+        assert torch.equal(outs[0][k * n:(k + 1) * n], psi.cpu()), k
+        assert torch.equal(outs[1][k * nb:(k + 1) * nb], coef.cpu()), k
+    ctx.close()
+
+
 def test_limiter_mode_normalize_matches_o8(torch_mod, efit, orc_mod):
     torch = torch_mod
     cfg = synth.small_config(65)
