@@ -235,10 +235,10 @@ int efit_interior_solve(efit_ctx* ctx, const double* d_pcurr, const double* d_ps
  *                                 upper X-point heights, lower X-point, upper X-point}; mask = the
  *                                 4-connected component of the axis node in {in-limiter, 0 <= psihat < 1}
  *                                 (private-flux regions excluded).  Every decision is plain IEEE fp64 in
- *                                 the reading's order (bit-reproducible).  Adds three launches per
+ *                                 the reading's order (bit-reproducible).  Adds five launches per
  *                                 iteration (the chained fit steps then normalise before every iteration).
- *                                 Needs 6 <= nw, nh and nw * ceil(nh/32) * 4 bytes of bitmap in shared
- *                                 memory (up to ~1025^2).  Applies to the attached batch slices too
+ *                                 Needs 6 <= nw, nh <= 2048 and nw * ceil(nh/64) * 8 bytes of component
+ *                                 bitmap in shared memory (up to ~1025^2).  Applies to the attached batch slices too
  *                                 (each slice normalises its own psi).
  * efit_set_steps: host-only switch (drops the cached fit-step graphs); EFIT_E_INVAL for a bad mode or
  *   a grid outside the limits above. */
