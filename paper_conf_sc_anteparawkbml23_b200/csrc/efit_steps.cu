@@ -10,12 +10,13 @@
 // This translation unit is compiled with -fmad=false: every floating-point expression below is a
 // sequence of plain IEEE fp64 operations in the written order (that of the reading), so every
 // discrete decision (candidate test, Newton acceptance, boundary choice, mask bit) is reproducible
-// bit for bit.  Three launches per normalisation:
-//   k_steps_scan   all CTAs: in-limiter argmax partials of s psi + X-point candidate list;
-//                  the last CTA: axis / X-point Newton searches, limiter value, boundary
-//   k_steps_bits   candidate bitmap {inlim, 0 <= psihat < 1}, one 32-bit word per warp (ballot)
+// bit for bit.  Five launches per normalisation (each programmatically behind its predecessor):
+//   k_steps_scan   all CTAs: in-limiter argmax partials of s psi + X-point candidate list
+//   k_steps_final  one CTA: axis / X-point Newton searches (one warp each), limiter value, boundary
+//   k_steps_bits   candidate bitmap {inlim, 0 <= psihat < 1}, 64-bit words (two ballots per warp)
 //   k_steps_fill   one CTA: bit-parallel flood fill from the axis node in shared memory (row runs by
-//                  carry propagation, column runs by a segmented scan), then the byte mask
+//                  carry propagation, column runs by a segmented warp scan, dirty rows / columns only)
+//   k_steps_mask   the component as the byte mask read by the basis / response / current kernels
 #include <cuda_runtime.h>
 #include <float.h>
 #include <limits.h>
