@@ -296,6 +296,10 @@ static void plan(Ctx& c, const efit_grid* g, const efit_basis* b, const efit_geo
         if (cost < best_cost) { best_cost = cost; best_mb = mb; }
     }
     t.resp_mb = best_mb;
+    if (const char* ev = getenv("EFIT_RESP_MB")) {  // tuning override (1..4)
+        const int mb = atoi(ev);
+        if (mb >= 1 && mb <= 4) t.resp_mb = mb;
+    }
 }
 
 // Per-iteration scratch (also the whole of a batch slice context).  batch: tb_part sized for the
