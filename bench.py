@@ -578,11 +578,19 @@ def gpu_arm(args, rank, world, local):
             except Exception:
                 flops = None
         fp64_peak = 148 * 64 * 2 * 1.965e9 / 1e12
+        fp64_src = "derived from unit counts (148 SMs x 64 FP64 FMA/clk x 2 x 1.965 GHz)"
+        pk = os.path.join(ROOT, "profiles", "fp64_peak.json")
+        if os.path.exists(pk):  # measured DFMA throughput on this pool (scripts/ubench/fp64_peak.cu)
+            try:
+                fp64_peak = float(json.load(open(pk))["fp64_tflops"])
+                fp64_src = "measured: profiles/fp64_peak.json (scripts/ubench/fp64_peak.cu, DFMA throughput)"
+            except Exception:
+                pass
         tf = flops / (tb_ms * 1e-3) / 1e12 if flops else None
         roof = {"kernel": key.replace("_otf", "") + " (on-the-fly)", "bound": "alu",
                 "achieved": round(tf, 2) if tf else None, "peak": round(fp64_peak, 2), "unit": "TFLOP/s",
                 "frac": round(tf / fp64_peak, 4) if tf else None, "traffic": None,
-                "peak_source": "derived from unit counts (no measured FP64 peak)",
+                "peak_source": fp64_src,
                 "fp64_flops_per_launch": flops}
     rb = None
     if rb_ms is not None:
